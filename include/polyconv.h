@@ -1,0 +1,170 @@
+/*
+ * polyconv.h — C-ABI of the B200 (sm_100a) PolyHankel forward convolution.
+ *
+ * The operation (PAPER.md = Xu et al., CGO'25; cited as P.<lines>):
+ *   y[n][k][oh][ow] = sum_c sum_i sum_j xpad[n][c][sh*oh+i][sw*ow+j] * w[k][c][i][j]
+ * computed as polynomial multiplication (§2.2):
+ *   A_{n,c}(t): the zero-padded input plane flattened row-major with row pitch
+ *               Wp = W + 2*pw  (Eq. 4, P.603-613; Eq. 10, P.941-950);
+ *   U_{k,c}(t): the reversed, gap-padded filter, coefficient of degree
+ *               e(i,j) = Wp*(R-1-i) + (S-1-j)  (Eq. 6, P.768-771; Eq. 11
+ *               P.954-964 as corrected in DESIGN.md reading R1; P.1365-1382);
+ *   p_{n,k}(t) = sum_c A_{n,c}(t) U_{k,c}(t)  (P.965; channel sum P.1350-1352);
+ *   y[n][k][oh][ow] = coefficient Wp*sh*oh + sw*ow + L_U - 1 of p_{n,k}
+ *               (Eq. 12, P.966-972; stride: DESIGN.md reading R4),
+ *   with L_A = Hp*Wp, L_U = (R-1)*Wp + S (KernelSize, P.1378-1380).
+ * Only the coefficients at the extraction degrees are computed.
+ *
+ * Problem parameters follow the paper's Table 1 (P.259-271): N, C, Ih=H,
+ * Iw=W, K, Kh=R, Kw=S, padding; "the same API design ... as cuDNN"
+ * (P.1444-1445).  Stride is an extension (reading R4).
+ *
+ * Conventions for every entry point:
+ *  - Tensors are plain device pointers, dense and contiguous:
+ *      x: [N][C][H][W]  w: [K][C][R][S]  y: [N][K][P][Q]  (NCHW, row-major),
+ *    element type = the plan's io dtype (fp32 or bf16), 16-byte aligned,
+ *    owned by the caller, on the plan's device.  y must not alias x or w.
+ *  - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
+ *    All work is enqueued asynchronously on it; no call synchronises except
+ *    polyconv_destroy.
+ *  - Errors are returned as polyconv_status_t; the library never aborts or
+ *    exits.  Argument errors are detected before any allocation or launch.
+ *  - A plan owns its device workspace (packed operands, tensor maps).  Calls on
+ *    one plan must be stream-ordered (one forward at a time).  Plans are not
+ *    thread-safe; different plans are independent.
+ */
+#ifndef POLYCONV_H_
+#define POLYCONV_H_
+
+#include <stddef.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define POLYCONV_ABI_VERSION 1
+
+typedef struct polyconv_plan_s *polyconv_plan_t; /* opaque, library-owned */
+
+typedef enum {
+    POLYCONV_STATUS_SUCCESS = 0,
+    POLYCONV_STATUS_BAD_PARAM = 1,        /* NULL pointer, dim < 1, stride < 1, pad < 0,
+                                             P < 1 or Q < 1, bad enum, unsupported combo */
+    POLYCONV_STATUS_NOT_SUPPORTED = 2,    /* no sm_100 device, tensor > 2^31 elements,
+                                             misaligned pointer, forced kernel cannot run */
+    POLYCONV_STATUS_ALLOC_FAILED = 3,     /* workspace cudaMalloc failed */
+    POLYCONV_STATUS_EXECUTION_FAILED = 4  /* CUDA launch/runtime error; see polyconv_last_error */
+} polyconv_status_t;
+
+/* Element type of x, w and y. */
+typedef enum { POLYCONV_F32 = 0, POLYCONV_BF16 = 1 } polyconv_dtype_t;
+
+/* Arithmetic of the coefficient multiply-accumulate (all accumulate in fp32).
+ *   FP32_FMA: fp32 operands, SIMT FFMA           (parity gate 1e-5 normwise)
+ *   TF32:     operands rounded fp32->tf32 (RNA) in packing, tcgen05 kind::tf32
+ *   BF16:     operands rounded fp32->bf16 (RNE) in packing, tcgen05 kind::f16
+ * io_dtype BF16 requires math BF16. */
+typedef enum {
+    POLYCONV_MATH_FP32_FMA = 0,
+    POLYCONV_MATH_TF32 = 1,
+    POLYCONV_MATH_BF16 = 2
+} polyconv_math_t;
+
+/* MAC kernel variant.  AUTO picks by shape and math; the others force one
+ * (ablations/tests).  TC = tcgen05/TMEM tensor-core contraction; FP32 = SIMT
+ * register-blocked FFMA; THIN = warp-per-output with shuffle reduction over
+ * C*R*S (tiny channel counts). */
+typedef enum {
+    POLYCONV_KERNEL_AUTO = 0,
+    POLYCONV_KERNEL_TC = 1,
+    POLYCONV_KERNEL_FP32 = 2,
+    POLYCONV_KERNEL_THIN = 3
+} polyconv_kernel_t;
+
+/* Packed-operand layouts exposed for bit-exact tests (a2/a3):
+ *   PLANAR      input:  [N][C][L_A]      A_{n,c}(t) coefficient vectors (Eq. 10)
+ *               filter: [K][C][L_U]      U_{k,c}(t) coefficient vectors (Eq. 11, R1)
+ *   INTERLEAVED input:  [N*L_A][Cp]      coefficient-major, channels innermost
+ *                                        (the tensor-core B/A operand layout)
+ *               filter: [R*S][Kp][Cp]    tap-major, channels innermost
+ * Storage words are the math mode's operand format: fp32 words (FP32_FMA),
+ * tf32-in-32-bit words with the low 13 bits zero (TF32), or bf16 (BF16).
+ * Cp/Kp are C/K rounded up as reported by polyconv_plan_info. */
+typedef enum { POLYCONV_LAYOUT_PLANAR = 0, POLYCONV_LAYOUT_INTERLEAVED = 1 } polyconv_layout_t;
+
+typedef struct {
+    int N, C, H, W, K, R, S, sh, sw, ph, pw;
+    int P, Q;          /* output height/width */
+    int Hp, Wp;        /* padded input height/width */
+    long long L_A;     /* input polynomial length Hp*Wp */
+    long long L_U;     /* kernel polynomial length (R-1)*Wp + S */
+    int Cp, Kp;        /* padded channel counts of the INTERLEAVED layouts */
+    int kernel;        /* polyconv_kernel_t the forward will run */
+    int tile_m, tile_n, stages; /* MAC tiling: positions x output channels, smem stages */
+    int launches;      /* kernel launches per polyconv_forward */
+    size_t workspace_bytes; /* device workspace the plan allocates at first use */
+} polyconv_info_t;
+
+/* Create a plan.  Validates every argument (no CUDA call happens on error).
+ * Device resources are allocated lazily at the first call that needs them,
+ * so planning works without a GPU (host-side tests).
+ *   N,C,H,W: x shape; K,R,S: w shape [K][C][R][S]; sh,sw >= 1; ph,pw >= 0;
+ *   io_dtype/math: see above; device: CUDA ordinal the pointers live on. */
+polyconv_status_t polyconv_plan(polyconv_plan_t *plan, int N, int C, int H, int W,
+                                int K, int R, int S, int stride_h, int stride_w,
+                                int pad_h, int pad_w, polyconv_dtype_t io_dtype,
+                                polyconv_math_t math, int device);
+
+/* Force a MAC variant (default AUTO).  BAD_PARAM if the variant cannot run
+ * this plan's math mode (TC needs TF32/BF16; FP32 needs FP32_FMA). */
+polyconv_status_t polyconv_plan_set_kernel(polyconv_plan_t plan, polyconv_kernel_t kernel);
+
+/* Output spatial size: P = (H+2ph-R)/sh + 1, Q = (W+2pw-S)/sw + 1. */
+polyconv_status_t polyconv_output_dims(polyconv_plan_t plan, int *P, int *Q);
+
+/* Sizes, chosen kernel and tiling (host only). */
+polyconv_status_t polyconv_plan_info(polyconv_plan_t plan, polyconv_info_t *info);
+
+/* The hot path: pack (a2,a3) -> coefficient MAC over channels (a4) with the
+ * extraction/strided NCHW store fused in its epilogue (a5).  y: [N][K][P][Q]. */
+polyconv_status_t polyconv_forward(polyconv_plan_t plan, const void *x, const void *w,
+                                   void *y, void *stream);
+
+/* a2 alone: write A_{n,c}(t) of x into dst in `layout` (see above).  dst must
+ * hold polyconv_packed_bytes(plan, 0, layout) bytes. */
+polyconv_status_t polyconv_pack_input(polyconv_plan_t plan, const void *x, void *dst,
+                                      polyconv_layout_t layout, void *stream);
+
+/* a3 alone: write U_{k,c}(t) of w into dst in `layout`. */
+polyconv_status_t polyconv_pack_filter(polyconv_plan_t plan, const void *w, void *dst,
+                                       polyconv_layout_t layout, void *stream);
+
+/* Bytes of a packed operand: which = 0 input, 1 filter. */
+polyconv_status_t polyconv_packed_bytes(polyconv_plan_t plan, int which,
+                                        polyconv_layout_t layout, size_t *bytes);
+
+/* a5 alone (standalone extraction, P.1396-1403): coeffs is the fp32 array of
+ * full product coefficients [N][K][L_A+L_U-1]; writes y[n][k][oh][ow] =
+ * coeffs[n][k][Wp*sh*oh + sw*ow + L_U-1] in the io dtype (bf16: RNE). */
+polyconv_status_t polyconv_extract(polyconv_plan_t plan, const float *coeffs, void *y,
+                                   void *stream);
+
+/* Synchronise the last stream used by the plan, free its workspace and the plan.
+ * NULL is accepted (no-op). */
+polyconv_status_t polyconv_destroy(polyconv_plan_t plan);
+
+/* Static description of a status code. */
+const char *polyconv_status_string(polyconv_status_t status);
+
+/* Text of the last failure on this plan ("" if none).  Valid until the next
+ * call on the plan. */
+const char *polyconv_last_error(polyconv_plan_t plan);
+
+/* POLYCONV_ABI_VERSION of the loaded library. */
+int polyconv_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* POLYCONV_H_ */

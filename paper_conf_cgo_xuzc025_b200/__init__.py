@@ -1,0 +1,246 @@
+"""PolyHankel forward convolution on B200 (sm_100a) — Python binding.
+
+A thin ctypes layer over the in-tree C-ABI library `_lib/libpolyconv.so`
+(include/polyconv.h).  It only marshals arguments: every step of the hot path
+(packing, coefficient MAC, extraction) runs in the library's CUDA kernels.
+PyTorch supplies device memory and streams.  There is no CPU fallback: if the
+library is missing the import of the binding fails loudly.
+
+    from paper_conf_cgo_xuzc025_b200 import Plan
+    plan = Plan((N, C, H, W), (K, C, R, S), stride=(1, 1), padding=(1, 1), math="bf16")
+    y = plan.forward(x, w)          # x, w: CUDA tensors (fp32, or bf16 with math="bf16")
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "_lib", "libpolyconv.so")
+
+SUCCESS, BAD_PARAM, NOT_SUPPORTED, ALLOC_FAILED, EXECUTION_FAILED = range(5)
+F32, BF16 = 0, 1
+MATH = {"fp32": 0, "tf32": 1, "bf16": 2}
+KERNEL = {"auto": 0, "tc": 1, "fp32": 2, "thin": 3}
+KERNEL_NAME = {v: k for k, v in KERNEL.items()}
+LAYOUT = {"planar": 0, "interleaved": 1}
+
+
+class PolyconvError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(msg)
+        self.status = status
+
+
+class Info(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_int) for n in "N C H W K R S sh sw ph pw P Q Hp Wp".split()] + [
+        ("L_A", ctypes.c_longlong), ("L_U", ctypes.c_longlong), ("Cp", ctypes.c_int), ("Kp", ctypes.c_int),
+        ("kernel", ctypes.c_int), ("tile_m", ctypes.c_int), ("tile_n", ctypes.c_int), ("stages", ctypes.c_int),
+        ("launches", ctypes.c_int), ("workspace_bytes", ctypes.c_size_t)]
+
+    def asdict(self):
+        d = {f: getattr(self, f) for f, _ in self._fields_}
+        d["kernel"] = KERNEL_NAME.get(d["kernel"], d["kernel"])
+        return d
+
+
+EXPORTS = ["polyconv_plan", "polyconv_plan_set_kernel", "polyconv_output_dims", "polyconv_plan_info",
+           "polyconv_forward", "polyconv_pack_input", "polyconv_pack_filter", "polyconv_packed_bytes",
+           "polyconv_extract", "polyconv_destroy", "polyconv_status_string", "polyconv_last_error",
+           "polyconv_abi_version"]
+
+_lib = None
+
+
+def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
+    """Load the C-ABI library (raises if it has not been built)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(path):
+        raise ImportError("polyconv CUDA library not built: %s missing (run `python -m "
+                          "paper_conf_cgo_xuzc025_b200.build` or __graft_entry__.build())" % path)
+    lib = ctypes.CDLL(path)
+    vp, ip, i = ctypes.c_void_p, ctypes.POINTER(ctypes.c_int), ctypes.c_int
+    P = ctypes.POINTER(ctypes.c_void_p)
+    lib.polyconv_plan.argtypes = [P] + [i] * 11 + [i, i, i]
+    lib.polyconv_plan_set_kernel.argtypes = [vp, i]
+    lib.polyconv_output_dims.argtypes = [vp, ip, ip]
+    lib.polyconv_plan_info.argtypes = [vp, ctypes.POINTER(Info)]
+    lib.polyconv_forward.argtypes = [vp, vp, vp, vp, vp]
+    lib.polyconv_pack_input.argtypes = [vp, vp, vp, i, vp]
+    lib.polyconv_pack_filter.argtypes = [vp, vp, vp, i, vp]
+    lib.polyconv_packed_bytes.argtypes = [vp, i, i, ctypes.POINTER(ctypes.c_size_t)]
+    lib.polyconv_extract.argtypes = [vp, vp, vp, vp]
+    lib.polyconv_destroy.argtypes = [vp]
+    lib.polyconv_status_string.argtypes = [i]
+    lib.polyconv_status_string.restype = ctypes.c_char_p
+    lib.polyconv_last_error.argtypes = [vp]
+    lib.polyconv_last_error.restype = ctypes.c_char_p
+    lib.polyconv_abi_version.argtypes = []
+    for name in EXPORTS:
+        if name not in ("polyconv_status_string", "polyconv_last_error"):
+            getattr(lib, name).restype = ctypes.c_int
+    _lib = lib
+    return lib
+
+
+def status_string(status: int) -> str:
+    return load_library().polyconv_status_string(status).decode()
+
+
+def _stream_ptr(stream):
+    import torch
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return ctypes.c_void_p(stream.cuda_stream)
+
+
+class Plan:
+    """One convolution problem (shapes, stride, padding, dtype, math) on one device.
+
+    math: "fp32" (SIMT FFMA), "tf32" or "bf16" (tcgen05 tensor cores).
+    io_dtype: "f32" or "bf16" (bf16 requires math="bf16").
+    kernel: "auto" | "tc" | "fp32" | "thin" (force a MAC variant).
+    """
+
+    def __init__(self, x_shape, w_shape, stride=(1, 1), padding=(0, 0), math="bf16", io_dtype="f32",
+                 device: int = 0, kernel: str = "auto"):
+        self._lib = load_library()
+        N, C, H, W = x_shape
+        K, C2, R, S = w_shape
+        if C != C2:
+            raise PolyconvError(BAD_PARAM, "channel mismatch")
+        self.x_shape, self.w_shape = tuple(x_shape), tuple(w_shape)
+        self.stride, self.padding = tuple(stride), tuple(padding)
+        self.math, self.io_dtype, self.device = math, io_dtype, device
+        h = ctypes.c_void_p()
+        st = self._lib.polyconv_plan(ctypes.byref(h), N, C, H, W, K, R, S, stride[0], stride[1], padding[0],
+                                     padding[1], BF16 if io_dtype == "bf16" else F32, MATH[math], device)
+        if st != SUCCESS:
+            raise PolyconvError(st, "polyconv_plan: %s" % status_string(st))
+        self._h = h
+        if kernel != "auto":
+            self._check(self._lib.polyconv_plan_set_kernel(self._h, KERNEL[kernel]), "set_kernel")
+        P, Q = ctypes.c_int(), ctypes.c_int()
+        self._check(self._lib.polyconv_output_dims(self._h, ctypes.byref(P), ctypes.byref(Q)), "output_dims")
+        self.P, self.Q = P.value, Q.value
+
+    # -- helpers ---------------------------------------------------------------
+    def _check(self, st, what):
+        if st != SUCCESS:
+            detail = self._lib.polyconv_last_error(self._h).decode() if getattr(self, "_h", None) else ""
+            raise PolyconvError(st, "polyconv_%s: %s %s" % (what, status_string(st), detail))
+
+    @property
+    def handle(self):
+        return self._h
+
+    @property
+    def output_shape(self):
+        return (self.x_shape[0], self.w_shape[0], self.P, self.Q)
+
+    def info(self) -> dict:
+        inf = Info()
+        self._check(self._lib.polyconv_plan_info(self._h, ctypes.byref(inf)), "plan_info")
+        return inf.asdict()
+
+    def _io_torch_dtype(self):
+        import torch
+        return torch.bfloat16 if self.io_dtype == "bf16" else torch.float32
+
+    def _check_tensor(self, t, shape, name):
+        import torch
+        if not isinstance(t, torch.Tensor) or not t.is_cuda:
+            raise PolyconvError(BAD_PARAM, "%s must be a CUDA tensor" % name)
+        if tuple(t.shape) != tuple(shape):
+            raise PolyconvError(BAD_PARAM, "%s shape %s != %s" % (name, tuple(t.shape), tuple(shape)))
+        if t.dtype != self._io_torch_dtype():
+            raise PolyconvError(BAD_PARAM, "%s dtype %s != %s" % (name, t.dtype, self._io_torch_dtype()))
+        if not t.is_contiguous():
+            raise PolyconvError(BAD_PARAM, "%s must be contiguous" % name)
+
+    # -- the hot path ------------------------------------------------------------
+    def forward(self, x, w, y=None, stream=None):
+        """y[N][K][P][Q] = conv(x, w) via pack -> coefficient MAC -> extraction."""
+        import torch
+        self._check_tensor(x, self.x_shape, "x")
+        self._check_tensor(w, self.w_shape, "w")
+        if y is None:
+            y = torch.empty(self.output_shape, dtype=self._io_torch_dtype(), device=x.device)
+        else:
+            self._check_tensor(y, self.output_shape, "y")
+        self._check(self._lib.polyconv_forward(self._h, ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(w.data_ptr()),
+                                               ctypes.c_void_p(y.data_ptr()), _stream_ptr(stream)), "forward")
+        return y
+
+    def forward_ptr(self, x_ptr: int, w_ptr: int, y_ptr: int, stream_ptr: int = 0):
+        """Raw-pointer forward (no checks beyond the library's)."""
+        self._check(self._lib.polyconv_forward(self._h, ctypes.c_void_p(x_ptr), ctypes.c_void_p(w_ptr),
+                                               ctypes.c_void_p(y_ptr), ctypes.c_void_p(stream_ptr)), "forward")
+
+    # -- single steps (bit-exact tests) ------------------------------------------------
+    def packed_bytes(self, which: str, layout: str) -> int:
+        b = ctypes.c_size_t()
+        self._check(self._lib.polyconv_packed_bytes(self._h, 0 if which == "input" else 1, LAYOUT[layout],
+                                                    ctypes.byref(b)), "packed_bytes")
+        return b.value
+
+    def pack_input(self, x, layout="planar", stream=None):
+        """a2: returns the packed A_{n,c}(t) words as a uint8 CUDA tensor."""
+        import torch
+        self._check_tensor(x, self.x_shape, "x")
+        out = torch.empty(self.packed_bytes("input", layout), dtype=torch.uint8, device=x.device)
+        self._check(self._lib.polyconv_pack_input(self._h, ctypes.c_void_p(x.data_ptr()),
+                                                  ctypes.c_void_p(out.data_ptr()), LAYOUT[layout],
+                                                  _stream_ptr(stream)), "pack_input")
+        return out
+
+    def pack_filter(self, w, layout="planar", stream=None):
+        """a3: returns the packed U_{k,c}(t) words as a uint8 CUDA tensor."""
+        import torch
+        self._check_tensor(w, self.w_shape, "w")
+        out = torch.empty(self.packed_bytes("filter", layout), dtype=torch.uint8, device=w.device)
+        self._check(self._lib.polyconv_pack_filter(self._h, ctypes.c_void_p(w.data_ptr()),
+                                                   ctypes.c_void_p(out.data_ptr()), LAYOUT[layout],
+                                                   _stream_ptr(stream)), "pack_filter")
+        return out
+
+    def extract(self, coeffs, stream=None):
+        """a5: y from the full fp32 product coefficients [N][K][L_A+L_U-1]."""
+        import torch
+        inf = self.info()
+        Lp = inf["L_A"] + inf["L_U"] - 1
+        if not coeffs.is_cuda or coeffs.dtype != torch.float32 or tuple(coeffs.shape) != (self.x_shape[0],
+                                                                                           self.w_shape[0], Lp):
+            raise PolyconvError(BAD_PARAM, "coeffs must be float32 CUDA [N][K][L_A+L_U-1]")
+        y = torch.empty(self.output_shape, dtype=self._io_torch_dtype(), device=coeffs.device)
+        self._check(self._lib.polyconv_extract(self._h, ctypes.c_void_p(coeffs.data_ptr()),
+                                               ctypes.c_void_p(y.data_ptr()), _stream_ptr(stream)), "extract")
+        return y
+
+    def close(self):
+        h = getattr(self, "_h", None)
+        if h:
+            self._lib.polyconv_destroy(h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def conv2d(x, w, stride=(1, 1), padding=(0, 0), math="bf16", kernel="auto"):
+    """One-shot convenience: plan + forward (the plan is cached per shape)."""
+    key = (tuple(x.shape), tuple(w.shape), tuple(stride), tuple(padding), math,
+           "bf16" if str(x.dtype) == "torch.bfloat16" else "f32", x.device.index or 0, kernel)
+    plan = _PLANS.get(key)
+    if plan is None:
+        plan = Plan(x.shape, w.shape, stride, padding, math, key[5], key[6], kernel)
+        _PLANS[key] = plan
+    return plan.forward(x, w)
+
+
+_PLANS: dict = {}

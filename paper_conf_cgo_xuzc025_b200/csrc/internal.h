@@ -1,0 +1,74 @@
+// internal.h — geometry shared by the host API (polyconv.cu) and the kernels.
+// Product code only; nothing here is used by oracle/.
+#pragma once
+#include <cstdint>
+#include <cstddef>
+#include <cuda_runtime.h>
+
+namespace polyconv {
+
+// Operand storage formats produced by packing (reading R11).
+enum Fmt : int { FMT_F32 = 0, FMT_TF32 = 1, FMT_BF16 = 2 };
+
+// Problem geometry, all derived once in polyconv_plan.
+struct Geom {
+  int N, C, H, W, K, R, S, sh, sw, ph, pw;
+  int P, Q;             // output size
+  int Hp, Wp;           // padded input size; Wp is the row pitch Iw of Eq. 10
+  long long L_A;        // Hp*Wp, input polynomial length (Eq. 10)
+  long long L_U;        // (R-1)*Wp + S, kernel polynomial length (P.1378-1380)
+  long long M_ext;      // positions per image that can hold an output:
+                        // (P-1)*sh*Wp + (Q-1)*sw + 1 (last extraction degree - (L_U-1) + 1)
+  int Cp, Kp;           // padded channel counts of the interleaved layouts
+};
+
+inline int fmt_bytes(int f) { return f == FMT_BF16 ? 2 : 4; }
+
+// ---- pack.cu ------------------------------------------------------------
+cudaError_t launch_pack_input_planar(const Geom& g, const void* x, bool x_bf16, void* dst,
+                                     int fmt, cudaStream_t st);
+cudaError_t launch_pack_input_interleaved(const Geom& g, const void* x, bool x_bf16, void* dst,
+                                          int fmt, cudaStream_t st);
+cudaError_t launch_pack_filter_planar(const Geom& g, const void* w, bool w_bf16, void* dst,
+                                      int fmt, cudaStream_t st);
+cudaError_t launch_pack_filter_tapmajor(const Geom& g, const void* w, bool w_bf16, void* dst,
+                                        int fmt, int Kp, int Cp, cudaStream_t st);
+// fused: input interleaved + filter tap-major in one launch
+cudaError_t launch_pack_both_interleaved(const Geom& g, const void* x, const void* w, bool io_bf16,
+                                         void* xdst, void* wdst, int fmt, cudaStream_t st);
+
+// ---- extract.cu -----------------------------------------------------------
+cudaError_t launch_extract(const Geom& g, const float* coeffs, void* y, bool y_bf16,
+                           cudaStream_t st);
+
+// ---- mac_thin.cu ----------------------------------------------------------
+// A: planar packed input [N][C][L_A] (fmt); U: tap-major packed filter [RS][Kp][Cp] (fmt)
+cudaError_t launch_mac_thin(const Geom& g, const void* A, const void* U, int Kp, int Cp, int fmt,
+                            void* y, bool y_bf16, cudaStream_t st);
+
+// ---- mac_fp32.cu ----------------------------------------------------------
+struct Fp32Tiling { int cc; int smem_bytes; int smax; };
+Fp32Tiling fp32_tiling(const Geom& g);
+cudaError_t launch_mac_fp32(const Geom& g, const Fp32Tiling& t, const float* A, const float* U,
+                            int Kp, int Cp, float* y, cudaStream_t st);
+inline int fp32_kp(int K) { return (K + 63) / 64 * 64; }
+
+// ---- mac_tc.cu ------------------------------------------------------------
+struct TcTiling {
+  int bm;          // positions per tile (UMMA M) = 128
+  int bn;          // output channels per tile (UMMA N), multiple of 32, <= 256
+  int kc;          // channels per k-block (row of the smem operand)
+  int row_bytes;   // kc * element bytes: 32, 64 or 128 (= swizzle width)
+  int stages;      // smem pipeline depth
+  int smem_bytes;  // dynamic shared memory
+  int tmem_cols;   // TMEM allocation (2 accumulators)
+  int num_m, num_n, kblocks;
+  int grid;        // persistent CTAs
+};
+bool tc_supported(const Geom& g, int fmt);
+TcTiling tc_tiling(const Geom& g, int fmt, int num_sms);
+// A: interleaved packed input [N*L_A][Cp]; U: tap-major packed filter [RS][Kp][Cp]
+cudaError_t launch_mac_tc(const Geom& g, const TcTiling& t, int fmt, const void* A, const void* U,
+                          void* y, bool y_bf16, cudaStream_t st, char* err, size_t errlen);
+
+}  // namespace polyconv

@@ -1,0 +1,351 @@
+// polyconv.cu — host side of the C-ABI (include/polyconv.h): argument
+// validation, the a1 plan/index math, kernel selection, workspace and launch
+// sequencing.  Every step of the hot path runs in the CUDA kernels of this
+// directory; there is no CPU compute path and no fallback to another library.
+#include <cuda_runtime.h>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <new>
+#include "../../include/polyconv.h"
+#include "internal.h"
+
+using namespace polyconv;
+
+struct polyconv_plan_s {
+  Geom g;
+  bool io_bf16;
+  int math;
+  int fmt;
+  int device;
+  int forced;
+  int kernel;  // resolved polyconv_kernel_t
+  TcTiling tc;
+  Fp32Tiling f32;
+  // workspace (lazy)
+  void* wsA = nullptr;
+  size_t wsA_bytes = 0;
+  void* wsU = nullptr;
+  size_t wsU_bytes = 0;
+  bool device_checked = false;
+  int num_sms = 148;
+  cudaStream_t last_stream = nullptr;
+  bool used = false;
+  char err[512];
+};
+
+namespace {
+
+const long long kMaxElems = (1LL << 31) - 1;
+
+void set_err(polyconv_plan_t p, const char* fmt_, const char* a = "", long long b = 0) {
+  if (p) snprintf(p->err, sizeof(p->err), fmt_, a, b);
+}
+
+// Resolve the MAC variant and fill the kernel-specific padded sizes.
+polyconv_status_t resolve(polyconv_plan_t p) {
+  Geom& g = p->g;
+  int k = p->forced;
+  const bool tc_math = p->math != POLYCONV_MATH_FP32_FMA;
+  if (k == POLYCONV_KERNEL_AUTO) {
+    if (tc_math)
+      k = (g.K >= 16 && tc_supported(g, p->fmt)) ? POLYCONV_KERNEL_TC : POLYCONV_KERNEL_THIN;
+    else
+      k = (g.K >= 16 && g.C * g.R * g.S >= 16 && fp32_tiling(g).smax > 0) ? POLYCONV_KERNEL_FP32
+                                                                          : POLYCONV_KERNEL_THIN;
+  }
+  if (k == POLYCONV_KERNEL_TC && (!tc_math || !tc_supported(g, p->fmt))) return POLYCONV_STATUS_BAD_PARAM;
+  if (k == POLYCONV_KERNEL_FP32 && (tc_math || fp32_tiling(g).smax == 0)) return POLYCONV_STATUS_BAD_PARAM;
+  p->kernel = k;
+  if (k == POLYCONV_KERNEL_TC) {
+    p->tc = tc_tiling(g, p->fmt, p->num_sms);
+    g.Cp = (g.C + p->tc.kc - 1) / p->tc.kc * p->tc.kc;
+    g.Kp = (g.K + p->tc.bn - 1) / p->tc.bn * p->tc.bn;
+  } else if (k == POLYCONV_KERNEL_FP32) {
+    p->f32 = fp32_tiling(g);
+    g.Cp = (g.C + p->f32.cc - 1) / p->f32.cc * p->f32.cc;
+    g.Kp = fp32_kp(g.K);
+  } else {
+    g.Cp = g.C;
+    g.Kp = g.K;
+  }
+  const int eb = fmt_bytes(p->fmt);
+  const size_t a_elems = (k == POLYCONV_KERNEL_TC) ? (size_t)g.N * g.L_A * g.Cp : (size_t)g.N * g.C * g.L_A;
+  p->wsA_bytes = a_elems * eb;
+  p->wsU_bytes = (size_t)g.R * g.S * g.Kp * g.Cp * eb;
+  return POLYCONV_STATUS_SUCCESS;
+}
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur;
+    if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+polyconv_status_t check_device(polyconv_plan_t p) {
+  if (p->device_checked) return POLYCONV_STATUS_SUCCESS;
+  cudaDeviceProp prop;
+  cudaError_t e = cudaGetDeviceProperties(&prop, p->device);
+  if (e != cudaSuccess) {
+    set_err(p, "no CUDA device: %s", cudaGetErrorString(e));
+    cudaGetLastError();
+    return POLYCONV_STATUS_NOT_SUPPORTED;
+  }
+  if (prop.major != 10 || prop.minor != 0) {
+    snprintf(p->err, sizeof(p->err), "device %d is sm_%d%d; this library is built for sm_100a only", p->device,
+             prop.major, prop.minor);
+    return POLYCONV_STATUS_NOT_SUPPORTED;
+  }
+  if (prop.multiProcessorCount != p->num_sms) {
+    p->num_sms = prop.multiProcessorCount;
+    resolve(p);
+  }
+  p->device_checked = true;
+  return POLYCONV_STATUS_SUCCESS;
+}
+
+polyconv_status_t ensure_workspace(polyconv_plan_t p) {
+  if (p->wsA && p->wsU) return POLYCONV_STATUS_SUCCESS;
+  if (!p->wsA && cudaMalloc(&p->wsA, p->wsA_bytes ? p->wsA_bytes : 16) != cudaSuccess) {
+    p->wsA = nullptr;
+    set_err(p, "cudaMalloc of %s workspace failed (%lld bytes)", "input", (long long)p->wsA_bytes);
+    cudaGetLastError();
+    return POLYCONV_STATUS_ALLOC_FAILED;
+  }
+  if (!p->wsU && cudaMalloc(&p->wsU, p->wsU_bytes ? p->wsU_bytes : 16) != cudaSuccess) {
+    p->wsU = nullptr;
+    set_err(p, "cudaMalloc of %s workspace failed (%lld bytes)", "filter", (long long)p->wsU_bytes);
+    cudaGetLastError();
+    return POLYCONV_STATUS_ALLOC_FAILED;
+  }
+  return POLYCONV_STATUS_SUCCESS;
+}
+
+polyconv_status_t finish(polyconv_plan_t p, cudaError_t e, const char* what) {
+  if (e != cudaSuccess) {
+    snprintf(p->err, sizeof(p->err), "%s: %s", what, cudaGetErrorString(e));
+    cudaGetLastError();
+    return POLYCONV_STATUS_EXECUTION_FAILED;
+  }
+  return POLYCONV_STATUS_SUCCESS;
+}
+
+bool aligned(const void* ptr, size_t a) { return (reinterpret_cast<uintptr_t>(ptr) % a) == 0; }
+
+#define PC_BEGIN(plan_)                                          \
+  if (!(plan_)) return POLYCONV_STATUS_BAD_PARAM;                \
+  (plan_)->err[0] = 0;                                           \
+  DeviceGuard guard_((plan_)->device);                           \
+  {                                                              \
+    polyconv_status_t s_ = check_device(plan_);                  \
+    if (s_ != POLYCONV_STATUS_SUCCESS) return s_;                \
+  }
+
+}  // namespace
+
+extern "C" {
+
+int polyconv_abi_version(void) { return POLYCONV_ABI_VERSION; }
+
+const char* polyconv_status_string(polyconv_status_t s) {
+  switch (s) {
+    case POLYCONV_STATUS_SUCCESS: return "POLYCONV_STATUS_SUCCESS";
+    case POLYCONV_STATUS_BAD_PARAM: return "POLYCONV_STATUS_BAD_PARAM";
+    case POLYCONV_STATUS_NOT_SUPPORTED: return "POLYCONV_STATUS_NOT_SUPPORTED";
+    case POLYCONV_STATUS_ALLOC_FAILED: return "POLYCONV_STATUS_ALLOC_FAILED";
+    case POLYCONV_STATUS_EXECUTION_FAILED: return "POLYCONV_STATUS_EXECUTION_FAILED";
+  }
+  return "POLYCONV_STATUS_UNKNOWN";
+}
+
+const char* polyconv_last_error(polyconv_plan_t plan) { return plan ? plan->err : ""; }
+
+polyconv_status_t polyconv_plan(polyconv_plan_t* plan, int N, int C, int H, int W, int K, int R, int S,
+                                int sh, int sw, int ph, int pw, polyconv_dtype_t io_dtype,
+                                polyconv_math_t math, int device) {
+  if (!plan) return POLYCONV_STATUS_BAD_PARAM;
+  *plan = nullptr;
+  if (N < 1 || C < 1 || H < 1 || W < 1 || K < 1 || R < 1 || S < 1 || sh < 1 || sw < 1 || ph < 0 || pw < 0 ||
+      device < 0)
+    return POLYCONV_STATUS_BAD_PARAM;
+  if (io_dtype != POLYCONV_F32 && io_dtype != POLYCONV_BF16) return POLYCONV_STATUS_BAD_PARAM;
+  if (math != POLYCONV_MATH_FP32_FMA && math != POLYCONV_MATH_TF32 && math != POLYCONV_MATH_BF16)
+    return POLYCONV_STATUS_BAD_PARAM;
+  if (io_dtype == POLYCONV_BF16 && math != POLYCONV_MATH_BF16) return POLYCONV_STATUS_BAD_PARAM;
+  const long long Hp = (long long)H + 2LL * ph, Wp = (long long)W + 2LL * pw;
+  if (Hp < R || Wp < S) return POLYCONV_STATUS_BAD_PARAM;  // P < 1 or Q < 1
+  const long long P = (Hp - R) / sh + 1, Q = (Wp - S) / sw + 1;
+  // every tensor (and every packed operand) must index with < 2^31 elements
+  if ((long long)N * C * H * W > kMaxElems || (long long)K * C * R * S > kMaxElems ||
+      (long long)N * K * P * Q > kMaxElems || Hp * Wp > kMaxElems || (long long)N * C * Hp * Wp > kMaxElems ||
+      (long long)N * Hp * Wp * ((C + 63) / 64 * 64) > kMaxElems)
+    return POLYCONV_STATUS_NOT_SUPPORTED;
+
+  polyconv_plan_t p = new (std::nothrow) polyconv_plan_s();
+  if (!p) return POLYCONV_STATUS_ALLOC_FAILED;
+  Geom& g = p->g;
+  g.N = N; g.C = C; g.H = H; g.W = W; g.K = K; g.R = R; g.S = S;
+  g.sh = sh; g.sw = sw; g.ph = ph; g.pw = pw;
+  g.Hp = (int)Hp; g.Wp = (int)Wp; g.P = (int)P; g.Q = (int)Q;
+  g.L_A = Hp * Wp;                          // Eq. 10
+  g.L_U = (long long)(R - 1) * Wp + S;      // KernelSize, P.1378-1380 (Iw := Wp)
+  g.M_ext = (P - 1) * sh * Wp + (Q - 1) * sw + 1;
+  p->io_bf16 = io_dtype == POLYCONV_BF16;
+  p->math = math;
+  p->fmt = math == POLYCONV_MATH_BF16 ? FMT_BF16 : (math == POLYCONV_MATH_TF32 ? FMT_TF32 : FMT_F32);
+  p->device = device;
+  p->forced = POLYCONV_KERNEL_AUTO;
+  p->err[0] = 0;
+  if (resolve(p) != POLYCONV_STATUS_SUCCESS) {
+    delete p;
+    return POLYCONV_STATUS_BAD_PARAM;
+  }
+  *plan = p;
+  return POLYCONV_STATUS_SUCCESS;
+}
+
+polyconv_status_t polyconv_plan_set_kernel(polyconv_plan_t p, polyconv_kernel_t kernel) {
+  if (!p) return POLYCONV_STATUS_BAD_PARAM;
+  if (kernel < POLYCONV_KERNEL_AUTO || kernel > POLYCONV_KERNEL_THIN) return POLYCONV_STATUS_BAD_PARAM;
+  const int old = p->forced;
+  p->forced = kernel;
+  if (resolve(p) != POLYCONV_STATUS_SUCCESS) {
+    p->forced = old;
+    resolve(p);
+    return POLYCONV_STATUS_BAD_PARAM;
+  }
+  // workspace sizes may have changed
+  if (p->wsA) { cudaFree(p->wsA); p->wsA = nullptr; }
+  if (p->wsU) { cudaFree(p->wsU); p->wsU = nullptr; }
+  return POLYCONV_STATUS_SUCCESS;
+}
+
+polyconv_status_t polyconv_output_dims(polyconv_plan_t p, int* P, int* Q) {
+  if (!p || !P || !Q) return POLYCONV_STATUS_BAD_PARAM;
+  *P = p->g.P;
+  *Q = p->g.Q;
+  return POLYCONV_STATUS_SUCCESS;
+}
+
+polyconv_status_t polyconv_plan_info(polyconv_plan_t p, polyconv_info_t* info) {
+  if (!p || !info) return POLYCONV_STATUS_BAD_PARAM;
+  const Geom& g = p->g;
+  info->N = g.N; info->C = g.C; info->H = g.H; info->W = g.W; info->K = g.K; info->R = g.R; info->S = g.S;
+  info->sh = g.sh; info->sw = g.sw; info->ph = g.ph; info->pw = g.pw;
+  info->P = g.P; info->Q = g.Q; info->Hp = g.Hp; info->Wp = g.Wp;
+  info->L_A = g.L_A; info->L_U = g.L_U; info->Cp = g.Cp; info->Kp = g.Kp;
+  info->kernel = p->kernel;
+  info->tile_m = p->kernel == POLYCONV_KERNEL_TC ? p->tc.bm : (p->kernel == POLYCONV_KERNEL_FP32 ? 256 : 1);
+  info->tile_n = p->kernel == POLYCONV_KERNEL_TC ? p->tc.bn : (p->kernel == POLYCONV_KERNEL_FP32 ? 64 : 1);
+  info->stages = p->kernel == POLYCONV_KERNEL_TC ? p->tc.stages : 1;
+  info->launches = p->kernel == POLYCONV_KERNEL_TC ? 2 : 3;
+  info->workspace_bytes = p->wsA_bytes + p->wsU_bytes;
+  return POLYCONV_STATUS_SUCCESS;
+}
+
+polyconv_status_t polyconv_forward(polyconv_plan_t p, const void* x, const void* w, void* y, void* stream) {
+  if (!p) return POLYCONV_STATUS_BAD_PARAM;
+  if (!x || !w || !y || x == y || w == y) return POLYCONV_STATUS_BAD_PARAM;
+  if (!aligned(x, 16) || !aligned(w, 16) || !aligned(y, 16)) return POLYCONV_STATUS_NOT_SUPPORTED;
+  PC_BEGIN(p);
+  polyconv_status_t s = ensure_workspace(p);
+  if (s != POLYCONV_STATUS_SUCCESS) return s;
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  p->last_stream = st;
+  p->used = true;
+  const Geom& g = p->g;
+  cudaError_t e;
+  if (p->kernel == POLYCONV_KERNEL_TC) {
+    // a2 + a3 in one launch (interleaved A, tap-major U), then the MAC (a4+a5)
+    e = launch_pack_both_interleaved(g, x, w, p->io_bf16, p->wsA, p->wsU, p->fmt, st);
+    if (e != cudaSuccess) return finish(p, e, "pack");
+    e = launch_mac_tc(g, p->tc, p->fmt, p->wsA, p->wsU, y, p->io_bf16, st, p->err, sizeof(p->err));
+    return finish(p, e, "mac_tc");
+  }
+  e = launch_pack_input_planar(g, x, p->io_bf16, p->wsA, p->fmt, st);
+  if (e != cudaSuccess) return finish(p, e, "pack_input");
+  e = launch_pack_filter_tapmajor(g, w, p->io_bf16, p->wsU, p->fmt, g.Kp, g.Cp, st);
+  if (e != cudaSuccess) return finish(p, e, "pack_filter");
+  if (p->kernel == POLYCONV_KERNEL_FP32) {
+    e = launch_mac_fp32(g, p->f32, (const float*)p->wsA, (const float*)p->wsU, g.Kp, g.Cp, (float*)y, st);
+    return finish(p, e, "mac_fp32");
+  }
+  e = launch_mac_thin(g, p->wsA, p->wsU, g.Kp, g.Cp, p->fmt, y, p->io_bf16, st);
+  return finish(p, e, "mac_thin");
+}
+
+polyconv_status_t polyconv_packed_bytes(polyconv_plan_t p, int which, polyconv_layout_t layout, size_t* bytes) {
+  if (!p || !bytes || (which != 0 && which != 1)) return POLYCONV_STATUS_BAD_PARAM;
+  if (layout != POLYCONV_LAYOUT_PLANAR && layout != POLYCONV_LAYOUT_INTERLEAVED) return POLYCONV_STATUS_BAD_PARAM;
+  const Geom& g = p->g;
+  const size_t eb = (size_t)fmt_bytes(p->fmt);
+  if (which == 0)
+    *bytes = eb * (layout == POLYCONV_LAYOUT_PLANAR ? (size_t)g.N * g.C * g.L_A : (size_t)g.N * g.L_A * g.Cp);
+  else
+    *bytes = eb * (layout == POLYCONV_LAYOUT_PLANAR ? (size_t)g.K * g.C * g.L_U : (size_t)g.R * g.S * g.Kp * g.Cp);
+  return POLYCONV_STATUS_SUCCESS;
+}
+
+polyconv_status_t polyconv_pack_input(polyconv_plan_t p, const void* x, void* dst, polyconv_layout_t layout,
+                                      void* stream) {
+  if (!p || !x || !dst) return POLYCONV_STATUS_BAD_PARAM;
+  if (layout != POLYCONV_LAYOUT_PLANAR && layout != POLYCONV_LAYOUT_INTERLEAVED) return POLYCONV_STATUS_BAD_PARAM;
+  if (!aligned(x, 16) || !aligned(dst, 16)) return POLYCONV_STATUS_NOT_SUPPORTED;
+  PC_BEGIN(p);
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  p->last_stream = st;
+  p->used = true;
+  cudaError_t e = layout == POLYCONV_LAYOUT_PLANAR
+                      ? launch_pack_input_planar(p->g, x, p->io_bf16, dst, p->fmt, st)
+                      : launch_pack_input_interleaved(p->g, x, p->io_bf16, dst, p->fmt, st);
+  return finish(p, e, "pack_input");
+}
+
+polyconv_status_t polyconv_pack_filter(polyconv_plan_t p, const void* w, void* dst, polyconv_layout_t layout,
+                                       void* stream) {
+  if (!p || !w || !dst) return POLYCONV_STATUS_BAD_PARAM;
+  if (layout != POLYCONV_LAYOUT_PLANAR && layout != POLYCONV_LAYOUT_INTERLEAVED) return POLYCONV_STATUS_BAD_PARAM;
+  if (!aligned(w, 16) || !aligned(dst, 16)) return POLYCONV_STATUS_NOT_SUPPORTED;
+  PC_BEGIN(p);
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  p->last_stream = st;
+  p->used = true;
+  cudaError_t e = layout == POLYCONV_LAYOUT_PLANAR
+                      ? launch_pack_filter_planar(p->g, w, p->io_bf16, dst, p->fmt, st)
+                      : launch_pack_filter_tapmajor(p->g, w, p->io_bf16, dst, p->fmt, p->g.Kp, p->g.Cp, st);
+  return finish(p, e, "pack_filter");
+}
+
+polyconv_status_t polyconv_extract(polyconv_plan_t p, const float* coeffs, void* y, void* stream) {
+  if (!p || !coeffs || !y) return POLYCONV_STATUS_BAD_PARAM;
+  if (!aligned(coeffs, 4) || !aligned(y, 16)) return POLYCONV_STATUS_NOT_SUPPORTED;
+  PC_BEGIN(p);
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  p->last_stream = st;
+  p->used = true;
+  return finish(p, launch_extract(p->g, coeffs, y, p->io_bf16, st), "extract");
+}
+
+polyconv_status_t polyconv_destroy(polyconv_plan_t p) {
+  if (!p) return POLYCONV_STATUS_SUCCESS;
+  polyconv_status_t s = POLYCONV_STATUS_SUCCESS;
+  if (p->used || p->wsA || p->wsU) {
+    DeviceGuard guard(p->device);
+    if (p->used && cudaStreamSynchronize(p->last_stream) != cudaSuccess) {
+      cudaGetLastError();
+      s = POLYCONV_STATUS_EXECUTION_FAILED;
+    }
+    if (p->wsA) cudaFree(p->wsA);
+    if (p->wsU) cudaFree(p->wsU);
+  }
+  delete p;
+  return s;
+}
+
+}  // extern "C"

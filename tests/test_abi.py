@@ -1,0 +1,95 @@
+"""CPU-side checks of the C-ABI library: it loads without a GPU, exports every
+symbol include/polyconv.h declares, and its host logic (argument validation,
+a1 size math, kernel selection, status strings) behaves as documented."""
+import ctypes
+import os
+import re
+
+import pytest
+
+import paper_conf_cgo_xuzc025_b200 as pc
+import oracle
+from oracle import poly_ref as pr
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def test_exports_every_declared_symbol():
+    hdr = open(os.path.join(ROOT, "include", "polyconv.h")).read()
+    declared = set(re.findall(r"\b(polyconv_\w+)\s*\(", hdr))
+    assert declared == set(pc.EXPORTS)
+    lib = pc.load_library()
+    for name in declared:
+        assert hasattr(lib, name), name
+    assert lib.polyconv_abi_version() == 1
+
+
+def test_status_strings():
+    for s in range(5):
+        assert pc.status_string(s).startswith("POLYCONV_STATUS_")
+
+
+@pytest.mark.parametrize("args", [
+    (0, 1, 8, 8, 1, 3, 3, 1, 1, 0, 0), (1, 1, 8, 8, 1, 3, 3, 0, 1, 0, 0), (1, 1, 8, 8, 1, 3, 3, 1, 1, -1, 0),
+    (1, 1, 2, 2, 1, 3, 3, 1, 1, 0, 0), (1, 0, 8, 8, 1, 3, 3, 1, 1, 0, 0), (1, 1, 8, 8, 0, 3, 3, 1, 1, 0, 0)])
+def test_plan_rejects_bad_params(args):
+    lib = pc.load_library()
+    h = ctypes.c_void_p()
+    st = lib.polyconv_plan(ctypes.byref(h), *args, 0, 2, 0)
+    assert st == pc.BAD_PARAM and not h.value
+
+
+def test_plan_rejects_bad_combos():
+    lib = pc.load_library()
+    h = ctypes.c_void_p()
+    assert lib.polyconv_plan(ctypes.byref(h), 1, 1, 8, 8, 1, 3, 3, 1, 1, 0, 0, 1, 0, 0) == pc.BAD_PARAM  # bf16 io, fp32 math
+    assert lib.polyconv_plan(ctypes.byref(h), 1, 1, 8, 8, 1, 3, 3, 1, 1, 0, 0, 0, 7, 0) == pc.BAD_PARAM  # bad math
+    assert lib.polyconv_plan(None, 1, 1, 8, 8, 1, 3, 3, 1, 1, 0, 0, 0, 0, 0) == pc.BAD_PARAM
+    # > 2^31 elements
+    assert lib.polyconv_plan(ctypes.byref(h), 4096, 512, 224, 224, 64, 3, 3, 1, 1, 1, 1, 0, 2, 0) == pc.NOT_SUPPORTED
+
+
+@pytest.mark.parametrize("H,W,R,S,s,p", [(8, 8, 3, 3, 1, 0), (28, 28, 3, 3, 1, 1), (224, 224, 7, 7, 2, 3),
+                                         (7, 11, 2, 5, 3, 2), (56, 56, 1, 1, 2, 0)])
+def test_plan_sizes_match_oracle(H, W, R, S, s, p):
+    plan = pc.Plan((2, 8, H, W), (16, 8, R, S), (s, s), (p, p), math="bf16")
+    inf = plan.info()
+    assert (inf["P"], inf["Q"]) == oracle.output_dims(H, W, R, S, (s, s), (p, p))
+    z = pr.sizes(H, W, R, S, s, s, p, p)
+    assert (inf["Hp"], inf["Wp"], inf["L_A"], inf["L_U"]) == (z["Hp"], z["Wp"], z["L_A"], z["L_U"])
+
+
+def test_kernel_selection_and_forcing():
+    assert pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="bf16").info()["kernel"] == "tc"
+    assert pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="tf32").info()["kernel"] == "tc"
+    assert pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="fp32").info()["kernel"] == "fp32"
+    assert pc.Plan((1, 1, 8, 8), (1, 1, 3, 3), math="fp32").info()["kernel"] == "thin"
+    assert pc.Plan((1, 1, 8, 8), (1, 1, 3, 3), math="bf16").info()["kernel"] == "thin"
+    with pytest.raises(pc.PolyconvError):
+        pc.Plan((1, 4, 8, 8), (16, 4, 3, 3), math="fp32", kernel="tc")
+    with pytest.raises(pc.PolyconvError):
+        pc.Plan((1, 4, 8, 8), (16, 4, 3, 3), math="bf16", kernel="fp32")
+    p = pc.Plan((1, 4, 8, 8), (16, 4, 3, 3), math="bf16", kernel="thin")
+    assert p.info()["kernel"] == "thin"
+
+
+def test_tc_tiling_choices():
+    inf = pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="bf16").info()
+    assert (inf["tile_m"], inf["tile_n"], inf["Cp"], inf["Kp"]) == (128, 128, 128, 128)
+    inf = pc.Plan((2, 3, 30, 30), (64, 3, 7, 7), (2, 2), (3, 3), math="bf16").info()
+    assert inf["Cp"] == 16 and inf["Kp"] == 64            # C=3 -> one 32-byte swizzle row
+    inf = pc.Plan((2, 3, 30, 30), (64, 3, 7, 7), (2, 2), (3, 3), math="tf32").info()
+    assert inf["Cp"] == 8
+    inf = pc.Plan((1, 64, 10, 10), (320, 64, 3, 3), (1, 1), (1, 1), math="bf16").info()
+    assert inf["tile_n"] == 256 and inf["Kp"] == 512
+
+
+def test_forward_without_gpu_fails_cleanly():
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("GPU present")
+    plan = pc.Plan((1, 4, 8, 8), (16, 4, 3, 3), math="bf16")
+    with pytest.raises(pc.PolyconvError) as e:
+        plan.forward_ptr(4096, 8192, 16384)
+    assert e.value.status == pc.NOT_SUPPORTED
+    assert plan._lib.polyconv_destroy(None) == pc.SUCCESS

@@ -1,0 +1,252 @@
+"""GPU parity: the CUDA path (through the C-ABI) against the fp64 oracle.
+
+Element-by-element on seeded inputs (synth/), at sizes the oracle finishes in
+seconds spanning several tiles and ragged tails, and at BASELINE sizes on
+sampled images.  Gates: normwise 1e-5 (FP32_FMA), 2e-2 (TF32/BF16); packing,
+extraction and integer-valued inputs bit-exact.
+"""
+import numpy as np
+import pytest
+
+import oracle
+from oracle import poly_ref as pr
+import synth
+from synth import ConvShape
+from helpers import GATE, normwise, bf16_round, gpu_forward
+
+pytestmark = pytest.mark.gpu
+
+MATH_KERNELS = [("fp32", "fp32"), ("fp32", "thin"), ("tf32", "tc"), ("bf16", "tc"), ("tf32", "thin"),
+                ("bf16", "thin")]
+
+SHAPES = [
+    ConvShape("tiny", 1, 1, 8, 8, 1, 3, 3),                      # BASELINE configs[0]
+    ConvShape("ragged", 2, 20, 13, 11, 40, 3, 3, 1, 1, 1, 1),   # C, K, plane all ragged
+    ConvShape("multi_tile", 3, 70, 17, 19, 80, 3, 3, 1, 1, 1, 1),
+    ConvShape("stride2", 2, 32, 15, 14, 64, 3, 3, 2, 2, 1, 1),
+    ConvShape("k5", 2, 16, 12, 12, 48, 5, 5, 1, 1, 2, 2),
+    ConvShape("k1", 2, 64, 9, 9, 96, 1, 1, 1, 1, 0, 0),
+    ConvShape("k1s2", 2, 48, 10, 10, 64, 1, 1, 2, 2, 0, 0),
+    ConvShape("stem", 1, 3, 30, 30, 64, 7, 7, 2, 2, 3, 3),
+    ConvShape("wideK", 1, 64, 10, 10, 320, 3, 3, 1, 1, 1, 1),   # 2 n-tiles, ragged last
+    ConvShape("rect", 2, 24, 7, 16, 32, 2, 4, 1, 1, 0, 1),
+    ConvShape("thinK", 2, 33, 9, 9, 8, 3, 3, 1, 1, 1, 1),
+]
+
+
+def _skip_unsupported(shape, math, kernel):
+    if kernel == "fp32" and max(shape.R, shape.S) > 7:
+        pytest.skip("fp32 kernel limited to S<=7")
+
+
+@pytest.mark.parametrize("shape", SHAPES, ids=lambda s: s.name)
+@pytest.mark.parametrize("math,kernel", MATH_KERNELS, ids=lambda v: str(v))
+def test_parity_uniform(shape, math, kernel):
+    _skip_unsupported(shape, math, kernel)
+    x, w = synth.make_inputs(shape, synth.seed_for(9, hash(shape.name) % 997), "uniform")
+    ref = oracle.conv2d(x, w, shape.stride, shape.padding)
+    y, plan = gpu_forward(shape, x, w, math=math, kernel=kernel)
+    assert plan.info()["kernel"] == kernel
+    assert y.shape == ref.shape
+    err = normwise(y, ref)
+    assert err <= GATE[math], f"normwise {err:.3e} > {GATE[math]} ({math}/{kernel})"
+
+
+@pytest.mark.parametrize("shape", SHAPES, ids=lambda s: s.name)
+@pytest.mark.parametrize("math,kernel", MATH_KERNELS, ids=lambda v: str(v))
+def test_integer_exact(shape, math, kernel):
+    """|x|<=8, |w|<=4: every product and partial sum is an integer < 2^24, so
+    every precision must reproduce the oracle bit for bit."""
+    _skip_unsupported(shape, math, kernel)
+    x, w = synth.make_inputs(shape, synth.seed_for(8, hash(shape.name) % 997), "int")
+    ref = oracle.conv2d(x, w, shape.stride, shape.padding)
+    y, _ = gpu_forward(shape, x, w, math=math, kernel=kernel)
+    assert np.array_equal(y, ref)
+
+
+@pytest.mark.parametrize("shape", [SHAPES[1], SHAPES[3], SHAPES[7]], ids=lambda s: s.name)
+def test_bf16_io(shape):
+    """bf16 in/out (math BF16): integer data -> output equals round_bf16(oracle);
+    uniform data within the 2e-2 gate against the fp32-input oracle."""
+    x, w = synth.make_inputs(shape, 77, "int")
+    ref = oracle.conv2d(x, w, shape.stride, shape.padding)
+    y, _ = gpu_forward(shape, x, w, math="bf16", io="bf16")
+    assert np.array_equal(y, bf16_round(ref))
+    x, w = synth.make_inputs(shape, 78, "uniform")
+    ref = oracle.conv2d(x, w, shape.stride, shape.padding)
+    y, _ = gpu_forward(shape, x, w, math="bf16", io="bf16")
+    assert normwise(y, ref) <= GATE["bf16"]
+
+
+@pytest.mark.parametrize("math,kernel", [("fp32", "fp32"), ("bf16", "tc"), ("tf32", "tc"), ("fp32", "thin")])
+def test_delta_filter_bit_exact(math, kernel):
+    """w[k][c][i][j] = [c == k mod C][i == i0][j == j0] -> y = shifted xpad,
+    bit-exact for every tap (checks each shift e(i,j) and the padding)."""
+    import torch
+    shape = ConvShape("delta", 2, 16, 9, 10, 32, 3, 3, 1, 1, 1, 1)
+    x, _ = synth.make_inputs(shape, 5, "uniform")
+    x = bf16_round(x)  # representable in every operand format
+    xp = np.pad(x, ((0, 0), (0, 0), (1, 1), (1, 1)))
+    for i0 in range(3):
+        for j0 in range(3):
+            w = np.zeros((32, 16, 3, 3), np.float32)
+            for k in range(32):
+                w[k, k % 16, i0, j0] = 1.0
+            y, _ = gpu_forward(shape, x, w, math=math, kernel=kernel)
+            want = xp[:, [k % 16 for k in range(32)], i0:i0 + 9, j0:j0 + 10]
+            assert np.array_equal(y, want), (i0, j0)
+
+
+@pytest.mark.parametrize("math", ["fp32", "tf32", "bf16"])
+def test_conv3x_full(math):
+    """BASELINE configs[1] (ResNet-50 conv3_x, N=32) in full against O1."""
+    shape = synth.CONV3X
+    x, w = synth.make_inputs(shape, synth.seed_for(1), "uniform")
+    ref = oracle.conv2d(x, w, shape.stride, shape.padding)
+    y, plan = gpu_forward(shape, x, w, math=math)
+    assert normwise(y, ref) <= GATE[math]
+
+
+def test_conv3x_bench_launch_config():
+    """The exact launch the bench times (conv3_x, bf16 in/out, math BF16, AUTO)."""
+    shape = synth.CONV3X
+    x, w = synth.make_inputs(shape, synth.seed_for(1), "uniform")
+    ref = oracle.conv2d(x, w, shape.stride, shape.padding)
+    y, plan = gpu_forward(shape, x, w, math="bf16", io="bf16")
+    assert plan.info()["kernel"] == "tc"
+    assert normwise(y, ref) <= GATE["bf16"]
+    xi, wi = synth.make_inputs(shape, synth.seed_for(1), "int")
+    y, _ = gpu_forward(shape, xi, wi, math="bf16", io="bf16", plan=plan)
+    assert np.array_equal(y, bf16_round(oracle.conv2d(xi, wi, shape.stride, shape.padding)))
+
+
+# --------------------------------------------------------------- single steps --
+
+PACK_SHAPES = [ConvShape("p1", 2, 5, 7, 6, 9, 3, 2, 1, 1, 1, 2), ConvShape("p2", 1, 70, 5, 5, 33, 3, 3, 1, 1, 1, 1),
+               ConvShape("p3", 3, 3, 11, 4, 64, 5, 5, 2, 2, 2, 2)]
+
+
+@pytest.mark.parametrize("shape", PACK_SHAPES, ids=lambda s: s.name)
+@pytest.mark.parametrize("math", ["fp32", "tf32", "bf16"])
+def test_pack_bit_exact(shape, math):
+    import torch
+    import paper_conf_cgo_xuzc025_b200 as pc
+    x, w = synth.make_inputs(shape, 4, "uniform")
+    xt, wt = torch.from_numpy(x).cuda(), torch.from_numpy(w).cuda()
+    plan = pc.Plan(x.shape, w.shape, shape.stride, shape.padding, math=math)
+    inf = plan.info()
+    wdt = np.uint16 if math == "bf16" else np.uint32
+    # planar input A_{n,c}(t) (Eq. 10)
+    got = plan.pack_input(xt, "planar").cpu().numpy().view(wdt)
+    want = pr.pack_input_planar(x, shape.padding, math)
+    assert np.array_equal(got, want.reshape(-1))
+    # interleaved input [N*L_A][Cp]: the same words, channels innermost, zero channel padding
+    got = plan.pack_input(xt, "interleaved").cpu().numpy().view(wdt).reshape(shape.N * inf["L_A"], inf["Cp"])
+    wi = np.zeros((shape.N, inf["L_A"], inf["Cp"]), wdt)
+    wi[:, :, :shape.C] = want.transpose(0, 2, 1)
+    assert np.array_equal(got, wi.reshape(-1, inf["Cp"]))
+    # planar filter U_{k,c}(t) (Eq. 6/11, reading R1)
+    got = plan.pack_filter(wt, "planar").cpu().numpy().view(wdt)
+    wantu = pr.pack_filter_planar(w, inf["Wp"], math)
+    assert np.array_equal(got, wantu.reshape(-1))
+    # tap-major filter [R*S][Kp][Cp]: the nonzero coefficients of U by degree e(i,j)
+    got = plan.pack_filter(wt, "interleaved").cpu().numpy().view(wdt).reshape(shape.R * shape.S, inf["Kp"], inf["Cp"])
+    tm = np.zeros_like(got)
+    for i in range(shape.R):
+        for j in range(shape.S):
+            e = pr.kernel_degree(i, j, shape.R, shape.S, inf["Wp"])
+            tm[i * shape.S + j, :shape.K, :shape.C] = wantu[:, :, e]
+    assert np.array_equal(got, tm)
+
+
+@pytest.mark.parametrize("shape", PACK_SHAPES + [synth.TINY], ids=lambda s: s.name)
+def test_extract_bit_exact(shape):
+    """a5 alone: (1) index-valued coefficients -> y holds exactly the Eq. 12
+    degrees; (2) the oracle's full product (np.convolve) -> y == O1."""
+    import torch
+    import paper_conf_cgo_xuzc025_b200 as pc
+    plan = pc.Plan((shape.N, shape.C, shape.H, shape.W), (shape.K, shape.C, shape.R, shape.S), shape.stride,
+                   shape.padding, math="fp32")
+    inf = plan.info()
+    Lp = inf["L_A"] + inf["L_U"] - 1
+    idx = np.arange(shape.N * shape.K * Lp, dtype=np.float32).reshape(shape.N, shape.K, Lp)  # exact < 2^24
+    y = plan.extract(torch.from_numpy(idx).cuda()).cpu().numpy()
+    for n in range(shape.N):
+        for k in range(shape.K):
+            deg = np.array([[pr.extraction_degree(oh, ow, shape.R, shape.S, inf["Wp"], shape.sh, shape.sw)
+                             for ow in range(inf["Q"])] for oh in range(inf["P"])])
+            assert np.array_equal(y[n, k], idx[n, k][deg])
+    if shape.sh == 1 and shape.sw == 1:
+        x, w = synth.make_inputs(shape, 6, "int")
+        fp = pr.full_product(x, w, shape.padding).astype(np.float32)
+        y = plan.extract(torch.from_numpy(fp).cuda()).cpu().numpy()
+        assert np.array_equal(y, oracle.conv2d(x, w, shape.stride, shape.padding))
+
+
+# ------------------------------------------------------- larger / sampled sizes --
+
+def _sampled(shape, math, io="f32", images=None, seed=0):
+    """Full-size launch; compare images {0, N-1} against O1 on those images."""
+    import torch
+    import paper_conf_cgo_xuzc025_b200 as pc
+    N = shape.N
+    images = images or sorted({0, N - 1})
+    dt = torch.bfloat16 if io == "bf16" else torch.float32
+    gen = torch.Generator(device="cuda").manual_seed(seed)
+    x = (torch.rand((N, shape.C, shape.H, shape.W), generator=gen, device="cuda") * 2 - 1)
+    w = (torch.rand((shape.K, shape.C, shape.R, shape.S), generator=gen, device="cuda") * 2 - 1) / np.sqrt(
+        shape.C * shape.R * shape.S)
+    x, w = x.to(dt), w.to(dt)
+    plan = pc.Plan(x.shape, w.shape, shape.stride, shape.padding, math=math, io_dtype=io)
+    y = plan.forward(x, w)
+    torch.cuda.synchronize()
+    xs = x[images].float().cpu().numpy()
+    ref = oracle.conv2d(xs, w.float().cpu().numpy(), shape.stride, shape.padding)
+    return normwise(y[images].float().cpu().numpy(), ref), plan
+
+
+@pytest.mark.parametrize("shape", [s for s in synth.RESNET50], ids=lambda s: s.name)
+def test_resnet50_sampled_bf16(shape):
+    err, plan = _sampled(shape, "bf16", io="bf16", seed=11)
+    assert err <= GATE["bf16"]
+
+
+@pytest.mark.parametrize("shape", [synth.VGG16[i] for i in (0, 1, 4, 8, 12)], ids=lambda s: s.name)
+@pytest.mark.parametrize("math", ["bf16", "tf32", "fp32"])
+def test_vgg16_sampled(shape, math):
+    err, plan = _sampled(shape, math, seed=12)
+    assert err <= GATE[math]
+
+
+@pytest.mark.parametrize("shape", [s for s in synth.SWEEP if s.flops() < 4e11][::3], ids=lambda s: s.name)
+def test_sweep_sampled_bf16(shape):
+    err, plan = _sampled(shape, "bf16", seed=13)
+    assert err <= GATE["bf16"]
+
+
+def test_batch_shard_bit_identical():
+    """Per-image results do not depend on the batch they are computed in
+    (reading R12): forward(x[a:b]) == forward(x)[a:b] bit for bit -- the basis
+    of the batch-sharded multi-GPU path."""
+    shape = ConvShape("shard", 8, 64, 14, 14, 128, 3, 3, 1, 1, 1, 1)
+    x, w = synth.make_inputs(shape, 21, "uniform")
+    for math in ("bf16", "tf32", "fp32"):
+        y_all, _ = gpu_forward(shape, x, w, math=math)
+        for a, b in [(0, 2), (2, 5), (5, 8)]:
+            ys, _ = gpu_forward(shape.with_batch(b - a), x[a:b], w, math=math)
+            assert np.array_equal(ys, y_all[a:b]), (math, a, b)
+
+
+def test_errors_on_device():
+    import torch
+    import paper_conf_cgo_xuzc025_b200 as pc
+    plan = pc.Plan((1, 4, 8, 8), (8, 4, 3, 3), math="bf16")
+    x = torch.zeros(1 * 4 * 8 * 8 + 1, device="cuda")
+    w = torch.zeros((8, 4, 3, 3), device="cuda")
+    y = torch.zeros((1, 8, 6, 6), device="cuda")
+    with pytest.raises(pc.PolyconvError) as e:
+        plan.forward_ptr(x.data_ptr() + 4, w.data_ptr(), y.data_ptr())   # misaligned x
+    assert e.value.status == pc.NOT_SUPPORTED
+    with pytest.raises(pc.PolyconvError) as e:
+        plan.forward_ptr(x.data_ptr(), w.data_ptr(), x.data_ptr())       # y aliases x
+    assert e.value.status == pc.BAD_PARAM
