@@ -130,6 +130,24 @@ polyconv_status_t polyconv_plan_info(polyconv_plan_t plan, polyconv_info_t *info
 polyconv_status_t polyconv_forward(polyconv_plan_t plan, const void *x, const void *w,
                                    void *y, void *stream);
 
+/* polyconv_forward from HOST buffers (the end-to-end call): x, w, y are host
+ * pointers (pinned for asynchronous copies; pageable works but serialises).
+ * Enqueues on `stream`: H2D copy of x and w into plan-owned device buffers
+ * (allocated at first use, freed by polyconv_destroy), polyconv_forward, D2H
+ * copy of y.  Does not synchronise: x, w, y must stay valid until `stream`
+ * is synchronised.  Errors as polyconv_forward (ALLOC_FAILED if the device
+ * buffers cannot be allocated). */
+polyconv_status_t polyconv_forward_host(polyconv_plan_t plan, const void *x, const void *w,
+                                        void *y, void *stream);
+
+/* Measurement hook: if both are non-NULL cudaEvent_t (passed as void*), every
+ * later forward records start_event just before and stop_event just after the
+ * coefficient-MAC launch (the dominant kernel) on the forward's stream.  NULL,
+ * NULL clears the hook.  BAD_PARAM if exactly one is NULL.  The events stay
+ * owned by the caller and must outlive their use. */
+polyconv_status_t polyconv_plan_set_timing_events(polyconv_plan_t plan, void *start_event,
+                                                  void *stop_event);
+
 /* a2 alone: write A_{n,c}(t) of x into dst in `layout` (see above).  dst must
  * hold polyconv_packed_bytes(plan, 0, layout) bytes. */
 polyconv_status_t polyconv_pack_input(polyconv_plan_t plan, const void *x, void *dst,

@@ -45,7 +45,7 @@ class Info(ctypes.Structure):
 
 
 EXPORTS = ["polyconv_plan", "polyconv_plan_set_kernel", "polyconv_output_dims", "polyconv_plan_info",
-           "polyconv_forward", "polyconv_pack_input", "polyconv_pack_filter", "polyconv_packed_bytes",
+           "polyconv_forward", "polyconv_forward_host", "polyconv_plan_set_timing_events", "polyconv_pack_input", "polyconv_pack_filter", "polyconv_packed_bytes",
            "polyconv_extract", "polyconv_destroy", "polyconv_status_string", "polyconv_last_error",
            "polyconv_abi_version"]
 
@@ -68,6 +68,8 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
     lib.polyconv_output_dims.argtypes = [vp, ip, ip]
     lib.polyconv_plan_info.argtypes = [vp, ctypes.POINTER(Info)]
     lib.polyconv_forward.argtypes = [vp, vp, vp, vp, vp]
+    lib.polyconv_forward_host.argtypes = [vp, vp, vp, vp, vp]
+    lib.polyconv_plan_set_timing_events.argtypes = [vp, vp, vp]
     lib.polyconv_pack_input.argtypes = [vp, vp, vp, i, vp]
     lib.polyconv_pack_filter.argtypes = [vp, vp, vp, i, vp]
     lib.polyconv_packed_bytes.argtypes = [vp, i, i, ctypes.POINTER(ctypes.c_size_t)]
@@ -173,6 +175,28 @@ class Plan:
         self._check(self._lib.polyconv_forward(self._h, ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(w.data_ptr()),
                                                ctypes.c_void_p(y.data_ptr()), _stream_ptr(stream)), "forward")
         return y
+
+    def forward_host(self, x, w, y, stream=None):
+        """End-to-end call: x, w, y are (pinned) CPU tensors; the library copies
+        them to/from its own device buffers on `stream` and runs the forward.
+        Asynchronous: synchronise the stream before reading y."""
+        for t, shp, nm in ((x, self.x_shape, "x"), (w, self.w_shape, "w"), (y, self.output_shape, "y")):
+            if t.is_cuda or tuple(t.shape) != tuple(shp) or t.dtype != self._io_torch_dtype() or not t.is_contiguous():
+                raise PolyconvError(BAD_PARAM, "%s must be a contiguous host tensor %s of %s" % (nm, shp, self.io_dtype))
+        self._check(self._lib.polyconv_forward_host(self._h, ctypes.c_void_p(x.data_ptr()),
+                                                    ctypes.c_void_p(w.data_ptr()), ctypes.c_void_p(y.data_ptr()),
+                                                    _stream_ptr(stream)), "forward_host")
+        return y
+
+    def set_timing_events(self, start, stop):
+        """Record torch.cuda.Event start/stop around the MAC kernel of every later
+        forward (None, None clears)."""
+        for ev in (start, stop):
+            if ev is not None and not ev.cuda_event:
+                ev.record()  # torch creates the underlying cudaEvent_t lazily
+        sp = ctypes.c_void_p(start.cuda_event) if start is not None else None
+        ep = ctypes.c_void_p(stop.cuda_event) if stop is not None else None
+        self._check(self._lib.polyconv_plan_set_timing_events(self._h, sp, ep), "set_timing_events")
 
     def forward_ptr(self, x_ptr: int, w_ptr: int, y_ptr: int, stream_ptr: int = 0):
         """Raw-pointer forward (no checks beyond the library's)."""

@@ -31,6 +31,13 @@ struct polyconv_plan_s {
   int num_sms = 148;
   cudaStream_t last_stream = nullptr;
   bool used = false;
+  // polyconv_forward_host: plan-owned device copies of x, w, y (lazy)
+  void* hx = nullptr;
+  void* hw = nullptr;
+  void* hy = nullptr;
+  // polyconv_plan_set_timing_events: recorded around the MAC launch
+  cudaEvent_t ev_start = nullptr;
+  cudaEvent_t ev_stop = nullptr;
   char err[512];
 };
 
@@ -265,19 +272,55 @@ polyconv_status_t polyconv_forward(polyconv_plan_t p, const void* x, const void*
     // a2 + a3 in one launch (interleaved A, tap-major U), then the MAC (a4+a5)
     e = launch_pack_both_interleaved(g, x, w, p->io_bf16, p->wsA, p->wsU, p->fmt, st);
     if (e != cudaSuccess) return finish(p, e, "pack");
+    if (p->ev_start) cudaEventRecord(p->ev_start, st);
     e = launch_mac_tc(g, p->tc, p->fmt, p->wsA, p->wsU, y, p->io_bf16, st, p->err, sizeof(p->err));
+    if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
     return finish(p, e, "mac_tc");
   }
   e = launch_pack_input_planar(g, x, p->io_bf16, p->wsA, p->fmt, st);
   if (e != cudaSuccess) return finish(p, e, "pack_input");
   e = launch_pack_filter_tapmajor(g, w, p->io_bf16, p->wsU, p->fmt, g.Kp, g.Cp, st);
   if (e != cudaSuccess) return finish(p, e, "pack_filter");
+  if (p->ev_start) cudaEventRecord(p->ev_start, st);
   if (p->kernel == POLYCONV_KERNEL_FP32) {
     e = launch_mac_fp32(g, p->f32, (const float*)p->wsA, (const float*)p->wsU, g.Kp, g.Cp, (float*)y, st);
+    if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
     return finish(p, e, "mac_fp32");
   }
   e = launch_mac_thin(g, p->wsA, p->wsU, g.Kp, g.Cp, p->fmt, y, p->io_bf16, st);
+  if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
   return finish(p, e, "mac_thin");
+}
+
+polyconv_status_t polyconv_forward_host(polyconv_plan_t p, const void* x, const void* w, void* y, void* stream) {
+  if (!p) return POLYCONV_STATUS_BAD_PARAM;
+  if (!x || !w || !y || x == y || w == y) return POLYCONV_STATUS_BAD_PARAM;
+  PC_BEGIN(p);
+  const Geom& g = p->g;
+  const size_t eb = p->io_bf16 ? 2 : 4;
+  const size_t xb = eb * g.N * g.C * g.H * g.W, wb = eb * g.K * g.C * g.R * g.S, yb = eb * g.N * g.K * g.P * g.Q;
+  if (!p->hx || !p->hw || !p->hy) {
+    if ((!p->hx && cudaMalloc(&p->hx, xb) != cudaSuccess) || (!p->hw && cudaMalloc(&p->hw, wb) != cudaSuccess) ||
+        (!p->hy && cudaMalloc(&p->hy, yb) != cudaSuccess)) {
+      cudaGetLastError();
+      set_err(p, "cudaMalloc of %s buffers failed", "host-path");
+      return POLYCONV_STATUS_ALLOC_FAILED;
+    }
+  }
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  cudaError_t e = cudaMemcpyAsync(p->hx, x, xb, cudaMemcpyHostToDevice, st);
+  if (e == cudaSuccess) e = cudaMemcpyAsync(p->hw, w, wb, cudaMemcpyHostToDevice, st);
+  if (e != cudaSuccess) return finish(p, e, "forward_host H2D");
+  polyconv_status_t s = polyconv_forward(p, p->hx, p->hw, p->hy, stream);
+  if (s != POLYCONV_STATUS_SUCCESS) return s;
+  return finish(p, cudaMemcpyAsync(y, p->hy, yb, cudaMemcpyDeviceToHost, st), "forward_host D2H");
+}
+
+polyconv_status_t polyconv_plan_set_timing_events(polyconv_plan_t p, void* start_event, void* stop_event) {
+  if (!p || (!start_event) != (!stop_event)) return POLYCONV_STATUS_BAD_PARAM;
+  p->ev_start = static_cast<cudaEvent_t>(start_event);
+  p->ev_stop = static_cast<cudaEvent_t>(stop_event);
+  return POLYCONV_STATUS_SUCCESS;
 }
 
 polyconv_status_t polyconv_packed_bytes(polyconv_plan_t p, int which, polyconv_layout_t layout, size_t* bytes) {
@@ -335,7 +378,7 @@ polyconv_status_t polyconv_extract(polyconv_plan_t p, const float* coeffs, void*
 polyconv_status_t polyconv_destroy(polyconv_plan_t p) {
   if (!p) return POLYCONV_STATUS_SUCCESS;
   polyconv_status_t s = POLYCONV_STATUS_SUCCESS;
-  if (p->used || p->wsA || p->wsU) {
+  if (p->used || p->wsA || p->wsU || p->hx || p->hw || p->hy) {
     DeviceGuard guard(p->device);
     if (p->used && cudaStreamSynchronize(p->last_stream) != cudaSuccess) {
       cudaGetLastError();
@@ -343,6 +386,9 @@ polyconv_status_t polyconv_destroy(polyconv_plan_t p) {
     }
     if (p->wsA) cudaFree(p->wsA);
     if (p->wsU) cudaFree(p->wsU);
+    if (p->hx) cudaFree(p->hx);
+    if (p->hw) cudaFree(p->hw);
+    if (p->hy) cudaFree(p->hy);
   }
   delete p;
   return s;
