@@ -71,14 +71,18 @@ typedef enum {
 } polyconv_math_t;
 
 /* MAC kernel variant.  AUTO picks by shape and math; the others force one
- * (ablations/tests).  TC = tcgen05/TMEM tensor-core contraction; FP32 = SIMT
- * register-blocked FFMA; THIN = warp-per-output with shuffle reduction over
- * C*R*S (tiny channel counts). */
+ * (ablations/tests).  TC = tcgen05/TMEM tensor-core contraction, filters as
+ * the M=128 operand, one position window per channel chunk reused by every
+ * tap (Hankel shift = descriptor offset); TC_PERTAP = the earlier tensor-core
+ * variant with positions as M and one TMA window load per tap (ablation);
+ * FP32 = SIMT register-blocked FFMA; THIN = warp-per-output with shuffle
+ * reduction over C*R*S (tiny channel counts). */
 typedef enum {
     POLYCONV_KERNEL_AUTO = 0,
     POLYCONV_KERNEL_TC = 1,
     POLYCONV_KERNEL_FP32 = 2,
-    POLYCONV_KERNEL_THIN = 3
+    POLYCONV_KERNEL_THIN = 3,
+    POLYCONV_KERNEL_TC_PERTAP = 4
 } polyconv_kernel_t;
 
 /* Packed-operand layouts exposed for bit-exact tests (a2/a3):

@@ -71,4 +71,24 @@ TcTiling tc_tiling(const Geom& g, int fmt, int num_sms);
 cudaError_t launch_mac_tc(const Geom& g, const TcTiling& t, int fmt, const void* A, const void* U,
                           void* y, bool y_bf16, cudaStream_t st, char* err, size_t errlen);
 
+// ---- mac_tc2.cu (default tensor-core path: window reuse across taps) ----------
+struct Tc2Tiling {
+  int nt;          // positions per tile (UMMA N), multiple of 16, <= 256
+  int kc;          // channels per chunk (one swizzle row)
+  int row_bytes;   // kc * element bytes: 32, 64 or 128
+  int nr;          // kernel rows served by one position window
+  int ngroups;     // ceil(R / nr)
+  int brows;       // rows of one position window (multiple of 32)
+  int num_mt, num_kt, num_tiles, nchunks;
+  int cs;          // cluster size (CTAs sharing multicast filter tiles)
+  int num_groups;  // cluster work items: ceil(num_mt / cs) * num_kt
+  int a_stages;    // filter-tile ring depth
+  int smem_bytes, acc_stride, tmem_cols, grid;
+};
+bool tc2_supported(const Geom& g, int fmt);
+Tc2Tiling tc2_tiling(const Geom& g, int fmt, int num_sms);
+// A: interleaved packed input [N*L_A][Cp]; U: tap-major packed filter [RS][Kp][Cp], Kp % 128 == 0
+cudaError_t launch_mac_tc2(const Geom& g, const Tc2Tiling& t, int fmt, const void* A, const void* U,
+                           void* y, bool y_bf16, cudaStream_t st, char* err, size_t errlen);
+
 }  // namespace polyconv

@@ -21,6 +21,7 @@ struct polyconv_plan_s {
   int forced;
   int kernel;  // resolved polyconv_kernel_t
   TcTiling tc;
+  Tc2Tiling tc2;
   Fp32Tiling f32;
   // workspace (lazy)
   void* wsA = nullptr;
@@ -56,15 +57,22 @@ polyconv_status_t resolve(polyconv_plan_t p) {
   const bool tc_math = p->math != POLYCONV_MATH_FP32_FMA;
   if (k == POLYCONV_KERNEL_AUTO) {
     if (tc_math)
-      k = (g.K >= 16 && tc_supported(g, p->fmt)) ? POLYCONV_KERNEL_TC : POLYCONV_KERNEL_THIN;
+      k = (g.K >= 16 && tc2_supported(g, p->fmt))  ? POLYCONV_KERNEL_TC
+          : (g.K >= 16 && tc_supported(g, p->fmt)) ? POLYCONV_KERNEL_TC_PERTAP
+                                                   : POLYCONV_KERNEL_THIN;
     else
       k = (g.K >= 16 && g.C * g.R * g.S >= 16 && fp32_tiling(g).smax > 0) ? POLYCONV_KERNEL_FP32
                                                                           : POLYCONV_KERNEL_THIN;
   }
-  if (k == POLYCONV_KERNEL_TC && (!tc_math || !tc_supported(g, p->fmt))) return POLYCONV_STATUS_BAD_PARAM;
+  if (k == POLYCONV_KERNEL_TC && (!tc_math || !tc2_supported(g, p->fmt))) return POLYCONV_STATUS_BAD_PARAM;
+  if (k == POLYCONV_KERNEL_TC_PERTAP && (!tc_math || !tc_supported(g, p->fmt))) return POLYCONV_STATUS_BAD_PARAM;
   if (k == POLYCONV_KERNEL_FP32 && (tc_math || fp32_tiling(g).smax == 0)) return POLYCONV_STATUS_BAD_PARAM;
   p->kernel = k;
   if (k == POLYCONV_KERNEL_TC) {
+    p->tc2 = tc2_tiling(g, p->fmt, p->num_sms);
+    g.Cp = (g.C + p->tc2.kc - 1) / p->tc2.kc * p->tc2.kc;
+    g.Kp = (g.K + 127) / 128 * 128;
+  } else if (k == POLYCONV_KERNEL_TC_PERTAP) {
     p->tc = tc_tiling(g, p->fmt, p->num_sms);
     g.Cp = (g.C + p->tc.kc - 1) / p->tc.kc * p->tc.kc;
     g.Kp = (g.K + p->tc.bn - 1) / p->tc.bn * p->tc.bn;
@@ -77,7 +85,7 @@ polyconv_status_t resolve(polyconv_plan_t p) {
     g.Kp = g.K;
   }
   const int eb = fmt_bytes(p->fmt);
-  const size_t a_elems = (k == POLYCONV_KERNEL_TC) ? (size_t)g.N * g.L_A * g.Cp : (size_t)g.N * g.C * g.L_A;
+  const size_t a_elems = (k == POLYCONV_KERNEL_TC || k == POLYCONV_KERNEL_TC_PERTAP) ? (size_t)g.N * g.L_A * g.Cp : (size_t)g.N * g.C * g.L_A;
   p->wsA_bytes = a_elems * eb;
   p->wsU_bytes = (size_t)g.R * g.S * g.Kp * g.Cp * eb;
   return POLYCONV_STATUS_SUCCESS;
@@ -219,7 +227,7 @@ polyconv_status_t polyconv_plan(polyconv_plan_t* plan, int N, int C, int H, int 
 
 polyconv_status_t polyconv_plan_set_kernel(polyconv_plan_t p, polyconv_kernel_t kernel) {
   if (!p) return POLYCONV_STATUS_BAD_PARAM;
-  if (kernel < POLYCONV_KERNEL_AUTO || kernel > POLYCONV_KERNEL_THIN) return POLYCONV_STATUS_BAD_PARAM;
+  if (kernel < POLYCONV_KERNEL_AUTO || kernel > POLYCONV_KERNEL_TC_PERTAP) return POLYCONV_STATUS_BAD_PARAM;
   const int old = p->forced;
   p->forced = kernel;
   if (resolve(p) != POLYCONV_STATUS_SUCCESS) {
@@ -248,10 +256,16 @@ polyconv_status_t polyconv_plan_info(polyconv_plan_t p, polyconv_info_t* info) {
   info->P = g.P; info->Q = g.Q; info->Hp = g.Hp; info->Wp = g.Wp;
   info->L_A = g.L_A; info->L_U = g.L_U; info->Cp = g.Cp; info->Kp = g.Kp;
   info->kernel = p->kernel;
-  info->tile_m = p->kernel == POLYCONV_KERNEL_TC ? p->tc.bm : (p->kernel == POLYCONV_KERNEL_FP32 ? 256 : 1);
-  info->tile_n = p->kernel == POLYCONV_KERNEL_TC ? p->tc.bn : (p->kernel == POLYCONV_KERNEL_FP32 ? 64 : 1);
-  info->stages = p->kernel == POLYCONV_KERNEL_TC ? p->tc.stages : 1;
-  info->launches = p->kernel == POLYCONV_KERNEL_TC ? 2 : 3;
+  switch (p->kernel) {
+    case POLYCONV_KERNEL_TC:  // tile = positions x output channels
+      info->tile_m = p->tc2.nt; info->tile_n = 128; info->stages = p->tc2.a_stages; info->launches = 2; break;
+    case POLYCONV_KERNEL_TC_PERTAP:
+      info->tile_m = p->tc.bm; info->tile_n = p->tc.bn; info->stages = p->tc.stages; info->launches = 2; break;
+    case POLYCONV_KERNEL_FP32:
+      info->tile_m = 256; info->tile_n = 64; info->stages = 1; info->launches = 3; break;
+    default:
+      info->tile_m = 1; info->tile_n = 1; info->stages = 1; info->launches = 3; break;
+  }
   info->workspace_bytes = p->wsA_bytes + p->wsU_bytes;
   return POLYCONV_STATUS_SUCCESS;
 }
@@ -268,12 +282,15 @@ polyconv_status_t polyconv_forward(polyconv_plan_t p, const void* x, const void*
   p->used = true;
   const Geom& g = p->g;
   cudaError_t e;
-  if (p->kernel == POLYCONV_KERNEL_TC) {
+  if (p->kernel == POLYCONV_KERNEL_TC || p->kernel == POLYCONV_KERNEL_TC_PERTAP) {
     // a2 + a3 in one launch (interleaved A, tap-major U), then the MAC (a4+a5)
     e = launch_pack_both_interleaved(g, x, w, p->io_bf16, p->wsA, p->wsU, p->fmt, st);
     if (e != cudaSuccess) return finish(p, e, "pack");
     if (p->ev_start) cudaEventRecord(p->ev_start, st);
-    e = launch_mac_tc(g, p->tc, p->fmt, p->wsA, p->wsU, y, p->io_bf16, st, p->err, sizeof(p->err));
+    if (p->kernel == POLYCONV_KERNEL_TC)
+      e = launch_mac_tc2(g, p->tc2, p->fmt, p->wsA, p->wsU, y, p->io_bf16, st, p->err, sizeof(p->err));
+    else
+      e = launch_mac_tc(g, p->tc, p->fmt, p->wsA, p->wsU, y, p->io_bf16, st, p->err, sizeof(p->err));
     if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
     return finish(p, e, "mac_tc");
   }

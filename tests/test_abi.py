@@ -74,13 +74,20 @@ def test_kernel_selection_and_forcing():
 
 
 def test_tc_tiling_choices():
+    # default TC: tile = nt positions x 128 output channels; conv3_x (G = 31*900 + 838
+    # positions) -> nt = 208 gives 139 tiles, one wave on 148 SMs
     inf = pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="bf16").info()
-    assert (inf["tile_m"], inf["tile_n"], inf["Cp"], inf["Kp"]) == (128, 128, 128, 128)
+    assert (inf["tile_m"], inf["tile_n"], inf["Cp"], inf["Kp"]) == (208, 128, 128, 128)
     inf = pc.Plan((2, 3, 30, 30), (64, 3, 7, 7), (2, 2), (3, 3), math="bf16").info()
-    assert inf["Cp"] == 16 and inf["Kp"] == 64            # C=3 -> one 32-byte swizzle row
+    assert inf["Cp"] == 16 and inf["Kp"] == 128           # C=3 -> one 32-byte swizzle row
     inf = pc.Plan((2, 3, 30, 30), (64, 3, 7, 7), (2, 2), (3, 3), math="tf32").info()
     assert inf["Cp"] == 8
     inf = pc.Plan((1, 64, 10, 10), (320, 64, 3, 3), (1, 1), (1, 1), math="bf16").info()
+    assert inf["tile_n"] == 128 and inf["Kp"] == 384
+    # TC_PERTAP (ablation): tile = 128 positions x bn output channels
+    inf = pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="bf16", kernel="tc_pertap").info()
+    assert (inf["tile_m"], inf["tile_n"], inf["Cp"], inf["Kp"]) == (128, 128, 128, 128)
+    inf = pc.Plan((1, 64, 10, 10), (320, 64, 3, 3), (1, 1), (1, 1), math="bf16", kernel="tc_pertap").info()
     assert inf["tile_n"] == 256 and inf["Kp"] == 512
 
 

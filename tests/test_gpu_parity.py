@@ -16,7 +16,8 @@ from helpers import GATE, normwise, bf16_round, gpu_forward
 
 pytestmark = pytest.mark.gpu
 
-MATH_KERNELS = [("fp32", "fp32"), ("fp32", "thin"), ("tf32", "tc"), ("bf16", "tc"), ("tf32", "thin"),
+MATH_KERNELS = [("fp32", "fp32"), ("fp32", "thin"), ("tf32", "tc"), ("bf16", "tc"), ("tf32", "tc_pertap"),
+                ("bf16", "tc_pertap"), ("tf32", "thin"),
                 ("bf16", "thin")]
 
 SHAPES = [
@@ -78,7 +79,8 @@ def test_bf16_io(shape):
     assert normwise(y, ref) <= GATE["bf16"]
 
 
-@pytest.mark.parametrize("math,kernel", [("fp32", "fp32"), ("bf16", "tc"), ("tf32", "tc"), ("fp32", "thin")])
+@pytest.mark.parametrize("math,kernel", [("fp32", "fp32"), ("bf16", "tc"), ("tf32", "tc"), ("fp32", "thin"),
+                                         ("bf16", "tc_pertap")])
 def test_delta_filter_bit_exact(math, kernel):
     """w[k][c][i][j] = [c == k mod C][i == i0][j == j0] -> y = shifted xpad,
     bit-exact for every tap (checks each shift e(i,j) and the padding)."""

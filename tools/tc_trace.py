@@ -1,0 +1,36 @@
+"""Per-CTA phase trace of the tensor-core MAC (globaltimer), conv3_x bench shape.
+Debug tool: POLYCONV_TC_DEBUG bit 8 makes mac_tc2 record timestamps."""
+import ctypes, os, sys
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np, torch
+import paper_conf_cgo_xuzc025_b200 as pc, synth
+
+shape = synth.CONV3X
+math = sys.argv[1] if len(sys.argv) > 1 else "bf16"
+modes = [int(m) for m in sys.argv[2:]] or [0]
+io = "bf16" if math == "bf16" else "f32"
+dt = torch.bfloat16 if io == "bf16" else torch.float32
+x, w = synth.make_inputs(shape, 1, "uniform")
+x, w = torch.from_numpy(x).cuda().to(dt), torch.from_numpy(w).cuda().to(dt)
+plan = pc.Plan(x.shape, w.shape, shape.stride, shape.padding, math=math, io_dtype=io)
+print(plan.info())
+lib = pc.load_library()
+buf = (ctypes.c_ulonglong * (160 * 8))()
+flush = torch.empty(64 << 20, device="cuda")
+names = ["setup", "first_B_full", "mma_issued", "epi_start", "epi_end", "producer_exit", "cta_end"]
+for mode in modes:
+    os.environ["POLYCONV_TC_DEBUG"] = str(8 | mode)
+    for it in range(3):
+        flush.zero_()
+        y = plan.forward(x, w)
+        torch.cuda.synchronize()
+    lib.polyconv_dbg_tc2_trace(buf)
+    a = np.array(buf, dtype=np.float64).reshape(160, 8)[: plan.info()["tile_m"] and 148]
+    a = a[a[:, 0] > 0]
+    t0 = a[:, 0].min()
+    rel = (a - t0) / 1e3
+    print("mode", mode, "CTAs", len(a), "start spread %.2f us" % (rel[:, 0].max()))
+    for k, nm in enumerate(names, 1):
+        col = rel[:, k]
+        print("  %-14s min %7.2f  med %7.2f  max %7.2f us" % (nm, col.min(), np.median(col), col.max()))
+os.environ["POLYCONV_TC_DEBUG"] = "0"
