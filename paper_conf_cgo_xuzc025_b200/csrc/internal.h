@@ -87,8 +87,12 @@ struct Tc2Tiling {
 };
 bool tc2_supported(const Geom& g, int fmt);
 Tc2Tiling tc2_tiling(const Geom& g, int fmt, int num_sms);
-// A: interleaved packed input [N*L_A][Cp]; U: tap-major packed filter [RS][Kp][Cp], Kp % 128 == 0
-cudaError_t launch_mac_tc2(const Geom& g, const Tc2Tiling& t, int fmt, const void* A, const void* U,
-                           void* y, bool y_bf16, cudaStream_t st, char* err, size_t errlen);
+// x: NCHW input (io dtype; packed on the fly, a2 fused); U: tap-major packed
+// filter [RS][Kp][Cp], Kp % 128 == 0.  pdl: launch as a programmatic dependent
+// of the preceding kernel (the filter pack), which it waits for before
+// reading U.
+cudaError_t launch_mac_tc2(const Geom& g, const Tc2Tiling& t, int fmt, const void* x, bool x_bf16,
+                           const void* U, void* y, bool y_bf16, bool pdl, cudaStream_t st, char* err,
+                           size_t errlen);
 
 }  // namespace polyconv

@@ -133,6 +133,9 @@ template <typename InT, int F>
 __global__ void __launch_bounds__(kThreads) pack_filter_tapmajor_kernel(Geom g, const InT* __restrict__ w,
                                                                         typename Word<F>::T* __restrict__ dst,
                                                                         int Kp, int Cp) {
+  // let a programmatic dependent (the tensor-core MAC) start its prologue now;
+  // it waits (griddepcontrol.wait) for this grid's completion before reading dst
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
   const long long total = (long long)g.R * g.S * Kp * Cp;
   for (long long idx = blockIdx.x * (long long)kThreads + threadIdx.x; idx < total;
        idx += (long long)gridDim.x * kThreads)

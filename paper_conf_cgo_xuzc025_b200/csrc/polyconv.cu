@@ -85,7 +85,11 @@ polyconv_status_t resolve(polyconv_plan_t p) {
     g.Kp = g.K;
   }
   const int eb = fmt_bytes(p->fmt);
-  const size_t a_elems = (k == POLYCONV_KERNEL_TC || k == POLYCONV_KERNEL_TC_PERTAP) ? (size_t)g.N * g.L_A * g.Cp : (size_t)g.N * g.C * g.L_A;
+  // TC packs the input on the fly (no input workspace); TC_PERTAP needs the
+  // interleaved copy, FP32/THIN the planar one
+  const size_t a_elems = k == POLYCONV_KERNEL_TC          ? 0
+                         : k == POLYCONV_KERNEL_TC_PERTAP ? (size_t)g.N * g.L_A * g.Cp
+                                                          : (size_t)g.N * g.C * g.L_A;
   p->wsA_bytes = a_elems * eb;
   p->wsU_bytes = (size_t)g.R * g.S * g.Kp * g.Cp * eb;
   return POLYCONV_STATUS_SUCCESS;
@@ -282,17 +286,24 @@ polyconv_status_t polyconv_forward(polyconv_plan_t p, const void* x, const void*
   p->used = true;
   const Geom& g = p->g;
   cudaError_t e;
-  if (p->kernel == POLYCONV_KERNEL_TC || p->kernel == POLYCONV_KERNEL_TC_PERTAP) {
+  if (p->kernel == POLYCONV_KERNEL_TC) {
+    // a3 (filter pack, tiny) then the fused a2+a4+a5 kernel, launched as its
+    // programmatic dependent so its prologue and input packing overlap the pack
+    if (p->ev_start) cudaEventRecord(p->ev_start, st);
+    e = launch_pack_filter_tapmajor(g, w, p->io_bf16, p->wsU, p->fmt, g.Kp, g.Cp, st);
+    if (e != cudaSuccess) return finish(p, e, "pack_filter");
+    e = launch_mac_tc2(g, p->tc2, p->fmt, x, p->io_bf16, p->wsU, y, p->io_bf16, true, st, p->err, sizeof(p->err));
+    if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
+    return finish(p, e, "mac_tc");
+  }
+  if (p->kernel == POLYCONV_KERNEL_TC_PERTAP) {
     // a2 + a3 in one launch (interleaved A, tap-major U), then the MAC (a4+a5)
     e = launch_pack_both_interleaved(g, x, w, p->io_bf16, p->wsA, p->wsU, p->fmt, st);
     if (e != cudaSuccess) return finish(p, e, "pack");
     if (p->ev_start) cudaEventRecord(p->ev_start, st);
-    if (p->kernel == POLYCONV_KERNEL_TC)
-      e = launch_mac_tc2(g, p->tc2, p->fmt, p->wsA, p->wsU, y, p->io_bf16, st, p->err, sizeof(p->err));
-    else
-      e = launch_mac_tc(g, p->tc, p->fmt, p->wsA, p->wsU, y, p->io_bf16, st, p->err, sizeof(p->err));
+    e = launch_mac_tc(g, p->tc, p->fmt, p->wsA, p->wsU, y, p->io_bf16, st, p->err, sizeof(p->err));
     if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
-    return finish(p, e, "mac_tc");
+    return finish(p, e, "mac_tc_pertap");
   }
   e = launch_pack_input_planar(g, x, p->io_bf16, p->wsA, p->fmt, st);
   if (e != cudaSuccess) return finish(p, e, "pack_input");

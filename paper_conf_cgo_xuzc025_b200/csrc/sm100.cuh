@@ -53,6 +53,29 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   } while (!done);
 }
 
+// mbar_wait for roles that wait long (epilogue, packers): back off with
+// __nanosleep between polls so the waiting warps leave the issue slots to the
+// warps doing work on the same SM sub-partition.
+__device__ __forceinline__ void mbar_wait_sleep(uint64_t* bar, uint32_t parity, uint32_t ns) {
+  const uint32_t a = smem_u32(bar);
+  uint32_t done;
+  uint64_t t0 = 0;
+  for (;;) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(done)
+        : "r"(a), "r"(parity)
+        : "memory");
+    if (done) return;
+    const uint64_t t = global_ns();
+    if (t0 == 0) t0 = t;
+    else if (t - t0 > 500000000ull) __trap();
+    __nanosleep(ns);
+  }
+}
+
 // One lane of the (fully active) warp returns true.  Issue loops run on the
 // whole warp so the compiler keeps their control values in uniform registers,
 // and only the elected lane issues TMA / tcgen05 instructions.

@@ -17,7 +17,7 @@ print(plan.info())
 lib = pc.load_library()
 buf = (ctypes.c_ulonglong * (160 * 8))()
 flush = torch.empty(64 << 20, device="cuda")
-names = ["setup", "first_B_full", "mma_issued", "epi_start", "epi_end", "producer_exit", "cta_end"]
+names = ["setup", "first_B_full", "mma_issued", "epi_start", "epi_end", "packer_win0", "cta_end"]
 for mode in modes:
     os.environ["POLYCONV_TC_DEBUG"] = str(8 | mode)
     for it in range(3):
@@ -29,8 +29,11 @@ for mode in modes:
     a = a[a[:, 0] > 0]
     t0 = a[:, 0].min()
     rel = (a - t0) / 1e3
+
     print("mode", mode, "CTAs", len(a), "start spread %.2f us" % (rel[:, 0].max()))
-    for k, nm in enumerate(names, 1):
+    nm_list = names if not (mode & 64) else ["setup", "pk_waited", "pk_zeroed", "pk_barrier", "pk_scattered",
+                                              "packer_win0", "cta_end"]
+    for k, nm in enumerate(nm_list, 1):
         col = rel[:, k]
         print("  %-14s min %7.2f  med %7.2f  max %7.2f us" % (nm, col.min(), np.median(col), col.max()))
 os.environ["POLYCONV_TC_DEBUG"] = "0"
