@@ -83,10 +83,12 @@ struct Tc2Tiling {
   int cs;          // cluster size (CTAs sharing multicast filter tiles)
   int num_groups;  // cluster work items: ceil(num_mt / cs) * num_kt
   int a_stages;    // filter-tile ring depth
+  bool tma_x;      // raw input staged by TMA (x as [N*C][H*W], 16-byte row pitch) vs direct loads
+  int box_bytes, stg_bytes;
   int smem_bytes, acc_stride, tmem_cols, grid;
 };
 bool tc2_supported(const Geom& g, int fmt);
-Tc2Tiling tc2_tiling(const Geom& g, int fmt, int num_sms);
+Tc2Tiling tc2_tiling(const Geom& g, int fmt, bool x_bf16, int num_sms);
 // x: NCHW input (io dtype; packed on the fly, a2 fused); U: tap-major packed
 // filter [RS][Kp][Cp], Kp % 128 == 0.  pdl: launch as a programmatic dependent
 // of the preceding kernel (the filter pack), which it waits for before

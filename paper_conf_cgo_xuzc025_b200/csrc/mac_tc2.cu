@@ -19,7 +19,11 @@
 //    the NCHW input -- coefficient r*Wp + s of A_{n,c}(t) is x[n][c][r-ph][s-pw]
 //    or 0 (Eq. 10, zero padding P.1353-1356) -- converting to the operand
 //    format (BF16 RNE / TF32 RNA, reading R11) and writing the swizzled
-//    K-major layout.  No packed copy of the input ever goes to HBM.
+//    K-major layout.  No packed copy of the input ever goes to HBM.  The raw
+//    input rows are brought in by TMA (boxes of 64 plane elements x kc channel
+//    planes, x viewed as [N*C][H*W]) into a staging buffer one window ahead,
+//    and transposed shared->shared; when H*W*elem is not a multiple of 16
+//    bytes (no TMA view) the packers load x directly (slow path).
 //  * Window reuse: one window of nt + (nr-1)*Wp + S-1 positions per channel
 //    chunk serves every tap (i,j) of nr kernel rows (all R when it fits): the
 //    tap's MMA reads it through a descriptor whose start is shifted by
@@ -32,16 +36,19 @@
 //    the loops run warp-wide so their control values stay in uniform
 //    registers -- issuing from a divergent lane-0 branch halved the MMA rate,
 //    tools/umma_rate.cu), warps 2-9 = packers, warps 10-17 = epilogue.
-//  * Epilogue (a5, fused): tcgen05.ld 32 channels x 64 positions -> shared
-//    transpose -> each lane owns two adjacent positions and stores them as one
-//    bf16x2 / float2 word per channel when they are adjacent output pixels;
-//    junk positions (off the Eq. 12 / R4 extraction lattice) are dropped.
+//  * Epilogue (a5, fused): tcgen05.ld.16x256b gives each lane two adjacent
+//    positions of four output channels; each pair is stored as one bf16x2 /
+//    float2 word per channel when it is two adjacent output pixels (8 lanes
+//    cover 16 consecutive pixels of a channel row); junk positions (off the
+//    Eq. 12 / R4 extraction lattice) are dropped.
 #include <cuda.h>
 #include <type_traits>
 #include "common.cuh"
 #include "sm100.cuh"
 #include <cstdio>
+#include <cstring>
 #include <cstdlib>
+#include <algorithm>
 
 namespace polyconv {
 
@@ -56,7 +63,8 @@ constexpr int kPackWarp0 = 2;
 constexpr int kEpiWarp0 = kPackWarp0 + kPackWarps;
 constexpr int kThreads = 32 * (kEpiWarp0 + kEpiWarps);
 constexpr int kBMaxRows = 384;           // max rows of one position window (48 KB at 128 B rows)
-constexpr int kTStride = 68;             // epilogue transpose row stride in floats (64 + 4 pad)
+constexpr int kBoxE = 64;                // plane elements per staging TMA box
+constexpr int kMaxSeg = 4;               // images one window may span on the TMA staging path
 
 struct Tc2Params {
   const void* x;    // NCHW input, io dtype
@@ -64,11 +72,14 @@ struct Tc2Params {
   long long NLA;    // N*L_A: positions that exist
   long long L_A, PQ, HW;
   int N, C, H, W, ph, pw, Hp;
+  int ealign;       // 16 / sizeof(input element): staging boxes start on this element multiple
   int Wp, P, Q, sh, sw, K, R, S;
   int nt, brows, nr, ngroups;
   int num_mt, num_kt, num_tiles, num_groups;
   int nchunks, kc, Kp;
   int a_stages;
+  uint32_t box_bytes;  // staging TMA box: kBoxE elements x kc planes
+  uint32_t stg_bytes;  // staging buffer (max boxes of any window)
   uint32_t idesc, a_bytes, b_bytes, row_bytes;
   int acc_stride, tmem_cols;
   void* y;          // NCHW output, io dtype (= the input's)
@@ -77,8 +88,6 @@ struct Tc2Params {
 
 // per-CTA phase timestamps (globaltimer ns) for POLYCONV_TC_DEBUG & 8
 __device__ unsigned long long g_tc2_trace[160 * 8];
-// packer fine trace (POLYCONV_TC_DEBUG & 16): clock64 per step of the first window, packer thread 0
-__device__ long long g_tc2_ptrace[160 * 16];
 
 // Input element -> operand word (reading R11: BF16 = RNE, TF32 = RNA).
 template <typename InT, bool kTf32>
@@ -98,22 +107,92 @@ struct ToWord<float, true> {
   __device__ __forceinline__ static uint32_t cvt(float v) { return to_tf32_rna(v); }
 };
 
-template <typename InT, bool kTf32, int CS, bool kVec>
+// ---- packer helpers (fused a2) ---------------------------------------------------
+struct Seg {
+  int n, e_lo, box0;  // image, first plane element staged, first staging box
+};
+
+// Position window wi of this CTA (in the MMA's order): first coefficient, first channel.
+template <int CS>
+__device__ __forceinline__ void tc2_window(const Tc2Params& p, int cl_id, int cl_num, uint32_t rank, int wi,
+                                           long long& wrow, int& cbase) {
+  const int wpg = p.nchunks * p.ngroups;
+  const int grp = cl_id + (wi / wpg) * cl_num, inner = wi % wpg;
+  const int ch = inner / p.ngroups, rg = inner - ch * p.ngroups;
+  const long long g0 = (long long)((grp / p.num_kt) * CS + (int)rank) * p.nt;
+  wrow = g0 + (long long)p.Wp * (rg * p.nr);
+  cbase = ch * p.kc;
+}
+
+// The x elements window wrow needs: per image segment q, plane elements
+// [e_lo, e_lo + boxes*kBoxE) of image sg[q].n (sg[q].n = -1: no rows of that
+// image).  Returns (segments) | (total boxes << 8).
+__device__ __forceinline__ int tc2_segments(const Tc2Params& p, long long wrow, Seg (&sg)[kMaxSeg]) {
+  int ns = 0, boxes = 0;
+#pragma unroll
+  for (int q = 0; q < kMaxSeg; ++q) sg[q].n = -1;
+  if (wrow >= p.NLA) return 0;
+  const int n_lo = (int)(wrow / p.L_A);
+  const int n_hi = (int)min((long long)p.N - 1, (wrow + p.brows - 1) / p.L_A);
+#pragma unroll
+  for (int q = 0; q < kMaxSeg; ++q) {  // unrolled: the segment table stays in registers
+    const int n = n_lo + q;
+    if (n > n_hi) continue;
+    const int base = (int)((long long)n * p.L_A - wrow);  // window row of coefficient 0 of image n
+    const int pr_lo = base >= 0 ? 0 : (-base) / p.Wp;
+    const int pr_hi = min(p.Hp - 1, (p.brows - 1 - base) / p.Wp);
+    const int h_lo = max(0, pr_lo - p.ph), h_hi = min(p.H - 1, pr_hi - p.ph);
+    if (h_lo > h_hi) continue;
+    // a TMA box must start 16-byte aligned in global memory: round the first
+    // element down to a multiple of 16/sizeof(elem) (planes start aligned)
+    const int e_lo = (h_lo * p.W) & ~(p.ealign - 1);
+    sg[q].n = n;
+    sg[q].e_lo = e_lo;
+    sg[q].box0 = boxes;
+    boxes += ((h_hi + 1) * p.W - e_lo + kBoxE - 1) / kBoxE;
+    ns = q + 1;
+  }
+  return ns | (boxes << 8);
+}
+
+// Staging TMA of window (wrow, cbase): boxes of kBoxE plane elements x kc planes.
+__device__ __forceinline__ void tc2_issue_staging(const Tc2Params& p, const CUtensorMap* tmX, uint8_t* sX,
+                                                  uint64_t* sfull, long long wrow, int cbase) {
+  Seg sg[kMaxSeg];
+  const int r = tc2_segments(p, wrow, sg);
+  const int boxes = r >> 8;
+  mbar_arrive_expect_tx(sfull, (uint32_t)boxes * p.box_bytes);
+#pragma unroll
+  for (int q = 0; q < kMaxSeg; ++q) {
+    if (sg[q].n < 0) continue;
+    int nxt = boxes;
+#pragma unroll
+    for (int q2 = kMaxSeg - 1; q2 > q; --q2)
+      if (sg[q2].n >= 0) nxt = sg[q2].box0;
+    for (int b = sg[q].box0; b < nxt; ++b)
+      tma_load_2d(sX + (size_t)b * p.box_bytes, tmX, sfull, sg[q].e_lo + (b - sg[q].box0) * kBoxE,
+                  sg[q].n * p.C + cbase);
+  }
+}
+
+template <typename InT, bool kTf32, int CS, bool kTmaX>
 __global__ void __launch_bounds__(kThreads, 1)
-    mac_tc2_kernel(const __grid_constant__ CUtensorMap tmW, const Tc2Params p) {
+    mac_tc2_kernel(const __grid_constant__ CUtensorMap tmW, const __grid_constant__ CUtensorMap tmX,
+                   const Tc2Params p) {
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw = smem_u32(smem_raw);
   uint8_t* smem = smem_raw + (((raw + 1023u) & ~1023u) - raw);
   uint8_t* sA = smem;                                        // filter tiles  [a_stages][128][row]
   uint8_t* sB = sA + (size_t)p.a_stages * p.a_bytes;         // position windows [2][brows][row]
-  float* sT = reinterpret_cast<float*>(sB + 2 * (size_t)p.b_bytes);  // [kEpiWarps][32][kTStride]
-  uint64_t* afull = reinterpret_cast<uint64_t*>(sT + kEpiWarps * 32 * kTStride);
+  uint8_t* sX = sB + 2 * (size_t)p.b_bytes;                  // raw-input staging (TMA path)
+  uint64_t* afull = reinterpret_cast<uint64_t*>(sX + (kTmaX ? (size_t)p.stg_bytes : 0));
   uint64_t* aempty = afull + p.a_stages;
   uint64_t* bfull = aempty + p.a_stages;
   uint64_t* bempty = bfull + 2;
   uint64_t* tfull = bempty + 2;
   uint64_t* tempty = tfull + 2;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+  uint64_t* sfull = tempty + 2;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(sfull + 1);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   // clusters of CS CTAs share one output-channel block: the filter tiles are
@@ -128,6 +207,7 @@ __global__ void __launch_bounds__(kThreads, 1)
 
   if (warp == 0 && lane == 0) {
     prefetch_tmap(&tmW);
+    if constexpr (kTmaX) prefetch_tmap(&tmX);
     for (int s = 0; s < p.a_stages; ++s) {
       mbar_init(afull + s, 1);
       mbar_init(aempty + s, CS);  // every CTA of the cluster reads the multicast filter tile
@@ -138,6 +218,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       mbar_init(tfull + s, 1);
       mbar_init(tempty + s, kEpiWarps);
     }
+    mbar_init(sfull, 1);
     fence_barrier_init();
   }
   if (warp == 1) tmem_alloc(tmem_slot, (uint32_t)p.tmem_cols);
@@ -235,209 +316,177 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
   } else if (warp < kEpiWarp0) {
     // ------------------------------------------- packers: fused a2 (Eq. 10 + padding)
-    // Window rows are coefficients gp = wrow + r of the concatenated input
-    // polynomials; coefficient pr*Wp + ps of A_{n,c} is x[n][c][pr-ph][ps-pw] or 0.
-    // Step 1 zeroes the window (padding coefficients, past N*L_A).  Step 2
-    // walks the x elements that land in it in units of EPC channels x V
-    // consecutive plane elements: EPC loads (one 16-byte vector per channel
-    // plane when kVec), a register transpose, and V 16-byte shared stores --
-    // one swizzled chunk (EPC channels of one coefficient) per element.  The 8
-    // lanes that share a segment cover the 8 chunks of one 128-byte row.
+    // Window row r is coefficient gp = wrow + r of the concatenated input
+    // polynomials; coefficient pr*Wp + ps of A_{n,c} is x[n][c][pr-ph][ps-pw],
+    // or 0 in the padding / past N*L_A.  Each packer thread builds whole rows:
+    // the kc channel words of one coefficient, as row_bytes/16 swizzled
+    // 16-byte chunks.  Consecutive lanes take consecutive rows.
     const int ptid = (warp - kPackWarp0) * 32 + lane;
-    constexpr int kEB = kTf32 ? 4 : 2;                          // operand word bytes
-    constexpr int EPC = 16 / kEB;                               // channels per 16-byte chunk
-    constexpr int V = kVec ? 16 / (int)sizeof(InT) : 1;         // plane elements per unit
+    constexpr int kNP = kPackWarps * 32;
+    constexpr int kEB = kTf32 ? 4 : 2;               // operand word bytes
+    constexpr int EPC = 16 / kEB;                    // channels per 16-byte chunk
     const uint32_t swmask = p.row_bytes / 16u - 1u;  // 128/64/32-byte swizzle: chunk ^= (addr>>7) & swmask
-    const int ncg = (int)p.row_bytes / 16;                      // chunks (channel groups) per row
+    const int ncg = (int)p.row_bytes / 16;           // chunks per row
     const InT* __restrict__ x = reinterpret_cast<const InT*>(p.x);
+    const InT* stg = reinterpret_cast<const InT*>(sX);
+    const int my_groups = p.num_groups > cl_id ? (p.num_groups - cl_id + cl_num - 1) / cl_num : 0;
+    const int nwin = my_groups * p.nchunks * p.ngroups;  // position windows this CTA packs
+    if constexpr (kTmaX) {
+      if (ptid == 0 && nwin > 0) {
+        long long wrow;
+        int cbase;
+        tc2_window<CS>(p, cl_id, cl_num, rank, 0, wrow, cbase);
+        tc2_issue_staging(p, &tmX, sX, sfull, wrow, cbase);
+      }
+    }
     int bs = 0;
-    uint32_t bph = 0;
-    for (int grp = cl_id; grp < p.num_groups; grp += cl_num) {
-      const long long g0 = (long long)((grp / p.num_kt) * CS + (int)rank) * p.nt;
-      for (int ch = 0; ch < p.nchunks; ++ch) {
-        const int cbase = ch * p.kc;
-        for (int rg = 0; rg < p.ngroups; ++rg) {
-          const long long wrow = g0 + (long long)p.Wp * (rg * p.nr);
-          const bool pt = (p.dbg & 16) && ptid == 0 && blockIdx.x < 160 && grp == cl_id && ch == 0 && rg == 0;
-          long long* ptr = g_tc2_ptrace + blockIdx.x * 16;
-          int npt = 0;
-          if (pt) ptr[npt++] = clock64();
-          mbar_wait_sleep(bempty + bs, bph ^ 1u, 64);
-          if (pt) ptr[npt++] = clock64();
-          uint8_t* dst = sB + (size_t)bs * p.b_bytes;
-          for (int i = ptid; i < (int)(p.b_bytes >> 4); i += kPackWarps * 32)
-            reinterpret_cast<uint4*>(dst)[i] = make_uint4(0u, 0u, 0u, 0u);
-          if (pt) ptr[npt++] = clock64();
-          asm volatile("bar.sync 1, %0;" ::"n"(kPackWarps * 32) : "memory");
-          if (pt) ptr[npt++] = clock64();
-          if (wrow < p.NLA) {
-            const int n_lo = (int)(wrow / p.L_A);
-            const int n_hi = (int)min((long long)p.N - 1, (wrow + p.brows - 1) / p.L_A);
-            for (int n = n_lo; n <= n_hi; ++n) {
-              const int base = (int)((long long)n * p.L_A - wrow);  // window row of coefficient 0 of image n
-              const int pr_lo = base >= 0 ? 0 : (-base) / p.Wp;
-              const int pr_hi = min(p.Hp - 1, (p.brows - 1 - base) / p.Wp);
-              const int h_lo = max(0, pr_lo - p.ph), h_hi = min(p.H - 1, pr_hi - p.ph);
-              if (h_lo > h_hi) continue;
-              const int e_lo = (h_lo * p.W) / V * V;
-              const int e_hi = min((int)p.HW, ((h_hi + 1) * p.W + V - 1) / V * V);
-              const int units = (e_hi - e_lo) / V * ncg;
-              const InT* xn = x + ((long long)n * p.C + cbase) * p.HW;
-              // kU units per thread per round, all loads issued before any use:
-              // the window's x bytes are in flight at once (memory-level parallelism)
-              constexpr int kU = 2;
-#pragma unroll 1
-              for (int u0 = ptid; u0 < units; u0 += kU * kPackWarps * 32) {
-                uint32_t L[kU][EPC][V];
+    uint32_t bph = 0, sph = 0;
+    for (int wi = 0; wi < nwin; ++wi) {
+      long long wrow;
+      int cbase;
+      tc2_window<CS>(p, cl_id, cl_num, rank, wi, wrow, cbase);
+      Seg sg[kMaxSeg];
+      int ns = 0;
+      if constexpr (kTmaX) ns = tc2_segments(p, wrow, sg) & 0xFF;
+      mbar_wait_sleep(bempty + bs, bph ^ 1u, 64);
+      if constexpr (kTmaX) {
+        mbar_wait(sfull, sph);
+        sph ^= 1u;
+      }
+      uint8_t* dst = sB + (size_t)bs * p.b_bytes;
+      for (int r = ptid; r < p.brows; r += kNP) {
+        const long long gp = wrow + r;
+        bool valid = gp < p.NLA;
+        int n = 0, e = 0;
+        if (valid) {
+          n = (int)(gp / p.L_A);
+          const int m = (int)(gp - (long long)n * p.L_A);
+          const int pr = m / p.Wp, ps = m - pr * p.Wp;
+          const int h = pr - p.ph, w = ps - p.pw;
+          valid = h >= 0 && h < p.H && w >= 0 && w < p.W;
+          e = h * p.W + w;
+        }
+        // source of channel c of this coefficient
+        long long src = 0;  // element index into stg (TMA path) or x (direct path)
+        if (valid) {
+          if constexpr (kTmaX) {
+            int e_lo = 0, box0 = 0;
 #pragma unroll
-                for (int t = 0; t < kU; ++t) {
-                  const int u = u0 + t * kPackWarps * 32;
-                  const int seg = u / ncg, cg = u - seg * ncg;
-                  const int e0 = e_lo + seg * V;
+            for (int q = 0; q < kMaxSeg; ++q)  // unrolled: the segment table stays in registers
+              if (q < ns && sg[q].n == n) { e_lo = sg[q].e_lo; box0 = sg[q].box0; }
+            const int de = e - e_lo;
+            src = (long long)(box0 + de / kBoxE) * p.kc * kBoxE + (de % kBoxE);
+          } else {
+            src = ((long long)n * p.C + cbase) * p.HW + e;
+          }
+        }
+        const long long cstride = kTmaX ? (long long)kBoxE : p.HW;
+        const uint32_t rowoff = (uint32_t)r * p.row_bytes;
+        for (int j = 0; j < ncg; ++j) {
+          uint32_t wv[EPC];
 #pragma unroll
-                  for (int e = 0; e < EPC; ++e) {
-                    const int c = cbase + cg * EPC + e;
-                    const InT* src = xn + (long long)(cg * EPC + e) * p.HW + e0;
-                    const bool ok = u < units && c < p.C;
-                    if constexpr (kVec) {
-                      const uint4 q = ok ? __ldg(reinterpret_cast<const uint4*>(src)) : make_uint4(0u, 0u, 0u, 0u);
-                      const uint32_t r4[4] = {q.x, q.y, q.z, q.w};
-#pragma unroll
-                      for (int k = 0; k < V; ++k) {
-                        if constexpr (sizeof(InT) == 2) L[t][e][k] = (r4[k >> 1] >> ((k & 1) * 16)) & 0xFFFFu;
-                        else L[t][e][k] = ToWord<InT, kTf32>::cvt(__uint_as_float(r4[k]));
-                      }
-                    } else {
-                      L[t][e][0] = ok ? ToWord<InT, kTf32>::cvt(__ldg(src)) : 0u;
-                    }
-                  }
-                }
-                if (pt && npt < 14) ptr[npt++] = clock64();
-#pragma unroll
-                for (int t = 0; t < kU; ++t) {
-                  const int u = u0 + t * kPackWarps * 32;
-                  if (u < units) {
-                    const int seg = u / ncg, cg = u - seg * ncg;
-                    const int e0 = e_lo + seg * V;
-                    // element e0 + k lands in window row base + (h+ph)*Wp + w+pw
-                    const int h0 = e0 / p.W;
-                    int w = e0 - h0 * p.W;
-                    int row = base + (h0 + p.ph) * p.Wp + (w + p.pw);
-#pragma unroll
-                    for (int k = 0; k < V; ++k) {
-                      if (row >= 0 && row < p.brows) {
-                        uint4 o;
-                        if constexpr (kEB == 2)
-                          o = make_uint4(L[t][0][k] | (L[t][1][k] << 16), L[t][2][k] | (L[t][3][k] << 16),
-                                         L[t][4][k] | (L[t][5][k] << 16), L[t][6][k] | (L[t][7][k] << 16));
-                        else
-                          o = make_uint4(L[t][0][k], L[t][1][k], L[t][2][k], L[t][3][k]);
-                        const uint32_t off = (uint32_t)row * p.row_bytes + 16u * cg;
-                        *reinterpret_cast<uint4*>(dst + (off ^ (((off >> 7) & swmask) << 4))) = o;
-                      }
-                      // next plane element: next column, or the next row (skipping the padding)
-                      if (++w == p.W) { w = 0; row += p.Wp - p.W + 1; } else { ++row; }
-                    }
-                  }
-                }
-                if (pt && npt < 14) ptr[npt++] = clock64();
-              }
+          for (int t = 0; t < EPC; ++t) {
+            const int c = j * EPC + t;
+            wv[t] = 0u;
+            if (valid && cbase + c < p.C) {
+              const InT v = kTmaX ? stg[src + c * cstride] : __ldg(x + src + c * cstride);
+              wv[t] = ToWord<InT, kTf32>::cvt(v);
             }
           }
-          if (pt) { ptr[npt < 15 ? npt : 15] = clock64(); ptr[15] = npt; }
-          // generic-proxy smem writes -> visible to the tensor core (async proxy)
-          asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-          __syncwarp();
-          if (trace && ptid == 0 && grp == cl_id && ch == 0 && rg == 0) tr[6] = global_ns();
-          if (lane == 0) mbar_arrive(bfull + bs);
-          if (++bs == 2) { bs = 0; bph ^= 1u; }
+          uint4 o;
+          if constexpr (kEB == 2)
+            o = make_uint4(wv[0] | (wv[1] << 16), wv[2] | (wv[3] << 16), wv[4] | (wv[5] << 16), wv[6] | (wv[7] << 16));
+          else
+            o = make_uint4(wv[0], wv[1], wv[2], wv[3]);
+          const uint32_t off = rowoff + 16u * j;
+          *reinterpret_cast<uint4*>(dst + (off ^ (((off >> 7) & swmask) << 4))) = o;
         }
       }
+      // generic-proxy smem writes -> visible to the tensor core (async proxy); every
+      // packer is done with the staging buffer before it is refilled for the next window
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      asm volatile("bar.sync 1, %0;" ::"n"(kNP) : "memory");
+      if constexpr (kTmaX) {
+        if (ptid == 0 && wi + 1 < nwin) {
+          long long wrow1;
+          int cbase1;
+          tc2_window<CS>(p, cl_id, cl_num, rank, wi + 1, wrow1, cbase1);
+          tc2_issue_staging(p, &tmX, sX, sfull, wrow1, cbase1);
+        }
+      }
+      if (trace && ptid == 0 && wi == 0) tr[6] = global_ns();
+      if (lane == 0) mbar_arrive(bfull + bs);
+      if (++bs == 2) { bs = 0; bph ^= 1u; }
     }
   } else {
     // -------------------------------------------------------------- epilogue
-    // warp w reads TMEM lane quadrant (w % 4); the two warps of a quadrant take
-    // alternate 64-column blocks of the accumulator.
+    // warp w reads TMEM lane quadrant (w % 4) (output channels kq..kq+31); the
+    // two warps of a quadrant take alternate 32-column (position) blocks.
+    // tcgen05.ld.16x256b: lane t holds positions c, c+1 (c = cb + 8r + 2(t%4))
+    // of channels kq + {t/4, t/4+8, t/4+16, t/4+24}.
     const int ew = warp - kEpiWarp0;
     const int quad = warp & 3;
     const int csub = ew >> 2, cstep = kEpiWarps / 4;
-    float* T = sT + ew * 32 * kTStride;
+    InT* __restrict__ y = reinterpret_cast<InT*>(p.y);
     int acc = 0;
     uint32_t accph = 0;
     for (int grp = cl_id; grp < p.num_groups; grp += cl_num) {
       const int mg = grp / p.num_kt, kt = grp - mg * p.num_kt;
       const long long g0 = (long long)(mg * CS + (int)rank) * p.nt;
-      const int kq = kt * BMK + quad * 32;  // first output channel of this warp's lanes
-      const int kmax = min(32, p.K - kq);
-      const long long n0 = g0 / p.L_A;      // decode the tile's first position once
+      const int kq = kt * BMK + quad * 32;
+      const int kl = kq + (lane >> 2);  // this lane's first channel; others +8, +16, +24
+      const long long n0 = g0 / p.L_A;  // decode the tile's first position once
       const int m0 = (int)(g0 - n0 * p.L_A);
       mbar_wait_sleep(tfull + acc, accph, 256);
       tc_fence_after();
       if (trace && ew == 0 && lane == 0) tr[4] = global_ns();
       const uint32_t taddr = tmem_base + ((uint32_t)(quad * 32) << 16) + (uint32_t)(acc * p.acc_stride);
-      for (int cb = csub * 64; cb < p.nt; cb += 64 * cstep) {
-        uint32_t v0[32], v1[32];
-        tmem_ld32(taddr + (uint32_t)cb, v0);
-        tmem_ld32(taddr + (uint32_t)cb + 32u, v1);
+      for (int cb = csub * 32; cb < p.nt; cb += 32 * cstep) {
+        uint32_t va[16], vb[16];
+        tmem_ld16x256b_x4(taddr + (uint32_t)cb, va);                  // lanes kq + 0..15
+        tmem_ld16x256b_x4(taddr + (16u << 16) + (uint32_t)cb, vb);    // lanes kq + 16..31
         tmem_ld_wait();
-        // T[channel lane][position 0..63]
-        float4* Trow = reinterpret_cast<float4*>(T + lane * kTStride);
 #pragma unroll
-        for (int q = 0; q < 8; ++q) {
-          Trow[q] = make_float4(__uint_as_float(v0[4 * q]), __uint_as_float(v0[4 * q + 1]),
-                                __uint_as_float(v0[4 * q + 2]), __uint_as_float(v0[4 * q + 3]));
-          Trow[8 + q] = make_float4(__uint_as_float(v1[4 * q]), __uint_as_float(v1[4 * q + 1]),
-                                    __uint_as_float(v1[4 * q + 2]), __uint_as_float(v1[4 * q + 3]));
-        }
-        __syncwarp();
-        // lane -> positions c, c+1 of the tile; a5: keep those on the extraction lattice
-        const int c = cb + 2 * lane;
-        long long n = n0;
-        int m = m0 + c;
-        while (m >= p.L_A) { m -= (int)p.L_A; ++n; }
-        const int r = m / p.Wp, s = m - r * p.Wp;
-        const int oh = r / p.sh, ow = s / p.sw;
-        const bool v0ok = c < p.nt && g0 + c < p.G && (r - oh * p.sh) == 0 && (s - ow * p.sw) == 0 &&
-                          oh < p.P && ow < p.Q;
-        int m1 = m + 1;
-        long long n1 = n;
-        if (m1 >= p.L_A) { m1 -= (int)p.L_A; ++n1; }
-        const int r1 = m1 / p.Wp, s1 = m1 - r1 * p.Wp;
-        const int oh1 = r1 / p.sh, ow1 = s1 / p.sw;
-        const bool v1ok = c + 1 < p.nt && g0 + c + 1 < p.G && (r1 - oh1 * p.sh) == 0 &&
-                          (s1 - ow1 * p.sw) == 0 && oh1 < p.P && ow1 < p.Q;
-        const long long y0 = (n * p.K + kq) * p.PQ + (long long)oh * p.Q + ow;
-        const long long y1 = (n1 * p.K + kq) * p.PQ + (long long)oh1 * p.Q + ow1;
-        // adjacent output pixels, even element offset -> one 2-element store per channel
-        const bool pair = v0ok && v1ok && y1 == y0 + 1 && (y0 & 1) == 0 && (p.PQ & 1) == 0;
-        if (v0ok || v1ok) {
-          const float2* Tcol = reinterpret_cast<const float2*>(T + 2 * lane);
-          InT* y = reinterpret_cast<InT*>(p.y);
-          if (pair) {
-            using Pair = typename std::conditional<sizeof(InT) == 2, __nv_bfloat162, float2>::type;
-            Pair* yp = reinterpret_cast<Pair*>(y + y0);
-            const long long st = p.PQ / 2;
-#pragma unroll 4
-            for (int q = 0; q < kmax; ++q) {
-              const float2 t = Tcol[q * (kTStride / 2)];
-              if constexpr (sizeof(InT) == 2) yp[q * st] = __float22bfloat162_rn(t);
-              else yp[q * st] = t;
-            }
-          } else {
-#pragma unroll 1
-            for (int q = 0; q < kmax; ++q) {
-              const float2 t = Tcol[q * (kTStride / 2)];
-              if constexpr (sizeof(InT) == 2) {
-                if (v0ok) y[y0 + q * p.PQ] = __float2bfloat16_rn(t.x);
-                if (v1ok) y[y1 + q * p.PQ] = __float2bfloat16_rn(t.y);
-              } else {
-                if (v0ok) y[y0 + q * p.PQ] = t.x;
-                if (v1ok) y[y1 + q * p.PQ] = t.y;
-              }
+        for (int rr = 0; rr < 4; ++rr) {
+          // a5: positions c, c+1 -> output pixels, kept iff on the extraction lattice
+          const int c = cb + 8 * rr + 2 * (lane & 3);
+          long long n = n0;
+          int m = m0 + c;
+          while (m >= p.L_A) { m -= (int)p.L_A; ++n; }
+          const int r = m / p.Wp, s = m - r * p.Wp;
+          const int oh = r / p.sh, ow = s / p.sw;
+          const bool v0 = c < p.nt && g0 + c < p.G && r == oh * p.sh && s == ow * p.sw && oh < p.P && ow < p.Q;
+          int m1 = m + 1;
+          long long n1 = n;
+          if (m1 >= p.L_A) { m1 -= (int)p.L_A; ++n1; }
+          const int r1 = m1 / p.Wp, s1 = m1 - r1 * p.Wp;
+          const int oh1 = r1 / p.sh, ow1 = s1 / p.sw;
+          const bool v1 = c + 1 < p.nt && g0 + c + 1 < p.G && r1 == oh1 * p.sh && s1 == ow1 * p.sw &&
+                          oh1 < p.P && ow1 < p.Q;
+          if (!(v0 || v1)) continue;
+          const long long y0 = (n * p.K + kl) * p.PQ + (long long)oh * p.Q + ow;
+          const long long y1 = (n1 * p.K + kl) * p.PQ + (long long)oh1 * p.Q + ow1;
+          // adjacent output pixels at an even element offset -> one 2-element store per channel
+          const bool pair = v0 && v1 && y1 == y0 + 1 && (y0 & 1) == 0 && (p.PQ & 1) == 0;
+#pragma unroll
+          for (int g = 0; g < 4; ++g) {
+            const int k = kl + 8 * g;
+            if (k >= p.K) continue;
+            const uint32_t* vv = g < 2 ? va : vb;
+            const float a0 = __uint_as_float(vv[4 * rr + 2 * (g & 1)]);
+            const float a1 = __uint_as_float(vv[4 * rr + 2 * (g & 1) + 1]);
+            const long long d = (long long)(8 * g) * p.PQ;
+            if (pair) {
+              if constexpr (sizeof(InT) == 2)
+                *reinterpret_cast<__nv_bfloat162*>(y + y0 + d) = __floats2bfloat162_rn(a0, a1);
+              else
+                *reinterpret_cast<float2*>(y + y0 + d) = make_float2(a0, a1);
+            } else {
+              if (v0) y[y0 + d] = (InT)a0;
+              if (v1) y[y1 + d] = (InT)a1;
             }
           }
         }
-        __syncwarp();
       }
       tc_fence_before();
       __syncwarp();
@@ -494,9 +543,9 @@ bool encode(CUtensorMap* map, const void* base, int fmt, uint64_t cols, uint64_t
 inline long long cdiv(long long a, long long b) { return (a + b - 1) / b; }
 
 template <typename InT, bool kTf32, int CS>
-cudaError_t launch_one(const Tc2Tiling& t, const CUtensorMap& tmW, const Tc2Params& p, bool vec, bool pdl,
-                       cudaStream_t st) {
-  auto kern = vec ? mac_tc2_kernel<InT, kTf32, CS, true> : mac_tc2_kernel<InT, kTf32, CS, false>;
+cudaError_t launch_one(const Tc2Tiling& t, const CUtensorMap& tmW, const CUtensorMap& tmX, const Tc2Params& p,
+                       bool pdl, cudaStream_t st) {
+  auto kern = t.tma_x ? mac_tc2_kernel<InT, kTf32, CS, true> : mac_tc2_kernel<InT, kTf32, CS, false>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, t.smem_bytes);
   if (e != cudaSuccess) return e;
   cudaLaunchConfig_t cfg = {};
@@ -513,7 +562,36 @@ cudaError_t launch_one(const Tc2Tiling& t, const CUtensorMap& tmW, const Tc2Para
   attr[1].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   cfg.numAttrs = pdl ? 2 : 1;
-  return cudaLaunchKernelEx(&cfg, kern, tmW, p);
+  return cudaLaunchKernelEx(&cfg, kern, tmW, tmX, p);
+}
+
+// Staging demand of the TMA input path: the most boxes (and image segments)
+// any position window needs -- the same walk the packers do.
+void staging_demand(const Geom& g, const Tc2Tiling& t, int eb_in, int& max_boxes, int& max_segs) {
+  max_boxes = 0;
+  max_segs = 0;
+  const long long NLA = (long long)g.N * g.L_A;
+  for (long long mt = 0; mt < (long long)t.num_groups / t.num_kt * t.cs; ++mt) {  // incl. dummy tiles
+    for (int rg = 0; rg < t.ngroups; ++rg) {
+      const long long wrow = mt * t.nt + (long long)g.Wp * (rg * t.nr);
+      if (wrow >= NLA) continue;
+      const int n_lo = (int)(wrow / g.L_A);
+      const int n_hi = (int)std::min((long long)g.N - 1, (wrow + t.brows - 1) / g.L_A);
+      int boxes = 0, segs = 0;
+      for (int n = n_lo; n <= n_hi; ++n) {
+        const int base = (int)((long long)n * g.L_A - wrow);
+        const int pr_lo = base >= 0 ? 0 : (-base) / g.Wp;
+        const int pr_hi = std::min(g.Hp - 1, (t.brows - 1 - base) / g.Wp);
+        const int h_lo = std::max(0, pr_lo - g.ph), h_hi = std::min(g.H - 1, pr_hi - g.ph);
+        if (h_lo > h_hi) continue;
+        const int e_lo = (h_lo * g.W) & ~(16 / eb_in - 1);
+        boxes += ((h_hi + 1) * g.W - e_lo + kBoxE - 1) / kBoxE;
+        ++segs;
+      }
+      max_boxes = std::max(max_boxes, boxes);
+      max_segs = std::max(max_segs, segs);
+    }
+  }
 }
 
 }  // namespace
@@ -525,7 +603,7 @@ bool tc2_supported(const Geom& g, int fmt) {
   return true;
 }
 
-Tc2Tiling tc2_tiling(const Geom& g, int fmt, int num_sms) {
+Tc2Tiling tc2_tiling(const Geom& g, int fmt, bool x_bf16, int num_sms) {
   Tc2Tiling t{};
   const int eb = fmt_bytes(fmt);
   int kc = 128 / eb;
@@ -566,7 +644,18 @@ Tc2Tiling tc2_tiling(const Geom& g, int fmt, int num_sms) {
   t.nchunks = (g.C + kc - 1) / kc;
   const int a_bytes = BMK * t.row_bytes;
   const int b_bytes = (int)cdiv((long long)t.brows * t.row_bytes, 1024) * 1024;
-  const int fixed = 1024 + 2 * b_bytes + kEpiWarps * 32 * kTStride * 4 + 512;
+  // input staging for the TMA path: x viewed as [N*C][H*W] needs a 16-byte row pitch
+  const int eb_in = x_bf16 ? 2 : 4;
+  t.box_bytes = kBoxE * kc * eb_in;
+  t.tma_x = ((long long)g.H * g.W * eb_in) % 16 == 0;
+  if (t.tma_x) {
+    int max_boxes, max_segs;
+    staging_demand(g, t, eb_in, max_boxes, max_segs);
+    t.stg_bytes = (int)cdiv((long long)std::max(1, max_boxes) * t.box_bytes, 1024) * 1024;
+    if (max_segs > kMaxSeg || 1024 + 2 * b_bytes + t.stg_bytes + 512 + 3 * a_bytes > 227 * 1024) t.tma_x = false;
+  }
+  if (!t.tma_x) t.stg_bytes = 0;
+  const int fixed = 1024 + 2 * b_bytes + t.stg_bytes + 512;
   int st = (227 * 1024 - fixed) / a_bytes;
   if (st > 12) st = 12;
   t.a_stages = st;
@@ -598,9 +687,31 @@ cudaError_t launch_mac_tc2(const Geom& g, const Tc2Tiling& t, int fmt, const voi
   p.PQ = (long long)g.P * g.Q;
   p.HW = (long long)g.H * g.W;
   p.N = g.N; p.C = g.C; p.H = g.H; p.W = g.W; p.ph = g.ph; p.pw = g.pw; p.Hp = g.Hp;
-  // packers load 16-byte vectors when every plane starts 16-byte aligned
-  const int eb_in = x_bf16 ? 2 : 4;
-  const bool vec = (p.HW % (16 / eb_in)) == 0 && (reinterpret_cast<uintptr_t>(x) % 16) == 0;
+  // staging TMA map over x as [N*C][H*W] (TMA path); its base must be 16-byte aligned
+  CUtensorMap tmX;
+  memset(&tmX, 0, sizeof(tmX));
+  if (t.tma_x) {
+    if ((reinterpret_cast<uintptr_t>(x) % 16) != 0) {
+      snprintf(err, errlen, "mac_tc2: x must be 16-byte aligned");
+      return cudaErrorInvalidValue;
+    }
+    EncodeTiledFn enc = get_encode2();
+    const int eb_in = x_bf16 ? 2 : 4;
+    cuuint64_t dims[2] = {(cuuint64_t)p.HW, (cuuint64_t)g.N * g.C};
+    cuuint64_t strides[1] = {(cuuint64_t)p.HW * eb_in};
+    cuuint32_t box[2] = {(cuuint32_t)kBoxE, (cuuint32_t)t.kc};
+    cuuint32_t estr[2] = {1, 1};
+    if (!enc || enc(&tmX, x_bf16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2,
+                    const_cast<void*>(x), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                    CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS) {
+      snprintf(err, errlen, "cuTensorMapEncodeTiled (input staging) failed");
+      return cudaErrorInvalidValue;
+    }
+  }
+  p.box_bytes = (uint32_t)t.box_bytes;
+  p.ealign = x_bf16 ? 8 : 4;
+  p.stg_bytes = (uint32_t)t.stg_bytes;
   p.Wp = g.Wp; p.P = g.P; p.Q = g.Q; p.sh = g.sh; p.sw = g.sw; p.K = g.K; p.R = g.R; p.S = g.S;
   p.nt = t.nt; p.brows = t.brows; p.nr = t.nr; p.ngroups = t.ngroups;
   p.num_mt = t.num_mt; p.num_kt = t.num_kt; p.num_tiles = t.num_tiles; p.num_groups = t.num_groups;
@@ -619,23 +730,20 @@ cudaError_t launch_mac_tc2(const Geom& g, const Tc2Tiling& t, int fmt, const voi
   p.dbg = dbg ? atoi(dbg) : 0;
   if (fmt == FMT_TF32) {
     if (x_bf16) return cudaErrorInvalidValue;
-    return t.cs == 1 ? launch_one<float, true, 1>(t, tmW, p, vec, pdl, st)
-                     : launch_one<float, true, 2>(t, tmW, p, vec, pdl, st);
+    return t.cs == 1 ? launch_one<float, true, 1>(t, tmW, tmX, p, pdl, st)
+                     : launch_one<float, true, 2>(t, tmW, tmX, p, pdl, st);
   }
   if (x_bf16)
-    return t.cs == 1 ? launch_one<__nv_bfloat16, false, 1>(t, tmW, p, vec, pdl, st)
-                     : launch_one<__nv_bfloat16, false, 2>(t, tmW, p, vec, pdl, st);
-  return t.cs == 1 ? launch_one<float, false, 1>(t, tmW, p, vec, pdl, st)
-                   : launch_one<float, false, 2>(t, tmW, p, vec, pdl, st);
+    return t.cs == 1 ? launch_one<__nv_bfloat16, false, 1>(t, tmW, tmX, p, pdl, st)
+                     : launch_one<__nv_bfloat16, false, 2>(t, tmW, tmX, p, pdl, st);
+  return t.cs == 1 ? launch_one<float, false, 1>(t, tmW, tmX, p, pdl, st)
+                   : launch_one<float, false, 2>(t, tmW, tmX, p, pdl, st);
 }
 
 }  // namespace polyconv
 
 // Debug only (not part of include/polyconv.h): copy the per-CTA phase trace of
 // the last POLYCONV_TC_DEBUG&8 launch to host (160 x 8 u64).
-extern "C" int polyconv_dbg_tc2_ptrace(long long* host) {
-  return (int)cudaMemcpyFromSymbol(host, polyconv::g_tc2_ptrace, sizeof(long long) * 160 * 16);
-}
 extern "C" int polyconv_dbg_tc2_trace(unsigned long long* host) {
   return (int)cudaMemcpyFromSymbol(host, polyconv::g_tc2_trace, sizeof(unsigned long long) * 160 * 8);
 }

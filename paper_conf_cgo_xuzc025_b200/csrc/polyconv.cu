@@ -69,7 +69,7 @@ polyconv_status_t resolve(polyconv_plan_t p) {
   if (k == POLYCONV_KERNEL_FP32 && (tc_math || fp32_tiling(g).smax == 0)) return POLYCONV_STATUS_BAD_PARAM;
   p->kernel = k;
   if (k == POLYCONV_KERNEL_TC) {
-    p->tc2 = tc2_tiling(g, p->fmt, p->num_sms);
+    p->tc2 = tc2_tiling(g, p->fmt, p->io_bf16, p->num_sms);
     g.Cp = (g.C + p->tc2.kc - 1) / p->tc2.kc * p->tc2.kc;
     g.Kp = (g.K + 127) / 128 * 128;
   } else if (k == POLYCONV_KERNEL_TC_PERTAP) {

@@ -3,6 +3,7 @@
 // (TMEM alloc, UMMA issue/commit, TMEM loads) and the UMMA descriptors.
 #pragma once
 #include <cstdint>
+#include <cstdio>
 
 namespace polyconv {
 namespace sm100 {
@@ -41,7 +42,10 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
     if ((++spins & 0xFFFu) == 0) {
       const uint64_t t = global_ns();
       if (t0 == 0) t0 = t;
-      else if (t - t0 > 500000000ull) __trap();
+      else if (t - t0 > 500000000ull) {
+        printf("polyconv watchdog: block %d thread %d bar %p parity %u\n", (int)blockIdx.x, (int)threadIdx.x, bar, parity);
+        __trap();
+      }
     }
     asm volatile(
         "{\n\t.reg .pred p;\n\t"
@@ -71,7 +75,10 @@ __device__ __forceinline__ void mbar_wait_sleep(uint64_t* bar, uint32_t parity, 
     if (done) return;
     const uint64_t t = global_ns();
     if (t0 == 0) t0 = t;
-    else if (t - t0 > 500000000ull) __trap();
+    else if (t - t0 > 500000000ull) {
+      printf("polyconv watchdog(sleep): block %d thread %d bar %p parity %u\n", (int)blockIdx.x, (int)threadIdx.x, bar, parity);
+      __trap();
+    }
     __nanosleep(ns);
   }
 }
@@ -184,6 +191,18 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&v)[32]) {
         "=r"(v[15]), "=r"(v[16]), "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]),
         "=r"(v[22]), "=r"(v[23]), "=r"(v[24]), "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]),
         "=r"(v[29]), "=r"(v[30]), "=r"(v[31])
+      : "r"(taddr)
+      : "memory");
+}
+// 16 lanes x 256 bits, repeated 4x along the columns (32 columns): thread t
+// gets, for repetition r, v[4r+0..1] = lane (base + t/4), columns 8r + 2(t%4)
+// and +1, and v[4r+2..3] = lane (base + 8 + t/4), the same columns.
+__device__ __forceinline__ void tmem_ld16x256b_x4(uint32_t taddr, uint32_t (&v)[16]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.16x256b.x4.b32 "
+      "{%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, %15}, [%16];"
+      : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
+        "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]), "=r"(v[15])
       : "r"(taddr)
       : "memory");
 }
