@@ -7,6 +7,22 @@
 
 namespace polyconv {
 
+// Division by a runtime-invariant divisor d >= 1 through a multiply-high
+// (round-up reciprocal; exact for 0 <= n < 2^31).  Set up on the host.
+struct FastDiv {
+  uint32_t d, mul, shr;
+  __host__ __device__ void init(uint32_t div) {
+    d = div;
+    if (div <= 1) { mul = 0; shr = 0; return; }
+    uint32_t l = 0;
+    while ((1ull << l) < div) ++l;  // ceil(log2(div))
+    const uint32_t p = 31 + l;
+    mul = (uint32_t)(((1ull << p) + div - 1) / div);
+    shr = p - 32;
+  }
+  __device__ __forceinline__ uint32_t div(uint32_t n) const { return d == 1 ? n : (__umulhi(n, mul) >> shr); }
+};
+
 __device__ __forceinline__ float load_io(const float* p, long long i) { return __ldg(p + i); }
 __device__ __forceinline__ float load_io(const __nv_bfloat16* p, long long i) {
   return __bfloat162float(p[i]);

@@ -84,6 +84,7 @@ struct Tc2Params {
   int acc_stride, tmem_cols;
   void* y;          // NCHW output, io dtype (= the input's)
   int dbg;          // POLYCONV_TC_DEBUG: 8 = per-CTA phase trace (g_tc2_trace)
+  FastDiv fLA, fWp, fsh, fsw;  // position decode: coefficient -> (n, r, s) -> (oh, ow)
 };
 
 // per-CTA phase timestamps (globaltimer ns) for POLYCONV_TC_DEBUG & 8
@@ -132,15 +133,15 @@ __device__ __forceinline__ int tc2_segments(const Tc2Params& p, long long wrow, 
 #pragma unroll
   for (int q = 0; q < kMaxSeg; ++q) sg[q].n = -1;
   if (wrow >= p.NLA) return 0;
-  const int n_lo = (int)(wrow / p.L_A);
-  const int n_hi = (int)min((long long)p.N - 1, (wrow + p.brows - 1) / p.L_A);
+  const int n_lo = (int)p.fLA.div((uint32_t)wrow);
+  const int n_hi = min(p.N - 1, (int)p.fLA.div((uint32_t)(wrow + p.brows - 1)));
 #pragma unroll
   for (int q = 0; q < kMaxSeg; ++q) {  // unrolled: the segment table stays in registers
     const int n = n_lo + q;
     if (n > n_hi) continue;
     const int base = (int)((long long)n * p.L_A - wrow);  // window row of coefficient 0 of image n
-    const int pr_lo = base >= 0 ? 0 : (-base) / p.Wp;
-    const int pr_hi = min(p.Hp - 1, (p.brows - 1 - base) / p.Wp);
+    const int pr_lo = base >= 0 ? 0 : (int)p.fWp.div((uint32_t)(-base));
+    const int pr_hi = min(p.Hp - 1, (int)p.fWp.div((uint32_t)(p.brows - 1 - base)));
     const int h_lo = max(0, pr_lo - p.ph), h_hi = min(p.H - 1, pr_hi - p.ph);
     if (h_lo > h_hi) continue;
     // a TMA box must start 16-byte aligned in global memory: round the first
@@ -185,7 +186,8 @@ __global__ void __launch_bounds__(kThreads, 1)
   uint8_t* sA = smem;                                        // filter tiles  [a_stages][128][row]
   uint8_t* sB = sA + (size_t)p.a_stages * p.a_bytes;         // position windows [2][brows][row]
   uint8_t* sX = sB + 2 * (size_t)p.b_bytes;                  // raw-input staging (TMA path)
-  uint64_t* afull = reinterpret_cast<uint64_t*>(sX + (kTmaX ? (size_t)p.stg_bytes : 0));
+  long long* sPos = reinterpret_cast<long long*>(sX + (kTmaX ? (size_t)p.stg_bytes : 0));  // [256] epilogue
+  uint64_t* afull = reinterpret_cast<uint64_t*>(sPos + 256);
   uint64_t* aempty = afull + p.a_stages;
   uint64_t* bfull = aempty + p.a_stages;
   uint64_t* bempty = bfull + 2;
@@ -359,9 +361,9 @@ __global__ void __launch_bounds__(kThreads, 1)
         bool valid = gp < p.NLA;
         int n = 0, e = 0;
         if (valid) {
-          n = (int)(gp / p.L_A);
+          n = (int)p.fLA.div((uint32_t)gp);
           const int m = (int)(gp - (long long)n * p.L_A);
-          const int pr = m / p.Wp, ps = m - pr * p.Wp;
+          const int pr = (int)p.fWp.div((uint32_t)m), ps = m - pr * p.Wp;
           const int h = pr - p.ph, w = ps - p.pw;
           valid = h >= 0 && h < p.H && w >= 0 && w < p.W;
           e = h * p.W + w;
@@ -435,12 +437,28 @@ __global__ void __launch_bounds__(kThreads, 1)
       const long long g0 = (long long)(mg * CS + (int)rank) * p.nt;
       const int kq = kt * BMK + quad * 32;
       const int kl = kq + (lane >> 2);  // this lane's first channel; others +8, +16, +24
-      const long long n0 = g0 / p.L_A;  // decode the tile's first position once
+      const long long n0 = g0 / p.L_A;  // the tile's first position: image n0, coefficient m0
       const int m0 = (int)(g0 - n0 * p.L_A);
       mbar_wait_sleep(tfull + acc, accph, 256);
       tc_fence_after();
       if (trace && ew == 0 && lane == 0) tr[4] = global_ns();
       const uint32_t taddr = tmem_base + ((uint32_t)(quad * 32) << 16) + (uint32_t)(acc * p.acc_stride);
+      // a5 for the tile's positions, once: sPos[c] = element offset of pixel
+      // (n, 0, oh, ow) in y (add k*PQ for channel k), or -1 off the Eq. 12 / R4 lattice
+      asm volatile("bar.sync 2, %0;" ::"n"(kEpiWarps * 32) : "memory");  // previous tile's table unused
+      for (int c = ew * 32 + lane; c < p.nt; c += kEpiWarps * 32) {
+        long long off = -1;
+        if (g0 + c < p.G) {
+          int n = (int)n0, m = m0 + c;
+          while (m >= p.L_A) { m -= (int)p.L_A; ++n; }
+          const int r = (int)p.fWp.div((uint32_t)m), s = m - r * p.Wp;
+          const int oh = (int)p.fsh.div((uint32_t)r), ow = (int)p.fsw.div((uint32_t)s);
+          if (r == oh * p.sh && s == ow * p.sw && oh < p.P && ow < p.Q)
+            off = (long long)n * p.K * p.PQ + (long long)oh * p.Q + ow;
+        }
+        sPos[c] = off;
+      }
+      asm volatile("bar.sync 2, %0;" ::"n"(kEpiWarps * 32) : "memory");
       for (int cb = csub * 32; cb < p.nt; cb += 32 * cstep) {
         uint32_t va[16], vb[16];
         tmem_ld16x256b_x4(taddr + (uint32_t)cb, va);                  // lanes kq + 0..15
@@ -448,42 +466,28 @@ __global__ void __launch_bounds__(kThreads, 1)
         tmem_ld_wait();
 #pragma unroll
         for (int rr = 0; rr < 4; ++rr) {
-          // a5: positions c, c+1 -> output pixels, kept iff on the extraction lattice
           const int c = cb + 8 * rr + 2 * (lane & 3);
-          long long n = n0;
-          int m = m0 + c;
-          while (m >= p.L_A) { m -= (int)p.L_A; ++n; }
-          const int r = m / p.Wp, s = m - r * p.Wp;
-          const int oh = r / p.sh, ow = s / p.sw;
-          const bool v0 = c < p.nt && g0 + c < p.G && r == oh * p.sh && s == ow * p.sw && oh < p.P && ow < p.Q;
-          int m1 = m + 1;
-          long long n1 = n;
-          if (m1 >= p.L_A) { m1 -= (int)p.L_A; ++n1; }
-          const int r1 = m1 / p.Wp, s1 = m1 - r1 * p.Wp;
-          const int oh1 = r1 / p.sh, ow1 = s1 / p.sw;
-          const bool v1 = c + 1 < p.nt && g0 + c + 1 < p.G && r1 == oh1 * p.sh && s1 == ow1 * p.sw &&
-                          oh1 < p.P && ow1 < p.Q;
-          if (!(v0 || v1)) continue;
-          const long long y0 = (n * p.K + kl) * p.PQ + (long long)oh * p.Q + ow;
-          const long long y1 = (n1 * p.K + kl) * p.PQ + (long long)oh1 * p.Q + ow1;
+          const long long o0 = c < p.nt ? sPos[c] : -1;
+          const long long o1 = c + 1 < p.nt ? sPos[c + 1] : -1;
+          if (o0 < 0 && o1 < 0) continue;
           // adjacent output pixels at an even element offset -> one 2-element store per channel
-          const bool pair = v0 && v1 && y1 == y0 + 1 && (y0 & 1) == 0 && (p.PQ & 1) == 0;
+          const bool pair = o0 >= 0 && o1 == o0 + 1 && (o0 & 1) == 0 && (p.PQ & 1) == 0;
+          const long long yk = (long long)kl * p.PQ;
 #pragma unroll
           for (int g = 0; g < 4; ++g) {
-            const int k = kl + 8 * g;
-            if (k >= p.K) continue;
+            if (kl + 8 * g >= p.K) continue;
             const uint32_t* vv = g < 2 ? va : vb;
             const float a0 = __uint_as_float(vv[4 * rr + 2 * (g & 1)]);
             const float a1 = __uint_as_float(vv[4 * rr + 2 * (g & 1) + 1]);
-            const long long d = (long long)(8 * g) * p.PQ;
+            const long long d = yk + (long long)(8 * g) * p.PQ;
             if (pair) {
               if constexpr (sizeof(InT) == 2)
-                *reinterpret_cast<__nv_bfloat162*>(y + y0 + d) = __floats2bfloat162_rn(a0, a1);
+                *reinterpret_cast<__nv_bfloat162*>(y + o0 + d) = __floats2bfloat162_rn(a0, a1);
               else
-                *reinterpret_cast<float2*>(y + y0 + d) = make_float2(a0, a1);
+                *reinterpret_cast<float2*>(y + o0 + d) = make_float2(a0, a1);
             } else {
-              if (v0) y[y0 + d] = (InT)a0;
-              if (v1) y[y1 + d] = (InT)a1;
+              if (o0 >= 0) y[o0 + d] = (InT)a0;
+              if (o1 >= 0) y[o1 + d] = (InT)a1;
             }
           }
         }
@@ -600,6 +604,7 @@ bool tc2_supported(const Geom& g, int fmt) {
   if (fmt != FMT_BF16 && fmt != FMT_TF32) return false;
   if ((long long)g.R * g.S * ((g.K + 127) / 128 * 128) >= (1LL << 31)) return false;  // TMA row coordinate
   if (g.S - 1 + 16 > kBMaxRows) return false;  // one kernel row must fit a window
+  if ((long long)g.N * g.L_A + 2 * kBMaxRows + 256 >= (1LL << 31)) return false;  // 32-bit position decode
   return true;
 }
 
@@ -652,10 +657,11 @@ Tc2Tiling tc2_tiling(const Geom& g, int fmt, bool x_bf16, int num_sms) {
     int max_boxes, max_segs;
     staging_demand(g, t, eb_in, max_boxes, max_segs);
     t.stg_bytes = (int)cdiv((long long)std::max(1, max_boxes) * t.box_bytes, 1024) * 1024;
-    if (max_segs > kMaxSeg || 1024 + 2 * b_bytes + t.stg_bytes + 512 + 3 * a_bytes > 227 * 1024) t.tma_x = false;
+    if (max_segs > kMaxSeg || 1024 + 2 * b_bytes + t.stg_bytes + 256 * 8 + 512 + 3 * a_bytes > 227 * 1024)
+      t.tma_x = false;
   }
   if (!t.tma_x) t.stg_bytes = 0;
-  const int fixed = 1024 + 2 * b_bytes + t.stg_bytes + 512;
+  const int fixed = 1024 + 2 * b_bytes + t.stg_bytes + 256 * 8 + 512;
   int st = (227 * 1024 - fixed) / a_bytes;
   if (st > 12) st = 12;
   t.a_stages = st;
@@ -711,6 +717,10 @@ cudaError_t launch_mac_tc2(const Geom& g, const Tc2Tiling& t, int fmt, const voi
   }
   p.box_bytes = (uint32_t)t.box_bytes;
   p.ealign = x_bf16 ? 8 : 4;
+  p.fLA.init((uint32_t)g.L_A);
+  p.fWp.init((uint32_t)g.Wp);
+  p.fsh.init((uint32_t)g.sh);
+  p.fsw.init((uint32_t)g.sw);
   p.stg_bytes = (uint32_t)t.stg_bytes;
   p.Wp = g.Wp; p.P = g.P; p.Q = g.Q; p.sh = g.sh; p.sw = g.sw; p.K = g.K; p.R = g.R; p.S = g.S;
   p.nt = t.nt; p.brows = t.brows; p.nr = t.nr; p.ngroups = t.ngroups;

@@ -1,0 +1,94 @@
+"""Multi-GPU sharding of the PolyHankel forward convolution.
+
+Images are independent units (Eq. 12 applies per batch item, P.1396-1403),
+and so are output channels (each (n,k) product polynomial is its own), so the
+path shards without any exchange in its arithmetic:
+
+  * batch mode (N >= world): rank r computes images [n0, n1) with the full
+    filters; the output shard stays on its rank (data-parallel inference) --
+    no collective on the data path.
+  * output-channel mode (N < world, e.g. N=1 layers): rank r computes filters
+    [k0, k1) for all images and the K-blocks are all-gathered (NCCL over
+    NVLink on GPUs).  For N=1, rank-ordered K blocks are exactly NCHW.
+
+One process per GPU (torch.distributed); PyTorch supplies the process group
+and the collective, the convolution itself runs in the C-ABI library.  The
+per-shard compute is injectable only so the CPU tests can drive the layout
+logic with gloo; the default is the CUDA path.
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass
+
+
+@dataclass(frozen=True)
+class Shard:
+    mode: str       # "batch" or "kshard"
+    n0: int
+    n1: int
+    k0: int
+    k1: int
+    k_pad: int      # K rounded up to a multiple of world (kshard mode), else K
+
+
+def shard_plan(N: int, K: int, world: int, rank: int) -> Shard:
+    """Which images / output channels rank `rank` of `world` computes."""
+    if world < 1 or not (0 <= rank < world) or N < 1 or K < 1:
+        raise ValueError("bad shard request")
+    if N >= world:
+        base, extra = divmod(N, world)  # uneven shards: the first `extra` ranks take one more image
+        n0 = rank * base + min(rank, extra)
+        n1 = n0 + base + (1 if rank < extra else 0)
+        return Shard("batch", n0, n1, 0, K, K)
+    kb = -(-K // world)  # equal blocks (all-gather needs equal sizes); the tail block is padded
+    k0 = min(rank * kb, K)
+    k1 = min(k0 + kb, K)
+    return Shard("kshard", 0, N, k0, k1, kb * world)
+
+
+def _cuda_compute(x, w, stride, padding, math):
+    from . import conv2d
+    return conv2d(x, w, stride=stride, padding=padding, math=math)
+
+
+def sharded_forward(x, w, stride=(1, 1), padding=(0, 0), math="bf16", group=None, compute=None):
+    """Distributed forward.  x: the FULL input batch [N][C][H][W] as seen by every
+    rank (batch mode slices it; pass only the local images with N >= world for
+    zero-copy use through `local_batch`), w: full filters.  Returns
+    (shard, y): in batch mode y is the local shard [n1-n0][K][P][Q]; in
+    output-channel mode y is the full gathered output [N][K][P][Q]."""
+    import torch
+    import torch.distributed as dist
+    compute = compute or _cuda_compute
+    world = dist.get_world_size(group) if dist.is_initialized() else 1
+    rank = dist.get_rank(group) if dist.is_initialized() else 0
+    N, K = x.shape[0], w.shape[0]
+    sh = shard_plan(N, K, world, rank)
+    if sh.mode == "batch":
+        return sh, compute(x[sh.n0:sh.n1].contiguous(), w, stride, padding, math)
+    kb = sh.k_pad // world
+    y_loc = compute(x, w[sh.k0:sh.k1].contiguous(), stride, padding, math) if sh.k1 > sh.k0 else None
+    P, Q = (y_loc.shape[2], y_loc.shape[3]) if y_loc is not None else _out_hw(x, w, stride, padding)
+    buf = torch.zeros((N, kb, P, Q), dtype=x.dtype, device=x.device)
+    if y_loc is not None:
+        buf[:, : sh.k1 - sh.k0] = y_loc
+    # gather the K blocks: [world][N][kb][P][Q] -> [N][K][P][Q]
+    if dist.is_initialized() and dist.get_backend(group) == "nccl":
+        out = torch.empty((world * N, kb, P, Q), dtype=x.dtype, device=x.device)
+        dist.all_gather_into_tensor(out, buf.reshape(N, kb, P, Q).contiguous(), group=group)
+        blocks = out.reshape(world, N, kb, P, Q)
+    else:
+        parts = [torch.empty_like(buf) for _ in range(world)]
+        if dist.is_initialized():
+            dist.all_gather(parts, buf, group=group)
+        else:
+            parts = [buf]
+        blocks = torch.stack(parts)
+    y = blocks.permute(1, 0, 2, 3, 4).reshape(N, world * kb, P, Q)[:, :K]
+    return sh, y.contiguous()
+
+
+def _out_hw(x, w, stride, padding):
+    H, W = x.shape[2], x.shape[3]
+    R, S = w.shape[2], w.shape[3]
+    return (H + 2 * padding[0] - R) // stride[0] + 1, (W + 2 * padding[1] - S) // stride[1] + 1
