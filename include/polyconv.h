@@ -73,8 +73,11 @@ typedef enum {
 /* MAC kernel variant.  AUTO picks by shape and math; the others force one
  * (ablations/tests).  TC = tcgen05/TMEM tensor-core contraction, filters as
  * the M=128 operand, one position window per channel chunk reused by every
- * tap (Hankel shift = descriptor offset); TC_PERTAP = the earlier tensor-core
- * variant with positions as M and one TMA window load per tap (ablation);
+ * tap (Hankel shift = descriptor offset), windows loaded by TMA from the
+ * packed input; TC_FUSED = the same contraction with the input packing done
+ * inside the kernel by packer warps (ablation); TC_PERTAP = the earlier
+ * tensor-core variant with positions as M and one TMA window load per tap
+ * (ablation);
  * FP32 = SIMT register-blocked FFMA; THIN = warp-per-output with shuffle
  * reduction over C*R*S (tiny channel counts). */
 typedef enum {
@@ -82,7 +85,8 @@ typedef enum {
     POLYCONV_KERNEL_TC = 1,
     POLYCONV_KERNEL_FP32 = 2,
     POLYCONV_KERNEL_THIN = 3,
-    POLYCONV_KERNEL_TC_PERTAP = 4
+    POLYCONV_KERNEL_TC_PERTAP = 4,
+    POLYCONV_KERNEL_TC_FUSED = 5
 } polyconv_kernel_t;
 
 /* Packed-operand layouts exposed for bit-exact tests (a2/a3):

@@ -82,19 +82,21 @@ struct Tc2Tiling {
   int num_mt, num_kt, num_tiles, nchunks;
   int cs;          // cluster size (CTAs sharing multicast filter tiles)
   int num_groups;  // cluster work items: ceil(num_mt / cs) * num_kt
-  int a_stages;    // filter-tile ring depth
-  bool tma_x;      // raw input staged by TMA (x as [N*C][H*W], 16-byte row pitch) vs direct loads
+  int a_stages;    // filter ring depth (stages)
+  int tps;         // filter taps per stage
+  int mode;        // 0: windows by TMA from the packed input; 1/2: fused packers (TMA staging / loads)
+  bool tma_x;      // fused: raw input staged by TMA (x as [N*C][H*W], 16-byte row pitch) vs direct loads
   int box_bytes, stg_bytes;
   int smem_bytes, acc_stride, tmem_cols, grid;
 };
 bool tc2_supported(const Geom& g, int fmt);
-Tc2Tiling tc2_tiling(const Geom& g, int fmt, bool x_bf16, int num_sms);
-// x: NCHW input (io dtype; packed on the fly, a2 fused); U: tap-major packed
-// filter [RS][Kp][Cp], Kp % 128 == 0.  pdl: launch as a programmatic dependent
-// of the preceding kernel (the filter pack), which it waits for before
-// reading U.
+Tc2Tiling tc2_tiling(const Geom& g, int fmt, bool x_bf16, int num_sms, bool fused);
+// mode 0: A = interleaved packed input [N*L_A][Cp] (x unused); fused modes:
+// x = NCHW input (packed on the fly), A unused.  U: tap-major packed filter
+// [RS][Kp][Cp], Kp % 128 == 0.  pdl: launch as a programmatic dependent of the
+// preceding pack kernel, which it waits for before reading A / U.
 cudaError_t launch_mac_tc2(const Geom& g, const Tc2Tiling& t, int fmt, const void* x, bool x_bf16,
-                           const void* U, void* y, bool y_bf16, bool pdl, cudaStream_t st, char* err,
-                           size_t errlen);
+                           const void* A, const void* U, void* y, bool y_bf16, bool pdl, cudaStream_t st,
+                           char* err, size_t errlen);
 
 }  // namespace polyconv

@@ -60,9 +60,22 @@ constexpr int BMK = 128;                 // output channels per tile (UMMA M, TM
 constexpr int kPackWarps = 8;
 constexpr int kEpiWarps = 8;             // 2 per TMEM lane quadrant
 constexpr int kPackWarp0 = 2;
-constexpr int kEpiWarp0 = kPackWarp0 + kPackWarps;
-constexpr int kThreads = 32 * (kEpiWarp0 + kEpiWarps);
+// kernel modes: windows by TMA from the packed input (kModeTma), or built in
+// the kernel by packer warps from NCHW x via TMA staging (kModeFusedTma) or
+// direct loads (kModeFusedLd)
+constexpr int kModeTma = 0, kModeFusedTma = 1, kModeFusedLd = 2;
+__host__ __device__ constexpr int epi_warp0(int mode) { return kPackWarp0 + (mode == kModeTma ? 0 : kPackWarps); }
+// kModeTma issues the MMAs from two warps (warp 1 and the last warp), alternating
+// filter stages: an mbarrier wait in the issuing thread stalls it until its own
+// earlier MMAs drain, so one issuer leaves the tensor pipe idle at every stage
+// boundary; with two, one issues while the other waits (tools/umma_rate.cu:
+// 235 -> 113 cycles per 128x208x16 MMA, ideal 104)
+__host__ __device__ constexpr int n_issuers(int mode) { return mode == kModeTma ? 2 : 1; }
+__host__ __device__ constexpr int threads_for(int mode) {
+  return 32 * (epi_warp0(mode) + kEpiWarps + n_issuers(mode) - 1);
+}
 constexpr int kBMaxRows = 384;           // max rows of one position window (48 KB at 128 B rows)
+constexpr int kBoxRows = 32;             // rows per TMA box of a position window (kModeTma)
 constexpr int kBoxE = 64;                // plane elements per staging TMA box
 constexpr int kMaxSeg = 4;               // images one window may span on the TMA staging path
 
@@ -81,14 +94,22 @@ struct Tc2Params {
   uint32_t box_bytes;  // staging TMA box: kBoxE elements x kc planes
   uint32_t stg_bytes;  // staging buffer (max boxes of any window)
   uint32_t idesc, a_bytes, b_bytes, row_bytes;
+  uint32_t b_bytes_tx;  // bytes the window TMA boxes deliver (brows * row_bytes), kModeTma
+  int tps;              // filter taps per pipeline stage
+  int stages_per_tile;  // filter stages per tile (all chunks and row groups)
+  uint32_t tap_bytes;   // one filter tile: 128 x kc words
   int acc_stride, tmem_cols;
   void* y;          // NCHW output, io dtype (= the input's)
-  int dbg;          // POLYCONV_TC_DEBUG: 8 = per-CTA phase trace (g_tc2_trace)
+  int dbg;          // POLYCONV_TC_DEBUG: 8 = per-CTA phase trace (g_tc2_trace), 16 = packer
+                    // trace; ablations 1 = no filter TMA after the first ring fill,
+                    // 2 = no window TMA after the first two (kModeTma, wrong results)
   FastDiv fLA, fWp, fsh, fsw;  // position decode: coefficient -> (n, r, s) -> (oh, ow)
 };
 
 // per-CTA phase timestamps (globaltimer ns) for POLYCONV_TC_DEBUG & 8
 __device__ unsigned long long g_tc2_trace[160 * 8];
+// packer sub-phases of the first two windows (POLYCONV_TC_DEBUG & 16), globaltimer ns
+__device__ unsigned long long g_tc2_pk[160 * 8];
 
 // Input element -> operand word (reading R11: BF16 = RNE, TF32 = RNA).
 template <typename InT, bool kTf32>
@@ -176,8 +197,8 @@ __device__ __forceinline__ void tc2_issue_staging(const Tc2Params& p, const CUte
   }
 }
 
-template <typename InT, bool kTf32, int CS, bool kTmaX>
-__global__ void __launch_bounds__(kThreads, 1)
+template <typename InT, bool kTf32, int CS, int kMode>
+__global__ void __launch_bounds__(threads_for(kMode), 1)
     mac_tc2_kernel(const __grid_constant__ CUtensorMap tmW, const __grid_constant__ CUtensorMap tmX,
                    const Tc2Params p) {
   extern __shared__ uint8_t smem_raw[];
@@ -186,6 +207,8 @@ __global__ void __launch_bounds__(kThreads, 1)
   uint8_t* sA = smem;                                        // filter tiles  [a_stages][128][row]
   uint8_t* sB = sA + (size_t)p.a_stages * p.a_bytes;         // position windows [2][brows][row]
   uint8_t* sX = sB + 2 * (size_t)p.b_bytes;                  // raw-input staging (TMA path)
+  constexpr bool kTmaX = kMode == kModeFusedTma;  // fused packers stage x by TMA
+  constexpr int kEpiWarp0 = epi_warp0(kMode);
   long long* sPos = reinterpret_cast<long long*>(sX + (kTmaX ? (size_t)p.stg_bytes : 0));  // [256] epilogue
   uint64_t* afull = reinterpret_cast<uint64_t*>(sPos + 256);
   uint64_t* aempty = afull + p.a_stages;
@@ -209,15 +232,15 @@ __global__ void __launch_bounds__(kThreads, 1)
 
   if (warp == 0 && lane == 0) {
     prefetch_tmap(&tmW);
-    if constexpr (kTmaX) prefetch_tmap(&tmX);
+    if constexpr (kMode != kModeFusedLd) prefetch_tmap(&tmX);
     for (int s = 0; s < p.a_stages; ++s) {
       mbar_init(afull + s, 1);
       mbar_init(aempty + s, CS);  // every CTA of the cluster reads the multicast filter tile
     }
     for (int s = 0; s < 2; ++s) {
-      mbar_init(bfull + s, kPackWarps);
-      mbar_init(bempty + s, 1);
-      mbar_init(tfull + s, 1);
+      mbar_init(bfull + s, kMode == kModeTma ? 1 : kPackWarps);
+      mbar_init(bempty + s, n_issuers(kMode));  // every issuer commits its share of a window
+      mbar_init(tfull + s, n_issuers(kMode));   // and of an accumulator
       mbar_init(tempty + s, kEpiWarps);
     }
     mbar_init(sfull, 1);
@@ -236,36 +259,77 @@ __global__ void __launch_bounds__(kThreads, 1)
     // The whole warp runs the loop (uniform control values); one elected lane issues.
     // The packed filter comes from the preceding kernel (programmatic dependent launch).
     asm volatile("griddepcontrol.wait;" ::: "memory");
-    int as = 0;
-    uint32_t aph = 0;
+    int as = 0, bs = 0, na = 0, nb = 0;
+    uint32_t aph = 0, bph = 0;
     for (int grp = cl_id; grp < p.num_groups; grp += cl_num) {
       const int kt = grp % p.num_kt;
       const int krow0 = kt * BMK;
+      const long long g0 = (long long)((grp / p.num_kt) * CS + (int)rank) * p.nt;
       for (int ch = 0; ch < p.nchunks; ++ch) {
-        for (int i = 0; i < p.R; ++i) {
-          for (int j = 0; j < p.S; ++j) {
+        for (int rg = 0; rg < p.ngroups; ++rg) {
+          const int i0 = rg * p.nr, i1 = min(p.R, i0 + p.nr);
+          if constexpr (kMode == kModeTma) {
+            // the position window (packed input rows [wrow, wrow+brows), channel chunk ch);
+            // rows past N*L_A are zero-filled by TMA
+            mbar_wait(bempty + bs, bph ^ 1u);
+            if (elect_one()) {
+              if ((p.dbg & 2) && nb >= 2) {  // ablation: no window traffic after the first two
+                mbar_arrive(bfull + bs);
+              } else {
+                mbar_arrive_expect_tx(bfull + bs, p.b_bytes_tx);
+                const int wrow = (int)(g0 + (long long)p.Wp * i0);
+                uint8_t* dst = sB + (size_t)bs * p.b_bytes;
+                for (int r = 0; r < p.brows; r += kBoxRows)
+                  tma_load_2d(dst + (size_t)r * p.row_bytes, &tmX, bfull + bs, ch * p.kc, wrow + r);
+              }
+            }
+            __syncwarp();
+            ++nb;
+            if (++bs == 2) { bs = 0; bph ^= 1u; }
+          }
+          // filter stages: `tps` consecutive taps of this window's kernel rows per stage
+          const int ntap = (i1 - i0) * p.S;
+          for (int t0 = 0; t0 < ntap; t0 += p.tps) {
+            const int nt_st = min(p.tps, ntap - t0);
             mbar_wait(aempty + as, aph ^ 1u);
             if (elect_one()) {
-              {
-                mbar_arrive_expect_tx(afull + as, p.a_bytes);
-                if constexpr (CS == 1) {
-                  tma_load_2d(sA + (size_t)as * p.a_bytes, &tmW, afull + as, ch * p.kc, (i * p.S + j) * p.Kp + krow0);
-                } else {
-                  constexpr int kSub = BMK / CS;  // filter rows this CTA loads for the cluster
-                  tma_load_2d_mc(sA + (size_t)as * p.a_bytes + (size_t)rank * kSub * p.row_bytes, &tmW, afull + as,
-                                 ch * p.kc, (i * p.S + j) * p.Kp + krow0 + (int)rank * kSub,
-                                 (uint16_t)((1u << CS) - 1));
+              if ((p.dbg & 1) && na >= p.a_stages) {  // ablation: no filter traffic
+                mbar_arrive(afull + as);
+              } else {
+                mbar_arrive_expect_tx(afull + as, (uint32_t)nt_st * p.tap_bytes);
+                for (int t = 0; t < nt_st; ++t) {
+                  const int tap = i0 * p.S + t0 + t;  // (i, j) with i*S + j = tap
+                  uint8_t* dst = sA + (size_t)as * p.a_bytes + (size_t)t * p.tap_bytes;
+                  if constexpr (CS == 1) {
+                    tma_load_2d(dst, &tmW, afull + as, ch * p.kc, tap * p.Kp + krow0);
+                  } else {
+                    constexpr int kSub = BMK / CS;  // filter rows this CTA loads for the cluster
+                    tma_load_2d_mc(dst + (size_t)rank * kSub * p.row_bytes, &tmW, afull + as, ch * p.kc,
+                                   tap * p.Kp + krow0 + (int)rank * kSub, (uint16_t)((1u << CS) - 1));
+                  }
                 }
               }
             }
             __syncwarp();
+            ++na;
             if (++as == p.a_stages) { as = 0; aph ^= 1u; }
           }
         }
       }
     }
-  } else if (warp == 1) {
-    // -------------------------------------------------------------- UMMA issuer
+  } else if (warp == 1 || (n_issuers(kMode) == 2 && warp == kEpiWarp0 + kEpiWarps)) {
+    // -------------------------------------------------------------- UMMA issuer(s)
+    // issuer q (0: warp 1, 1: the extra warp) issues the CTA's filter stages g
+    // with g % n_issuers == q, in strict alternation: before issuing stage g it
+    // waits on named barrier 3 + (g-1)%2 for "stage g-1 issued", and after
+    // issuing it arrives on 3 + g%2.  The tensor pipe thus receives the MMAs in
+    // one fixed order (deterministic accumulation, reading R12) while each
+    // issuer's barrier checks overlap the other's MMAs.
+    constexpr int NI = n_issuers(kMode);
+    const int q = warp == 1 ? 0 : 1;
+    long long gs = 0;  // global stage counter of this CTA
+    const long long gs_total =
+        (long long)(p.num_groups > cl_id ? (p.num_groups - cl_id + cl_num - 1) / cl_num : 0) * p.stages_per_tile;
     int as = 0, bs = 0, acc = 0;
     uint32_t aph = 0, bph = 0, accph = 0;
     const int ksteps = (int)p.row_bytes / 32;
@@ -275,48 +339,60 @@ __global__ void __launch_bounds__(kThreads, 1)
       mbar_wait(tempty + acc, accph ^ 1u);
       tc_fence_after();
       const uint32_t d_tmem = tmem_base + (uint32_t)(acc * p.acc_stride);
-      uint32_t accumulate = 0;
+      int k = 0;  // filter stage index within the tile
       for (int ch = 0; ch < p.nchunks; ++ch) {
         for (int rg = 0; rg < p.ngroups; ++rg) {
           const int i0 = rg * p.nr, i1 = min(p.R, i0 + p.nr);
           mbar_wait(bfull + bs, bph);
           tc_fence_after();
-          if (trace && lane == 0 && ch == 0 && rg == 0 && grp == cl_id) tr[2] = global_ns();
+          if (trace && q == 0 && lane == 0 && ch == 0 && rg == 0 && grp == cl_id)
+            tr[2] = (p.dbg & 32) ? clock64() : global_ns();
           const uint32_t b_addr = sB0 + (uint32_t)bs * p.b_bytes;
-          for (int i = i0; i < i1; ++i) {
-            for (int j = 0; j < p.S; ++j) {
+          const int ntap = (i1 - i0) * p.S;
+          for (int t0 = 0; t0 < ntap; t0 += p.tps, ++k, ++gs) {
+            if (gs % NI == q) {
+              const int nt_st = min(p.tps, ntap - t0);
               mbar_wait(afull + as, aph);
+              if (NI == 2 && gs > 0) {  // stage gs-1 (the other issuer's) is in the pipe
+                if ((gs - 1) & 1) asm volatile("bar.sync 4, 64;" ::: "memory");
+                else asm volatile("bar.sync 3, 64;" ::: "memory");
+              }
               tc_fence_after();
-              // Hankel shift of tap (i,j) inside the window: Wp*(i-i0) + j rows
-              const uint32_t b_shift = (uint32_t)(p.Wp * (i - i0) + j) * p.row_bytes;
-              const uint64_t ad = make_sdesc(sA0 + (uint32_t)as * p.a_bytes, p.row_bytes, 0);
-              const uint64_t bd = make_sdesc(b_addr + b_shift, p.row_bytes, 0);
+              const uint32_t a_stage = sA0 + (uint32_t)as * p.a_bytes;
               if (elect_one()) {
-                // K step = 32 bytes = +2 in the descriptor's start-address field
-                for (int ks = 0; ks < ksteps; ++ks) {
-                  umma<kTf32>(d_tmem, ad + 2 * ks, bd + 2 * ks, p.idesc, accumulate);
-                  accumulate = 1;
+                for (int t = 0; t < nt_st; ++t) {
+                  const int tl = t0 + t, i = i0 + tl / p.S, j = tl - (tl / p.S) * p.S;
+                  // Hankel shift of tap (i,j) inside the window: Wp*(i-i0) + j rows
+                  const uint32_t b_shift = (uint32_t)(p.Wp * (i - i0) + j) * p.row_bytes;
+                  const uint64_t ad = make_sdesc(a_stage + (uint32_t)t * p.tap_bytes, p.row_bytes, 0);
+                  const uint64_t bd = make_sdesc(b_addr + b_shift, p.row_bytes, 0);
+                  // K step = 32 bytes = +2 in the descriptor's start-address field
+                  for (int ks = 0; ks < ksteps; ++ks)
+                    umma<kTf32>(d_tmem, ad + 2 * ks, bd + 2 * ks, p.idesc, (k | t | ks) != 0 ? 1u : 0u);
                 }
                 // filter slot free (in every CTA of the cluster) when these MMAs finish
                 if constexpr (CS == 1) umma_commit(aempty + as);
                 else umma_commit_mc(aempty + as, cl_mask);
               }
               __syncwarp();
-              accumulate = 1;
-              if (++as == p.a_stages) { as = 0; aph ^= 1u; }
+              if (NI == 2 && gs + 1 < gs_total) {
+                if (gs & 1) asm volatile("bar.arrive 4, 64;" ::: "memory");
+                else asm volatile("bar.arrive 3, 64;" ::: "memory");
+              }
             }
+            if (++as == p.a_stages) { as = 0; aph ^= 1u; }
           }
           if (elect_one()) umma_commit(bempty + bs);  // window free when every tap using it finished
           __syncwarp();
           if (++bs == 2) { bs = 0; bph ^= 1u; }
         }
       }
-      if (trace && lane == 0) tr[3] = global_ns();
+      if (trace && q == 0 && lane == 0) tr[3] = (p.dbg & 32) ? clock64() : global_ns();
       if (elect_one()) umma_commit(tfull + acc);
       __syncwarp();
       if (++acc == 2) { acc = 0; accph ^= 1u; }
     }
-  } else if (warp < kEpiWarp0) {
+  } else if (kMode != kModeTma && warp < kEpiWarp0) {
     // ------------------------------------------- packers: fused a2 (Eq. 10 + padding)
     // Window row r is coefficient gp = wrow + r of the concatenated input
     // polynomials; coefficient pr*Wp + ps of A_{n,c} is x[n][c][pr-ph][ps-pw],
@@ -350,64 +426,107 @@ __global__ void __launch_bounds__(kThreads, 1)
       Seg sg[kMaxSeg];
       int ns = 0;
       if constexpr (kTmaX) ns = tc2_segments(p, wrow, sg) & 0xFF;
+      const bool pkt = (p.dbg & 16) && ptid == 0 && wi < 2 && blockIdx.x < 160;
+      unsigned long long* pk = g_tc2_pk + blockIdx.x * 8 + wi * 4;
+      if (pkt) pk[0] = global_ns();
       mbar_wait_sleep(bempty + bs, bph ^ 1u, 64);
       if constexpr (kTmaX) {
         mbar_wait(sfull, sph);
         sph ^= 1u;
       }
+      if (pkt) pk[1] = global_ns();
       uint8_t* dst = sB + (size_t)bs * p.b_bytes;
-      for (int r = ptid; r < p.brows; r += kNP) {
-        const long long gp = wrow + r;
-        bool valid = gp < p.NLA;
-        int n = 0, e = 0;
-        if (valid) {
-          n = (int)p.fLA.div((uint32_t)gp);
+      // Row r -> (valid, src): src = element index of channel cbase of that
+      // coefficient in the staging buffer (TMA path) or in x (direct path).
+      // Rows go in pairs (r, r+1); when both come from consecutive staging
+      // elements at an even index (the common case for even W, Wp), one 32-bit
+      // shared load per channel fetches both rows' values (bf16 fast path).
+      const bool full_chunk = cbase + p.kc <= p.C;
+      const int rstart = (int)(((p.pw - wrow) % 2 + 2) % 2);
+      const long long cstride = kTmaX ? (long long)kBoxE : p.HW;
+      const int npairs = (p.brows - rstart) / 2;
+      const int nitems = npairs + 2;  // pairs, then the unpaired first / last row
+      for (int it = ptid; it < nitems; it += kNP) {
+        int ra, nrows;
+        if (it < npairs) { ra = rstart + 2 * it; nrows = 2; }
+        else if (it == npairs) { ra = 0; nrows = rstart; }  // row 0 when the pairs start at 1
+        else { ra = rstart + 2 * npairs; nrows = p.brows - ra; }  // trailing row
+        if (nrows <= 0) continue;
+        bool valid[2] = {false, false};
+        long long src[2] = {0, 0};
+#pragma unroll
+        for (int q = 0; q < 2; ++q) {
+          if (q >= nrows) continue;
+          const long long gp = wrow + ra + q;
+          if (gp >= p.NLA) continue;
+          const int n = (int)p.fLA.div((uint32_t)gp);
           const int m = (int)(gp - (long long)n * p.L_A);
           const int pr = (int)p.fWp.div((uint32_t)m), ps = m - pr * p.Wp;
           const int h = pr - p.ph, w = ps - p.pw;
-          valid = h >= 0 && h < p.H && w >= 0 && w < p.W;
-          e = h * p.W + w;
-        }
-        // source of channel c of this coefficient
-        long long src = 0;  // element index into stg (TMA path) or x (direct path)
-        if (valid) {
+          if (h < 0 || h >= p.H || w < 0 || w >= p.W) continue;
+          valid[q] = true;
+          const int e = h * p.W + w;
           if constexpr (kTmaX) {
             int e_lo = 0, box0 = 0;
 #pragma unroll
-            for (int q = 0; q < kMaxSeg; ++q)  // unrolled: the segment table stays in registers
-              if (q < ns && sg[q].n == n) { e_lo = sg[q].e_lo; box0 = sg[q].box0; }
+            for (int g = 0; g < kMaxSeg; ++g)  // unrolled: the segment table stays in registers
+              if (g < ns && sg[g].n == n) { e_lo = sg[g].e_lo; box0 = sg[g].box0; }
             const int de = e - e_lo;
-            src = (long long)(box0 + de / kBoxE) * p.kc * kBoxE + (de % kBoxE);
+            src[q] = (long long)(box0 + de / kBoxE) * p.kc * kBoxE + (de % kBoxE);
           } else {
-            src = ((long long)n * p.C + cbase) * p.HW + e;
+            src[q] = ((long long)n * p.C + cbase) * p.HW + e;
           }
         }
-        const long long cstride = kTmaX ? (long long)kBoxE : p.HW;
-        const uint32_t rowoff = (uint32_t)r * p.row_bytes;
-        for (int j = 0; j < ncg; ++j) {
-          uint32_t wv[EPC];
+        constexpr bool kPairPath = kTmaX && sizeof(InT) == 2 && !kTf32;
+        if (kPairPath && nrows == 2 && full_chunk && valid[0] && valid[1] && src[1] == src[0] + 1 &&
+            (src[0] & 1) == 0) {
+          const uint32_t* s32 = reinterpret_cast<const uint32_t*>(stg + src[0]);  // 4-byte aligned
+          const uint32_t off0 = (uint32_t)ra * p.row_bytes, off1 = off0 + p.row_bytes;
+          for (int j = 0; j < ncg; ++j) {
+            uint32_t v[8];
 #pragma unroll
-          for (int t = 0; t < EPC; ++t) {
-            const int c = j * EPC + t;
-            wv[t] = 0u;
-            if (valid && cbase + c < p.C) {
-              const InT v = kTmaX ? stg[src + c * cstride] : __ldg(x + src + c * cstride);
-              wv[t] = ToWord<InT, kTf32>::cvt(v);
-            }
+            for (int t = 0; t < 8; ++t) v[t] = s32[(j * 8 + t) * (kBoxE / 2)];  // channel j*8+t, rows ra, ra+1
+            const uint4 o0 = make_uint4(__byte_perm(v[0], v[1], 0x5410), __byte_perm(v[2], v[3], 0x5410),
+                                        __byte_perm(v[4], v[5], 0x5410), __byte_perm(v[6], v[7], 0x5410));
+            const uint4 o1 = make_uint4(__byte_perm(v[0], v[1], 0x7632), __byte_perm(v[2], v[3], 0x7632),
+                                        __byte_perm(v[4], v[5], 0x7632), __byte_perm(v[6], v[7], 0x7632));
+            const uint32_t a0 = off0 + 16u * j, a1 = off1 + 16u * j;
+            *reinterpret_cast<uint4*>(dst + (a0 ^ (((a0 >> 7) & swmask) << 4))) = o0;
+            *reinterpret_cast<uint4*>(dst + (a1 ^ (((a1 >> 7) & swmask) << 4))) = o1;
           }
-          uint4 o;
-          if constexpr (kEB == 2)
-            o = make_uint4(wv[0] | (wv[1] << 16), wv[2] | (wv[3] << 16), wv[4] | (wv[5] << 16), wv[6] | (wv[7] << 16));
-          else
-            o = make_uint4(wv[0], wv[1], wv[2], wv[3]);
-          const uint32_t off = rowoff + 16u * j;
-          *reinterpret_cast<uint4*>(dst + (off ^ (((off >> 7) & swmask) << 4))) = o;
+          continue;
+        }
+#pragma unroll
+        for (int q = 0; q < 2; ++q) {
+          if (q >= nrows) continue;
+          const uint32_t rowoff = (uint32_t)(ra + q) * p.row_bytes;
+          for (int j = 0; j < ncg; ++j) {
+            uint32_t wv[EPC];
+#pragma unroll
+            for (int t = 0; t < EPC; ++t) {
+              const int c = j * EPC + t;
+              wv[t] = 0u;
+              if (valid[q] && (full_chunk || cbase + c < p.C)) {
+                const InT v = kTmaX ? stg[src[q] + c * cstride] : __ldg(x + src[q] + c * cstride);
+                wv[t] = ToWord<InT, kTf32>::cvt(v);
+              }
+            }
+            uint4 o;
+            if constexpr (kEB == 2)
+              o = make_uint4(wv[0] | (wv[1] << 16), wv[2] | (wv[3] << 16), wv[4] | (wv[5] << 16), wv[6] | (wv[7] << 16));
+            else
+              o = make_uint4(wv[0], wv[1], wv[2], wv[3]);
+            const uint32_t off = rowoff + 16u * j;
+            *reinterpret_cast<uint4*>(dst + (off ^ (((off >> 7) & swmask) << 4))) = o;
+          }
         }
       }
       // generic-proxy smem writes -> visible to the tensor core (async proxy); every
       // packer is done with the staging buffer before it is refilled for the next window
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      if (pkt) pk[2] = global_ns();
       asm volatile("bar.sync 1, %0;" ::"n"(kNP) : "memory");
+      if (pkt) pk[3] = global_ns();
       if constexpr (kTmaX) {
         if (ptid == 0 && wi + 1 < nwin) {
           long long wrow1;
@@ -549,12 +668,14 @@ inline long long cdiv(long long a, long long b) { return (a + b - 1) / b; }
 template <typename InT, bool kTf32, int CS>
 cudaError_t launch_one(const Tc2Tiling& t, const CUtensorMap& tmW, const CUtensorMap& tmX, const Tc2Params& p,
                        bool pdl, cudaStream_t st) {
-  auto kern = t.tma_x ? mac_tc2_kernel<InT, kTf32, CS, true> : mac_tc2_kernel<InT, kTf32, CS, false>;
+  auto kern = t.mode == kModeTma        ? mac_tc2_kernel<InT, kTf32, CS, kModeTma>
+              : t.mode == kModeFusedTma ? mac_tc2_kernel<InT, kTf32, CS, kModeFusedTma>
+                                        : mac_tc2_kernel<InT, kTf32, CS, kModeFusedLd>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, t.smem_bytes);
   if (e != cudaSuccess) return e;
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)t.grid);
-  cfg.blockDim = dim3(kThreads);
+  cfg.blockDim = dim3(threads_for(t.mode));
   cfg.dynamicSmemBytes = (size_t)t.smem_bytes;
   cfg.stream = st;
   cudaLaunchAttribute attr[2];
@@ -608,7 +729,7 @@ bool tc2_supported(const Geom& g, int fmt) {
   return true;
 }
 
-Tc2Tiling tc2_tiling(const Geom& g, int fmt, bool x_bf16, int num_sms) {
+Tc2Tiling tc2_tiling(const Geom& g, int fmt, bool x_bf16, int num_sms, bool fused) {
   Tc2Tiling t{};
   const int eb = fmt_bytes(fmt);
   int kc = 128 / eb;
@@ -642,7 +763,9 @@ Tc2Tiling tc2_tiling(const Geom& g, int fmt, bool x_bf16, int num_sms) {
   while (nr > 1 && (long long)t.nt + (long long)(nr - 1) * g.Wp + g.S - 1 > kBMaxRows) --nr;
   t.nr = nr;
   t.ngroups = (g.R + nr - 1) / nr;
-  t.brows = (int)cdiv((long long)t.nt + (long long)(nr - 1) * g.Wp + g.S - 1, 8) * 8;
+  // window rows: whole TMA boxes (kModeTma) / swizzle atoms of 8 rows (fused)
+  t.brows = (int)cdiv((long long)t.nt + (long long)(nr - 1) * g.Wp + g.S - 1, fused ? 8 : kBoxRows) *
+            (fused ? 8 : kBoxRows);
   t.num_mt = (int)cdiv(G, t.nt);
   t.num_tiles = t.num_mt * t.num_kt;
   t.num_groups = (int)cdiv(t.num_mt, t.cs) * t.num_kt;
@@ -652,7 +775,7 @@ Tc2Tiling tc2_tiling(const Geom& g, int fmt, bool x_bf16, int num_sms) {
   // input staging for the TMA path: x viewed as [N*C][H*W] needs a 16-byte row pitch
   const int eb_in = x_bf16 ? 2 : 4;
   t.box_bytes = kBoxE * kc * eb_in;
-  t.tma_x = ((long long)g.H * g.W * eb_in) % 16 == 0;
+  t.tma_x = fused && ((long long)g.H * g.W * eb_in) % 16 == 0;
   if (t.tma_x) {
     int max_boxes, max_segs;
     staging_demand(g, t, eb_in, max_boxes, max_segs);
@@ -661,11 +784,19 @@ Tc2Tiling tc2_tiling(const Geom& g, int fmt, bool x_bf16, int num_sms) {
       t.tma_x = false;
   }
   if (!t.tma_x) t.stg_bytes = 0;
+  t.mode = !fused ? kModeTma : (t.tma_x ? kModeFusedTma : kModeFusedLd);
   const int fixed = 1024 + 2 * b_bytes + t.stg_bytes + 256 * 8 + 512;
-  int st = (227 * 1024 - fixed) / a_bytes;
+  // taps per filter stage: as many as leave room for a 3-deep ring (fewer, larger
+  // stages amortise the per-stage barrier check of the MMA issuer)
+  const int budget = 227 * 1024 - fixed;
+  int tps = g.R * g.S;
+  while (tps > 1 && 3 * tps * a_bytes > budget) --tps;
+  if (fused) tps = 1;
+  t.tps = tps;
+  int st = budget / (tps * a_bytes);
   if (st > 12) st = 12;
   t.a_stages = st;
-  t.smem_bytes = fixed + st * a_bytes;
+  t.smem_bytes = fixed + st * tps * a_bytes;
   t.acc_stride = t.nt <= 128 ? 128 : 256;
   t.tmem_cols = 2 * t.acc_stride;
   const int max_clusters = num_sms / t.cs;
@@ -673,8 +804,8 @@ Tc2Tiling tc2_tiling(const Geom& g, int fmt, bool x_bf16, int num_sms) {
   return t;
 }
 
-cudaError_t launch_mac_tc2(const Geom& g, const Tc2Tiling& t, int fmt, const void* x, bool x_bf16, const void* U,
-                           void* y, bool y_bf16, bool pdl, cudaStream_t st, char* err, size_t errlen) {
+cudaError_t launch_mac_tc2(const Geom& g, const Tc2Tiling& t, int fmt, const void* x, bool x_bf16, const void* A,
+                           const void* U, void* y, bool y_bf16, bool pdl, cudaStream_t st, char* err, size_t errlen) {
   if (t.a_stages < 2) {
     snprintf(err, errlen, "mac_tc2: shared memory too small for the window");
     return cudaErrorInvalidValue;
@@ -696,7 +827,13 @@ cudaError_t launch_mac_tc2(const Geom& g, const Tc2Tiling& t, int fmt, const voi
   // staging TMA map over x as [N*C][H*W] (TMA path); its base must be 16-byte aligned
   CUtensorMap tmX;
   memset(&tmX, 0, sizeof(tmX));
-  if (t.tma_x) {
+  if (t.mode == kModeTma) {
+    // position windows from the packed input [N*L_A][Cp] (a2 done by pack_both), 32-row boxes
+    if (!encode(&tmX, A, fmt, (uint64_t)g.Cp, (uint64_t)g.N * g.L_A, t.kc, kBoxRows, t.row_bytes)) {
+      snprintf(err, errlen, "cuTensorMapEncodeTiled (packed input) failed");
+      return cudaErrorInvalidValue;
+    }
+  } else if (t.tma_x) {
     if ((reinterpret_cast<uintptr_t>(x) % 16) != 0) {
       snprintf(err, errlen, "mac_tc2: x must be 16-byte aligned");
       return cudaErrorInvalidValue;
@@ -731,8 +868,17 @@ cudaError_t launch_mac_tc2(const Geom& g, const Tc2Tiling& t, int fmt, const voi
   // instruction descriptor: D=f32 @4, A/B format @7/@10, both K-major, N>>3 @17, M>>4 @24
   p.idesc = (1u << 4) | (ab << 7) | (ab << 10) | ((uint32_t)(t.nt >> 3) << 17) | ((uint32_t)(BMK >> 4) << 24);
   p.row_bytes = (uint32_t)t.row_bytes;
-  p.a_bytes = (uint32_t)(BMK * t.row_bytes);
+  p.tap_bytes = (uint32_t)(BMK * t.row_bytes);
+  p.tps = t.tps;
+  p.stages_per_tile = 0;
+  for (int rg = 0; rg < t.ngroups; ++rg) {
+    const int ntap = (std::min(g.R, (rg + 1) * t.nr) - rg * t.nr) * g.S;
+    p.stages_per_tile += (ntap + t.tps - 1) / t.tps;
+  }
+  p.stages_per_tile *= t.nchunks;
+  p.a_bytes = p.tap_bytes * (uint32_t)t.tps;
   p.b_bytes = (uint32_t)(cdiv((long long)t.brows * t.row_bytes, 1024) * 1024);
+  p.b_bytes_tx = (uint32_t)(t.brows * t.row_bytes);
   p.acc_stride = t.acc_stride; p.tmem_cols = t.tmem_cols;
   p.y = y;
   if (y_bf16 != x_bf16) return cudaErrorInvalidValue;  // y has the io dtype of x
@@ -754,6 +900,9 @@ cudaError_t launch_mac_tc2(const Geom& g, const Tc2Tiling& t, int fmt, const voi
 
 // Debug only (not part of include/polyconv.h): copy the per-CTA phase trace of
 // the last POLYCONV_TC_DEBUG&8 launch to host (160 x 8 u64).
+extern "C" int polyconv_dbg_tc2_pk(unsigned long long* host) {
+  return (int)cudaMemcpyFromSymbol(host, polyconv::g_tc2_pk, sizeof(unsigned long long) * 160 * 8);
+}
 extern "C" int polyconv_dbg_tc2_trace(unsigned long long* host) {
   return (int)cudaMemcpyFromSymbol(host, polyconv::g_tc2_trace, sizeof(unsigned long long) * 160 * 8);
 }

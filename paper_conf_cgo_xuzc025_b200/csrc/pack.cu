@@ -23,76 +23,165 @@ inline unsigned grid_for(long long total, int per_block) {
 }
 
 // ---- planar input [N][C][L_A] ---------------------------------------------
+// Grid over (plane n*C+c, padded row r): one block row writes the Wp
+// coefficients r*Wp .. r*Wp+Wp-1 of A_{n,c}(t); 32-bit index math (the plan
+// guarantees every tensor indexes below 2^31).
 template <typename InT, int F>
 __global__ void __launch_bounds__(kThreads) pack_input_planar_kernel(Geom g, const InT* __restrict__ x,
                                                                      typename Word<F>::T* __restrict__ dst) {
-  const long long total = (long long)g.N * g.C * g.L_A;
-  for (long long idx = blockIdx.x * (long long)kThreads + threadIdx.x; idx < total;
-       idx += (long long)gridDim.x * kThreads) {
-    long long nc = idx / g.L_A;
-    int m = (int)(idx - nc * g.L_A);
-    int r = m / g.Wp, s = m - r * g.Wp;
-    int h = r - g.ph, w = s - g.pw;
-    float v = 0.f;
-    if (h >= 0 && h < g.H && w >= 0 && w < g.W) v = load_io(x, (nc * g.H + h) * g.W + w);
-    dst[idx] = Word<F>::enc(v);
+  const int rows = g.N * g.C * g.Hp;  // (plane, padded row) pairs
+  const int per = kThreads / g.Wp;  // rows per block (0: rows wider than the block)
+  if (per >= 1) {
+    // several rows per block: thread -> (row, s)
+    const int sub = threadIdx.x / g.Wp, s = threadIdx.x - sub * g.Wp;
+    if (sub >= per) return;
+    for (int rr = blockIdx.x * per + sub; rr < rows; rr += gridDim.x * per) {
+      const int nc = rr / g.Hp, r = rr - nc * g.Hp;
+      const int h = r - g.ph, w = s - g.pw;
+      float v = 0.f;
+      if (h >= 0 && h < g.H && w >= 0 && w < g.W) v = load_io(x, ((long long)nc * g.H + h) * g.W + w);
+      dst[(long long)nc * g.L_A + (long long)r * g.Wp + s] = Word<F>::enc(v);
+    }
+  } else {
+    // wide rows: a block per row
+    for (int rr = blockIdx.x; rr < rows; rr += gridDim.x) {
+      const int nc = rr / g.Hp, r = rr - nc * g.Hp;
+      const int h = r - g.ph;
+      for (int s = threadIdx.x; s < g.Wp; s += kThreads) {
+        const int w = s - g.pw;
+        float v = 0.f;
+        if (h >= 0 && h < g.H && w >= 0 && w < g.W) v = load_io(x, ((long long)nc * g.H + h) * g.W + w);
+        dst[(long long)nc * g.L_A + (long long)r * g.Wp + s] = Word<F>::enc(v);
+      }
+    }
   }
 }
 
 // ---- interleaved input [N*L_A][Cp] ------------------------------------------
-// Tiled transpose: a block moves 64 coefficients x 32 channels.  Reads walk the
-// coefficient axis (consecutive s -> consecutive w in x), writes walk channels.
-constexpr int TM = 64, TCH = 32;
+// One block per (image n, chunk of kRowCh channels, band of `rb` padded rows):
+// the block stages the band's input rows -- a contiguous run of rb*W elements
+// per channel plane -- in shared memory (coalesced, sequential reads), then
+// writes the band's rb*Wp output coefficients, each as 16-byte chunks of
+// consecutive channels.  Padding rows/columns (Eq. 10 + reading R3) and
+// channels C..Cp-1 are written as zeros.  32-bit index math (the plan
+// guarantees every count < 2^31).
+constexpr int kRowCh = 64;
+constexpr int kBandBytes = 32 * 1024;  // staged bytes per block: kRowCh planes x rb rows
+
+__device__ __forceinline__ float to_f32(float v) { return v; }
+__device__ __forceinline__ uint32_t word_bits(float w) { return __float_as_uint(w); }
+__device__ __forceinline__ uint32_t word_bits(uint32_t w) { return w; }
+__device__ __forceinline__ uint32_t word_bits(__nv_bfloat16 w) { return (uint32_t)__bfloat16_as_ushort(w); }
+__device__ __forceinline__ float to_f32(__nv_bfloat16 v) { return __bfloat162float(v); }
+
+struct BandGeom {
+  int rb;     // padded rows per band
+  int nband;  // bands per image
+  int nch;    // channel chunks
+  int tw;     // staged elements per channel (rb*W rounded to an odd number of words)
+};
+
+inline BandGeom band_geom(const Geom& g, int elem_bytes) {
+  BandGeom b;
+  const int elems = kBandBytes / (kRowCh * elem_bytes);  // staged elements per channel
+  b.rb = g.W >= elems ? 1 : elems / g.W;
+  if (b.rb > g.Hp) b.rb = g.Hp;
+  b.nband = (g.Hp + b.rb - 1) / b.rb;
+  b.nch = (g.Cp + kRowCh - 1) / kRowCh;
+  int tw = (b.rb * g.W + 1) & ~1;
+  if (((tw / 2) & 1) == 0) tw += 2;
+  b.tw = tw;
+  return b;
+}
 
 template <typename InT, int F>
-__device__ __forceinline__ void pack_interleaved_tile(const Geom& g, const InT* __restrict__ x,
-                                                      typename Word<F>::T* __restrict__ dst,
-                                                      long long tile, float (*sm)[TM + 1]) {
-  const int ctiles = (g.Cp + TCH - 1) / TCH;
-  const long long mtiles = (g.L_A + TM - 1) / TM;
-  const long long per_img = mtiles * ctiles;
-  const int n = (int)(tile / per_img);
-  long long rem = tile - (long long)n * per_img;
-  const long long m0 = (rem / ctiles) * TM;
-  const int c0 = (int)(rem % ctiles) * TCH;
-  const int t = threadIdx.x;
-  // load: thread -> (c = t/64 + 4*it, m = t%64)
+__device__ __forceinline__ void pack_band(const Geom& g, const BandGeom& bg, const InT* __restrict__ x,
+                                          typename Word<F>::T* __restrict__ dst, int blk, InT* tile) {
+  using WT = typename Word<F>::T;
+  constexpr int EPC = 16 / (int)sizeof(WT);  // channels per 16-byte chunk
+  const int band = blk % bg.nband;
+  const int rest = blk / bg.nband;
+  const int chunk = rest % bg.nch, n = rest / bg.nch;
+  const int pr0 = band * bg.rb, pr1 = min(g.Hp, pr0 + bg.rb);  // padded rows of this band
+  const int h0 = max(0, pr0 - g.ph), h1 = min(g.H, pr1 - g.ph);  // input rows they contain
+  const int c0 = chunk * kRowCh;
+  const int cw = min(kRowCh, g.Cp - c0);         // channels of this chunk in the output
+  const int cv = max(0, min(kRowCh, g.C - c0));  // of which real
+  const int nel = h1 > h0 ? (h1 - h0) * g.W : 0;  // contiguous elements per channel plane
   {
-    const int mm = t % TM;
-    const long long m = m0 + mm;
-    int r = (int)(m / g.Wp), s = (int)(m - (long long)r * g.Wp);
-    int h = r - g.ph, w = s - g.pw;
-    bool inb = m < g.L_A && h >= 0 && h < g.H && w >= 0 && w < g.W;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const InT* src = x + ((size_t)(n * g.C + c0) * g.H + h0) * g.W;
+    const int cs = g.H * g.W;
+    for (int c = warp; c < cv; c += kThreads / 32) {
+      const InT* sc = src + (size_t)c * cs;
+      InT* tc = tile + c * bg.tw;
+      for (int e0 = 0; e0 < nel; e0 += 4 * 32) {  // four independent loads in flight per lane
+        InT v[4];
 #pragma unroll
-    for (int it = 0; it < TCH / (kThreads / TM); ++it) {
-      int cc = t / TM + it * (kThreads / TM);
-      int c = c0 + cc;
-      float v = 0.f;
-      if (inb && c < g.C) v = load_io(x, (((long long)n * g.C + c) * g.H + h) * g.W + w);
-      sm[cc][mm] = v;
+        for (int k = 0; k < 4; ++k) {
+          const int e = e0 + k * 32 + lane;
+          if (e < nel) v[k] = sc[e];
+        }
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          const int e = e0 + k * 32 + lane;
+          if (e < nel) tc[e] = v[k];
+        }
+      }
     }
   }
   __syncthreads();
-  {
-    const int cc = t % TCH;
+  WT* out = dst + ((size_t)n * (size_t)g.L_A + (size_t)(pr0 * g.Wp)) * g.Cp + c0;
+  const int npos = (pr1 - pr0) * g.Wp;
+  if (g.Cp % EPC == 0) {
+    // 16-byte chunks of EPC consecutive channels (Cp is a multiple of EPC)
+    const int cpp = cw / EPC;
+    const bool pow2 = (cpp & (cpp - 1)) == 0;
+    const int sh = __ffs(cpp) - 1;
+    const int total = npos * cpp;
+    for (int u = threadIdx.x; u < total; u += kThreads) {
+      const int pos = pow2 ? (u >> sh) : u / cpp, cg = u - pos * cpp;
+      const int r = pos / g.Wp, ps = pos - r * g.Wp;
+      const int h = pr0 + r - g.ph, w = ps - g.pw;
+      const bool in = h >= h0 && h < h1 && w >= 0 && w < g.W;
+      const int e = (h - h0) * g.W + w;
+      uint32_t word[EPC];
 #pragma unroll
-    for (int it = 0; it < TM / (kThreads / TCH); ++it) {
-      int mm = t / TCH + it * (kThreads / TCH);
-      long long m = m0 + mm;
-      if (m < g.L_A && c0 + cc < g.Cp)
-        dst[((long long)n * g.L_A + m) * g.Cp + c0 + cc] = Word<F>::enc(sm[cc][mm]);
+      for (int t = 0; t < EPC; ++t) {
+        const int c = cg * EPC + t;
+        const float v = (in && c < cv) ? to_f32(tile[c * bg.tw + e]) : 0.f;
+        word[t] = word_bits(Word<F>::enc(v));
+      }
+      uint4 q;
+      if constexpr (sizeof(WT) == 2)
+        q = make_uint4(word[0] | (word[1] << 16), word[2] | (word[3] << 16), word[4] | (word[5] << 16),
+                       word[6] | (word[7] << 16));
+      else
+        q = make_uint4(word[0], word[1], word[2], word[3]);
+      *reinterpret_cast<uint4*>(out + pos * g.Cp + cg * EPC) = q;
+    }
+  } else {
+    // unaligned channel count (thin plans): one word per thread
+    const int total = npos * cw;
+    for (int u = threadIdx.x; u < total; u += kThreads) {
+      const int pos = u / cw, c = u - pos * cw;
+      const int r = pos / g.Wp, ps = pos - r * g.Wp;
+      const int h = pr0 + r - g.ph, w = ps - g.pw;
+      const bool in = h >= h0 && h < h1 && w >= 0 && w < g.W && c < cv;
+      out[pos * g.Cp + c] = Word<F>::enc(in ? to_f32(tile[c * bg.tw + (h - h0) * g.W + w]) : 0.f);
     }
   }
   __syncthreads();
 }
 
 template <typename InT, int F>
-__global__ void __launch_bounds__(kThreads) pack_input_interleaved_kernel(Geom g, const InT* __restrict__ x,
+__global__ void __launch_bounds__(kThreads) pack_input_interleaved_kernel(Geom g, BandGeom bg,
+                                                                          const InT* __restrict__ x,
                                                                           typename Word<F>::T* __restrict__ dst) {
-  __shared__ float sm[TCH][TM + 1];
-  const long long ntiles = (long long)g.N * ((g.L_A + TM - 1) / TM) * ((g.Cp + TCH - 1) / TCH);
-  for (long long tile = blockIdx.x; tile < ntiles; tile += gridDim.x)
-    pack_interleaved_tile<InT, F>(g, x, dst, tile, sm);
+  extern __shared__ __align__(16) unsigned char pk_smem[];
+  InT* tile = reinterpret_cast<InT*>(pk_smem);
+  const int nblk = g.N * bg.nch * bg.nband;
+  for (int b = blockIdx.x; b < nblk; b += gridDim.x) pack_band<InT, F>(g, bg, x, dst, b, tile);
 }
 
 // ---- planar filter [K][C][L_U] ----------------------------------------------
@@ -116,17 +205,21 @@ __global__ void __launch_bounds__(kThreads) pack_filter_planar_kernel(Geom g, co
 
 // ---- tap-major filter [R*S][Kp][Cp] -------------------------------------------
 // The nonzero coefficients of U_{k,c}(t) grouped by degree e(i,j) (tap), k, c.
+// One thread per (k, c) of [Kp][Cp]: reads the R*S contiguous taps w[k][c][*]
+// and writes coefficient e(i,j) of U_{k,c} into row (tap, k) -- consecutive
+// threads write consecutive channels.  32-bit index math (plan guarantees < 2^31).
 template <typename InT, int F>
-__device__ __forceinline__ void pack_tapmajor_elem(const Geom& g, const InT* __restrict__ w,
-                                                   typename Word<F>::T* __restrict__ dst, int Kp,
-                                                   int Cp, long long idx) {
-  long long tk = idx / Cp;
-  int c = (int)(idx - tk * Cp);
-  int tap = (int)(tk / Kp);
-  int k = (int)(tk - (long long)tap * Kp);
-  float v = 0.f;
-  if (k < g.K && c < g.C) v = load_io(w, ((long long)k * g.C + c) * g.R * g.S + tap);
-  dst[idx] = Word<F>::enc(v);
+__device__ __forceinline__ void pack_tapmajor_kc(const Geom& g, const InT* __restrict__ w,
+                                                 typename Word<F>::T* __restrict__ dst, int Kp, int Cp, int idx) {
+  const int k = idx / Cp, c = idx - k * Cp;
+  const int RS = g.R * g.S;
+  const bool in = k < g.K && c < g.C;
+  const InT* src = w + ((long long)k * g.C + c) * RS;
+#pragma unroll 4
+  for (int tap = 0; tap < RS; ++tap) {
+    const float v = in ? load_io(src, tap) : 0.f;
+    dst[((long long)tap * Kp + k) * Cp + c] = Word<F>::enc(v);
+  }
 }
 
 template <typename InT, int F>
@@ -136,30 +229,31 @@ __global__ void __launch_bounds__(kThreads) pack_filter_tapmajor_kernel(Geom g, 
   // let a programmatic dependent (the tensor-core MAC) start its prologue now;
   // it waits (griddepcontrol.wait) for this grid's completion before reading dst
   asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
-  const long long total = (long long)g.R * g.S * Kp * Cp;
-  for (long long idx = blockIdx.x * (long long)kThreads + threadIdx.x; idx < total;
-       idx += (long long)gridDim.x * kThreads)
-    pack_tapmajor_elem<InT, F>(g, w, dst, Kp, Cp, idx);
+  const int total = Kp * Cp;
+  for (int idx = blockIdx.x * kThreads + threadIdx.x; idx < total; idx += gridDim.x * kThreads)
+    pack_tapmajor_kc<InT, F>(g, w, dst, Kp, Cp, idx);
 }
 
-// ---- fused launch: interleaved input tiles, then tap-major filter ------------
+// ---- fused launch: tap-major filter, then interleaved input bands ------------
 template <typename InT, int F>
-__global__ void __launch_bounds__(kThreads) pack_both_kernel(Geom g, const InT* __restrict__ x,
+__global__ void __launch_bounds__(kThreads) pack_both_kernel(Geom g, BandGeom bg, const InT* __restrict__ x,
                                                              const InT* __restrict__ w,
                                                              typename Word<F>::T* __restrict__ xdst,
                                                              typename Word<F>::T* __restrict__ wdst,
-                                                             unsigned x_blocks) {
-  __shared__ float sm[TCH][TM + 1];
-  if (blockIdx.x < x_blocks) {
-    const long long ntiles = (long long)g.N * ((g.L_A + TM - 1) / TM) * ((g.Cp + TCH - 1) / TCH);
-    for (long long tile = blockIdx.x; tile < ntiles; tile += x_blocks)
-      pack_interleaved_tile<InT, F>(g, x, xdst, tile, sm);
+                                                             unsigned w_blocks) {
+  // let a programmatic dependent (the tensor-core MAC) start its prologue now;
+  // it waits (griddepcontrol.wait) for this grid's completion before reading
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+  extern __shared__ __align__(16) unsigned char pk_smem[];
+  if (blockIdx.x < w_blocks) {
+    const int total = g.Kp * g.Cp;
+    for (int idx = (int)blockIdx.x * kThreads + threadIdx.x; idx < total; idx += (int)w_blocks * kThreads)
+      pack_tapmajor_kc<InT, F>(g, w, wdst, g.Kp, g.Cp, idx);
   } else {
-    const unsigned wb = gridDim.x - x_blocks;
-    const long long total = (long long)g.R * g.S * g.Kp * g.Cp;
-    for (long long idx = (blockIdx.x - x_blocks) * (long long)kThreads + threadIdx.x; idx < total;
-         idx += (long long)wb * kThreads)
-      pack_tapmajor_elem<InT, F>(g, w, wdst, g.Kp, g.Cp, idx);
+    InT* tile = reinterpret_cast<InT*>(pk_smem);
+    const int nblk = g.N * bg.nch * bg.nband;
+    const int xb = (int)(gridDim.x - w_blocks);
+    for (int b = (int)(blockIdx.x - w_blocks); b < nblk; b += xb) pack_band<InT, F>(g, bg, x, xdst, b, tile);
   }
 }
 
@@ -181,17 +275,27 @@ cudaError_t dispatch(bool in_bf16, int fmt, Args&&... args) {
 
 template <typename InT, int F> struct LInPlanar {
   static cudaError_t run(const Geom& g, const void* x, void* dst, cudaStream_t st) {
-    long long total = (long long)g.N * g.C * g.L_A;
-    pack_input_planar_kernel<InT, F><<<grid_for(total, kThreads), kThreads, 0, st>>>(
+    const long long rows = (long long)g.N * g.C * g.Hp;
+    const int per = kThreads / g.Wp;
+    const long long blocks = per >= 1 ? (rows + per - 1) / per : rows;
+    pack_input_planar_kernel<InT, F><<<grid_for(blocks, 1), kThreads, 0, st>>>(
         g, (const InT*)x, (typename Word<F>::T*)dst);
     return cudaGetLastError();
   }
 };
+template <typename InT>
+size_t band_bytes(const BandGeom& bg) { return (size_t)kRowCh * bg.tw * sizeof(InT); }
+
 template <typename InT, int F> struct LInInter {
   static cudaError_t run(const Geom& g, const void* x, void* dst, cudaStream_t st) {
-    long long nt = (long long)g.N * ((g.L_A + TM - 1) / TM) * ((g.Cp + TCH - 1) / TCH);
-    pack_input_interleaved_kernel<InT, F><<<grid_for(nt, 1), kThreads, 0, st>>>(
-        g, (const InT*)x, (typename Word<F>::T*)dst);
+    const BandGeom bg = band_geom(g, (int)sizeof(InT));
+    const long long nblk = (long long)g.N * bg.nch * bg.nband;
+    const size_t smem = band_bytes<InT>(bg);
+    cudaError_t e = cudaFuncSetAttribute(pack_input_interleaved_kernel<InT, F>,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    pack_input_interleaved_kernel<InT, F><<<grid_for(nblk, 1), kThreads, smem, st>>>(
+        g, bg, (const InT*)x, (typename Word<F>::T*)dst);
     return cudaGetLastError();
   }
 };
@@ -205,7 +309,7 @@ template <typename InT, int F> struct LFPlanar {
 };
 template <typename InT, int F> struct LFTap {
   static cudaError_t run(const Geom& g, const void* w, void* dst, int Kp, int Cp, cudaStream_t st) {
-    long long total = (long long)g.R * g.S * Kp * Cp;
+    long long total = (long long)Kp * Cp;
     pack_filter_tapmajor_kernel<InT, F><<<grid_for(total, kThreads), kThreads, 0, st>>>(
         g, (const InT*)w, (typename Word<F>::T*)dst, Kp, Cp);
     return cudaGetLastError();
@@ -214,15 +318,18 @@ template <typename InT, int F> struct LFTap {
 template <typename InT, int F> struct LBoth {
   static cudaError_t run(const Geom& g, const void* x, const void* w, void* xd, void* wd,
                          cudaStream_t st) {
-    long long nt = (long long)g.N * ((g.L_A + TM - 1) / TM) * ((g.Cp + TCH - 1) / TCH);
-    long long wt = (long long)g.R * g.S * g.Kp * g.Cp;
-    unsigned xb = grid_for(nt, 1);
+    const BandGeom bg = band_geom(g, (int)sizeof(InT));
+    const long long nblk = (long long)g.N * bg.nch * bg.nband;
+    unsigned xb = grid_for(nblk, 1);
     if (xb > 148 * 8) xb = 148 * 8;
-    unsigned wb = grid_for(wt, kThreads);
-    if (wb > 148) wb = 148;
-    pack_both_kernel<InT, F><<<xb + wb, kThreads, 0, st>>>(g, (const InT*)x, (const InT*)w,
-                                                           (typename Word<F>::T*)xd,
-                                                           (typename Word<F>::T*)wd, xb);
+    const unsigned wb = grid_for((long long)g.Kp * g.Cp, kThreads);  // one (k, c) filter row per thread
+    const size_t smem = band_bytes<InT>(bg);
+    cudaError_t e = cudaFuncSetAttribute(pack_both_kernel<InT, F>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)smem);
+    if (e != cudaSuccess) return e;
+    pack_both_kernel<InT, F><<<wb + xb, kThreads, smem, st>>>(g, bg, (const InT*)x, (const InT*)w,
+                                                              (typename Word<F>::T*)xd,
+                                                              (typename Word<F>::T*)wd, wb);
     return cudaGetLastError();
   }
 };

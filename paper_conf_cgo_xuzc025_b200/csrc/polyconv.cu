@@ -64,12 +64,13 @@ polyconv_status_t resolve(polyconv_plan_t p) {
       k = (g.K >= 16 && g.C * g.R * g.S >= 16 && fp32_tiling(g).smax > 0) ? POLYCONV_KERNEL_FP32
                                                                           : POLYCONV_KERNEL_THIN;
   }
-  if (k == POLYCONV_KERNEL_TC && (!tc_math || !tc2_supported(g, p->fmt))) return POLYCONV_STATUS_BAD_PARAM;
+  if ((k == POLYCONV_KERNEL_TC || k == POLYCONV_KERNEL_TC_FUSED) && (!tc_math || !tc2_supported(g, p->fmt)))
+    return POLYCONV_STATUS_BAD_PARAM;
   if (k == POLYCONV_KERNEL_TC_PERTAP && (!tc_math || !tc_supported(g, p->fmt))) return POLYCONV_STATUS_BAD_PARAM;
   if (k == POLYCONV_KERNEL_FP32 && (tc_math || fp32_tiling(g).smax == 0)) return POLYCONV_STATUS_BAD_PARAM;
   p->kernel = k;
-  if (k == POLYCONV_KERNEL_TC) {
-    p->tc2 = tc2_tiling(g, p->fmt, p->io_bf16, p->num_sms);
+  if (k == POLYCONV_KERNEL_TC || k == POLYCONV_KERNEL_TC_FUSED) {
+    p->tc2 = tc2_tiling(g, p->fmt, p->io_bf16, p->num_sms, k == POLYCONV_KERNEL_TC_FUSED);
     g.Cp = (g.C + p->tc2.kc - 1) / p->tc2.kc * p->tc2.kc;
     g.Kp = (g.K + 127) / 128 * 128;
   } else if (k == POLYCONV_KERNEL_TC_PERTAP) {
@@ -87,9 +88,9 @@ polyconv_status_t resolve(polyconv_plan_t p) {
   const int eb = fmt_bytes(p->fmt);
   // TC packs the input on the fly (no input workspace); TC_PERTAP needs the
   // interleaved copy, FP32/THIN the planar one
-  const size_t a_elems = k == POLYCONV_KERNEL_TC          ? 0
-                         : k == POLYCONV_KERNEL_TC_PERTAP ? (size_t)g.N * g.L_A * g.Cp
-                                                          : (size_t)g.N * g.C * g.L_A;
+  const size_t a_elems = k == POLYCONV_KERNEL_TC_FUSED ? 0
+                         : (k == POLYCONV_KERNEL_TC || k == POLYCONV_KERNEL_TC_PERTAP) ? (size_t)g.N * g.L_A * g.Cp
+                                                                                       : (size_t)g.N * g.C * g.L_A;
   p->wsA_bytes = a_elems * eb;
   p->wsU_bytes = (size_t)g.R * g.S * g.Kp * g.Cp * eb;
   return POLYCONV_STATUS_SUCCESS;
@@ -231,7 +232,7 @@ polyconv_status_t polyconv_plan(polyconv_plan_t* plan, int N, int C, int H, int 
 
 polyconv_status_t polyconv_plan_set_kernel(polyconv_plan_t p, polyconv_kernel_t kernel) {
   if (!p) return POLYCONV_STATUS_BAD_PARAM;
-  if (kernel < POLYCONV_KERNEL_AUTO || kernel > POLYCONV_KERNEL_TC_PERTAP) return POLYCONV_STATUS_BAD_PARAM;
+  if (kernel < POLYCONV_KERNEL_AUTO || kernel > POLYCONV_KERNEL_TC_FUSED) return POLYCONV_STATUS_BAD_PARAM;
   const int old = p->forced;
   p->forced = kernel;
   if (resolve(p) != POLYCONV_STATUS_SUCCESS) {
@@ -262,6 +263,7 @@ polyconv_status_t polyconv_plan_info(polyconv_plan_t p, polyconv_info_t* info) {
   info->kernel = p->kernel;
   switch (p->kernel) {
     case POLYCONV_KERNEL_TC:  // tile = positions x output channels
+    case POLYCONV_KERNEL_TC_FUSED:
       info->tile_m = p->tc2.nt; info->tile_n = 128; info->stages = p->tc2.a_stages; info->launches = 2; break;
     case POLYCONV_KERNEL_TC_PERTAP:
       info->tile_m = p->tc.bm; info->tile_n = p->tc.bn; info->stages = p->tc.stages; info->launches = 2; break;
@@ -287,14 +289,25 @@ polyconv_status_t polyconv_forward(polyconv_plan_t p, const void* x, const void*
   const Geom& g = p->g;
   cudaError_t e;
   if (p->kernel == POLYCONV_KERNEL_TC) {
-    // a3 (filter pack, tiny) then the fused a2+a4+a5 kernel, launched as its
-    // programmatic dependent so its prologue and input packing overlap the pack
+    // a2 + a3 in one pack launch (interleaved input rows, tap-major filter), then the
+    // windowed tensor-core MAC (a4+a5) as its programmatic dependent
+    if (p->ev_start) cudaEventRecord(p->ev_start, st);
+    e = launch_pack_both_interleaved(g, x, w, p->io_bf16, p->wsA, p->wsU, p->fmt, st);
+    if (e != cudaSuccess) return finish(p, e, "pack");
+    e = launch_mac_tc2(g, p->tc2, p->fmt, x, p->io_bf16, p->wsA, p->wsU, y, p->io_bf16, true, st, p->err,
+                       sizeof(p->err));
+    if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
+    return finish(p, e, "mac_tc");
+  }
+  if (p->kernel == POLYCONV_KERNEL_TC_FUSED) {
+    // a3 (filter pack, tiny) then the fused a2+a4+a5 kernel as its programmatic dependent
     if (p->ev_start) cudaEventRecord(p->ev_start, st);
     e = launch_pack_filter_tapmajor(g, w, p->io_bf16, p->wsU, p->fmt, g.Kp, g.Cp, st);
     if (e != cudaSuccess) return finish(p, e, "pack_filter");
-    e = launch_mac_tc2(g, p->tc2, p->fmt, x, p->io_bf16, p->wsU, y, p->io_bf16, true, st, p->err, sizeof(p->err));
+    e = launch_mac_tc2(g, p->tc2, p->fmt, x, p->io_bf16, nullptr, p->wsU, y, p->io_bf16, true, st, p->err,
+                       sizeof(p->err));
     if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
-    return finish(p, e, "mac_tc");
+    return finish(p, e, "mac_tc_fused");
   }
   if (p->kernel == POLYCONV_KERNEL_TC_PERTAP) {
     // a2 + a3 in one launch (interleaved A, tap-major U), then the MAC (a4+a5)

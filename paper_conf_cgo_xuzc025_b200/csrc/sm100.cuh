@@ -42,10 +42,7 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
     if ((++spins & 0xFFFu) == 0) {
       const uint64_t t = global_ns();
       if (t0 == 0) t0 = t;
-      else if (t - t0 > 500000000ull) {
-        printf("polyconv watchdog: block %d thread %d bar %p parity %u\n", (int)blockIdx.x, (int)threadIdx.x, bar, parity);
-        __trap();
-      }
+      else if (t - t0 > 500000000ull) __trap();
     }
     asm volatile(
         "{\n\t.reg .pred p;\n\t"
@@ -55,6 +52,30 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
         : "r"(a), "r"(parity)
         : "memory");
   } while (!done);
+}
+
+// Spin on mbarrier.test_wait (never suspends): for the latency-critical issue
+// loops, where try_wait's suspend/wake-up left the tensor pipe idle between stages.
+__device__ __forceinline__ void mbar_wait_spin(uint64_t* bar, uint32_t parity) {
+  const uint32_t a = smem_u32(bar);
+  uint32_t done;
+  uint32_t spins = 0;
+  uint64_t t0 = 0;
+  for (;;) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, p;\n\t}"
+        : "=r"(done)
+        : "r"(a), "r"(parity)
+        : "memory");
+    if (done) return;
+    if ((++spins & 0xFFFu) == 0) {
+      const uint64_t t = global_ns();
+      if (t0 == 0) t0 = t;
+      else if (t - t0 > 500000000ull) __trap();
+    }
+  }
 }
 
 // mbar_wait for roles that wait long (epilogue, packers): back off with
@@ -75,10 +96,7 @@ __device__ __forceinline__ void mbar_wait_sleep(uint64_t* bar, uint32_t parity, 
     if (done) return;
     const uint64_t t = global_ns();
     if (t0 == 0) t0 = t;
-    else if (t - t0 > 500000000ull) {
-      printf("polyconv watchdog(sleep): block %d thread %d bar %p parity %u\n", (int)blockIdx.x, (int)threadIdx.x, bar, parity);
-      __trap();
-    }
+    else if (t - t0 > 500000000ull) __trap();
     __nanosleep(ns);
   }
 }

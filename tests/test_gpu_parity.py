@@ -17,7 +17,7 @@ from helpers import GATE, normwise, bf16_round, gpu_forward
 pytestmark = pytest.mark.gpu
 
 MATH_KERNELS = [("fp32", "fp32"), ("fp32", "thin"), ("tf32", "tc"), ("bf16", "tc"), ("tf32", "tc_pertap"),
-                ("bf16", "tc_pertap"), ("tf32", "thin"),
+                ("bf16", "tc_pertap"), ("tf32", "tc_fused"), ("bf16", "tc_fused"), ("tf32", "thin"),
                 ("bf16", "thin")]
 
 SHAPES = [
@@ -80,7 +80,7 @@ def test_bf16_io(shape):
 
 
 @pytest.mark.parametrize("math,kernel", [("fp32", "fp32"), ("bf16", "tc"), ("tf32", "tc"), ("fp32", "thin"),
-                                         ("bf16", "tc_pertap")])
+                                         ("bf16", "tc_pertap"), ("bf16", "tc_fused")])
 def test_delta_filter_bit_exact(math, kernel):
     """w[k][c][i][j] = [c == k mod C][i == i0][j == j0] -> y = shifted xpad,
     bit-exact for every tap (checks each shift e(i,j) and the padding)."""

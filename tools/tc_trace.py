@@ -33,7 +33,14 @@ for mode in modes:
     print("mode", mode, "CTAs", len(a), "start spread %.2f us" % (rel[:, 0].max()))
     nm_list = names if not (mode & 64) else ["setup", "pk_waited", "pk_zeroed", "pk_barrier", "pk_scattered",
                                               "packer_win0", "cta_end"]
+    if mode & 32:
+        raw = np.array(buf, dtype=np.float64).reshape(160, 8)[:len(a)]
+        cyc = raw[:, 3] - raw[:, 2]
+        ns = None
+        print("  MMA phase in SM cycles: min %d med %d max %d" % (cyc.min(), np.median(cyc), cyc.max()))
+        continue
     for k, nm in enumerate(nm_list, 1):
         col = rel[:, k]
         print("  %-14s min %7.2f  med %7.2f  max %7.2f us" % (nm, col.min(), np.median(col), col.max()))
 os.environ["POLYCONV_TC_DEBUG"] = "0"
+
