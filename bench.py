@@ -231,6 +231,7 @@ def main():
     ap.add_argument("--math", default="bf16", choices=["bf16", "tf32", "fp32"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-cudnn", action="store_true")
+    ap.add_argument("--kernel", default="auto", help="force a MAC variant (ablation; default auto)")
     args = ap.parse_args()
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -259,7 +260,8 @@ def main():
     w_host = torch.from_numpy(w_np).to(tdt).pin_memory()
     x = x_host.to(dev)
     w = w_host.to(dev)
-    plan = pc.Plan(x.shape, w.shape, shape.stride, shape.padding, math=args.math, io_dtype=io, device=local)
+    plan = pc.Plan(x.shape, w.shape, shape.stride, shape.padding, math=args.math, io_dtype=io, device=local,
+                   kernel=args.kernel)
     info = plan.info()
     y = torch.empty(plan.output_shape, dtype=tdt, device=dev)
     flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.float32, device=dev)

@@ -20,6 +20,9 @@ struct Geom {
   long long M_ext;      // positions per image that can hold an output:
                         // (P-1)*sh*Wp + (Q-1)*sw + 1 (last extraction degree - (L_U-1) + 1)
   int Cp, Kp;           // padded channel counts of the interleaved layouts
+  int urep;             // copies of the tap-major filter in the plan workspace (>= 1): the
+                        // tensor-core MAC spreads its filter reads over them (every CTA
+                        // streams the whole filter; one copy is an L2 hot spot)
 };
 
 inline int fmt_bytes(int f) { return f == FMT_BF16 ? 2 : 4; }

@@ -63,16 +63,29 @@ constexpr int kPackWarp0 = 2;
 // kernel modes: windows by TMA from the packed input (kModeTma), or built in
 // the kernel by packer warps from NCHW x via TMA staging (kModeFusedTma) or
 // direct loads (kModeFusedLd)
-constexpr int kModeTma = 0, kModeFusedTma = 1, kModeFusedLd = 2;
-__host__ __device__ constexpr int epi_warp0(int mode) { return kPackWarp0 + (mode == kModeTma ? 0 : kPackWarps); }
+// kModeFusedMx: packer warps transpose TMA-staged boxes of x with 8x8 matrix
+// moves (ldmatrix.trans -> stmatrix) fed by a ring of kRing staged boxes and a
+// dedicated staging-producer warp (bf16 input and math)
+constexpr int kModeTma = 0, kModeFusedTma = 1, kModeFusedLd = 2, kModeFusedMx = 3;
+#ifndef MX_PACK_WARPS
+#define MX_PACK_WARPS 8
+#endif
+constexpr int kMxPackWarps = MX_PACK_WARPS;
+constexpr int kRing = 6;                 // staged x boxes in flight (kModeFusedMx)
+__host__ __device__ constexpr int pack_warps(int mode) {
+  return mode == kModeTma ? 0 : (mode == kModeFusedMx ? kMxPackWarps : kPackWarps);
+}
+__host__ __device__ constexpr int epi_warp0(int mode) { return kPackWarp0 + pack_warps(mode); }
 // kModeTma issues the MMAs from two warps (warp 1 and the last warp), alternating
 // filter stages: an mbarrier wait in the issuing thread stalls it until its own
 // earlier MMAs drain, so one issuer leaves the tensor pipe idle at every stage
 // boundary; with two, one issues while the other waits (tools/umma_rate.cu:
 // 235 -> 113 cycles per 128x208x16 MMA, ideal 104)
-__host__ __device__ constexpr int n_issuers(int mode) { return mode == kModeTma ? 2 : 1; }
+__host__ __device__ constexpr int n_issuers(int mode) { return mode == kModeTma || mode == kModeFusedMx ? 2 : 1; }
+// kModeFusedMx: the staging producer is the warp after the epilogue / second issuer
+__host__ __device__ constexpr int xld_warp(int mode) { return epi_warp0(mode) + kEpiWarps + n_issuers(mode) - 1; }
 __host__ __device__ constexpr int threads_for(int mode) {
-  return 32 * (epi_warp0(mode) + kEpiWarps + n_issuers(mode) - 1);
+  return 32 * (xld_warp(mode) + (mode == kModeFusedMx ? 1 : 0));
 }
 constexpr int kBMaxRows = 384;           // max rows of one position window (48 KB at 128 B rows)
 constexpr int kBoxRows = 32;             // rows per TMA box of a position window (kModeTma)
@@ -96,6 +109,7 @@ struct Tc2Params {
   uint32_t idesc, a_bytes, b_bytes, row_bytes;
   uint32_t b_bytes_tx;  // bytes the window TMA boxes deliver (brows * row_bytes), kModeTma
   int tps;              // filter taps per pipeline stage
+  int urep;             // filter copies; cluster c reads copy c % urep
   int stages_per_tile;  // filter stages per tile (all chunks and row groups)
   uint32_t tap_bytes;   // one filter tile: 128 x kc words
   int acc_stride, tmem_cols;
@@ -104,6 +118,7 @@ struct Tc2Params {
                     // trace; ablations 1 = no filter TMA after the first ring fill,
                     // 2 = no window TMA after the first two (kModeTma, wrong results)
   FastDiv fLA, fWp, fsh, fsw;  // position decode: coefficient -> (n, r, s) -> (oh, ow)
+  FastDiv fW;                  // plane element -> (h, w) (kModeFusedMx)
 };
 
 // per-CTA phase timestamps (globaltimer ns) for POLYCONV_TC_DEBUG & 8
@@ -208,16 +223,20 @@ __global__ void __launch_bounds__(threads_for(kMode), 1)
   uint8_t* sB = sA + (size_t)p.a_stages * p.a_bytes;         // position windows [2][brows][row]
   uint8_t* sX = sB + 2 * (size_t)p.b_bytes;                  // raw-input staging (TMA path)
   constexpr bool kTmaX = kMode == kModeFusedTma;  // fused packers stage x by TMA
+  constexpr bool kStage = kTmaX || kMode == kModeFusedMx;
   constexpr int kEpiWarp0 = epi_warp0(kMode);
-  long long* sPos = reinterpret_cast<long long*>(sX + (kTmaX ? (size_t)p.stg_bytes : 0));  // [256] epilogue
-  uint64_t* afull = reinterpret_cast<uint64_t*>(sPos + 256);
+  long long* sPos = reinterpret_cast<long long*>(sX + (kStage ? (size_t)p.stg_bytes : 0));  // [256] epilogue
+  uint8_t* sDummy = reinterpret_cast<uint8_t*>(sPos + 256);  // 128 B sink for dropped stmatrix rows
+  uint64_t* afull = reinterpret_cast<uint64_t*>(sDummy + 128);
   uint64_t* aempty = afull + p.a_stages;
   uint64_t* bfull = aempty + p.a_stages;
   uint64_t* bempty = bfull + 2;
   uint64_t* tfull = bempty + 2;
   uint64_t* tempty = tfull + 2;
   uint64_t* sfull = tempty + 2;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(sfull + 1);
+  uint64_t* rfull = sfull + 1;       // [kRing] staged box landed (kModeFusedMx)
+  uint64_t* rempty = rfull + kRing;  // [kRing] staged box transposed
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(rempty + kRing);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   // clusters of CS CTAs share one output-channel block: the filter tiles are
@@ -228,6 +247,8 @@ __global__ void __launch_bounds__(threads_for(kMode), 1)
   const int cl_id = (int)blockIdx.x / CS, cl_num = (int)gridDim.x / CS;
   const bool trace = (p.dbg & 8) && blockIdx.x < 160;
   unsigned long long* tr = g_tc2_trace + blockIdx.x * 8;
+  const bool ptrace = (p.dbg & 16) && blockIdx.x < 160;  // MX sub-phases (g_tc2_pk)
+  unsigned long long* pk = g_tc2_pk + blockIdx.x * 8;
   if (trace && threadIdx.x == 0) tr[0] = global_ns();
 
   if (warp == 0 && lane == 0) {
@@ -238,12 +259,16 @@ __global__ void __launch_bounds__(threads_for(kMode), 1)
       mbar_init(aempty + s, CS);  // every CTA of the cluster reads the multicast filter tile
     }
     for (int s = 0; s < 2; ++s) {
-      mbar_init(bfull + s, kMode == kModeTma ? 1 : kPackWarps);
+      mbar_init(bfull + s, kMode == kModeTma ? 1 : pack_warps(kMode));
       mbar_init(bempty + s, n_issuers(kMode));  // every issuer commits its share of a window
       mbar_init(tfull + s, n_issuers(kMode));   // and of an accumulator
       mbar_init(tempty + s, kEpiWarps);
     }
     mbar_init(sfull, 1);
+    for (int s = 0; s < kRing; ++s) {
+      mbar_init(rfull + s, 1);
+      mbar_init(rempty + s, 1);
+    }
     fence_barrier_init();
   }
   if (warp == 1) tmem_alloc(tmem_slot, (uint32_t)p.tmem_cols);
@@ -263,7 +288,7 @@ __global__ void __launch_bounds__(threads_for(kMode), 1)
     uint32_t aph = 0, bph = 0;
     for (int grp = cl_id; grp < p.num_groups; grp += cl_num) {
       const int kt = grp % p.num_kt;
-      const int krow0 = kt * BMK;
+      const int krow0 = kt * BMK + (cl_id % p.urep) * p.R * p.S * p.Kp;  // this cluster's filter copy
       const long long g0 = (long long)((grp / p.num_kt) * CS + (int)rank) * p.nt;
       for (int ch = 0; ch < p.nchunks; ++ch) {
         for (int rg = 0; rg < p.ngroups; ++rg) {
@@ -392,7 +417,157 @@ __global__ void __launch_bounds__(threads_for(kMode), 1)
       __syncwarp();
       if (++acc == 2) { acc = 0; accph ^= 1u; }
     }
-  } else if (kMode != kModeTma && warp < kEpiWarp0) {
+  } else if (kMode == kModeFusedMx && warp == xld_warp(kMode)) {
+    // ------------------------------------------- staging producer (kModeFusedMx)
+    // Boxes of kBoxE plane elements x kc channel planes of x (viewed as
+    // [N*C][H*W], 128-byte swizzle) for every window, in window order, into a
+    // ring of kRing slots.  x is the caller's input, not produced by the
+    // preceding (PDL primary) kernel, so this starts without griddepcontrol.wait.
+    const int my_groups = p.num_groups > cl_id ? (p.num_groups - cl_id + cl_num - 1) / cl_num : 0;
+    const int nwin = my_groups * p.nchunks * p.ngroups;
+    long long gb = 0;
+    for (int wi = 0; wi < nwin; ++wi) {
+      long long wrow;
+      int cbase;
+      tc2_window<CS>(p, cl_id, cl_num, rank, wi, wrow, cbase);
+      Seg sg[kMaxSeg];
+      const int r = tc2_segments(p, wrow, sg);
+      const int nbox = r >> 8;
+#pragma unroll
+      for (int q = 0; q < kMaxSeg; ++q) {
+        if (sg[q].n < 0) continue;
+        int nxt = nbox;
+#pragma unroll
+        for (int q2 = kMaxSeg - 1; q2 > q; --q2)
+          if (sg[q2].n >= 0) nxt = sg[q2].box0;
+        for (int b = sg[q].box0; b < nxt; ++b, ++gb) {
+          const int slot = (int)(gb % kRing);
+          mbar_wait(rempty + slot, (uint32_t)((gb / kRing) & 1) ^ 1u);
+          if (elect_one()) {
+            mbar_arrive_expect_tx(rfull + slot, p.box_bytes);
+            tma_load_2d(sX + (size_t)slot * p.box_bytes, &tmX, rfull + slot,
+                        sg[q].e_lo + (b - sg[q].box0) * kBoxE, sg[q].n * p.C + cbase);
+          }
+          __syncwarp();
+        }
+      }
+      if (ptrace && lane == 0 && wi == 0) pk[7] = global_ns();
+    }
+  } else if (kMode == kModeFusedMx && warp < kEpiWarp0) {
+    // ------------------------------ packers (kModeFusedMx): fused a2, Eq. 10 + padding
+    // Each staged box holds kBoxE consecutive plane elements of kc channels
+    // (rows = channels, 128-byte swizzled).  One warp transposes a box as 8x8
+    // blocks: ldmatrix.trans reads 8 channels x 8 elements, stmatrix writes 8
+    // window rows (the elements' coefficients r*Wp + s of A_{n,c}(t), Eq. 10)
+    // of 8 channel words each into the swizzled K-major window.  Elements
+    // outside the window go to a dummy row.  Window rows that are padding
+    // (reading R3) or past N*L_A are written as zeros.  Boxes of a window are
+    // dealt round-robin to the packer warps.
+    constexpr int NPW = pack_warps(kMode);
+    const int pw = warp - kPackWarp0;
+    const uint32_t swmask = p.row_bytes / 16u - 1u;
+    const int ncg = (int)p.row_bytes / 16;  // 8-channel groups per window row
+    const uint32_t sB0 = smem_u32(sB), sX0 = smem_u32(sX), sD = smem_u32(sDummy);
+    const int my_groups = p.num_groups > cl_id ? (p.num_groups - cl_id + cl_num - 1) / cl_num : 0;
+    const int nwin = my_groups * p.nchunks * p.ngroups;
+    int bs = 0;
+    uint32_t bph = 0;
+    long long gb0 = 0;  // ring index of the window's first box
+    for (int wi = 0; wi < nwin; ++wi) {
+      long long wrow;
+      int cbase;
+      tc2_window<CS>(p, cl_id, cl_num, rank, wi, wrow, cbase);
+      Seg sg[kMaxSeg];
+      const int r = tc2_segments(p, wrow, sg);
+      const int nbox = r >> 8;
+      const bool trace0 = trace && pw == 0 && lane == 0 && wi == 0;
+      mbar_wait(bempty + bs, bph ^ 1u);
+      const uint32_t wbase = sB0 + (uint32_t)bs * p.b_bytes;
+      const int cvalid = p.C - cbase;  // channels of this chunk that exist
+      for (int j = pw; j < nbox; j += NPW) {
+        int n = 0, e0 = 0;
+#pragma unroll
+        for (int q = 0; q < kMaxSeg; ++q)
+          if (sg[q].n >= 0 && j >= sg[q].box0) { n = sg[q].n; e0 = sg[q].e_lo + (j - sg[q].box0) * kBoxE; }
+        const long long gb = gb0 + j;
+        const int slot = (int)(gb % kRing);
+        mbar_wait(rfull + slot, (uint32_t)((gb / kRing) & 1));
+        if (ptrace && wi == 0 && j < 4 && lane == 0) pk[j] = global_ns();  // box j of window 0 landed
+        const uint32_t sbase = sX0 + (uint32_t)slot * p.box_bytes;
+        const long long nbase = (long long)n * p.L_A - wrow;  // window row of coefficient 0 of image n
+        const long long c_t0 = clock64();
+        // this lane's stmatrix rows: element e0 + 8 eg + (lane & 7) -> window row (or -1)
+        int prow[kBoxE / 8];
+#pragma unroll
+        for (int eg = 0; eg < kBoxE / 8; ++eg) {
+          const int e = e0 + 8 * eg + (lane & 7);
+          prow[eg] = -1;
+          if (e < (int)p.HW) {
+            const int h = (int)p.fW.div((uint32_t)e), w = e - h * p.W;
+            const long long pos = nbase + (long long)(h + p.ph) * p.Wp + (w + p.pw);
+            if (pos >= 0 && pos < p.brows) prow[eg] = (int)pos;
+          }
+        }
+        for (int cq = 0; cq < ncg; cq += 4) {
+          // 8 independent 8x8 loads in flight, then 8 stores (a single warp is latency-bound otherwise)
+          const int c = (cq + (lane >> 3)) * 8 + (lane & 7);  // staging row (channel) this lane addresses
+          const uint32_t srow = sbase + (uint32_t)c * 128u;
+          uint32_t d[kBoxE / 8][4];
+#pragma unroll
+          for (int eg = 0; eg < kBoxE / 8; ++eg)
+            ldsm_x4_trans(srow + 16u * (uint32_t)(eg ^ (c & 7)), d[eg][0], d[eg][1], d[eg][2], d[eg][3]);
+          if (cvalid < p.kc) {  // partial chunk: channels >= C are zero
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+              const int c2 = (cq + q) * 8 + 2 * (lane & 3);
+              const uint32_t m = (c2 >= cvalid ? 0u : 0x0000FFFFu) | (c2 + 1 >= cvalid ? 0u : 0xFFFF0000u);
+#pragma unroll
+              for (int eg = 0; eg < kBoxE / 8; ++eg) d[eg][q] &= m;
+            }
+          }
+          const uint32_t cgoff = 16u * (uint32_t)(cq + (lane >> 3));
+#pragma unroll
+          for (int eg = 0; eg < kBoxE / 8; ++eg) {
+            uint32_t dst = sD + 16u * (uint32_t)(lane & 7);
+            if (prow[eg] >= 0) {
+              const uint32_t off = (uint32_t)prow[eg] * p.row_bytes + cgoff;
+              dst = wbase + (off ^ (((off >> 7) & swmask) << 4));
+            }
+            stsm_x4(dst, d[eg][0], d[eg][1], d[eg][2], d[eg][3]);
+          }
+        }
+        __syncwarp();
+        if (ptrace && wi == 0 && j == 0 && lane == 0) pk[5] = (unsigned long long)(clock64() - c_t0);
+        if (ptrace && wi == 1 && j == 0 && lane == 0) pk[4] = (unsigned long long)(clock64() - c_t0);
+        if (lane == 0) mbar_arrive(rempty + slot);
+      }
+      // zero rows: padding coefficients (Eq. 10, reading R3) and rows past N*L_A
+      for (int pp = pw * 32 + lane; pp < p.brows; pp += NPW * 32) {
+        const long long gp = wrow + pp;
+        bool pad = gp >= p.NLA;
+        if (!pad) {
+          const int n = (int)p.fLA.div((uint32_t)gp);
+          const int m = (int)(gp - (long long)n * p.L_A);
+          const int pr = (int)p.fWp.div((uint32_t)m), ps = m - pr * p.Wp;
+          const int h = pr - p.ph, w = ps - p.pw;
+          pad = h < 0 || h >= p.H || w < 0 || w >= p.W;
+        }
+        if (pad)
+          for (int cg = 0; cg < ncg; ++cg) {
+            const uint32_t off = (uint32_t)pp * p.row_bytes + 16u * (uint32_t)cg;
+            sts128_zero(wbase + (off ^ (((off >> 7) & swmask) << 4)));
+          }
+      }
+      // generic-proxy smem writes -> visible to the tensor core (async proxy)
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      __syncwarp();
+      if (trace0) tr[6] = global_ns();
+      if (ptrace && wi == 0 && pw == 0 && lane == 0) pk[6] = global_ns();
+      if (lane == 0) mbar_arrive(bfull + bs);
+      gb0 += nbox;
+      if (++bs == 2) { bs = 0; bph ^= 1u; }
+    }
+  } else if ((kMode == kModeFusedTma || kMode == kModeFusedLd) && warp < kEpiWarp0) {
     // ------------------------------------------- packers: fused a2 (Eq. 10 + padding)
     // Window row r is coefficient gp = wrow + r of the concatenated input
     // polynomials; coefficient pr*Wp + ps of A_{n,c} is x[n][c][pr-ph][ps-pw],
@@ -400,7 +575,7 @@ __global__ void __launch_bounds__(threads_for(kMode), 1)
     // the kc channel words of one coefficient, as row_bytes/16 swizzled
     // 16-byte chunks.  Consecutive lanes take consecutive rows.
     const int ptid = (warp - kPackWarp0) * 32 + lane;
-    constexpr int kNP = kPackWarps * 32;
+    constexpr int kNP = pack_warps(kMode) * 32;
     constexpr int kEB = kTf32 ? 4 : 2;               // operand word bytes
     constexpr int EPC = 16 / kEB;                    // channels per 16-byte chunk
     const uint32_t swmask = p.row_bytes / 16u - 1u;  // 128/64/32-byte swizzle: chunk ^= (addr>>7) & swmask
@@ -583,6 +758,13 @@ __global__ void __launch_bounds__(threads_for(kMode), 1)
         tmem_ld16x256b_x4(taddr + (uint32_t)cb, va);                  // lanes kq + 0..15
         tmem_ld16x256b_x4(taddr + (16u << 16) + (uint32_t)cb, vb);    // lanes kq + 16..31
         tmem_ld_wait();
+        if (p.dbg & 64) {  // ablation: TMEM reads only, no output stores (wrong results)
+          uint32_t acc_bits = 0;
+#pragma unroll
+          for (int t = 0; t < 16; ++t) acc_bits ^= va[t] ^ vb[t];
+          if (acc_bits == 0x7fbfffffu) y[0] = (InT)0.f;
+          continue;
+        }
 #pragma unroll
         for (int rr = 0; rr < 4; ++rr) {
           const int c = cb + 8 * rr + 2 * (lane & 3);
@@ -671,6 +853,8 @@ cudaError_t launch_one(const Tc2Tiling& t, const CUtensorMap& tmW, const CUtenso
   auto kern = t.mode == kModeTma        ? mac_tc2_kernel<InT, kTf32, CS, kModeTma>
               : t.mode == kModeFusedTma ? mac_tc2_kernel<InT, kTf32, CS, kModeFusedTma>
                                         : mac_tc2_kernel<InT, kTf32, CS, kModeFusedLd>;
+  if constexpr (std::is_same<InT, __nv_bfloat16>::value && !kTf32)
+    if (t.mode == kModeFusedMx) kern = mac_tc2_kernel<InT, kTf32, CS, kModeFusedMx>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, t.smem_bytes);
   if (e != cudaSuccess) return e;
   cudaLaunchConfig_t cfg = {};
@@ -785,13 +969,19 @@ Tc2Tiling tc2_tiling(const Geom& g, int fmt, bool x_bf16, int num_sms, bool fuse
   }
   if (!t.tma_x) t.stg_bytes = 0;
   t.mode = !fused ? kModeTma : (t.tma_x ? kModeFusedTma : kModeFusedLd);
-  const int fixed = 1024 + 2 * b_bytes + t.stg_bytes + 256 * 8 + 512;
+  // bf16 input and math with a TMA view: ring-staged 8x8-transpose packers
+  if (fused && t.tma_x && x_bf16 && fmt == FMT_BF16 && kc >= 32 && !getenv("POLYCONV_TC_NO_MX")) {
+    t.mode = kModeFusedMx;
+    t.stg_bytes = kRing * t.box_bytes;
+  }
+  const int fixed = 1024 + 2 * b_bytes + t.stg_bytes + 256 * 8 + 128 + 768;
   // taps per filter stage: as many as leave room for a 3-deep ring (fewer, larger
   // stages amortise the per-stage barrier check of the MMA issuer)
   const int budget = 227 * 1024 - fixed;
   int tps = g.R * g.S;
   while (tps > 1 && 3 * tps * a_bytes > budget) --tps;
   if (fused) tps = 1;
+  if (const char* f = getenv("POLYCONV_TC_TPS")) tps = std::max(1, std::min(tps, atoi(f)));  // experiments only
   t.tps = tps;
   int st = budget / (tps * a_bytes);
   if (st > 12) st = 12;
@@ -812,7 +1002,7 @@ cudaError_t launch_mac_tc2(const Geom& g, const Tc2Tiling& t, int fmt, const voi
   }
   CUtensorMap tmW;
   // filter box = the 128/cs rows one CTA loads and multicasts to its cluster
-  if (!encode(&tmW, U, fmt, (uint64_t)g.Cp, (uint64_t)g.R * g.S * g.Kp, t.kc, BMK / t.cs, t.row_bytes)) {
+  if (!encode(&tmW, U, fmt, (uint64_t)g.Cp, (uint64_t)g.urep * g.R * g.S * g.Kp, t.kc, BMK / t.cs, t.row_bytes)) {
     snprintf(err, errlen, "cuTensorMapEncodeTiled failed");
     return cudaErrorInvalidValue;
   }
@@ -831,6 +1021,23 @@ cudaError_t launch_mac_tc2(const Geom& g, const Tc2Tiling& t, int fmt, const voi
     // position windows from the packed input [N*L_A][Cp] (a2 done by pack_both), 32-row boxes
     if (!encode(&tmX, A, fmt, (uint64_t)g.Cp, (uint64_t)g.N * g.L_A, t.kc, kBoxRows, t.row_bytes)) {
       snprintf(err, errlen, "cuTensorMapEncodeTiled (packed input) failed");
+      return cudaErrorInvalidValue;
+    }
+  } else if (t.mode == kModeFusedMx) {
+    // staging boxes of kBoxE elements x kc planes of x viewed as [N*C][H*W], 128-byte swizzle
+    if ((reinterpret_cast<uintptr_t>(x) % 16) != 0) {
+      snprintf(err, errlen, "mac_tc2: x must be 16-byte aligned");
+      return cudaErrorInvalidValue;
+    }
+    EncodeTiledFn enc = get_encode2();
+    cuuint64_t dims[2] = {(cuuint64_t)p.HW, (cuuint64_t)g.N * g.C};
+    cuuint64_t strides[1] = {(cuuint64_t)p.HW * 2};
+    cuuint32_t box[2] = {(cuuint32_t)kBoxE, (cuuint32_t)t.kc};
+    cuuint32_t estr[2] = {1, 1};
+    if (!enc || enc(&tmX, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(x), dims, strides, box, estr,
+                    CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS) {
+      snprintf(err, errlen, "cuTensorMapEncodeTiled (input staging, swizzled) failed");
       return cudaErrorInvalidValue;
     }
   } else if (t.tma_x) {
@@ -858,6 +1065,7 @@ cudaError_t launch_mac_tc2(const Geom& g, const Tc2Tiling& t, int fmt, const voi
   p.fWp.init((uint32_t)g.Wp);
   p.fsh.init((uint32_t)g.sh);
   p.fsw.init((uint32_t)g.sw);
+  p.fW.init((uint32_t)g.W);
   p.stg_bytes = (uint32_t)t.stg_bytes;
   p.Wp = g.Wp; p.P = g.P; p.Q = g.Q; p.sh = g.sh; p.sw = g.sw; p.K = g.K; p.R = g.R; p.S = g.S;
   p.nt = t.nt; p.brows = t.brows; p.nr = t.nr; p.ngroups = t.ngroups;
@@ -870,6 +1078,7 @@ cudaError_t launch_mac_tc2(const Geom& g, const Tc2Tiling& t, int fmt, const voi
   p.row_bytes = (uint32_t)t.row_bytes;
   p.tap_bytes = (uint32_t)(BMK * t.row_bytes);
   p.tps = t.tps;
+  p.urep = g.urep;
   p.stages_per_tile = 0;
   for (int rg = 0; rg < t.ngroups; ++rg) {
     const int ntap = (std::min(g.R, (rg + 1) * t.nr) - rg * t.nr) * g.S;

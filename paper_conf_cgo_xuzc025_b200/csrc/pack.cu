@@ -8,7 +8,11 @@
 // Conversion to the math mode's operand format happens here (reading R11):
 // fp32 stays fp32, TF32 = cvt.rna, BF16 = RNE.  All kernels are pure copies
 // with index math (HBM-bound); the outputs are bit-exact by construction.
+#include <cuda.h>
+#include <algorithm>
+#include <cstdlib>
 #include "common.cuh"
+#include "sm100.cuh"
 
 namespace polyconv {
 
@@ -215,10 +219,11 @@ __device__ __forceinline__ void pack_tapmajor_kc(const Geom& g, const InT* __res
   const int RS = g.R * g.S;
   const bool in = k < g.K && c < g.C;
   const InT* src = w + ((long long)k * g.C + c) * RS;
+  const long long rep_stride = (long long)RS * Kp * Cp;
 #pragma unroll 4
   for (int tap = 0; tap < RS; ++tap) {
-    const float v = in ? load_io(src, tap) : 0.f;
-    dst[((long long)tap * Kp + k) * Cp + c] = Word<F>::enc(v);
+    const auto v = Word<F>::enc(in ? load_io(src, tap) : 0.f);
+    for (int r = 0; r < g.urep; ++r) dst[r * rep_stride + ((long long)tap * Kp + k) * Cp + c] = v;
   }
 }
 
@@ -234,7 +239,140 @@ __global__ void __launch_bounds__(kThreads) pack_filter_tapmajor_kernel(Geom g, 
     pack_tapmajor_kc<InT, F>(g, w, dst, Kp, Cp, idx);
 }
 
+// ---- interleaved input, TMA band path (the hot-path pack) -------------------
+// One block per (image n, band of rb padded rows, chunk of kc2 channels).
+//  1. One TMA 2-D load brings the band's input rows of kc2 channel planes
+//     (x viewed as [N*C][H*W]: plane elements [e_lo, e_lo+seg) of planes
+//     n*C + c0 ..) into S1 = [kc2][seg]; elements past H*W / planes past N*C
+//     are zero-filled by the TMA unit.
+//  2. Transpose S1 -> S2 = [rb*Wp positions][kc2 words]: thread (position p,
+//     16-byte chunk j) reads the chunk's channels at p's input element (zero in
+//     the padding, Eq. 10 + reading R3, and for channels >= C), converts them to
+//     the operand format (reading R11) and stores one 16-byte chunk, XOR-swizzled
+//     by p so that neither the S1 reads nor the S2 writes conflict in banks.
+//  3. Coalesced copy-out: each position's kc2 words are one contiguous run of
+//     the interleaved layout [N*L_A][Cp].
+struct TBand {
+  int rb;     // padded rows per block
+  int nband;  // bands per image
+  int kc2;    // channels per block
+  int nch;    // Cp / kc2
+  int seg;    // staged plane elements per channel (TMA box dim 0)
+  int ealign; // 16 / sizeof(input element)
+};
+
+template <typename InT, int F>
+__device__ __forceinline__ void pack_tband(const Geom& g, const TBand& b, const CUtensorMap* tmX,
+                                           typename Word<F>::T* __restrict__ dst, int blk, unsigned char* smem) {
+  using WT = typename Word<F>::T;
+  constexpr int EPC = 16 / (int)sizeof(WT);  // channels per 16-byte chunk
+  const int band = blk % b.nband;
+  const int rest = blk / b.nband;
+  const int ch = rest % b.nch, n = rest / b.nch;
+  const int pr0 = band * b.rb, pr1 = min(g.Hp, pr0 + b.rb);
+  const int h0 = max(0, pr0 - g.ph), h1 = min(g.H, pr1 - g.ph);
+  const int e_lo = (h0 * g.W) & ~(b.ealign - 1);
+  const int c0 = ch * b.kc2;
+  const InT* S1 = reinterpret_cast<const InT*>(smem);
+  const size_t s1_bytes = ((size_t)b.kc2 * b.seg * sizeof(InT) + 127) & ~(size_t)127;
+  unsigned char* S2 = smem + s1_bytes;
+  uint64_t* bar = reinterpret_cast<uint64_t*>(S2 + (size_t)b.rb * g.Wp * b.kc2 * sizeof(WT));
+  const bool has = h1 > h0;
+  if (threadIdx.x == 0 && has) {
+    sm100::mbar_init(bar, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    sm100::mbar_arrive_expect_tx(bar, (uint32_t)(b.kc2 * b.seg * sizeof(InT)));
+    sm100::tma_load_2d(smem, tmX, bar, e_lo, n * g.C + c0);
+  }
+  __syncthreads();
+  if (has) sm100::mbar_wait(bar, 0);
+  const int npos = (pr1 - pr0) * g.Wp;
+  const int ncg = b.kc2 / EPC;              // 16-byte chunks per position
+  const int rowb = b.kc2 * (int)sizeof(WT);  // bytes per position in S2
+  const int cv = min(b.kc2, g.C - c0);       // real channels of this chunk
+  for (int i = threadIdx.x; i < npos * ncg; i += kThreads) {
+    const int j = i / npos, p = i - j * npos;  // consecutive threads: consecutive positions
+    const int r = p / g.Wp, ps = p - r * g.Wp;
+    const int h = pr0 + r - g.ph, w = ps - g.pw;
+    const bool in = h >= 0 && h < g.H && w >= 0 && w < g.W;
+    const int e = h * g.W + w - e_lo;
+    uint32_t word[EPC];
+#pragma unroll
+    for (int t = 0; t < EPC; ++t) {
+      const int c = j * EPC + t;
+      const float v = (in && c < cv) ? to_f32(S1[c * b.seg + e]) : 0.f;
+      word[t] = word_bits(Word<F>::enc(v));
+    }
+    uint4 q;
+    if constexpr (sizeof(WT) == 2)
+      q = make_uint4(word[0] | (word[1] << 16), word[2] | (word[3] << 16), word[4] | (word[5] << 16),
+                     word[6] | (word[7] << 16));
+    else
+      q = make_uint4(word[0], word[1], word[2], word[3]);
+    *reinterpret_cast<uint4*>(S2 + p * rowb + 16 * (j ^ (p & (ncg - 1)))) = q;
+  }
+  __syncthreads();
+  WT* out = dst + ((size_t)n * (size_t)g.L_A + (size_t)pr0 * g.Wp) * g.Cp + c0;
+  for (int i = threadIdx.x; i < npos * ncg; i += kThreads) {
+    const int p = i / ncg, j = i - p * ncg;  // consecutive threads: the chunks of one position
+    const uint4 q = *reinterpret_cast<const uint4*>(S2 + p * rowb + 16 * (j ^ (p & (ncg - 1))));
+    *reinterpret_cast<uint4*>(out + (size_t)p * g.Cp + j * EPC) = q;
+  }
+  __syncthreads();  // S1/S2/bar reused by the block's next band
+  if (threadIdx.x == 0 && has) asm volatile("mbarrier.inval.shared::cta.b64 [%0];" ::"r"(sm100::smem_u32(bar)) : "memory");
+  __syncthreads();
+}
+
+inline size_t tband_smem(const Geom& g, const TBand& b, int in_bytes, int word_bytes) {
+  return (((size_t)b.kc2 * b.seg * in_bytes + 127) & ~(size_t)127) + (size_t)b.rb * g.Wp * b.kc2 * word_bytes + 16;
+}
+
+// Band geometry of the TMA path; rb = 0 when the shape has no TMA view of x
+// (H*W*elem not a multiple of 16 bytes) or a band does not fit one box.
+inline TBand tband_geom(const Geom& g, int in_bytes, int word_bytes, int num_sms) {
+  TBand b{};
+  b.ealign = 16 / in_bytes;
+  if (((long long)g.H * g.W * in_bytes) % 16 != 0) return b;
+  b.kc2 = std::min(g.Cp, 128 / word_bytes);
+  if (g.Cp % b.kc2 != 0 || (b.kc2 * word_bytes) % 16 != 0) return b;
+  b.nch = g.Cp / b.kc2;
+  auto seg_of = [&](int rb) { return (rb * g.W + b.ealign - 1 + b.ealign - 1) / b.ealign * b.ealign; };
+  int rb = std::min(g.Hp, 256 / g.Wp);
+  while (rb > 1 && (seg_of(rb) > 256 || tband_smem(g, TBand{rb, 0, b.kc2, 0, seg_of(rb), b.ealign}, in_bytes,
+                                                   word_bytes) > 64 * 1024))
+    --rb;
+  // at least ~2 blocks per SM when the problem allows it
+  while (rb > 1 && (long long)g.N * b.nch * ((g.Hp + rb - 1) / rb) < 2LL * num_sms) --rb;
+  if (rb < 1 || seg_of(rb) > 256 || g.Wp > 256) return TBand{};
+  b.rb = rb;
+  b.seg = seg_of(rb);
+  b.nband = (g.Hp + rb - 1) / rb;
+  return b;
+}
+
 // ---- fused launch: tap-major filter, then interleaved input bands ------------
+template <typename InT, int F>
+__global__ void __launch_bounds__(kThreads) pack_both_tma_kernel(const __grid_constant__ CUtensorMap tmX, Geom g,
+                                                                 TBand b, const InT* __restrict__ w,
+                                                                 typename Word<F>::T* __restrict__ xdst,
+                                                                 typename Word<F>::T* __restrict__ wdst,
+                                                                 unsigned w_blocks) {
+  // let a programmatic dependent (the tensor-core MAC) start its prologue now;
+  // it waits (griddepcontrol.wait) for this grid's completion before reading
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+  extern __shared__ __align__(128) unsigned char pk_smem[];
+  if (blockIdx.x < w_blocks) {
+    const int total = g.Kp * g.Cp;
+    for (int idx = (int)blockIdx.x * kThreads + threadIdx.x; idx < total; idx += (int)w_blocks * kThreads)
+      pack_tapmajor_kc<InT, F>(g, w, wdst, g.Kp, g.Cp, idx);
+  } else {
+    const int nblk = g.N * b.nch * b.nband;
+    const int xb = (int)(gridDim.x - w_blocks);
+    for (int blk = (int)(blockIdx.x - w_blocks); blk < nblk; blk += xb)
+      pack_tband<InT, F>(g, b, &tmX, xdst, blk, pk_smem);
+  }
+}
+
 template <typename InT, int F>
 __global__ void __launch_bounds__(kThreads) pack_both_kernel(Geom g, BandGeom bg, const InT* __restrict__ x,
                                                              const InT* __restrict__ w,
@@ -286,8 +424,63 @@ template <typename InT, int F> struct LInPlanar {
 template <typename InT>
 size_t band_bytes(const BandGeom& bg) { return (size_t)kRowCh * bg.tw * sizeof(InT); }
 
+typedef CUresult (*EncodeTiledFnP)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                   const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                   CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+// TMA view of x as [N*C][H*W] with boxes of b.seg elements x b.kc2 planes.
+template <typename InT>
+bool encode_x_bands(CUtensorMap* m, const Geom& g, const TBand& b, const void* x) {
+  static EncodeTiledFnP fn = nullptr;
+  if (!fn) {
+    void* f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess)
+      return false;
+    fn = reinterpret_cast<EncodeTiledFnP>(f);
+  }
+  if ((reinterpret_cast<uintptr_t>(x) & 15) != 0) return false;
+  cuuint64_t dims[2] = {(cuuint64_t)g.H * g.W, (cuuint64_t)g.N * g.C};
+  cuuint64_t strides[1] = {(cuuint64_t)g.H * g.W * sizeof(InT)};
+  cuuint32_t box[2] = {(cuuint32_t)b.seg, (cuuint32_t)b.kc2};
+  cuuint32_t estr[2] = {1, 1};
+  const CUtensorMapDataType dt =
+      sizeof(InT) == 2 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32;
+  return fn(m, dt, 2, const_cast<void*>(x), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+            CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+// Interleaved pack (+ tap-major filter pack when w != nullptr) by the TMA band
+// kernel; returns cudaErrorNotSupported when the shape has no TMA view.
+template <typename InT, int F>
+cudaError_t launch_tband(const Geom& g, const void* x, const void* w, void* xd, void* wd, cudaStream_t st) {
+  int nsm = 148;
+  int dev;
+  if (cudaGetDevice(&dev) == cudaSuccess) cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+  const TBand b = tband_geom(g, (int)sizeof(InT), (int)sizeof(typename Word<F>::T), nsm);
+  if (b.rb == 0) return cudaErrorNotSupported;
+  CUtensorMap tm;
+  if (!encode_x_bands<InT>(&tm, g, b, x)) return cudaErrorNotSupported;
+  const size_t smem = tband_smem(g, b, (int)sizeof(InT), (int)sizeof(typename Word<F>::T));
+  const long long nblk = (long long)g.N * b.nch * b.nband;
+  unsigned xb = grid_for(nblk, 1);
+  const unsigned wb = w ? grid_for((long long)g.Kp * g.Cp, kThreads) : 0u;
+  cudaError_t e = cudaFuncSetAttribute(pack_both_tma_kernel<InT, F>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       (int)smem);
+  if (e != cudaSuccess) return e;
+  pack_both_tma_kernel<InT, F><<<wb + xb, kThreads, smem, st>>>(tm, g, b, (const InT*)w, (typename Word<F>::T*)xd,
+                                                                (typename Word<F>::T*)wd, wb);
+  return cudaGetLastError();
+}
+
 template <typename InT, int F> struct LInInter {
   static cudaError_t run(const Geom& g, const void* x, void* dst, cudaStream_t st) {
+    if (!getenv("POLYCONV_PACK_LEGACY")) {
+      const cudaError_t e = launch_tband<InT, F>(g, x, nullptr, dst, nullptr, st);
+      if (e != cudaErrorNotSupported) return e;
+    }
     const BandGeom bg = band_geom(g, (int)sizeof(InT));
     const long long nblk = (long long)g.N * bg.nch * bg.nband;
     const size_t smem = band_bytes<InT>(bg);
@@ -318,6 +511,10 @@ template <typename InT, int F> struct LFTap {
 template <typename InT, int F> struct LBoth {
   static cudaError_t run(const Geom& g, const void* x, const void* w, void* xd, void* wd,
                          cudaStream_t st) {
+    if (!getenv("POLYCONV_PACK_LEGACY")) {
+      const cudaError_t e = launch_tband<InT, F>(g, x, w, xd, wd, st);
+      if (e != cudaErrorNotSupported) return e;
+    }
     const BandGeom bg = band_geom(g, (int)sizeof(InT));
     const long long nblk = (long long)g.N * bg.nch * bg.nband;
     unsigned xb = grid_for(nblk, 1);

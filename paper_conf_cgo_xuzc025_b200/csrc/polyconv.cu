@@ -92,7 +92,15 @@ polyconv_status_t resolve(polyconv_plan_t p) {
                          : (k == POLYCONV_KERNEL_TC || k == POLYCONV_KERNEL_TC_PERTAP) ? (size_t)g.N * g.L_A * g.Cp
                                                                                        : (size_t)g.N * g.C * g.L_A;
   p->wsA_bytes = a_elems * eb;
-  p->wsU_bytes = (size_t)g.R * g.S * g.Kp * g.Cp * eb;
+  g.urep = 1;
+  if (k == POLYCONV_KERNEL_TC || k == POLYCONV_KERNEL_TC_FUSED) {
+    const char* r = getenv("POLYCONV_FILTER_REP");  // experiments only
+    g.urep = r ? atoi(r) : 8;
+    if (g.urep < 1) g.urep = 1;
+    if (g.urep > 64) g.urep = 64;
+    if ((long long)g.urep * g.R * g.S * g.Kp >= (1LL << 31)) g.urep = 1;  // TMA row coordinate
+  }
+  p->wsU_bytes = (size_t)g.urep * g.R * g.S * g.Kp * g.Cp * eb;
   return POLYCONV_STATUS_SUCCESS;
 }
 
@@ -400,9 +408,11 @@ polyconv_status_t polyconv_pack_filter(polyconv_plan_t p, const void* w, void* d
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   p->last_stream = st;
   p->used = true;
+  Geom g1 = p->g;
+  g1.urep = 1;  // the caller's buffer holds one copy
   cudaError_t e = layout == POLYCONV_LAYOUT_PLANAR
-                      ? launch_pack_filter_planar(p->g, w, p->io_bf16, dst, p->fmt, st)
-                      : launch_pack_filter_tapmajor(p->g, w, p->io_bf16, dst, p->fmt, p->g.Kp, p->g.Cp, st);
+                      ? launch_pack_filter_planar(g1, w, p->io_bf16, dst, p->fmt, st)
+                      : launch_pack_filter_tapmajor(g1, w, p->io_bf16, dst, p->fmt, g1.Kp, g1.Cp, st);
   return finish(p, e, "pack_filter");
 }
 

@@ -246,3 +246,28 @@ __device__ __forceinline__ uint64_t make_sdesc(uint32_t saddr, uint32_t row_byte
 
 }  // namespace sm100
 }  // namespace polyconv
+
+namespace polyconv {
+namespace sm100 {
+// ---- 8x8 b16 matrix moves (fused input packing) ---------------------------------
+// ldmatrix .trans: lane l addresses row (l&7) of matrix (l>>3); thread t receives,
+// per matrix q, dq = {T[t/4][2(t%4)], T[t/4][2(t%4)+1]} of the transposed matrix.
+__device__ __forceinline__ void ldsm_x4_trans(uint32_t saddr, uint32_t& d0, uint32_t& d1, uint32_t& d2,
+                                              uint32_t& d3) {
+  asm volatile("ldmatrix.sync.aligned.m8n8.x4.trans.shared.b16 {%0, %1, %2, %3}, [%4];"
+               : "=r"(d0), "=r"(d1), "=r"(d2), "=r"(d3)
+               : "r"(saddr)
+               : "memory");
+}
+// stmatrix: lane l addresses row (l&7) of matrix (l>>3); thread t supplies, per
+// matrix q, row t/4, columns 2(t%4) and 2(t%4)+1 in dq.
+__device__ __forceinline__ void stsm_x4(uint32_t saddr, uint32_t d0, uint32_t d1, uint32_t d2, uint32_t d3) {
+  asm volatile("stmatrix.sync.aligned.m8n8.x4.shared.b16 [%0], {%1, %2, %3, %4};" ::"r"(saddr), "r"(d0), "r"(d1),
+               "r"(d2), "r"(d3)
+               : "memory");
+}
+__device__ __forceinline__ void sts128_zero(uint32_t saddr) {
+  asm volatile("st.shared.v4.b32 [%0], {%1, %1, %1, %1};" ::"r"(saddr), "r"(0) : "memory");
+}
+}  // namespace sm100
+}  // namespace polyconv

@@ -79,6 +79,41 @@ def test_bf16_io(shape):
     assert normwise(y, ref) <= GATE["bf16"]
 
 
+# bf16 in/out shapes with a TMA view of x (H*W*2 % 16 == 0): the fused tensor-core
+# kernel takes its ring-staged 8x8-transpose packing mode on these
+MX_SHAPES = [
+    ConvShape("mx_a", 3, 64, 12, 12, 128, 3, 3, 1, 1, 1, 1),
+    ConvShape("mx_partial", 2, 80, 16, 10, 96, 3, 3, 1, 1, 1, 1),   # second channel chunk partial
+    ConvShape("mx_s2", 2, 48, 20, 20, 64, 3, 3, 2, 2, 1, 1),        # C < kc, stride 2
+    ConvShape("mx_k5", 2, 32, 16, 16, 48, 5, 5, 1, 1, 2, 2),        # kc = 32 (64-byte swizzle)
+    ConvShape("mx_k1", 2, 64, 8, 8, 64, 1, 1, 1, 1, 0, 0),
+    ConvShape("mx_many", 9, 64, 8, 8, 128, 3, 3, 1, 1, 1, 1),       # windows span several images
+    ConvShape("mx_asym", 2, 64, 14, 20, 72, 3, 5, 1, 1, 0, 2),
+]
+
+
+@pytest.mark.parametrize("shape", MX_SHAPES, ids=lambda s: s.name)
+@pytest.mark.parametrize("kernel", ["tc_fused", "tc"])
+def test_bf16_io_fused_packing(shape, kernel):
+    """bf16 in/out, BF16 math: integer data bit-exact against round_bf16(O1);
+    uniform data within the BF16 gate."""
+    x, w = synth.make_inputs(shape, synth.seed_for(7, hash(shape.name) % 997), "int")
+    y, plan = gpu_forward(shape, x, w, math="bf16", io="bf16", kernel=kernel)
+    assert plan.info()["kernel"] == kernel
+    assert np.array_equal(y, bf16_round(oracle.conv2d(x, w, shape.stride, shape.padding)))
+    x, w = synth.make_inputs(shape, synth.seed_for(7, hash(shape.name) % 991), "uniform")
+    y, _ = gpu_forward(shape, x, w, math="bf16", io="bf16", kernel=kernel)
+    assert normwise(y, oracle.conv2d(x, w, shape.stride, shape.padding)) <= GATE["bf16"]
+
+
+def test_conv3x_fused_bf16_io():
+    """BASELINE configs[1] in full, bf16 in/out, the fused kernel."""
+    shape = synth.CONV3X
+    xi, wi = synth.make_inputs(shape, synth.seed_for(1), "int")
+    y, plan = gpu_forward(shape, xi, wi, math="bf16", io="bf16", kernel="tc_fused")
+    assert np.array_equal(y, bf16_round(oracle.conv2d(xi, wi, shape.stride, shape.padding)))
+
+
 @pytest.mark.parametrize("math,kernel", [("fp32", "fp32"), ("bf16", "tc"), ("tf32", "tc"), ("fp32", "thin"),
                                          ("bf16", "tc_pertap"), ("bf16", "tc_fused")])
 def test_delta_filter_bit_exact(math, kernel):
@@ -125,7 +160,9 @@ def test_conv3x_bench_launch_config():
 # --------------------------------------------------------------- single steps --
 
 PACK_SHAPES = [ConvShape("p1", 2, 5, 7, 6, 9, 3, 2, 1, 1, 1, 2), ConvShape("p2", 1, 70, 5, 5, 33, 3, 3, 1, 1, 1, 1),
-               ConvShape("p3", 3, 3, 11, 4, 64, 5, 5, 2, 2, 2, 2)]
+               ConvShape("p3", 3, 3, 11, 4, 64, 5, 5, 2, 2, 2, 2),
+               # H*W*elem a multiple of 16 bytes: the TMA band pack path
+               ConvShape("p4", 2, 70, 8, 12, 16, 3, 3, 1, 1, 1, 1), ConvShape("p5", 3, 130, 16, 16, 8, 3, 3, 1, 1, 2, 1)]
 
 
 @pytest.mark.parametrize("shape", PACK_SHAPES, ids=lambda s: s.name)

@@ -12,7 +12,7 @@ io = "bf16" if math == "bf16" else "f32"
 dt = torch.bfloat16 if io == "bf16" else torch.float32
 x, w = synth.make_inputs(shape, 1, "uniform")
 x, w = torch.from_numpy(x).cuda().to(dt), torch.from_numpy(w).cuda().to(dt)
-plan = pc.Plan(x.shape, w.shape, shape.stride, shape.padding, math=math, io_dtype=io)
+plan = pc.Plan(x.shape, w.shape, shape.stride, shape.padding, math=math, io_dtype=io, kernel=os.environ.get("KERN", "auto"))
 print(plan.info())
 lib = pc.load_library()
 buf = (ctypes.c_ulonglong * (160 * 8))()
@@ -39,6 +39,19 @@ for mode in modes:
         ns = None
         print("  MMA phase in SM cycles: min %d med %d max %d" % (cyc.min(), np.median(cyc), cyc.max()))
         continue
+    if mode & 16:
+        pkb = (ctypes.c_ulonglong * (160 * 8))()
+        lib.polyconv_dbg_tc2_pk(pkb)
+        pk = np.array(pkb, dtype=np.float64).reshape(160, 8)[:len(a)]
+        pkn = ["box0_landed", "box1_landed", "box2_landed", "box3_landed", "box4_landed", "box5_landed",
+               "win0_packed_pw0", "xld_win0_issued"]
+        print("  pk box0 transpose cycles: med %d max %d; window-1 box0: med %d max %d" % (
+            np.median(pk[:, 5]), pk[:, 5].max(), np.median(pk[:, 4]), pk[:, 4].max()))
+        for k, nm in enumerate(pkn):
+            if k in (4, 5): continue
+            col = (pk[:, k] - t0) / 1e3
+            col = col[pk[:, k] > 0] if (pk[:, k] > 0).any() else col
+            print("  pk %-16s min %7.2f  med %7.2f  max %7.2f us" % (nm, col.min(), np.median(col), col.max()))
     for k, nm in enumerate(nm_list, 1):
         col = rel[:, k]
         print("  %-14s min %7.2f  med %7.2f  max %7.2f us" % (nm, col.min(), np.median(col), col.max()))
