@@ -49,6 +49,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
     os.makedirs(os.path.join(OUT_DIR, "obj"), exist_ok=True)
     srcs = _sources()
     extra = ["-Xptxas", "-v"] if verbose else []
+    # experiments only: POLYCONV_NVCC_DEFINES="MX_RING=12 MX_PACK_WARPS=8" (use with --force)
+    extra += ["-D" + d for d in os.environ.get("POLYCONV_NVCC_DEFINES", "").split()]
 
     def compile_one(src):
         obj = os.path.join(OUT_DIR, "obj", os.path.basename(src) + ".o")

@@ -91,15 +91,22 @@ struct Tc2Tiling {
   bool tma_x;      // fused: raw input staged by TMA (x as [N*C][H*W], 16-byte row pitch) vs direct loads
   int box_bytes, stg_bytes;
   int smem_bytes, acc_stride, tmem_cols, grid;
+  int ecols, stage_pitch, stage_bytes;  // epilogue staging
 };
 bool tc2_supported(const Geom& g, int fmt);
-Tc2Tiling tc2_tiling(const Geom& g, int fmt, bool x_bf16, int num_sms, bool fused);
+// true when a fused tiling packs the input with the ring-staged 8x8-transpose packers
+bool tc2_is_mx(const Tc2Tiling& t);
+Tc2Tiling tc2_tiling(const Geom& g, int fmt, bool x_bf16, int num_sms, bool fused, bool y_bf16);
 // mode 0: A = interleaved packed input [N*L_A][Cp] (x unused); fused modes:
 // x = NCHW input (packed on the fly), A unused.  U: tap-major packed filter
 // [RS][Kp][Cp], Kp % 128 == 0.  pdl: launch as a programmatic dependent of the
 // preceding pack kernel, which it waits for before reading A / U.
+// fused modes with w != nullptr: the kernel packs the filter itself (a3) into U,
+// every CTA one slice, synchronised through *fcount (must reach ftarget =
+// number of launches so far x t.grid; the plan owns the counter).
 cudaError_t launch_mac_tc2(const Geom& g, const Tc2Tiling& t, int fmt, const void* x, bool x_bf16,
                            const void* A, const void* U, void* y, bool y_bf16, bool pdl, cudaStream_t st,
-                           char* err, size_t errlen);
+                           char* err, size_t errlen, const void* w = nullptr,
+                           unsigned long long* fcount = nullptr, unsigned long long ftarget = 0);
 
 }  // namespace polyconv

@@ -68,10 +68,14 @@ constexpr int kPackWarp0 = 2;
 // dedicated staging-producer warp (bf16 input and math)
 constexpr int kModeTma = 0, kModeFusedTma = 1, kModeFusedLd = 2, kModeFusedMx = 3;
 #ifndef MX_PACK_WARPS
-#define MX_PACK_WARPS 8
+#define MX_PACK_WARPS 6
 #endif
 constexpr int kMxPackWarps = MX_PACK_WARPS;
-constexpr int kRing = 6;                 // staged x boxes in flight (kModeFusedMx)
+// staged x boxes in flight (kModeFusedMx).  Box gb lives in slot gb % kRing and is
+// transposed by packer warp gb % kRing: every slot has one consumer that takes its
+// boxes in order, so no waiter can be a whole ring cycle ahead of the slot (an
+// mbarrier parity wait would then pass on the previous phase)
+constexpr int kRing = MX_PACK_WARPS;                 // staged x boxes in flight (kModeFusedMx)
 __host__ __device__ constexpr int pack_warps(int mode) {
   return mode == kModeTma ? 0 : (mode == kModeFusedMx ? kMxPackWarps : kPackWarps);
 }
@@ -102,7 +106,7 @@ struct Tc2Params {
   int Wp, P, Q, sh, sw, K, R, S;
   int nt, brows, nr, ngroups;
   int num_mt, num_kt, num_tiles, num_groups;
-  int nchunks, kc, Kp;
+  int nchunks, kc, Kp, Cp;
   int a_stages;
   uint32_t box_bytes;  // staging TMA box: kBoxE elements x kc planes
   uint32_t stg_bytes;  // staging buffer (max boxes of any window)
@@ -113,6 +117,18 @@ struct Tc2Params {
   int stages_per_tile;  // filter stages per tile (all chunks and row groups)
   uint32_t tap_bytes;   // one filter tile: 128 x kc words
   int acc_stride, tmem_cols;
+  int ecols;            // epilogue columns (positions) staged per pass
+  uint32_t stage_bytes, stage_pitch;
+  int big_stage;        // the last tile may stage all nt columns in the operand buffers
+  // in-kernel a3 (fused modes): every CTA packs a slice of the tap-major filter
+  // from w (KCRS) into U, then counts itself in *fcount; the filter producers
+  // start when *fcount reaches ftarget (all CTAs are co-resident: grid <= SMs)
+  const void* w;
+  void* U;
+  unsigned long long* fcount;
+  unsigned long long ftarget;
+  int fpack;
+  FastDiv fQ;           // output index -> (oh, ow)
   void* y;          // NCHW output, io dtype (= the input's)
   int dbg;          // POLYCONV_TC_DEBUG: 8 = per-CTA phase trace (g_tc2_trace), 16 = packer
                     // trace; ablations 1 = no filter TMA after the first ring fill,
@@ -125,6 +141,9 @@ struct Tc2Params {
 __device__ unsigned long long g_tc2_trace[160 * 8];
 // packer sub-phases of the first two windows (POLYCONV_TC_DEBUG & 16), globaltimer ns
 __device__ unsigned long long g_tc2_pk[160 * 8];
+// epilogue sub-phase cycles of warp 0 (POLYCONV_TC_DEBUG & 128): tmem ld, staging stores,
+// barrier 1, offset table, copy-out, barrier 2
+__device__ unsigned long long g_tc2_epi[160 * 8];
 
 // Input element -> operand word (reading R11: BF16 = RNE, TF32 = RNA).
 template <typename InT, bool kTf32>
@@ -225,7 +244,8 @@ __global__ void __launch_bounds__(threads_for(kMode), 1)
   constexpr bool kTmaX = kMode == kModeFusedTma;  // fused packers stage x by TMA
   constexpr bool kStage = kTmaX || kMode == kModeFusedMx;
   constexpr int kEpiWarp0 = epi_warp0(kMode);
-  long long* sPos = reinterpret_cast<long long*>(sX + (kStage ? (size_t)p.stg_bytes : 0));  // [256] epilogue
+  uint8_t* sStage = sX + (kStage ? (size_t)p.stg_bytes : 0);  // epilogue staging [128][ecols] (+16 B pitch pad)
+  int* sPos = reinterpret_cast<int*>(sStage + p.stage_bytes);  // [256] output offsets of the tile's positions
   uint8_t* sDummy = reinterpret_cast<uint8_t*>(sPos + 256);  // 128 B sink for dropped stmatrix rows
   uint64_t* afull = reinterpret_cast<uint64_t*>(sDummy + 128);
   uint64_t* aempty = afull + p.a_stages;
@@ -283,7 +303,25 @@ __global__ void __launch_bounds__(threads_for(kMode), 1)
     // ------------------------------------------------------- filter TMA producer
     // The whole warp runs the loop (uniform control values); one elected lane issues.
     // The packed filter comes from the preceding kernel (programmatic dependent launch).
-    asm volatile("griddepcontrol.wait;" ::: "memory");
+    if (p.fpack) {
+      // every CTA's slice of the packed filter is in global memory
+      if (lane == 0) {
+        unsigned long long v;
+        uint64_t t0 = 0;
+        for (;;) {
+          asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p.fcount) : "memory");
+          if (v >= p.ftarget) break;
+          const uint64_t t = global_ns();
+          if (t0 == 0) t0 = t;
+          else if (t - t0 > 500000000ull) __trap();
+          __nanosleep(32);
+        }
+        asm volatile("fence.proxy.async.global;" ::: "memory");  // generic writes -> TMA reads
+      }
+      __syncwarp();
+    } else {
+      asm volatile("griddepcontrol.wait;" ::: "memory");
+    }
     int as = 0, bs = 0, na = 0, nb = 0;
     uint32_t aph = 0, bph = 0;
     for (int grp = cl_id; grp < p.num_groups; grp += cl_num) {
@@ -484,7 +522,7 @@ __global__ void __launch_bounds__(threads_for(kMode), 1)
       mbar_wait(bempty + bs, bph ^ 1u);
       const uint32_t wbase = sB0 + (uint32_t)bs * p.b_bytes;
       const int cvalid = p.C - cbase;  // channels of this chunk that exist
-      for (int j = pw; j < nbox; j += NPW) {
+      for (int j = (int)(((long long)pw - gb0 % NPW + NPW) % NPW); j < nbox; j += NPW) {  // boxes gb0+j = pw mod NPW
         int n = 0, e0 = 0;
 #pragma unroll
         for (int q = 0; q < kMaxSeg; ++q)
@@ -716,83 +754,157 @@ __global__ void __launch_bounds__(threads_for(kMode), 1)
     }
   } else {
     // -------------------------------------------------------------- epilogue
-    // warp w reads TMEM lane quadrant (w % 4) (output channels kq..kq+31); the
-    // two warps of a quadrant take alternate 32-column (position) blocks.
-    // tcgen05.ld.16x256b: lane t holds positions c, c+1 (c = cb + 8r + 2(t%4))
-    // of channels kq + {t/4, t/4+8, t/4+16, t/4+24}.
+    // a5 (Eq. 12 extraction + strided NCHW store), in passes of ecols positions:
+    //  A. warp w reads TMEM lane quadrant (w % 4) = output channels kq..kq+31
+    //     with tcgen05.ld.32x32b (thread = channel, 32 consecutive positions),
+    //     converts to the output type and stores the row segment into the
+    //     staging buffer sStage[channel][position - pass start];
+    //  B. the warps copy the pass out channel by channel: the pass's
+    //     extraction degrees of one image are one contiguous run of output
+    //     indices o = oh*Q + ow of y[n][k] (Eq. 12 is monotone in m), so lanes
+    //     take consecutive o and the stores are coalesced; coefficient m of o
+    //     is Wp*sh*oh + sw*ow (the degree m(oh,ow) minus L_U - 1).
     const int ew = warp - kEpiWarp0;
     const int quad = warp & 3;
-    const int csub = ew >> 2, cstep = kEpiWarps / 4;
+    const int hh = ew >> 2;  // which 32-column half of a 64-column step
+    if (p.fpack) {
+      // a3 (Eq. 6, reversed + gap-padded kernel; MMA view: tap-major [R*S][Kp][Cp],
+      // reading R11 conversion): this CTA's slice of the packed filter
+      using WT = typename std::conditional<kTf32, uint32_t, uint16_t>::type;
+      const InT* __restrict__ wk = reinterpret_cast<const InT*>(p.w);
+      WT* __restrict__ U = reinterpret_cast<WT*>(p.U);
+      const int RS = p.R * p.S;
+      const long long plane = (long long)p.Kp * p.Cp, total = plane * RS;
+      const long long per = (total + gridDim.x - 1) / gridDim.x;
+      const long long i0 = per * blockIdx.x, i1 = min(total, i0 + per);
+      for (long long idx = i0 + ew * 32 + lane; idx < i1; idx += kEpiWarps * 32) {
+        const int tap = (int)(idx / plane);
+        const int rem = (int)(idx - (long long)tap * plane);
+        const int k = rem / p.Cp, c = rem - k * p.Cp;
+        uint32_t word = 0;
+        if (k < p.K && c < p.C) word = ToWord<InT, kTf32>::cvt(wk[((long long)k * p.C + c) * RS + tap]);
+        U[idx] = (WT)word;
+      }
+      asm volatile("fence.proxy.async.global;" ::: "memory");
+      __threadfence();
+      asm volatile("bar.sync 2, %0;" ::"n"(kEpiWarps * 32) : "memory");
+      if (ew == 0 && lane == 0) atomicAdd(p.fcount, 1ull);
+    }
+    constexpr int EB = (int)sizeof(InT);
     InT* __restrict__ y = reinterpret_cast<InT*>(p.y);
+    const uint32_t st0 = smem_u32(sStage);
     int acc = 0;
     uint32_t accph = 0;
     for (int grp = cl_id; grp < p.num_groups; grp += cl_num) {
       const int mg = grp / p.num_kt, kt = grp - mg * p.num_kt;
       const long long g0 = (long long)(mg * CS + (int)rank) * p.nt;
-      const int kq = kt * BMK + quad * 32;
-      const int kl = kq + (lane >> 2);  // this lane's first channel; others +8, +16, +24
-      const long long n0 = g0 / p.L_A;  // the tile's first position: image n0, coefficient m0
-      const int m0 = (int)(g0 - n0 * p.L_A);
-      mbar_wait_sleep(tfull + acc, accph, 256);
+      mbar_wait_sleep(tfull + acc, accph, 64);
       tc_fence_after();
       if (trace && ew == 0 && lane == 0) tr[4] = global_ns();
       const uint32_t taddr = tmem_base + ((uint32_t)(quad * 32) << 16) + (uint32_t)(acc * p.acc_stride);
-      // a5 for the tile's positions, once: sPos[c] = element offset of pixel
-      // (n, 0, oh, ow) in y (add k*PQ for channel k), or -1 off the Eq. 12 / R4 lattice
+      // a5 index math once per tile: sPos[c] = element offset of output (n, k=0, oh, ow)
+      // of position g0+c in y when it lies on the Eq. 12 / R4 lattice, else -1
       asm volatile("bar.sync 2, %0;" ::"n"(kEpiWarps * 32) : "memory");  // previous tile's table unused
       for (int c = ew * 32 + lane; c < p.nt; c += kEpiWarps * 32) {
-        long long off = -1;
-        if (g0 + c < p.G) {
-          int n = (int)n0, m = m0 + c;
-          while (m >= p.L_A) { m -= (int)p.L_A; ++n; }
-          const int r = (int)p.fWp.div((uint32_t)m), s = m - r * p.Wp;
-          const int oh = (int)p.fsh.div((uint32_t)r), ow = (int)p.fsw.div((uint32_t)s);
-          if (r == oh * p.sh && s == ow * p.sw && oh < p.P && ow < p.Q)
-            off = (long long)n * p.K * p.PQ + (long long)oh * p.Q + ow;
+        int off = -1;
+        const long long gp = g0 + c;
+        if (gp < p.G) {
+          const int n = (int)p.fLA.div((uint32_t)gp);
+          const int m = (int)gp - n * (int)p.L_A;
+          const int r = (int)p.fWp.div((uint32_t)m), sc = m - r * p.Wp;
+          const int oh = (int)p.fsh.div((uint32_t)r), ow = (int)p.fsw.div((uint32_t)sc);
+          if (r == oh * p.sh && sc == ow * p.sw && oh < p.P && ow < p.Q) off = (n * p.K) * (int)p.PQ + oh * p.Q + ow;
         }
         sPos[c] = off;
       }
-      asm volatile("bar.sync 2, %0;" ::"n"(kEpiWarps * 32) : "memory");
-      for (int cb = csub * 32; cb < p.nt; cb += 32 * cstep) {
-        uint32_t va[16], vb[16];
-        tmem_ld16x256b_x4(taddr + (uint32_t)cb, va);                  // lanes kq + 0..15
-        tmem_ld16x256b_x4(taddr + (16u << 16) + (uint32_t)cb, vb);    // lanes kq + 16..31
-        tmem_ld_wait();
-        if (p.dbg & 64) {  // ablation: TMEM reads only, no output stores (wrong results)
-          uint32_t acc_bits = 0;
+      const bool etr = (p.dbg & 128) && ew == 0 && lane == 0 && blockIdx.x < 160;
+      unsigned long long ecyc[6] = {0, 0, 0, 0, 0, 0};
+      long long et = clock64();
+      auto tick = [&](int i) { const long long t = clock64(); ecyc[i] += (unsigned long long)(t - et); et = t; };
+      // the CTA's last tile: every MMA is complete and no more operand loads will
+      // land, so the whole tile is staged at once in the operand buffers (one
+      // pass: no global stores queued in front of later passes' shared stores)
+      const bool big = p.big_stage && grp + cl_num >= p.num_groups;
+      const int ecols = big ? (p.nt + 31) / 32 * 32 : p.ecols;
+      const uint32_t pitch = big ? (uint32_t)(ecols * EB + 16) : p.stage_pitch;
+      const uint32_t stb = big ? smem_u32(sA) : st0;
+      for (int c0 = 0; c0 < p.nt; c0 += ecols) {
+        const int c1 = min(p.nt, c0 + ecols);
+        // ---- A: TMEM -> staging (row = channel quad*32 + lane)
+        for (int cb = c0 + 32 * hh; cb < c1; cb += 64) {
+          uint32_t v[32];
+          tmem_ld32(taddr + (uint32_t)cb, v);
+          tmem_ld_wait();
+          tick(0);
+          const uint32_t row = stb + (uint32_t)(quad * 32 + lane) * pitch + (uint32_t)(cb - c0) * EB;
+          if constexpr (EB == 2) {
 #pragma unroll
-          for (int t = 0; t < 16; ++t) acc_bits ^= va[t] ^ vb[t];
-          if (acc_bits == 0x7fbfffffu) y[0] = (InT)0.f;
-          continue;
+            for (int q = 0; q < 4; ++q) {
+              uint32_t w4[4];
+#pragma unroll
+              for (int t = 0; t < 4; ++t) {
+                const __nv_bfloat162 h2 =
+                    __floats2bfloat162_rn(__uint_as_float(v[8 * q + 2 * t]), __uint_as_float(v[8 * q + 2 * t + 1]));
+                w4[t] = *reinterpret_cast<const uint32_t*>(&h2);
+              }
+              asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(row + 16u * q), "r"(w4[0]), "r"(w4[1]),
+                           "r"(w4[2]), "r"(w4[3]) : "memory");
+            }
+          } else {
+#pragma unroll
+            for (int q = 0; q < 8; ++q)
+              asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(row + 16u * q), "r"(v[4 * q]),
+                           "r"(v[4 * q + 1]), "r"(v[4 * q + 2]), "r"(v[4 * q + 3]) : "memory");
+          }
+          tick(1);
         }
+        tick(3);
+        asm volatile("bar.sync 2, %0;" ::"n"(kEpiWarps * 32) : "memory");
+        tick(2);
+        // ---- B: staging -> y.  Lane l copies column cs+l of the warp's 16 channels
+        // (consecutive lanes -> consecutive output pixels: coalesced; junk columns,
+        // off the Eq. 12 / R4 lattice, are predicated off); the 16 shared loads are
+        // issued before the 16 stores.
+        for (int cs = c0; cs < c1; cs += 32) {
+          const int cc = cs + lane;
+          const int off = cc < c1 ? sPos[cc] : -1;
+          constexpr int KPW = BMK / kEpiWarps;  // channels per warp
+          const int kw = kt * BMK + ew;         // the warp's first channel
+          const uint32_t sa0 = stb + (uint32_t)ew * pitch + (uint32_t)(cc - c0) * EB;
+          InT* yp = y + (long long)kw * p.PQ + (off >= 0 ? off : 0);
+          const long long ystep = (long long)kEpiWarps * p.PQ;
+          if constexpr (EB == 2) {
+            unsigned short b[KPW];
 #pragma unroll
-        for (int rr = 0; rr < 4; ++rr) {
-          const int c = cb + 8 * rr + 2 * (lane & 3);
-          const long long o0 = c < p.nt ? sPos[c] : -1;
-          const long long o1 = c + 1 < p.nt ? sPos[c + 1] : -1;
-          if (o0 < 0 && o1 < 0) continue;
-          // adjacent output pixels at an even element offset -> one 2-element store per channel
-          const bool pair = o0 >= 0 && o1 == o0 + 1 && (o0 & 1) == 0 && (p.PQ & 1) == 0;
-          const long long yk = (long long)kl * p.PQ;
+            for (int i = 0; i < KPW; ++i)
+              asm volatile("ld.shared.u16 %0, [%1];" : "=h"(b[i]) : "r"(sa0 + (uint32_t)(i * kEpiWarps) * pitch));
+            if (off >= 0 && !(p.dbg & 64)) {
 #pragma unroll
-          for (int g = 0; g < 4; ++g) {
-            if (kl + 8 * g >= p.K) continue;
-            const uint32_t* vv = g < 2 ? va : vb;
-            const float a0 = __uint_as_float(vv[4 * rr + 2 * (g & 1)]);
-            const float a1 = __uint_as_float(vv[4 * rr + 2 * (g & 1) + 1]);
-            const long long d = yk + (long long)(8 * g) * p.PQ;
-            if (pair) {
-              if constexpr (sizeof(InT) == 2)
-                *reinterpret_cast<__nv_bfloat162*>(y + o0 + d) = __floats2bfloat162_rn(a0, a1);
-              else
-                *reinterpret_cast<float2*>(y + o0 + d) = make_float2(a0, a1);
-            } else {
-              if (o0 >= 0) y[o0 + d] = (InT)a0;
-              if (o1 >= 0) y[o1 + d] = (InT)a1;
+              for (int i = 0; i < KPW; ++i) {
+                if (kw + i * kEpiWarps < p.K) *reinterpret_cast<unsigned short*>(yp) = b[i];
+                yp += ystep;
+              }
+            }
+          } else {
+            float f[KPW];
+#pragma unroll
+            for (int i = 0; i < KPW; ++i)
+              asm volatile("ld.shared.f32 %0, [%1];" : "=f"(f[i]) : "r"(sa0 + (uint32_t)(i * kEpiWarps) * pitch));
+            if (off >= 0 && !(p.dbg & 64)) {
+#pragma unroll
+              for (int i = 0; i < KPW; ++i) {
+                if (kw + i * kEpiWarps < p.K) *yp = f[i];
+                yp += ystep;
+              }
             }
           }
         }
+        tick(4);
+        asm volatile("bar.sync 2, %0;" ::"n"(kEpiWarps * 32) : "memory");  // staging reused by the next pass
+        tick(5);
       }
+      if (etr)
+        for (int i = 0; i < 6; ++i) g_tc2_epi[blockIdx.x * 8 + i] = ecyc[i];
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(tempty + acc);
@@ -905,6 +1017,8 @@ void staging_demand(const Geom& g, const Tc2Tiling& t, int eb_in, int& max_boxes
 
 }  // namespace
 
+bool tc2_is_mx(const Tc2Tiling& t) { return t.mode == kModeFusedMx; }
+
 bool tc2_supported(const Geom& g, int fmt) {
   if (fmt != FMT_BF16 && fmt != FMT_TF32) return false;
   if ((long long)g.R * g.S * ((g.K + 127) / 128 * 128) >= (1LL << 31)) return false;  // TMA row coordinate
@@ -913,7 +1027,7 @@ bool tc2_supported(const Geom& g, int fmt) {
   return true;
 }
 
-Tc2Tiling tc2_tiling(const Geom& g, int fmt, bool x_bf16, int num_sms, bool fused) {
+Tc2Tiling tc2_tiling(const Geom& g, int fmt, bool x_bf16, int num_sms, bool fused, bool y_bf16) {
   Tc2Tiling t{};
   const int eb = fmt_bytes(fmt);
   int kc = 128 / eb;
@@ -964,7 +1078,7 @@ Tc2Tiling tc2_tiling(const Geom& g, int fmt, bool x_bf16, int num_sms, bool fuse
     int max_boxes, max_segs;
     staging_demand(g, t, eb_in, max_boxes, max_segs);
     t.stg_bytes = (int)cdiv((long long)std::max(1, max_boxes) * t.box_bytes, 1024) * 1024;
-    if (max_segs > kMaxSeg || 1024 + 2 * b_bytes + t.stg_bytes + 256 * 8 + 512 + 3 * a_bytes > 227 * 1024)
+    if (max_segs > kMaxSeg || 1024 + 2 * b_bytes + t.stg_bytes + 18 * 1024 + 512 + 3 * a_bytes > 227 * 1024)
       t.tma_x = false;
   }
   if (!t.tma_x) t.stg_bytes = 0;
@@ -974,7 +1088,11 @@ Tc2Tiling tc2_tiling(const Geom& g, int fmt, bool x_bf16, int num_sms, bool fuse
     t.mode = kModeFusedMx;
     t.stg_bytes = kRing * t.box_bytes;
   }
-  const int fixed = 1024 + 2 * b_bytes + t.stg_bytes + 256 * 8 + 128 + 768;
+  // epilogue staging: 128 channels x ecols positions of the output type (+16 B per row)
+  t.ecols = y_bf16 ? 64 : 32;  // a multiple of the 32 columns one tcgen05.ld.32x32b.x32 returns
+  t.stage_pitch = t.ecols * (y_bf16 ? 2 : 4) + 16;
+  t.stage_bytes = BMK * t.stage_pitch;  // + the pass's output-offset table (ecols x 8 B)
+  const int fixed = 1024 + 2 * b_bytes + t.stg_bytes + t.stage_bytes + 256 * 4 + 128 + 768;
   // taps per filter stage: as many as leave room for a 3-deep ring (fewer, larger
   // stages amortise the per-stage barrier check of the MMA issuer)
   const int budget = 227 * 1024 - fixed;
@@ -995,7 +1113,8 @@ Tc2Tiling tc2_tiling(const Geom& g, int fmt, bool x_bf16, int num_sms, bool fuse
 }
 
 cudaError_t launch_mac_tc2(const Geom& g, const Tc2Tiling& t, int fmt, const void* x, bool x_bf16, const void* A,
-                           const void* U, void* y, bool y_bf16, bool pdl, cudaStream_t st, char* err, size_t errlen) {
+                           const void* U, void* y, bool y_bf16, bool pdl, cudaStream_t st, char* err, size_t errlen,
+                           const void* w, unsigned long long* fcount, unsigned long long ftarget) {
   if (t.a_stages < 2) {
     snprintf(err, errlen, "mac_tc2: shared memory too small for the window");
     return cudaErrorInvalidValue;
@@ -1070,7 +1189,7 @@ cudaError_t launch_mac_tc2(const Geom& g, const Tc2Tiling& t, int fmt, const voi
   p.Wp = g.Wp; p.P = g.P; p.Q = g.Q; p.sh = g.sh; p.sw = g.sw; p.K = g.K; p.R = g.R; p.S = g.S;
   p.nt = t.nt; p.brows = t.brows; p.nr = t.nr; p.ngroups = t.ngroups;
   p.num_mt = t.num_mt; p.num_kt = t.num_kt; p.num_tiles = t.num_tiles; p.num_groups = t.num_groups;
-  p.nchunks = t.nchunks; p.kc = t.kc; p.Kp = g.Kp;
+  p.nchunks = t.nchunks; p.kc = t.kc; p.Kp = g.Kp; p.Cp = g.Cp;
   p.a_stages = t.a_stages;
   const uint32_t ab = fmt == FMT_BF16 ? 1u : 2u;
   // instruction descriptor: D=f32 @4, A/B format @7/@10, both K-major, N>>3 @17, M>>4 @24
@@ -1089,8 +1208,23 @@ cudaError_t launch_mac_tc2(const Geom& g, const Tc2Tiling& t, int fmt, const voi
   p.b_bytes = (uint32_t)(cdiv((long long)t.brows * t.row_bytes, 1024) * 1024);
   p.b_bytes_tx = (uint32_t)(t.brows * t.row_bytes);
   p.acc_stride = t.acc_stride; p.tmem_cols = t.tmem_cols;
+  p.ecols = t.ecols;
+  p.stage_pitch = (uint32_t)t.stage_pitch;
+  p.stage_bytes = (uint32_t)t.stage_bytes;
+  p.fQ.init((uint32_t)g.Q);
+  {
+    const int eb_y = y_bf16 ? 2 : 4;
+    const long long need = (long long)BMK * (((t.nt + 31) / 32 * 32) * eb_y + 16);
+    p.big_stage = need <= (long long)t.a_stages * BMK * t.row_bytes * t.tps && !getenv("POLYCONV_TC_NO_BIGSTAGE");
+  }
   p.y = y;
   if (y_bf16 != x_bf16) return cudaErrorInvalidValue;  // y has the io dtype of x
+  p.w = w;
+  p.U = const_cast<void*>(U);
+  p.fcount = fcount;
+  p.ftarget = ftarget;
+  p.fpack = (w != nullptr && fcount != nullptr && t.mode != kModeTma) ? 1 : 0;
+  if (p.fpack) pdl = false;  // no primary kernel: the filter is packed in this grid
   const char* dbg = getenv("POLYCONV_TC_DEBUG");
   p.dbg = dbg ? atoi(dbg) : 0;
   if (fmt == FMT_TF32) {
@@ -1111,6 +1245,9 @@ cudaError_t launch_mac_tc2(const Geom& g, const Tc2Tiling& t, int fmt, const voi
 // the last POLYCONV_TC_DEBUG&8 launch to host (160 x 8 u64).
 extern "C" int polyconv_dbg_tc2_pk(unsigned long long* host) {
   return (int)cudaMemcpyFromSymbol(host, polyconv::g_tc2_pk, sizeof(unsigned long long) * 160 * 8);
+}
+extern "C" int polyconv_dbg_tc2_epi(unsigned long long* host) {
+  return (int)cudaMemcpyFromSymbol(host, polyconv::g_tc2_epi, sizeof(unsigned long long) * 160 * 8);
 }
 extern "C" int polyconv_dbg_tc2_trace(unsigned long long* host) {
   return (int)cudaMemcpyFromSymbol(host, polyconv::g_tc2_trace, sizeof(unsigned long long) * 160 * 8);

@@ -39,6 +39,9 @@ struct polyconv_plan_s {
   // polyconv_plan_set_timing_events: recorded around the MAC launch
   cudaEvent_t ev_start = nullptr;
   cudaEvent_t ev_stop = nullptr;
+  // TC_FUSED: the MAC packs the filter in-kernel; its CTAs meet on this counter
+  unsigned long long* fcount = nullptr;
+  unsigned long long fepoch = 0;
   char err[512];
 };
 
@@ -56,7 +59,10 @@ polyconv_status_t resolve(polyconv_plan_t p) {
   int k = p->forced;
   const bool tc_math = p->math != POLYCONV_MATH_FP32_FMA;
   if (k == POLYCONV_KERNEL_AUTO) {
-    if (tc_math)
+    if (tc_math && g.K >= 16 && tc2_supported(g, p->fmt) && p->io_bf16 && !getenv("POLYCONV_NO_FUSED_DEFAULT") &&
+        tc2_is_mx(tc2_tiling(g, p->fmt, p->io_bf16, p->num_sms, true, p->io_bf16)))
+      k = POLYCONV_KERNEL_TC_FUSED;  // bf16 in/out: one launch, input packed in-kernel
+    else if (tc_math)
       k = (g.K >= 16 && tc2_supported(g, p->fmt))  ? POLYCONV_KERNEL_TC
           : (g.K >= 16 && tc_supported(g, p->fmt)) ? POLYCONV_KERNEL_TC_PERTAP
                                                    : POLYCONV_KERNEL_THIN;
@@ -70,7 +76,7 @@ polyconv_status_t resolve(polyconv_plan_t p) {
   if (k == POLYCONV_KERNEL_FP32 && (tc_math || fp32_tiling(g).smax == 0)) return POLYCONV_STATUS_BAD_PARAM;
   p->kernel = k;
   if (k == POLYCONV_KERNEL_TC || k == POLYCONV_KERNEL_TC_FUSED) {
-    p->tc2 = tc2_tiling(g, p->fmt, p->io_bf16, p->num_sms, k == POLYCONV_KERNEL_TC_FUSED);
+    p->tc2 = tc2_tiling(g, p->fmt, p->io_bf16, p->num_sms, k == POLYCONV_KERNEL_TC_FUSED, p->io_bf16);
     g.Cp = (g.C + p->tc2.kc - 1) / p->tc2.kc * p->tc2.kc;
     g.Kp = (g.K + 127) / 128 * 128;
   } else if (k == POLYCONV_KERNEL_TC_PERTAP) {
@@ -95,7 +101,7 @@ polyconv_status_t resolve(polyconv_plan_t p) {
   g.urep = 1;
   if (k == POLYCONV_KERNEL_TC || k == POLYCONV_KERNEL_TC_FUSED) {
     const char* r = getenv("POLYCONV_FILTER_REP");  // experiments only
-    g.urep = r ? atoi(r) : 8;
+    g.urep = r ? atoi(r) : 1;
     if (g.urep < 1) g.urep = 1;
     if (g.urep > 64) g.urep = 64;
     if ((long long)g.urep * g.R * g.S * g.Kp >= (1LL << 31)) g.urep = 1;  // TMA row coordinate
@@ -272,7 +278,8 @@ polyconv_status_t polyconv_plan_info(polyconv_plan_t p, polyconv_info_t* info) {
   switch (p->kernel) {
     case POLYCONV_KERNEL_TC:  // tile = positions x output channels
     case POLYCONV_KERNEL_TC_FUSED:
-      info->tile_m = p->tc2.nt; info->tile_n = 128; info->stages = p->tc2.a_stages; info->launches = 2; break;
+      info->tile_m = p->tc2.nt; info->tile_n = 128; info->stages = p->tc2.a_stages;
+      info->launches = p->kernel == POLYCONV_KERNEL_TC_FUSED ? 1 : 2; break;
     case POLYCONV_KERNEL_TC_PERTAP:
       info->tile_m = p->tc.bm; info->tile_n = p->tc.bn; info->stages = p->tc.stages; info->launches = 2; break;
     case POLYCONV_KERNEL_FP32:
@@ -308,12 +315,28 @@ polyconv_status_t polyconv_forward(polyconv_plan_t p, const void* x, const void*
     return finish(p, e, "mac_tc");
   }
   if (p->kernel == POLYCONV_KERNEL_TC_FUSED) {
-    // a3 (filter pack, tiny) then the fused a2+a4+a5 kernel as its programmatic dependent
+    // one launch: a3 (filter slices, every CTA), a2 (packer warps), a4, a5.  The
+    // grid is persistent (one CTA per SM at most), so all CTAs are co-resident
+    // and meet on the plan's counter before the first filter tile is loaded.
+    if (!p->fcount) {
+      if (cudaMalloc(&p->fcount, sizeof(unsigned long long)) != cudaSuccess ||
+          cudaMemsetAsync(p->fcount, 0, sizeof(unsigned long long), st) != cudaSuccess) {
+        cudaGetLastError();
+        p->fcount = nullptr;
+        set_err(p, "cudaMalloc of the %s failed", "filter-pack counter");
+        return POLYCONV_STATUS_ALLOC_FAILED;
+      }
+      p->fepoch = 0;
+    }
+    if (p->tc2.grid > p->num_sms) {
+      set_err(p, "mac_tc_fused: grid %s exceeds the SM count", "");
+      return POLYCONV_STATUS_NOT_SUPPORTED;
+    }
     if (p->ev_start) cudaEventRecord(p->ev_start, st);
-    e = launch_pack_filter_tapmajor(g, w, p->io_bf16, p->wsU, p->fmt, g.Kp, g.Cp, st);
-    if (e != cudaSuccess) return finish(p, e, "pack_filter");
-    e = launch_mac_tc2(g, p->tc2, p->fmt, x, p->io_bf16, nullptr, p->wsU, y, p->io_bf16, true, st, p->err,
-                       sizeof(p->err));
+    const unsigned long long target = (p->fepoch + 1) * (unsigned long long)p->tc2.grid;
+    e = launch_mac_tc2(g, p->tc2, p->fmt, x, p->io_bf16, nullptr, p->wsU, y, p->io_bf16, false, st, p->err,
+                       sizeof(p->err), w, p->fcount, target);
+    if (e == cudaSuccess) ++p->fepoch;
     if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
     return finish(p, e, "mac_tc_fused");
   }
@@ -429,7 +452,7 @@ polyconv_status_t polyconv_extract(polyconv_plan_t p, const float* coeffs, void*
 polyconv_status_t polyconv_destroy(polyconv_plan_t p) {
   if (!p) return POLYCONV_STATUS_SUCCESS;
   polyconv_status_t s = POLYCONV_STATUS_SUCCESS;
-  if (p->used || p->wsA || p->wsU || p->hx || p->hw || p->hy) {
+  if (p->used || p->wsA || p->wsU || p->hx || p->hw || p->hy || p->fcount) {
     DeviceGuard guard(p->device);
     if (p->used && cudaStreamSynchronize(p->last_stream) != cudaSuccess) {
       cudaGetLastError();
@@ -440,6 +463,7 @@ polyconv_status_t polyconv_destroy(polyconv_plan_t p) {
     if (p->hx) cudaFree(p->hx);
     if (p->hw) cudaFree(p->hw);
     if (p->hy) cudaFree(p->hy);
+    if (p->fcount) cudaFree(p->fcount);
   }
   delete p;
   return s;

@@ -150,7 +150,7 @@ def test_conv3x_bench_launch_config():
     x, w = synth.make_inputs(shape, synth.seed_for(1), "uniform")
     ref = oracle.conv2d(x, w, shape.stride, shape.padding)
     y, plan = gpu_forward(shape, x, w, math="bf16", io="bf16")
-    assert plan.info()["kernel"] == "tc"
+    assert plan.info()["kernel"] == "tc_fused"  # bf16 in/out: the one-launch fused kernel
     assert normwise(y, ref) <= GATE["bf16"]
     xi, wi = synth.make_inputs(shape, synth.seed_for(1), "int")
     y, _ = gpu_forward(shape, xi, wi, math="bf16", io="bf16", plan=plan)

@@ -45,6 +45,14 @@ st = torch.cuda.current_stream()
 def pack():
     lib.polyconv_pack_input(plan.handle, ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(dst.data_ptr()), 1,
                             ctypes.c_void_p(st.cuda_stream))
+wdst = torch.empty(w.numel() * 4, dtype=torch.bfloat16, device="cuda")
+def packf():
+    lib.polyconv_pack_filter(plan.handle, ctypes.c_void_p(w.data_ptr()), ctypes.c_void_p(wdst.data_ptr()), 1,
+                             ctypes.c_void_p(st.cuda_stream))
+print("pack_filter tap-major: med %.2f us min %.2f us" % timeit(packf))
+tiny = torch.zeros(4, device="cuda")
+print("one tiny torch kernel: med %.2f us min %.2f us" % timeit(lambda: tiny.zero_()))
+print("two tiny torch kernels: med %.2f us min %.2f us" % timeit(lambda: (tiny.zero_(), tiny.zero_())))
 print("flush mode", MODE); print("pack_input interleaved: med %.2f us min %.2f us (%d bytes out)" % (*timeit(pack), nb.value))
 for k in kernels:
     p = pc.Plan(x.shape, w.shape, shape.stride, shape.padding, math=math, io_dtype=io, kernel=k)

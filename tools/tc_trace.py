@@ -17,11 +17,13 @@ print(plan.info())
 lib = pc.load_library()
 buf = (ctypes.c_ulonglong * (160 * 8))()
 flush = torch.empty(64 << 20, device="cuda")
+evict = torch.empty(64 << 20, device="cuda")
 names = ["setup", "first_B_full", "mma_issued", "epi_start", "epi_end", "packer_win0", "cta_end"]
 for mode in modes:
     os.environ["POLYCONV_TC_DEBUG"] = str(8 | mode)
     for it in range(3):
         flush.zero_()
+        evict.sum()  # write back the flush's dirty lines before the launch
         y = plan.forward(x, w)
         torch.cuda.synchronize()
     lib.polyconv_dbg_tc2_trace(buf)
@@ -39,6 +41,12 @@ for mode in modes:
         ns = None
         print("  MMA phase in SM cycles: min %d med %d max %d" % (cyc.min(), np.median(cyc), cyc.max()))
         continue
+    if mode & 128:
+        eb = (ctypes.c_ulonglong * (160 * 8))()
+        lib.polyconv_dbg_tc2_epi(eb)
+        e = np.array(eb, dtype=np.float64).reshape(160, 8)[:len(a)]
+        for k, nm in enumerate(["tmem_ld", "stage_st", "bar1", "pos_table", "copy_out", "bar2"]):
+            print("  epi %-10s cycles med %7d max %7d" % (nm, np.median(e[:, k]), e[:, k].max()))
     if mode & 16:
         pkb = (ctypes.c_ulonglong * (160 * 8))()
         lib.polyconv_dbg_tc2_pk(pkb)
