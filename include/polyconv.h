@@ -77,7 +77,13 @@ typedef enum {
  * packed input; TC_FUSED = the same contraction with the input packing done
  * inside the kernel by packer warps (ablation); TC_PERTAP = the earlier
  * tensor-core variant with positions as M and one TMA window load per tap
- * (ablation);
+ * (ablation); TC_PAIR = the BF16 default: ONE launch that packs the input
+ * and filter polynomials (a2, a3) into the plan workspace, then runs the
+ * contraction on CTA pairs (tcgen05 cta_group::2, 256 positions x up to 256
+ * output channels per pair tile) with the filter resident in shared memory
+ * and the extraction (a5) fused into its epilogue (bf16 math, K <= 256 and a
+ * filter half that fits shared memory; polyconv_plan_set_kernel returns
+ * POLYCONV_STATUS_BAD_PARAM otherwise);
  * FP32 = SIMT register-blocked FFMA; THIN = warp-per-output with shuffle
  * reduction over C*R*S (tiny channel counts). */
 typedef enum {
@@ -86,7 +92,8 @@ typedef enum {
     POLYCONV_KERNEL_FP32 = 2,
     POLYCONV_KERNEL_THIN = 3,
     POLYCONV_KERNEL_TC_PERTAP = 4,
-    POLYCONV_KERNEL_TC_FUSED = 5
+    POLYCONV_KERNEL_TC_FUSED = 5,
+    POLYCONV_KERNEL_TC_PAIR = 6
 } polyconv_kernel_t;
 
 /* Packed-operand layouts exposed for bit-exact tests (a2/a3):

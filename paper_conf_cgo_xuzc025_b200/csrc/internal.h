@@ -109,4 +109,24 @@ cudaError_t launch_mac_tc2(const Geom& g, const Tc2Tiling& t, int fmt, const voi
                            char* err, size_t errlen, const void* w = nullptr,
                            unsigned long long* fcount = nullptr, unsigned long long ftarget = 0);
 
+// ---- mac_pair.cu (bf16 default: one launch, CTA pairs, resident filter) -------
+struct PairTiling {
+  bool ok;              // shape supported (bf16 math, K <= 256, filter half + 2 windows fit)
+  int kc, row_bytes;    // channels per chunk (one swizzle row of kc bf16 words)
+  int Cp, NN;           // padded channels (multiple of kc); MMA N = padded output channels
+  int nchunks, RS, nblk;
+  int box_rows, nbox;   // position window: nbox TMA boxes of box_rows rows
+  int wbytes, wbytes_tx, fbytes;
+  int ring;             // window ring depth
+  int smem_bytes, tmem_cols;
+  int num_tiles, num_pairs, grid;
+  int rb, nb, nunits, spitch;  // packing bands (rb padded rows, nb per image), staging pitch
+};
+PairTiling pair_tiling(const Geom& g, int fmt, int num_sms);
+// One launch: packs w -> U [R*S][NN][Cp] and x -> A [N*L_A][Cp] (bf16, plan workspace),
+// meets on *fcount (must reach ftarget = launches so far x t.grid), then the pair MAC.
+cudaError_t launch_mac_pair(const Geom& g, const PairTiling& t, const void* x, const void* w, bool io_bf16,
+                            void* A, void* U, void* y, unsigned long long* fcount, unsigned long long ftarget,
+                            cudaStream_t st, char* err, size_t errlen);
+
 }  // namespace polyconv

@@ -23,6 +23,7 @@ struct polyconv_plan_s {
   TcTiling tc;
   Tc2Tiling tc2;
   Fp32Tiling f32;
+  PairTiling pair;
   // workspace (lazy)
   void* wsA = nullptr;
   size_t wsA_bytes = 0;
@@ -58,8 +59,11 @@ polyconv_status_t resolve(polyconv_plan_t p) {
   Geom& g = p->g;
   int k = p->forced;
   const bool tc_math = p->math != POLYCONV_MATH_FP32_FMA;
+  if (k == POLYCONV_KERNEL_AUTO || k == POLYCONV_KERNEL_TC_PAIR) p->pair = pair_tiling(g, p->fmt, p->num_sms);
   if (k == POLYCONV_KERNEL_AUTO) {
-    if (tc_math && g.K >= 16 && tc2_supported(g, p->fmt) && p->io_bf16 && !getenv("POLYCONV_NO_FUSED_DEFAULT") &&
+    if (tc_math && g.K >= 16 && p->pair.ok && !getenv("POLYCONV_NO_PAIR_DEFAULT"))
+      k = POLYCONV_KERNEL_TC_PAIR;  // bf16: one launch, CTA pairs, resident filter
+    else if (tc_math && g.K >= 16 && tc2_supported(g, p->fmt) && p->io_bf16 && !getenv("POLYCONV_NO_FUSED_DEFAULT") &&
         tc2_is_mx(tc2_tiling(g, p->fmt, p->io_bf16, p->num_sms, true, p->io_bf16)))
       k = POLYCONV_KERNEL_TC_FUSED;  // bf16 in/out: one launch, input packed in-kernel
     else if (tc_math)
@@ -72,10 +76,14 @@ polyconv_status_t resolve(polyconv_plan_t p) {
   }
   if ((k == POLYCONV_KERNEL_TC || k == POLYCONV_KERNEL_TC_FUSED) && (!tc_math || !tc2_supported(g, p->fmt)))
     return POLYCONV_STATUS_BAD_PARAM;
+  if (k == POLYCONV_KERNEL_TC_PAIR && (!tc_math || !p->pair.ok)) return POLYCONV_STATUS_BAD_PARAM;
   if (k == POLYCONV_KERNEL_TC_PERTAP && (!tc_math || !tc_supported(g, p->fmt))) return POLYCONV_STATUS_BAD_PARAM;
   if (k == POLYCONV_KERNEL_FP32 && (tc_math || fp32_tiling(g).smax == 0)) return POLYCONV_STATUS_BAD_PARAM;
   p->kernel = k;
-  if (k == POLYCONV_KERNEL_TC || k == POLYCONV_KERNEL_TC_FUSED) {
+  if (k == POLYCONV_KERNEL_TC_PAIR) {
+    g.Cp = p->pair.Cp;
+    g.Kp = p->pair.NN;
+  } else if (k == POLYCONV_KERNEL_TC || k == POLYCONV_KERNEL_TC_FUSED) {
     p->tc2 = tc2_tiling(g, p->fmt, p->io_bf16, p->num_sms, k == POLYCONV_KERNEL_TC_FUSED, p->io_bf16);
     g.Cp = (g.C + p->tc2.kc - 1) / p->tc2.kc * p->tc2.kc;
     g.Kp = (g.K + 127) / 128 * 128;
@@ -95,7 +103,7 @@ polyconv_status_t resolve(polyconv_plan_t p) {
   // TC packs the input on the fly (no input workspace); TC_PERTAP needs the
   // interleaved copy, FP32/THIN the planar one
   const size_t a_elems = k == POLYCONV_KERNEL_TC_FUSED ? 0
-                         : (k == POLYCONV_KERNEL_TC || k == POLYCONV_KERNEL_TC_PERTAP) ? (size_t)g.N * g.L_A * g.Cp
+                         : (k == POLYCONV_KERNEL_TC || k == POLYCONV_KERNEL_TC_PERTAP || k == POLYCONV_KERNEL_TC_PAIR) ? (size_t)g.N * g.L_A * g.Cp
                                                                                        : (size_t)g.N * g.C * g.L_A;
   p->wsA_bytes = a_elems * eb;
   g.urep = 1;
@@ -246,7 +254,7 @@ polyconv_status_t polyconv_plan(polyconv_plan_t* plan, int N, int C, int H, int 
 
 polyconv_status_t polyconv_plan_set_kernel(polyconv_plan_t p, polyconv_kernel_t kernel) {
   if (!p) return POLYCONV_STATUS_BAD_PARAM;
-  if (kernel < POLYCONV_KERNEL_AUTO || kernel > POLYCONV_KERNEL_TC_FUSED) return POLYCONV_STATUS_BAD_PARAM;
+  if (kernel < POLYCONV_KERNEL_AUTO || kernel > POLYCONV_KERNEL_TC_PAIR) return POLYCONV_STATUS_BAD_PARAM;
   const int old = p->forced;
   p->forced = kernel;
   if (resolve(p) != POLYCONV_STATUS_SUCCESS) {
@@ -254,7 +262,8 @@ polyconv_status_t polyconv_plan_set_kernel(polyconv_plan_t p, polyconv_kernel_t 
     resolve(p);
     return POLYCONV_STATUS_BAD_PARAM;
   }
-  // workspace sizes may have changed
+  // workspace sizes (and the grid the pack counter counts) may have changed
+  if (p->fcount) { cudaFree(p->fcount); p->fcount = nullptr; }
   if (p->wsA) { cudaFree(p->wsA); p->wsA = nullptr; }
   if (p->wsU) { cudaFree(p->wsU); p->wsU = nullptr; }
   return POLYCONV_STATUS_SUCCESS;
@@ -280,6 +289,8 @@ polyconv_status_t polyconv_plan_info(polyconv_plan_t p, polyconv_info_t* info) {
     case POLYCONV_KERNEL_TC_FUSED:
       info->tile_m = p->tc2.nt; info->tile_n = 128; info->stages = p->tc2.a_stages;
       info->launches = p->kernel == POLYCONV_KERNEL_TC_FUSED ? 1 : 2; break;
+    case POLYCONV_KERNEL_TC_PAIR:  // pair tile = 256 positions x NN output channels
+      info->tile_m = 256; info->tile_n = p->pair.NN; info->stages = p->pair.ring; info->launches = 1; break;
     case POLYCONV_KERNEL_TC_PERTAP:
       info->tile_m = p->tc.bm; info->tile_n = p->tc.bn; info->stages = p->tc.stages; info->launches = 2; break;
     case POLYCONV_KERNEL_FP32:
@@ -313,6 +324,27 @@ polyconv_status_t polyconv_forward(polyconv_plan_t p, const void* x, const void*
                        sizeof(p->err));
     if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
     return finish(p, e, "mac_tc");
+  }
+  if (p->kernel == POLYCONV_KERNEL_TC_PAIR) {
+    // one launch: a3 + a2 into the workspace (every CTA a slice), grid counter,
+    // then a4 + a5 on CTA pairs.  All CTAs are co-resident (checked at launch).
+    if (!p->fcount) {
+      if (cudaMalloc(&p->fcount, sizeof(unsigned long long)) != cudaSuccess ||
+          cudaMemsetAsync(p->fcount, 0, sizeof(unsigned long long), st) != cudaSuccess) {
+        cudaGetLastError();
+        p->fcount = nullptr;
+        set_err(p, "cudaMalloc of the %s failed", "pack counter");
+        return POLYCONV_STATUS_ALLOC_FAILED;
+      }
+      p->fepoch = 0;
+    }
+    if (p->ev_start) cudaEventRecord(p->ev_start, st);
+    const unsigned long long target = (p->fepoch + 1) * (unsigned long long)p->pair.grid;
+    e = launch_mac_pair(g, p->pair, x, w, p->io_bf16, p->wsA, p->wsU, y, p->fcount, target, st, p->err,
+                        sizeof(p->err));
+    if (e == cudaSuccess) ++p->fepoch;
+    if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
+    return finish(p, e, "mac_pair");
   }
   if (p->kernel == POLYCONV_KERNEL_TC_FUSED) {
     // one launch: a3 (filter slices, every CTA), a2 (packer warps), a4, a5.  The

@@ -60,7 +60,13 @@ def test_plan_sizes_match_oracle(H, W, R, S, s, p):
 
 
 def test_kernel_selection_and_forcing():
-    assert pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="bf16").info()["kernel"] == "tc"
+    assert pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="bf16").info()["kernel"] == "tc_pair"
+    # K > 256 (two output-channel tiles): the single-CTA tensor-core kernel
+    assert pc.Plan((1, 64, 10, 10), (320, 64, 3, 3), padding=(1, 1), math="bf16").info()["kernel"] == "tc"
+    with pytest.raises(pc.PolyconvError):
+        pc.Plan((1, 64, 10, 10), (320, 64, 3, 3), padding=(1, 1), math="bf16", kernel="tc_pair")
+    with pytest.raises(pc.PolyconvError):
+        pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="tf32", kernel="tc_pair")
     assert pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="tf32").info()["kernel"] == "tc"
     assert pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="fp32").info()["kernel"] == "fp32"
     assert pc.Plan((1, 1, 8, 8), (1, 1, 3, 3), math="fp32").info()["kernel"] == "thin"
@@ -76,14 +82,22 @@ def test_kernel_selection_and_forcing():
 def test_tc_tiling_choices():
     # default TC: tile = nt positions x 128 output channels; conv3_x (G = 31*900 + 838
     # positions) -> nt = 208 gives 139 tiles, one wave on 148 SMs
-    inf = pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="bf16").info()
+    inf = pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="bf16", kernel="tc").info()
     assert (inf["tile_m"], inf["tile_n"], inf["Cp"], inf["Kp"]) == (208, 128, 128, 128)
-    inf = pc.Plan((2, 3, 30, 30), (64, 3, 7, 7), (2, 2), (3, 3), math="bf16").info()
+    inf = pc.Plan((2, 3, 30, 30), (64, 3, 7, 7), (2, 2), (3, 3), math="bf16", kernel="tc").info()
     assert inf["Cp"] == 16 and inf["Kp"] == 128           # C=3 -> one 32-byte swizzle row
     inf = pc.Plan((2, 3, 30, 30), (64, 3, 7, 7), (2, 2), (3, 3), math="tf32").info()
     assert inf["Cp"] == 8
     inf = pc.Plan((1, 64, 10, 10), (320, 64, 3, 3), (1, 1), (1, 1), math="bf16").info()
     assert inf["tile_n"] == 128 and inf["Kp"] == 384
+    # TC_PAIR (bf16 default): pair tile = 256 positions x NN output channels (NN = K
+    # rounded up to 64), channels in chunks of 64/32/16; one launch
+    inf = pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="bf16").info()
+    assert (inf["tile_m"], inf["tile_n"], inf["Cp"], inf["Kp"], inf["launches"]) == (256, 128, 128, 128, 1)
+    inf = pc.Plan((2, 3, 30, 30), (64, 3, 7, 7), (2, 2), (3, 3), math="bf16").info()
+    assert (inf["kernel"], inf["Cp"], inf["Kp"]) == ("tc_pair", 16, 64)
+    inf = pc.Plan((2, 40, 9, 9), (72, 40, 3, 3), (1, 1), (1, 1), math="bf16").info()
+    assert (inf["kernel"], inf["Cp"], inf["Kp"]) == ("tc_pair", 64, 128)
     # TC_PERTAP (ablation): tile = 128 positions x bn output channels
     inf = pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="bf16", kernel="tc_pertap").info()
     assert (inf["tile_m"], inf["tile_n"], inf["Cp"], inf["Kp"]) == (128, 128, 128, 128)

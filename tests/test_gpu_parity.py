@@ -18,7 +18,7 @@ pytestmark = pytest.mark.gpu
 
 MATH_KERNELS = [("fp32", "fp32"), ("fp32", "thin"), ("tf32", "tc"), ("bf16", "tc"), ("tf32", "tc_pertap"),
                 ("bf16", "tc_pertap"), ("tf32", "tc_fused"), ("bf16", "tc_fused"), ("tf32", "thin"),
-                ("bf16", "thin")]
+                ("bf16", "thin"), ("bf16", "tc_pair")]
 
 SHAPES = [
     ConvShape("tiny", 1, 1, 8, 8, 1, 3, 3),                      # BASELINE configs[0]
@@ -38,6 +38,8 @@ SHAPES = [
 def _skip_unsupported(shape, math, kernel):
     if kernel == "fp32" and max(shape.R, shape.S) > 7:
         pytest.skip("fp32 kernel limited to S<=7")
+    if kernel == "tc_pair" and shape.K > 256:
+        pytest.skip("tc_pair: one output-channel tile (K <= 256)")
 
 
 @pytest.mark.parametrize("shape", SHAPES, ids=lambda s: s.name)
@@ -93,7 +95,7 @@ MX_SHAPES = [
 
 
 @pytest.mark.parametrize("shape", MX_SHAPES, ids=lambda s: s.name)
-@pytest.mark.parametrize("kernel", ["tc_fused", "tc"])
+@pytest.mark.parametrize("kernel", ["tc_fused", "tc", "tc_pair"])
 def test_bf16_io_fused_packing(shape, kernel):
     """bf16 in/out, BF16 math: integer data bit-exact against round_bf16(O1);
     uniform data within the BF16 gate."""
@@ -106,16 +108,18 @@ def test_bf16_io_fused_packing(shape, kernel):
     assert normwise(y, oracle.conv2d(x, w, shape.stride, shape.padding)) <= GATE["bf16"]
 
 
-def test_conv3x_fused_bf16_io():
-    """BASELINE configs[1] in full, bf16 in/out, the fused kernel."""
+@pytest.mark.parametrize("kernel", ["tc_fused", "tc_pair"])
+def test_conv3x_fused_bf16_io(kernel):
+    """BASELINE configs[1] in full, bf16 in/out, the one-launch kernels."""
     shape = synth.CONV3X
     xi, wi = synth.make_inputs(shape, synth.seed_for(1), "int")
-    y, plan = gpu_forward(shape, xi, wi, math="bf16", io="bf16", kernel="tc_fused")
+    y, plan = gpu_forward(shape, xi, wi, math="bf16", io="bf16", kernel=kernel)
     assert np.array_equal(y, bf16_round(oracle.conv2d(xi, wi, shape.stride, shape.padding)))
 
 
 @pytest.mark.parametrize("math,kernel", [("fp32", "fp32"), ("bf16", "tc"), ("tf32", "tc"), ("fp32", "thin"),
-                                         ("bf16", "tc_pertap"), ("bf16", "tc_fused")])
+                                         ("bf16", "tc_pertap"), ("bf16", "tc_fused"),
+                                         ("bf16", "tc_pair")])
 def test_delta_filter_bit_exact(math, kernel):
     """w[k][c][i][j] = [c == k mod C][i == i0][j == j0] -> y = shifted xpad,
     bit-exact for every tap (checks each shift e(i,j) and the padding)."""
@@ -150,7 +154,7 @@ def test_conv3x_bench_launch_config():
     x, w = synth.make_inputs(shape, synth.seed_for(1), "uniform")
     ref = oracle.conv2d(x, w, shape.stride, shape.padding)
     y, plan = gpu_forward(shape, x, w, math="bf16", io="bf16")
-    assert plan.info()["kernel"] == "tc_fused"  # bf16 in/out: the one-launch fused kernel
+    assert plan.info()["kernel"] == "tc_pair"  # bf16: the one-launch CTA-pair kernel
     assert normwise(y, ref) <= GATE["bf16"]
     xi, wi = synth.make_inputs(shape, synth.seed_for(1), "int")
     y, _ = gpu_forward(shape, xi, wi, math="bf16", io="bf16", plan=plan)
