@@ -121,8 +121,12 @@ struct PairTiling {
   int smem_bytes, tmem_cols;
   int num_tiles, num_pairs, grid;
   int rb, nb, nunits, spitch;  // packing bands (rb padded rows, nb per image), staging pitch
+  int pack_tma;                // bands in/out by TMA (x band box ne_box x C; A boxes 64 ch x rb*Wp rows)
+  int ne_box, last_rows, in_bytes, obox_bytes, obox_bytes2;
+  int tr, tpi, ntile;          // row-aligned CTA tiles: tr output rows of one image each
+  int epi_tma, estage_bytes;   // epilogue staged in shared memory and written by TMA stores
 };
-PairTiling pair_tiling(const Geom& g, int fmt, int num_sms);
+PairTiling pair_tiling(const Geom& g, int fmt, bool io_bf16, int num_sms);
 // One launch: packs w -> U [R*S][NN][Cp] and x -> A [N*L_A][Cp] (bf16, plan workspace),
 // meets on *fcount (must reach ftarget = launches so far x t.grid), then the pair MAC.
 cudaError_t launch_mac_pair(const Geom& g, const PairTiling& t, const void* x, const void* w, bool io_bf16,

@@ -75,6 +75,17 @@ struct PairParams {
   int rb, nb, nunits, spitch;
   FastDiv fLA, fWp, fsh, fsw;
   int dbg;
+  // TMA pack path (pack_tma): x band [C rows][ne_box elements] in by TMA, the band's
+  // A rows out by TMA stores of 64-channel SW128 boxes (rb*Wp rows; the last band
+  // of an image through the second map)
+  int pack_tma, ne_box, last_rows;
+  uint32_t in_bytes, obox_bytes, obox_bytes2;
+  // row-aligned tiles: a CTA tile = tr output rows of one image (tpi tiles per image,
+  // ntile CTA tiles in all); epilogue by TMA stores of [32 channels][tr*Q pixels]
+  // boxes staged in shared memory (epi_tma) or by direct stores
+  int tr, tpi, ntile, epi_tma;
+  uint32_t estage_bytes;
+  FastDiv ftpi;
 };
 
 // per-CTA phase trace (POLYCONV_PAIR_DEBUG & 8), globaltimer ns:
@@ -84,7 +95,8 @@ struct PairParams {
 // (leader), 15 last window TMA issued (producer)
 constexpr int kTr = 16;
 __device__ unsigned long long g_pair_trace[160 * kTr];
-__device__ unsigned long long g_pair_clk[160 * 2];  // clock64 at tr[0] and tr[13]: SM clock = cycles / ns
+__device__ unsigned long long g_pair_clk[160 * 2];
+__device__ unsigned long long g_pair_pk[160 * 4];  // pack sub-phases: filter done, band staged, band written  // clock64 at tr[0] and tr[13]: SM clock = cycles / ns
 
 // ---- pair-specific PTX ---------------------------------------------------------
 __device__ __forceinline__ uint32_t mapa_rank0(uint32_t local) {
@@ -167,9 +179,10 @@ __device__ __forceinline__ uint16_t to_bf16_bits<__nv_bfloat16>(__nv_bfloat16 v)
 
 // ---- phase 1: a3 + a2 into the workspace ----------------------------------------
 template <typename IoT>
-__device__ __forceinline__ void pair_pack(const PairParams& p, uint16_t* stg) {
+__device__ __forceinline__ void pair_pack(const PairParams& p, uint16_t* stg, bool x_too) {
   const int tid = threadIdx.x;
   const int nth = blockDim.x;
+  const bool ptr = (p.dbg & 8) && blockIdx.x < 160 && tid == 0;
   // a3: U[tap][k][c] = w[k][c][tap] (tap = i*S + j; k >= K or c >= C: 0)
   {
     const IoT* w = static_cast<const IoT*>(p.w);
@@ -183,6 +196,8 @@ __device__ __forceinline__ void pair_pack(const PairParams& p, uint16_t* stg) {
         U[((long long)t * p.NN + k) * p.Cp + c] = ok ? to_bf16_bits<IoT>(src[t]) : (uint16_t)0;
     }
   }
+  if (ptr) g_pair_pk[blockIdx.x * 4] = global_ns();
+  if (!x_too) return;
   // a2: bands of rb padded rows of one image: stage the band's input rows of
   // every channel (contiguous in NCHW), then write each position's Cp channel
   // words as 16-byte chunks (coalesced: consecutive threads, consecutive chunks)
@@ -254,6 +269,7 @@ __device__ __forceinline__ void pair_pack(const PairParams& p, uint16_t* stg) {
       }
     }
     __syncthreads();
+    if (ptr) g_pair_pk[blockIdx.x * 4 + 1] = global_ns();
     const int npos = (r1 - r0) * p.Wp;
     uint4* dst = A4 + ((long long)n * p.L_A + (long long)r0 * p.Wp) * ncg;
     for (int idx = tid; idx < npos * ncg; idx += nth) {
@@ -274,26 +290,126 @@ __device__ __forceinline__ void pair_pack(const PairParams& p, uint16_t* stg) {
       dst[idx] = make_uint4(v[0], v[1], v[2], v[3]);
     }
     __syncthreads();
+    if (ptr) g_pair_pk[blockIdx.x * 4 + 2] = global_ns();
+  }
+}
+
+// a2 by TMA: one 2-D TMA box brings the band's input rows of all C channel planes
+// (x viewed as [N*C][H*W]; elements past the plane / planes past N*C are
+// zero-filled or ignored), the warps transpose it into the band's rows of the
+// interleaved layout (coefficient r*Wp + s of A_{n,c}(t) = xpad[n][c][r][s],
+// Eq. 10, zero padding P.1353-1356), 128-byte swizzled per 64 channels, and TMA
+// stores write them out.  Consecutive threads take consecutive positions, so the
+// staging reads are conflict-free and the swizzled 16-byte writes are too.
+__device__ __forceinline__ void tma_store_2d(const void* tmap, uint32_t src, int c0, int c1) {
+  asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
+                   reinterpret_cast<uint64_t>(tmap)),
+               "r"(src), "r"(c0), "r"(c1)
+               : "memory");
+}
+
+template <typename IoT>
+__device__ __forceinline__ void pair_pack_x_tma(const PairParams& p, uint8_t* stage, uint64_t* pbar,
+                                                const CUtensorMap* tmX, const CUtensorMap* tmS,
+                                                const CUtensorMap* tmS2, bool first_issued) {
+  const int tid = threadIdx.x;
+  const int nth = blockDim.x;
+  const bool ptr = (p.dbg & 8) && blockIdx.x < 160 && tid == 0;
+  const IoT* in = reinterpret_cast<const IoT*>(stage);
+  uint8_t* out = stage + p.in_bytes;
+  int it = 0;
+  for (int u = blockIdx.x; u < p.nunits; u += gridDim.x, ++it) {
+    const int n = u / p.nb, b = u - (u / p.nb) * p.nb;
+    const int r0 = b * p.rb, r1 = min(p.Hp, r0 + p.rb);
+    const int h0 = min(max(r0 - p.ph, 0), p.H), h1 = min(max(r1 - p.ph, 0), p.H);
+    const bool any = h1 > h0;
+    if (tid == 0 && any && !(it == 0 && first_issued)) {
+      mbar_arrive_expect_tx(pbar, p.C * p.ne_box * (uint32_t)sizeof(IoT));
+      tma_load_2d(stage, tmX, pbar, (h0 * p.W) & ~(16 / (int)sizeof(IoT) - 1), n * p.C);
+    }
+    if (any) mbar_wait(pbar, (uint32_t)(it & 1));
+    if (ptr) g_pair_pk[blockIdx.x * 4 + 1] = global_ns();
+    const int npos = (r1 - r0) * p.Wp;
+    FastDiv fnp;
+    fnp.init((uint32_t)npos);
+    const uint32_t obox = (r1 - r0 == p.rb) ? p.obox_bytes : p.obox_bytes2;
+    const int nbx = p.Cp / 64;
+    const int eoff = (h0 * p.W) & (16 / (int)sizeof(IoT) - 1);  // the box starts at h0*W rounded down
+    // one item = one position's 64 channels = one 128-byte row of box bx; consecutive
+    // threads take consecutive positions (conflict-free staging reads and swizzled writes)
+    for (int idx = tid; idx < nbx * npos; idx += nth) {
+      const int bx = (int)fnp.div((uint32_t)idx), pos = idx - bx * npos;
+      const int rr = (int)p.fWp.div((uint32_t)pos);
+      const int h = r0 + rr - p.ph, ww = pos - rr * p.Wp - p.pw;
+      uint8_t* drow = out + (size_t)bx * obox + (size_t)pos * 128;
+      const uint32_t sw = (uint32_t)(pos & 7);
+      if (h >= 0 && h < p.H && ww >= 0 && ww < p.W) {
+        const IoT* src = in + (size_t)(bx * 64) * p.ne_box + (h - h0) * p.W + ww + eoff;
+        const int cbase = bx * 64;
+#pragma unroll
+        for (int q8 = 0; q8 < 8; ++q8) {
+          const int c0 = cbase + q8 * 8;
+          uint32_t v[4];
+          if (c0 + 8 <= p.C) {
+            uint32_t hv[8];
+#pragma unroll
+            for (int k = 0; k < 8; ++k) hv[k] = to_bf16_bits<IoT>(src[(q8 * 8 + k) * p.ne_box]);
+#pragma unroll
+            for (int m = 0; m < 4; ++m) v[m] = hv[2 * m] | (hv[2 * m + 1] << 16);
+          } else {
+#pragma unroll
+            for (int m = 0; m < 4; ++m) {
+              const int c = c0 + 2 * m;
+              const uint32_t lo = c < p.C ? (uint32_t)to_bf16_bits<IoT>(src[(q8 * 8 + 2 * m) * p.ne_box]) : 0u;
+              const uint32_t hi =
+                  c + 1 < p.C ? (uint32_t)to_bf16_bits<IoT>(src[(q8 * 8 + 2 * m + 1) * p.ne_box]) : 0u;
+              v[m] = lo | (hi << 16);
+            }
+          }
+          *reinterpret_cast<uint4*>(drow + (((uint32_t)q8 ^ sw) << 4)) = make_uint4(v[0], v[1], v[2], v[3]);
+        }
+      } else {
+#pragma unroll
+        for (int q8 = 0; q8 < 8; ++q8)
+          *reinterpret_cast<uint4*>(drow + (((uint32_t)q8 ^ sw) << 4)) = make_uint4(0u, 0u, 0u, 0u);
+      }
+    }
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // staging -> TMA store / next load
+    __syncthreads();
+    if (ptr) g_pair_pk[blockIdx.x * 4 + 3] = global_ns();
+    if (tid == 0) {
+      const CUtensorMap* m = (r1 - r0 == p.rb) ? tmS : tmS2;
+      for (int bx = 0; bx < p.Cp / 64; ++bx)
+        tma_store_2d(m, smem_u32(out + (size_t)bx * obox), bx * 64, (int)((long long)n * p.L_A + (long long)r0 * p.Wp));
+      asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+      asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");  // written (before the grid counter / reuse)
+    }
+    __syncthreads();
+    if (ptr) g_pair_pk[blockIdx.x * 4 + 2] = global_ns();
   }
 }
 
 template <typename IoT>
 __global__ void __launch_bounds__(kPairThreads, 1)
     mac_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmU,
+                    const __grid_constant__ CUtensorMap tmX, const __grid_constant__ CUtensorMap tmS,
+                    const __grid_constant__ CUtensorMap tmS2, const __grid_constant__ CUtensorMap tmY,
                     const PairParams p) {
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw = smem_u32(smem_raw);
   uint8_t* smem = smem_raw + (((raw + 1023u) & ~1023u) - raw);
   uint8_t* sF = smem;                                        // filter blocks [nblk][NN/2][row]
   uint8_t* sWin = sF + (size_t)p.nblk * p.fbytes;            // window ring [ring][rows][row]
-  uint64_t* bars = reinterpret_cast<uint64_t*>(sWin + (size_t)p.ring * p.wbytes);
+  uint8_t* sEpi = sWin + (size_t)p.ring * p.wbytes;          // epilogue staging [NN][tr*Q] bf16
+  uint64_t* bars = reinterpret_cast<uint64_t*>(sEpi + p.estage_bytes);
   uint64_t* ffull = bars;                 // [kMaxBlk] filter block landed (leader: both halves)
   uint64_t* wfull = ffull + kMaxBlk;      // [ring] window landed (leader: both CTAs' windows)
   uint64_t* wempty = wfull + 8;           // [ring] window consumed (both CTAs, MMA commit)
   uint64_t* tfull = wempty + 8;           // [2] accumulator ready (both CTAs, MMA commit)
   uint64_t* tempty = tfull + 2;           // [2] accumulator drained (leader: 16 epilogue warps)
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
-  uint32_t* mtab = tmem_slot + 4;  // [kMaxBlk][2]: per rotated tap, A shift and B offset (16-byte units)
+  uint32_t* mtab = tmem_slot + 4;  // [kMaxBlk][2]: per tap, A shift and B offset (16-byte units)
+  uint64_t* pbar = reinterpret_cast<uint64_t*>(mtab + 2 * kMaxBlk);  // pack: x band landed
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t rank = cluster_ctarank();
@@ -317,16 +433,41 @@ __global__ void __launch_bounds__(kPairThreads, 1)
       mbar_init(tfull + s, 1);
       mbar_init(tempty + s, 2 * 8);
     }
+    mbar_init(pbar, 1);
     fence_barrier_init();
   }
   if (warp == 1) tmem_alloc2(tmem_slot, (uint32_t)p.tmem_cols);
+  __syncthreads();  // pbar initialised
 
   // phase 1: packing (all warps); the window ring and filter area are the staging buffer
-  if (!(p.dbg & 2)) pair_pack<IoT>(p, reinterpret_cast<uint16_t*>(sF));  // dbg&2: skip (timing only)
+  if (!(p.dbg & 2)) {  // dbg&2: skip the packing (timing experiments only)
+    if (p.pack_tma) {
+      // the first band's input load flies while the filter is packed
+      const bool first = (int)blockIdx.x < p.nunits;
+      bool issued = false;
+      if (threadIdx.x == 0 && first) {
+        const int n = (int)blockIdx.x / p.nb, b = (int)blockIdx.x - n * p.nb;
+        const int r0 = b * p.rb, r1 = min(p.Hp, r0 + p.rb);
+        const int h0 = min(max(r0 - p.ph, 0), p.H), h1 = min(max(r1 - p.ph, 0), p.H);
+        if (h1 > h0) {
+          prefetch_tmap(&tmX);
+          mbar_arrive_expect_tx(pbar, p.C * p.ne_box * (uint32_t)sizeof(IoT));
+          // a TMA box must start 16-byte aligned in global memory: round down
+          tma_load_2d(sF, &tmX, pbar, (h0 * p.W) & ~(16 / (int)sizeof(IoT) - 1), n * p.C);
+        }
+      }
+      issued = first;
+      pair_pack<IoT>(p, nullptr, false);
+      pair_pack_x_tma<IoT>(p, sF, pbar, &tmX, &tmS, &tmS2, issued);
+    } else {
+      pair_pack<IoT>(p, reinterpret_cast<uint16_t*>(sF), true);
+    }
+  }
   // the staging area is overwritten by TMA (async proxy) next
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
   __syncthreads();
   if (threadIdx.x == 0) {
+    asm volatile("fence.proxy.async.global;" ::: "memory");  // TMA-stored A -> generic release
     __threadfence();
     atomicAdd(p.fcount, 1ull);
   }
@@ -369,11 +510,15 @@ __global__ void __launch_bounds__(kPairThreads, 1)
     __syncwarp();
     int wi = 0, lt = 0;
     for (int t = pair; t < p.num_tiles; t += p.num_pairs, ++lt) {
-      const int g0 = t * (2 * kTileM) + (int)rank * kTileM;
+      // CTA tile 2t + rank = output rows [blk*tr, blk*tr + tr) of image n; its positions
+      // start at coefficient n*L_A + blk*tr*sh*Wp (Eq. 12 base of output (blk*tr, 0))
+      const int ct = 2 * t + (int)rank;
+      const int tn = (int)p.ftpi.div((uint32_t)ct), tb = ct - tn * p.tpi;
+      const int g0 = tn * (int)p.L_A + tb * p.tr * p.sh * p.Wp;
       for (int ci = 0; ci < p.nchunks; ++ci, ++wi) {
-        // every pair walks the (chunk, tap) blocks in its own rotated order, so
-        // that the 148 CTAs do not all stream the same filter lines at once
-        const int ch = (ci + pair) % p.nchunks;
+        // one fixed (chunk, tap) order everywhere: every output sees the same
+        // accumulation order whatever tile or batch it is computed in (reading R12)
+        const int ch = ci;
         const int slot = wi % p.ring;
         mbar_wait_cl(wempty + slot, (uint32_t)((wi / p.ring) & 1) ^ 1u, (p.dbg & 16) ? 500u : 0u);
         if (elect_one()) {
@@ -383,7 +528,7 @@ __global__ void __launch_bounds__(kPairThreads, 1)
                              lead_wfull + 8u * (uint32_t)slot, ch * p.kc, g0 + b * p.box_rows);
           if (lt == 0 && !(p.dbg & 1)) {  // the filter blocks of this chunk: loaded once, resident
             for (int ti = 0; ti < p.RS; ++ti) {
-              const int tap = (ti + pair) % p.RS;
+              const int tap = ti;
               const int blk = ch * p.RS + tap;
               if (rank == 0) mbar_arrive_expect_tx(ffull + blk, 2u * p.fbytes);
               tma_load_2d_pair(sF0 + (uint32_t)blk * p.fbytes, &tmU, lead_ffull + 8u * (uint32_t)blk, ch * p.kc,
@@ -400,10 +545,10 @@ __global__ void __launch_bounds__(kPairThreads, 1)
     if (rank == 0) {
       const uint32_t sW0 = smem_u32(sWin), sF0 = smem_u32(sF);
       const int ksteps = p.row_bytes / 32;
-      // descriptor offsets of the pair's rotated tap order, so that the issue loop
-      // is a few uniform adds per tap (divisions in it left the tensor pipe idle)
+      // descriptor offsets per tap, so that the issue loop is a few uniform adds
+      // per tap (divisions in it left the tensor pipe idle)
       for (int ti = lane; ti < p.RS; ti += 32) {
-        const int tap = (ti + pair) % p.RS;
+        const int tap = ti;
         const int i = tap / p.S, j = tap - (tap / p.S) * p.S;
         mtab[2 * ti] = ((uint32_t)(p.Wp * i + j) * (uint32_t)p.row_bytes) >> 4;
         mtab[2 * ti + 1] = ((uint32_t)tap * p.fbytes) >> 4;
@@ -416,7 +561,7 @@ __global__ void __launch_bounds__(kPairThreads, 1)
         tc_fence_after();
         const uint32_t d_tmem = tmem_base + (uint32_t)(a * p.NN);
         for (int ci = 0; ci < p.nchunks; ++ci, ++wi) {
-          const int ch = (ci + pair) % p.nchunks;  // the producer's rotated order
+          const int ch = ci;  // the producer's order
           const int slot = wi % p.ring;
           if (!(p.dbg & 4)) mbar_wait_cl(wfull + slot, (uint32_t)((wi / p.ring) & 1));
           tc_fence_after();
@@ -457,49 +602,69 @@ __global__ void __launch_bounds__(kPairThreads, 1)
     const int h = e >> 2;         // channel half
     const int half = p.NN / 2;
     const uint32_t lead_tempty = mapa_rank0(smem_u32(tempty));
-    IoT* y = static_cast<IoT*>(p.y);
     int lt = 0;
     for (int t = pair; t < p.num_tiles; t += p.num_pairs, ++lt) {
       const int a = lt & 1;
       mbar_wait_cl(tfull + a, (uint32_t)((lt >> 1) & 1), (p.dbg & 16) ? 1000u : 64u);
       tc_fence_after();
       if (trace && threadIdx.x == kEpi0 * 32 && lt < 2) tr[9 + 2 * lt] = global_ns();
-      // this lane's position -> output pixel (Eq. 12 with stride, reading R4)
-      const long long gpos = (long long)t * (2 * kTileM) + rank * kTileM + q * 32 + lane;
-      long long base = -1;
-      if (gpos < p.G) {
-        const int n = (int)p.fLA.div((uint32_t)gpos);
-        const int rem = (int)(gpos - (long long)n * p.L_A);
-        const int r = (int)p.fWp.div((uint32_t)rem), s = rem - r * p.Wp;
-        const int oh = (int)p.fsh.div((uint32_t)r), ow = (int)p.fsw.div((uint32_t)s);
-        if (oh * p.sh == r && ow * p.sw == s && oh < p.P && ow < p.Q)
-          base = (long long)n * p.K * p.PQ + (long long)oh * p.Q + ow;
-      }
+      // this lane's position m (tile-relative coefficient) -> output pixel (Eq. 12 with
+      // stride, reading R4): row r = m / Wp, column s; valid on the stride lattice
+      const int ct = 2 * t + (int)rank;
+      const int tn = (int)p.ftpi.div((uint32_t)ct), tb = ct - tn * p.tpi;
+      const int m = q * 32 + lane;
+      const int r = (int)p.fWp.div((uint32_t)m), sc = m - r * p.Wp;
+      const int ohr = (int)p.fsh.div((uint32_t)r), ow = (int)p.fsw.div((uint32_t)sc);
+      const bool valid = ct < p.ntile && ohr * p.sh == r && ow * p.sw == sc && ohr < p.tr &&
+                         tb * p.tr + ohr < p.P && ow < p.Q;
+      const int j = ohr * p.Q + ow;  // pixel within the tile's run [tb*tr*Q, (tb*tr + tr)*Q)
       const uint32_t taddr = tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)(a * p.NN + h * half);
-      for (int cc = 0; cc < half; cc += 32) {
-        uint32_t v[32];
-        tmem_ld32(taddr + (uint32_t)cc, v);
-        tmem_ld_wait();
-        if (cc + 32 >= half) {  // every TMEM read of this accumulator done: release it
-          tc_fence_before();
-          __syncwarp();
-          if (lane == 0) mbar_arrive_remote(lead_tempty + 8u * (uint32_t)a);
-        }
-        const int k0 = h * half + cc;
-        if (base >= 0) {
+      uint32_t v[64];
+      tmem_ld32(taddr, *reinterpret_cast<uint32_t(*)[32]>(&v[0]));
+      if (half > 32) tmem_ld32(taddr + 32u, *reinterpret_cast<uint32_t(*)[32]>(&v[32]));
+      tmem_ld_wait();
+      tc_fence_before();  // every TMEM read of this accumulator done: release it
+      __syncwarp();
+      if (lane == 0) mbar_arrive_remote(lead_tempty + 8u * (uint32_t)a);
+      if (p.epi_tma) {
+        // stage this half's channels [64][tr*Q] (bf16), then one thread stores the
+        // 32-channel boxes; the staging is free once the previous stores were read
+        const int trq = p.tr * p.Q;
+        __nv_bfloat16* st = reinterpret_cast<__nv_bfloat16*>(sEpi) + (size_t)h * half * trq;
+        const bool issuer = (e & 3) == 0 && lane == 0;
+        if (issuer) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+        asm volatile("bar.sync %0, 128;" ::"r"(1 + h) : "memory");
+        if (valid) {
 #pragma unroll
-          for (int jj = 0; jj < 32; ++jj) {
-            const int k = k0 + jj;
-            if (k < p.K) {
-              const float f = __uint_as_float(v[jj]);
-              if constexpr (std::is_same<IoT, float>::value) y[base + (long long)k * p.PQ] = f;
-              else y[base + (long long)k * p.PQ] = __float2bfloat16_rn(f);
-            }
+          for (int jj = 0; jj < 64; ++jj)
+            if (jj < half) st[jj * trq + j] = __float2bfloat16_rn(__uint_as_float(v[jj]));
+        }
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        asm volatile("bar.sync %0, 128;" ::"r"(1 + h) : "memory");
+        if (issuer && ct < p.ntile) {
+          for (int b = 0; b < half / 32; ++b) {
+            const int k0 = h * half + b * 32;
+            if (k0 >= p.K) break;
+            tma_store_2d(&tmY, smem_u32(st + (size_t)b * 32 * trq), tb * trq, tn * p.K + k0);
+          }
+          asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+        }
+      } else if (valid) {
+        IoT* y = static_cast<IoT*>(p.y);
+        const long long base = (long long)tn * p.K * p.PQ + (long long)(tb * p.tr + ohr) * p.Q + ow;
+#pragma unroll
+        for (int jj = 0; jj < 64; ++jj) {
+          const int k = h * half + jj;
+          if (jj < half && k < p.K) {
+            const float f = __uint_as_float(v[jj]);
+            if constexpr (std::is_same<IoT, float>::value) y[base + (long long)k * p.PQ] = f;
+            else y[base + (long long)k * p.PQ] = __float2bfloat16_rn(f);
           }
         }
       }
       if (trace && threadIdx.x == kEpi0 * 32 && lt < 2) tr[10 + 2 * lt] = global_ns();
     }
+    if (p.epi_tma && (e & 3) == 0 && lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
   }
 
   tc_fence_before();
@@ -555,11 +720,11 @@ inline long long cdivp(long long a, long long b) { return (a + b - 1) / b; }
 
 }  // namespace
 
-PairTiling pair_tiling(const Geom& g, int fmt, int num_sms) {
+PairTiling pair_tiling(const Geom& g, int fmt, bool io_bf16, int num_sms) {
   PairTiling t{};
   t.ok = false;
   if (fmt != FMT_BF16) return t;
-  if (g.K > 256) return t;
+  if (g.K > 128) return t;  // one output-channel tile of NN <= 128 (64 per CTA of the pair)
   t.kc = g.C >= 64 ? 64 : (g.C >= 32 ? 32 : 16);
   t.row_bytes = t.kc * 2;
   t.Cp = (int)cdivp(g.C, t.kc) * t.kc;
@@ -581,21 +746,38 @@ PairTiling pair_tiling(const Geom& g, int fmt, int num_sms) {
   t.wbytes_tx = t.nbox * t.box_rows * t.row_bytes;
   t.fbytes = t.NN / 2 * t.row_bytes;
   const long long fil = (long long)t.nblk * t.fbytes;
+  // row-aligned tiles: tr output rows of one image per CTA tile, every valid output
+  // inside the 128 TMEM lanes: (tr-1)*sh*Wp + (Q-1)*sw + 1 <= 128
+  if ((long long)(g.Q - 1) * g.sw + 1 > kTileM) return t;
+  t.tr = 1;
+  while ((long long)t.tr * g.sh * g.Wp + (long long)(g.Q - 1) * g.sw + 1 <= kTileM && t.tr < g.P) ++t.tr;
+  t.tpi = (int)cdivp(g.P, t.tr);
+  if ((long long)g.N * t.tpi >= (1LL << 30)) return t;
+  t.ntile = g.N * t.tpi;
+  // epilogue by TMA stores: y viewed as [N*K][P*Q] bf16, boxes of tr*Q pixels x 32 channels
+  const long long trq = (long long)t.tr * g.Q;
+  t.epi_tma = io_bf16 && g.K % 32 == 0 && (trq * 2) % 16 == 0 && ((long long)g.P * g.Q * 2) % 16 == 0 &&
+              trq <= 256 && !getenv("POLYCONV_PAIR_EPI_ST");
+  t.estage_bytes = t.epi_tma ? (int)(cdivp((long long)t.NN * trq * 2, 1024) * 1024) : 0;
   const long long budget = 227LL * 1024 - 1024 - 2048;  // alignment slack, barriers + tap table
-  const long long left = budget - fil;
-  if (left < 2LL * t.wbytes) return t;
-  t.ring = (int)std::min(4LL, left / t.wbytes);
-  t.smem_bytes = (int)(1024 + fil + (long long)t.ring * t.wbytes + 2048);
+  const long long left = budget - fil - t.estage_bytes;
+  if (left < 2LL * t.wbytes) {
+    if (!t.epi_tma) return t;
+    t.epi_tma = 0;  // no room to stage the epilogue: direct stores
+    t.estage_bytes = 0;
+    if (budget - fil < 2LL * t.wbytes) return t;
+  }
+  t.ring = (int)std::min(4LL, (budget - fil - t.estage_bytes) / t.wbytes);
+  t.smem_bytes = (int)(1024 + fil + (long long)t.ring * t.wbytes + t.estage_bytes + 2048);
   t.tmem_cols = 64;
   while (t.tmem_cols < 2 * t.NN) t.tmem_cols *= 2;
   if (t.tmem_cols > 512) return t;
-  const long long G = (long long)(g.N - 1) * g.L_A + g.M_ext;
   if ((long long)g.N * g.L_A + 4096 >= (1LL << 31)) return t;  // 32-bit TMA row coordinates / decode
-  t.num_tiles = (int)cdivp(G, 2 * kTileM);
+  t.num_tiles = (int)cdivp(t.ntile, 2);
   t.num_pairs = std::min(t.num_tiles, num_sms / 2);
   t.grid = 2 * t.num_pairs;
   // packing bands: about one band per CTA, staged in the (then unused) operand area
-  const long long stage_cap = fil + (long long)t.ring * t.wbytes;
+  const long long stage_cap = fil + (long long)t.ring * t.wbytes + t.estage_bytes;
   t.nb = std::max(1, t.grid / g.N);
   if (t.nb > g.Hp) t.nb = g.Hp;
   for (;;) {
@@ -607,6 +789,37 @@ PairTiling pair_tiling(const Geom& g, int fmt, int num_sms) {
   if ((long long)t.Cp * t.spitch * 2 > stage_cap) return t;
   t.nb = (int)cdivp(g.Hp, t.rb);
   t.nunits = g.N * t.nb;
+  // TMA pack path: x band by one TMA box, A rows out by TMA stores (64-channel SW128 boxes)
+  t.pack_tma = 0;
+  {
+    const int eb_in = io_bf16 ? 2 : 4;
+    const int ve = 16 / eb_in;
+    int nb2 = std::max(1, t.grid / g.N);
+    if (nb2 > g.Hp) nb2 = g.Hp;
+    int rb2 = (int)cdivp(g.Hp, nb2);
+    const int rb_cap = std::min(256 / g.Wp, 256 / g.W);
+    if (rb2 > rb_cap) rb2 = rb_cap;
+    if (rb2 >= 1 && t.Cp % 64 == 0 && g.C <= 256 && ((long long)g.H * g.W * eb_in) % 16 == 0 &&
+        !getenv("POLYCONV_PAIR_PACK_LD")) {
+      const int nbb = (int)cdivp(g.Hp, rb2);
+      const int last = g.Hp - (nbb - 1) * rb2;
+      const int ne_box = (int)cdivp((long long)rb2 * g.W + ve - 1, ve) * ve;  // + the start's rounding
+      const long long in_b = cdivp((long long)g.C * ne_box * eb_in, 1024) * 1024;
+      const long long ob = cdivp((long long)rb2 * g.Wp * 128, 1024) * 1024;
+      const long long ob2 = cdivp((long long)last * g.Wp * 128, 1024) * 1024;
+      if (ne_box <= 256 && in_b + (long long)(t.Cp / 64) * ob <= stage_cap) {
+        t.pack_tma = 1;
+        t.rb = rb2;
+        t.nb = nbb;
+        t.nunits = g.N * nbb;
+        t.last_rows = last;
+        t.ne_box = ne_box;
+        t.in_bytes = (int)in_b;
+        t.obox_bytes = (int)ob;
+        t.obox_bytes2 = (int)ob2;
+      }
+    }
+  }
   t.ok = true;
   return t;
 }
@@ -624,8 +837,50 @@ cudaError_t launch_mac_pair(const Geom& g, const PairTiling& t, const void* x, c
     snprintf(err, errlen, "mac_pair: cuTensorMapEncodeTiled failed");
     return cudaErrorInvalidValue;
   }
+  CUtensorMap tmX, tmS, tmS2;
+  memset(&tmX, 0, sizeof(tmX));
+  memset(&tmS, 0, sizeof(tmS));
+  memset(&tmS2, 0, sizeof(tmS2));
+  if (t.pack_tma) {
+    EncodeTiledFnPair enc = get_encode_pair();
+    const int eb_in = io_bf16 ? 2 : 4;
+    cuuint64_t dims[2] = {(cuuint64_t)g.H * g.W, (cuuint64_t)g.N * g.C};
+    cuuint64_t strides[1] = {(cuuint64_t)g.H * g.W * eb_in};
+    cuuint32_t box[2] = {(cuuint32_t)t.ne_box, (cuuint32_t)g.C};
+    cuuint32_t estr[2] = {1, 1};
+    bool ok = enc && enc(&tmX, io_bf16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2,
+                         const_cast<void*>(x), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                         CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                         CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+    ok = ok && encode_bf16(&tmS, A, (uint64_t)t.Cp, (uint64_t)g.N * g.L_A, 64, (uint32_t)(t.rb * g.Wp)) &&
+         encode_bf16(&tmS2, A, (uint64_t)t.Cp, (uint64_t)g.N * g.L_A, 64, (uint32_t)(t.last_rows * g.Wp));
+    if (!ok) {
+      snprintf(err, errlen, "mac_pair: cuTensorMapEncodeTiled (pack) failed");
+      return cudaErrorInvalidValue;
+    }
+  }
+  CUtensorMap tmY;
+  memset(&tmY, 0, sizeof(tmY));
+  if (t.epi_tma) {
+    EncodeTiledFnPair enc = get_encode_pair();
+    cuuint64_t dims[2] = {(cuuint64_t)g.P * g.Q, (cuuint64_t)g.N * g.K};
+    cuuint64_t strides[1] = {(cuuint64_t)g.P * g.Q * 2};
+    cuuint32_t box[2] = {(cuuint32_t)(t.tr * g.Q), 32};
+    cuuint32_t estr[2] = {1, 1};
+    if (!enc || enc(&tmY, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, y, dims, strides, box, estr,
+                    CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_NONE,
+                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS) {
+      snprintf(err, errlen, "mac_pair: cuTensorMapEncodeTiled (output) failed");
+      return cudaErrorInvalidValue;
+    }
+  }
   PairParams p{};
   p.x = x; p.w = w; p.A = A; p.U = U; p.y = y;
+  p.tr = t.tr; p.tpi = t.tpi; p.ntile = t.ntile; p.epi_tma = t.epi_tma;
+  p.estage_bytes = (uint32_t)t.estage_bytes;
+  p.ftpi.init((uint32_t)t.tpi);
+  p.pack_tma = t.pack_tma; p.ne_box = t.ne_box; p.last_rows = t.last_rows;
+  p.in_bytes = (uint32_t)t.in_bytes; p.obox_bytes = (uint32_t)t.obox_bytes; p.obox_bytes2 = (uint32_t)t.obox_bytes2;
   p.fcount = fcount; p.ftarget = ftarget;
   p.L_A = g.L_A;
   p.G = (long long)(g.N - 1) * g.L_A + g.M_ext;
@@ -670,13 +925,16 @@ cudaError_t launch_mac_pair(const Geom& g, const PairTiling& t, const void* x, c
     return cudaErrorInvalidConfiguration;
   }
   cudaGetLastError();
-  return cudaLaunchKernelEx(&cfg, kern, tmA, tmU, p);
+  return cudaLaunchKernelEx(&cfg, kern, tmA, tmU, tmX, tmS, tmS2, tmY, p);
 }
 
 }  // namespace polyconv
 
 // Debug only (not part of include/polyconv.h): the per-CTA phase trace of the
 // last POLYCONV_PAIR_DEBUG&8 launch (160 x 16 u64).
+extern "C" int polyconv_dbg_pair_pk(unsigned long long* host) {
+  return (int)cudaMemcpyFromSymbol(host, polyconv::g_pair_pk, sizeof(unsigned long long) * 160 * 4);
+}
 extern "C" int polyconv_dbg_pair_clk(unsigned long long* host) {
   return (int)cudaMemcpyFromSymbol(host, polyconv::g_pair_clk, sizeof(unsigned long long) * 160 * 2);
 }

@@ -59,7 +59,7 @@ polyconv_status_t resolve(polyconv_plan_t p) {
   Geom& g = p->g;
   int k = p->forced;
   const bool tc_math = p->math != POLYCONV_MATH_FP32_FMA;
-  if (k == POLYCONV_KERNEL_AUTO || k == POLYCONV_KERNEL_TC_PAIR) p->pair = pair_tiling(g, p->fmt, p->num_sms);
+  if (k == POLYCONV_KERNEL_AUTO || k == POLYCONV_KERNEL_TC_PAIR) p->pair = pair_tiling(g, p->fmt, p->io_bf16, p->num_sms);
   if (k == POLYCONV_KERNEL_AUTO) {
     if (tc_math && g.K >= 16 && p->pair.ok && !getenv("POLYCONV_NO_PAIR_DEFAULT"))
       k = POLYCONV_KERNEL_TC_PAIR;  // bf16: one launch, CTA pairs, resident filter

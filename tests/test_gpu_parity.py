@@ -38,8 +38,8 @@ SHAPES = [
 def _skip_unsupported(shape, math, kernel):
     if kernel == "fp32" and max(shape.R, shape.S) > 7:
         pytest.skip("fp32 kernel limited to S<=7")
-    if kernel == "tc_pair" and shape.K > 256:
-        pytest.skip("tc_pair: one output-channel tile (K <= 256)")
+    if kernel == "tc_pair" and (shape.K > 128 or (shape.Q - 1) * shape.stride[1] + 1 > 128):
+        pytest.skip("tc_pair: one output-channel tile (K <= 128), an output row within 128 positions")
 
 
 @pytest.mark.parametrize("shape", SHAPES, ids=lambda s: s.name)

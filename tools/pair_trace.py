@@ -42,3 +42,13 @@ c = np.array(clk, dtype=np.float64).reshape(160, 2)[: len(a)]
 raw = np.array(buf, dtype=np.float64).reshape(160, 16)[: len(a)]
 mhz = (c[:, 1] - c[:, 0]) / (raw[:, 13] - raw[:, 0]) * 1e3
 print("  SM clock during the kernel: med %.0f MHz (min %.0f, max %.0f)" % (np.median(mhz), mhz.min(), mhz.max()))
+
+pk = (ctypes.c_ulonglong * (160 * 4))()
+lib.polyconv_dbg_pair_pk(pk)
+k = np.array(pk, dtype=np.float64).reshape(160, 4)[: len(a)]
+for col, nm in enumerate(["pk_filter_done", "pk_band_staged", "pk_band_written", "pk_band_gathered"]):
+    v = k[:, col]
+    v = v[v > 0]
+    if len(v):
+        rel = (v - t0) / 1e3
+        print("  %-16s n=%3d min %7.2f  med %7.2f  max %7.2f us" % (nm, len(v), rel.min(), np.median(rel), rel.max()))
