@@ -129,8 +129,14 @@ struct PairTiling {
 PairTiling pair_tiling(const Geom& g, int fmt, bool io_bf16, int num_sms);
 // One launch: packs w -> U [R*S][NN][Cp] and x -> A [N*L_A][Cp] (bf16, plan workspace),
 // meets on *fcount (must reach ftarget = launches so far x t.grid), then the pair MAC.
+// fcount: filter-slice counter (ftarget = launches so far x t.grid); bflag: [N*t.nb] band
+// flags (zeroed once; band u is published as `epoch` = launches so far); state: launch
+// cache from pair_state_new() (tensor maps + parameters per pointer set), or nullptr
 cudaError_t launch_mac_pair(const Geom& g, const PairTiling& t, const void* x, const void* w, bool io_bf16,
                             void* A, void* U, void* y, unsigned long long* fcount, unsigned long long ftarget,
-                            cudaStream_t st, char* err, size_t errlen);
+                            unsigned long long* bflag, unsigned long long epoch, cudaStream_t st, char* err,
+                            size_t errlen, void* state);
+void* pair_state_new();
+void pair_state_free(void* s);
 
 }  // namespace polyconv

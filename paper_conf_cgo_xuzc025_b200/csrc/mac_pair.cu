@@ -42,6 +42,7 @@
 #include <cstring>
 #include <algorithm>
 #include <type_traits>
+#include <new>
 #include "common.cuh"
 #include "sm100.cuh"
 
@@ -62,8 +63,10 @@ struct PairParams {
   void* A;  // interleaved input polynomial [N*L_A][Cp] bf16 (plan workspace)
   void* U;  // tap-major filter [R*S][NN][Cp] bf16 (plan workspace)
   void* y;
-  unsigned long long* fcount;
+  unsigned long long* fcount;   // filter slices packed (all CTAs): reaches ftarget
   unsigned long long ftarget;
+  unsigned long long* bflag;    // [N*nb] band u of A written in launch epoch
+  unsigned long long epoch;
   long long L_A, G, NLA;
   int N, C, H, W, K, R, S, sh, sw, ph, pw, Hp, Wp, P, Q, PQ;
   int Cp, NN, kc, row_bytes, nchunks, RS, nblk;
@@ -183,17 +186,31 @@ __device__ __forceinline__ void pair_pack(const PairParams& p, uint16_t* stg, bo
   const int tid = threadIdx.x;
   const int nth = blockDim.x;
   const bool ptr = (p.dbg & 8) && blockIdx.x < 160 && tid == 0;
-  // a3: U[tap][k][c] = w[k][c][tap] (tap = i*S + j; k >= K or c >= C: 0)
+  // a3: U[tap][k][c] = w[k][c][tap] (tap = i*S + j; k >= K or c >= C: 0).  One flat
+  // pass over U spread over every thread of the grid (consecutive threads write
+  // consecutive channels), four loads in flight per thread
   {
     const IoT* w = static_cast<const IoT*>(p.w);
     uint16_t* U = static_cast<uint16_t*>(p.U);
-    const int nkc = p.NN * p.Cp;
-    for (int idx = blockIdx.x * nth + tid; idx < nkc; idx += gridDim.x * nth) {
-      const int k = idx / p.Cp, c = idx - (idx / p.Cp) * p.Cp;
-      const bool ok = k < p.K && c < p.C;
-      const IoT* src = w + ((long long)k * p.C + c) * p.RS;
-      for (int t = 0; t < p.RS; ++t)
-        U[((long long)t * p.NN + k) * p.Cp + c] = ok ? to_bf16_bits<IoT>(src[t]) : (uint16_t)0;
+    const int total = p.RS * p.NN * p.Cp;
+    const int stride = gridDim.x * nth;
+    for (int base = blockIdx.x * nth + tid; base < total; base += 4 * stride) {
+      uint16_t v[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const int idx = base + u * stride;
+        v[u] = 0;
+        if (idx < total) {
+          const int c = idx % p.Cp, tk = idx / p.Cp;
+          const int k = tk % p.NN, tap = tk / p.NN;
+          if (k < p.K && c < p.C) v[u] = to_bf16_bits<IoT>(w[((long long)k * p.C + c) * p.RS + tap]);
+        }
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const int idx = base + u * stride;
+        if (idx < total) U[idx] = v[u];
+      }
     }
   }
   if (ptr) g_pair_pk[blockIdx.x * 4] = global_ns();
@@ -308,6 +325,29 @@ __device__ __forceinline__ void tma_store_2d(const void* tmap, uint32_t src, int
                : "memory");
 }
 
+// Publish band u of this launch (epoch): its A rows are in global memory.
+__device__ __forceinline__ void publish_band(const PairParams& p, int u) {
+  asm volatile("fence.proxy.async.global;" ::: "memory");  // TMA-stored rows -> generic release
+  __threadfence();
+  asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p.bflag + u), "l"(p.epoch) : "memory");
+}
+
+// x-box bx (64 channel planes) of the band of unit u: TMA load, 16-byte aligned start
+template <typename IoT>
+__device__ __forceinline__ void pack_load(const PairParams& p, const CUtensorMap* tmX, uint8_t* stage,
+                                          uint64_t* pbar, int u, int bx) {
+  const int n = u / p.nb, b = u - (u / p.nb) * p.nb;
+  const int r0 = b * p.rb;
+  const int h0 = min(max(r0 - p.ph, 0), p.H);
+  const uint32_t bytes = 64u * p.ne_box * (uint32_t)sizeof(IoT);
+  mbar_arrive_expect_tx(pbar + bx, bytes);
+  tma_load_2d(stage + (size_t)bx * bytes, tmX, pbar + bx, (h0 * p.W) & ~(16 / (int)sizeof(IoT) - 1),
+              n * p.C + bx * 64);
+}
+
+// band units of this CTA: x boxes of 64 channel planes in by TMA (the first unit's
+// already issued), each transposed into its 128-byte swizzled box of A rows and
+// stored by TMA as soon as it is done, then the band is published.
 template <typename IoT>
 __device__ __forceinline__ void pair_pack_x_tma(const PairParams& p, uint8_t* stage, uint64_t* pbar,
                                                 const CUtensorMap* tmX, const CUtensorMap* tmS,
@@ -315,77 +355,78 @@ __device__ __forceinline__ void pair_pack_x_tma(const PairParams& p, uint8_t* st
   const int tid = threadIdx.x;
   const int nth = blockDim.x;
   const bool ptr = (p.dbg & 8) && blockIdx.x < 160 && tid == 0;
-  const IoT* in = reinterpret_cast<const IoT*>(stage);
+  const int nbx = p.Cp / 64;
+  const uint32_t xbox = 64u * p.ne_box * (uint32_t)sizeof(IoT);
   uint8_t* out = stage + p.in_bytes;
   int it = 0;
   for (int u = blockIdx.x; u < p.nunits; u += gridDim.x, ++it) {
     const int n = u / p.nb, b = u - (u / p.nb) * p.nb;
     const int r0 = b * p.rb, r1 = min(p.Hp, r0 + p.rb);
     const int h0 = min(max(r0 - p.ph, 0), p.H), h1 = min(max(r1 - p.ph, 0), p.H);
-    const bool any = h1 > h0;
-    if (tid == 0 && any && !(it == 0 && first_issued)) {
-      mbar_arrive_expect_tx(pbar, p.C * p.ne_box * (uint32_t)sizeof(IoT));
-      tma_load_2d(stage, tmX, pbar, (h0 * p.W) & ~(16 / (int)sizeof(IoT) - 1), n * p.C);
-    }
-    if (any) mbar_wait(pbar, (uint32_t)(it & 1));
-    if (ptr) g_pair_pk[blockIdx.x * 4 + 1] = global_ns();
+    const bool any = h1 > h0 && !(p.dbg & 2);
+    if (tid == 0 && any && !(it == 0 && first_issued))
+      for (int bx = 0; bx < nbx; ++bx) pack_load<IoT>(p, tmX, stage, pbar, u, bx);
     const int npos = (r1 - r0) * p.Wp;
-    FastDiv fnp;
-    fnp.init((uint32_t)npos);
     const uint32_t obox = (r1 - r0 == p.rb) ? p.obox_bytes : p.obox_bytes2;
-    const int nbx = p.Cp / 64;
     const int eoff = (h0 * p.W) & (16 / (int)sizeof(IoT) - 1);  // the box starts at h0*W rounded down
-    // one item = one position's 64 channels = one 128-byte row of box bx; consecutive
-    // threads take consecutive positions (conflict-free staging reads and swizzled writes)
-    for (int idx = tid; idx < nbx * npos; idx += nth) {
-      const int bx = (int)fnp.div((uint32_t)idx), pos = idx - bx * npos;
-      const int rr = (int)p.fWp.div((uint32_t)pos);
-      const int h = r0 + rr - p.ph, ww = pos - rr * p.Wp - p.pw;
-      uint8_t* drow = out + (size_t)bx * obox + (size_t)pos * 128;
-      const uint32_t sw = (uint32_t)(pos & 7);
-      if (h >= 0 && h < p.H && ww >= 0 && ww < p.W) {
-        const IoT* src = in + (size_t)(bx * 64) * p.ne_box + (h - h0) * p.W + ww + eoff;
-        const int cbase = bx * 64;
+    const CUtensorMap* m = (r1 - r0 == p.rb) ? tmS : tmS2;
+    for (int bx = 0; bx < nbx; ++bx) {
+      if (any) mbar_wait(pbar + bx, (uint32_t)(it & 1));
+      if (ptr && bx == 0) g_pair_pk[blockIdx.x * 4 + 1] = global_ns();
+      const IoT* in = reinterpret_cast<const IoT*>(stage + (size_t)bx * xbox);
+      uint8_t* dbox = out + (size_t)bx * obox;
+      const int cbase = bx * 64;
+      // one item = one position's 64 channels = one 128-byte row of the box; consecutive
+      // threads take consecutive positions (conflict-free staging reads, swizzled writes)
+      for (int pos = tid; pos < npos; pos += nth) {
+        const int rr = (int)p.fWp.div((uint32_t)pos);
+        const int h = r0 + rr - p.ph, ww = pos - rr * p.Wp - p.pw;
+        uint8_t* drow = dbox + (size_t)pos * 128;
+        const uint32_t sw = (uint32_t)(pos & 7);
+        if (any && h >= 0 && h < p.H && ww >= 0 && ww < p.W) {
+          const IoT* src = in + (h - h0) * p.W + ww + eoff;
 #pragma unroll
-        for (int q8 = 0; q8 < 8; ++q8) {
-          const int c0 = cbase + q8 * 8;
-          uint32_t v[4];
-          if (c0 + 8 <= p.C) {
-            uint32_t hv[8];
+          for (int q8 = 0; q8 < 8; ++q8) {
+            const int c0 = cbase + q8 * 8;
+            uint32_t v[4];
+            if (c0 + 8 <= p.C) {
+              uint32_t hv[8];
 #pragma unroll
-            for (int k = 0; k < 8; ++k) hv[k] = to_bf16_bits<IoT>(src[(q8 * 8 + k) * p.ne_box]);
+              for (int k = 0; k < 8; ++k) hv[k] = to_bf16_bits<IoT>(src[(q8 * 8 + k) * p.ne_box]);
 #pragma unroll
-            for (int m = 0; m < 4; ++m) v[m] = hv[2 * m] | (hv[2 * m + 1] << 16);
-          } else {
+              for (int mm = 0; mm < 4; ++mm) v[mm] = hv[2 * mm] | (hv[2 * mm + 1] << 16);
+            } else {
 #pragma unroll
-            for (int m = 0; m < 4; ++m) {
-              const int c = c0 + 2 * m;
-              const uint32_t lo = c < p.C ? (uint32_t)to_bf16_bits<IoT>(src[(q8 * 8 + 2 * m) * p.ne_box]) : 0u;
-              const uint32_t hi =
-                  c + 1 < p.C ? (uint32_t)to_bf16_bits<IoT>(src[(q8 * 8 + 2 * m + 1) * p.ne_box]) : 0u;
-              v[m] = lo | (hi << 16);
+              for (int mm = 0; mm < 4; ++mm) {
+                const int c = c0 + 2 * mm;
+                const uint32_t lo = c < p.C ? (uint32_t)to_bf16_bits<IoT>(src[(q8 * 8 + 2 * mm) * p.ne_box]) : 0u;
+                const uint32_t hi =
+                    c + 1 < p.C ? (uint32_t)to_bf16_bits<IoT>(src[(q8 * 8 + 2 * mm + 1) * p.ne_box]) : 0u;
+                v[mm] = lo | (hi << 16);
+              }
             }
+            *reinterpret_cast<uint4*>(drow + (((uint32_t)q8 ^ sw) << 4)) = make_uint4(v[0], v[1], v[2], v[3]);
           }
-          *reinterpret_cast<uint4*>(drow + (((uint32_t)q8 ^ sw) << 4)) = make_uint4(v[0], v[1], v[2], v[3]);
-        }
-      } else {
+        } else {
 #pragma unroll
-        for (int q8 = 0; q8 < 8; ++q8)
-          *reinterpret_cast<uint4*>(drow + (((uint32_t)q8 ^ sw) << 4)) = make_uint4(0u, 0u, 0u, 0u);
+          for (int q8 = 0; q8 < 8; ++q8)
+            *reinterpret_cast<uint4*>(drow + (((uint32_t)q8 ^ sw) << 4)) = make_uint4(0u, 0u, 0u, 0u);
+        }
+      }
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // staging -> TMA store / next load
+      __syncthreads();
+      if (tid == 0) {
+        if (ptr && bx == nbx - 1) g_pair_pk[blockIdx.x * 4 + 3] = global_ns();
+        tma_store_2d(m, smem_u32(dbox), bx * 64, (int)((long long)n * p.L_A + (long long)r0 * p.Wp));
+        asm volatile("cp.async.bulk.commit_group;" ::: "memory");
       }
     }
-    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // staging -> TMA store / next load
-    __syncthreads();
-    if (ptr) g_pair_pk[blockIdx.x * 4 + 3] = global_ns();
     if (tid == 0) {
-      const CUtensorMap* m = (r1 - r0 == p.rb) ? tmS : tmS2;
-      for (int bx = 0; bx < p.Cp / 64; ++bx)
-        tma_store_2d(m, smem_u32(out + (size_t)bx * obox), bx * 64, (int)((long long)n * p.L_A + (long long)r0 * p.Wp));
-      asm volatile("cp.async.bulk.commit_group;" ::: "memory");
-      asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");  // written (before the grid counter / reuse)
+      asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");  // written (before publishing / reuse)
+      publish_band(p, u);
+      if (ptr) g_pair_pk[blockIdx.x * 4 + 2] = global_ns();
     }
     __syncthreads();
-    if (ptr) g_pair_pk[blockIdx.x * 4 + 2] = global_ns();
   }
 }
 
@@ -409,7 +450,7 @@ __global__ void __launch_bounds__(kPairThreads, 1)
   uint64_t* tempty = tfull + 2;           // [2] accumulator drained (leader: 16 epilogue warps)
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
   uint32_t* mtab = tmem_slot + 4;  // [kMaxBlk][2]: per tap, A shift and B offset (16-byte units)
-  uint64_t* pbar = reinterpret_cast<uint64_t*>(mtab + 2 * kMaxBlk);  // pack: x band landed
+  uint64_t* pbar = reinterpret_cast<uint64_t*>(mtab + 2 * kMaxBlk);  // [4] pack: x box landed
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t rank = cluster_ctarank();
@@ -420,6 +461,7 @@ __global__ void __launch_bounds__(kPairThreads, 1)
     tr[0] = global_ns();
     g_pair_clk[blockIdx.x * 2] = clock64();
   }
+  if (p.dbg & 32) return;  // timing experiment: launch + teardown cost of this configuration
 
   if (warp == 0 && lane == 0) {
     prefetch_tmap(&tmA);
@@ -433,44 +475,48 @@ __global__ void __launch_bounds__(kPairThreads, 1)
       mbar_init(tfull + s, 1);
       mbar_init(tempty + s, 2 * 8);
     }
-    mbar_init(pbar, 1);
+    for (int i = 0; i < 4; ++i) mbar_init(pbar + i, 1);
     fence_barrier_init();
   }
   if (warp == 1) tmem_alloc2(tmem_slot, (uint32_t)p.tmem_cols);
   __syncthreads();  // pbar initialised
 
-  // phase 1: packing (all warps); the window ring and filter area are the staging buffer
-  if (!(p.dbg & 2)) {  // dbg&2: skip the packing (timing experiments only)
-    if (p.pack_tma) {
-      // the first band's input load flies while the filter is packed
-      const bool first = (int)blockIdx.x < p.nunits;
-      bool issued = false;
-      if (threadIdx.x == 0 && first) {
-        const int n = (int)blockIdx.x / p.nb, b = (int)blockIdx.x - n * p.nb;
-        const int r0 = b * p.rb, r1 = min(p.Hp, r0 + p.rb);
-        const int h0 = min(max(r0 - p.ph, 0), p.H), h1 = min(max(r1 - p.ph, 0), p.H);
-        if (h1 > h0) {
-          prefetch_tmap(&tmX);
-          mbar_arrive_expect_tx(pbar, p.C * p.ne_box * (uint32_t)sizeof(IoT));
-          // a TMA box must start 16-byte aligned in global memory: round down
-          tma_load_2d(sF, &tmX, pbar, (h0 * p.W) & ~(16 / (int)sizeof(IoT) - 1), n * p.C);
-        }
+  // phase 1: packing (all warps); the window ring and filter area are the staging buffer.
+  // The filter slices meet on the grid counter *fcount; every band of A is published
+  // on its own flag, so a tile's window waits only for the bands it reads.
+  if (p.pack_tma) {
+    // the first band's input boxes fly while the filter is packed
+    const bool first = (int)blockIdx.x < p.nunits;
+    if (threadIdx.x == 0 && first && !(p.dbg & 2)) {
+      const int u = (int)blockIdx.x;
+      const int n = u / p.nb, b = u - n * p.nb;
+      const int r0 = b * p.rb, r1 = min(p.Hp, r0 + p.rb);
+      const int h0 = min(max(r0 - p.ph, 0), p.H), h1 = min(max(r1 - p.ph, 0), p.H);
+      if (h1 > h0) {
+        prefetch_tmap(&tmX);
+        for (int bx = 0; bx < p.Cp / 64; ++bx) pack_load<IoT>(p, &tmX, sF, pbar, u, bx);
       }
-      issued = first;
-      pair_pack<IoT>(p, nullptr, false);
-      pair_pack_x_tma<IoT>(p, sF, pbar, &tmX, &tmS, &tmS2, issued);
-    } else {
-      pair_pack<IoT>(p, reinterpret_cast<uint16_t*>(sF), true);
+    }
+    if (!(p.dbg & 2)) pair_pack<IoT>(p, nullptr, false);  // dbg&2: no packing (timing experiments only)
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      __threadfence();
+      atomicAdd(p.fcount, 1ull);
+    }
+    pair_pack_x_tma<IoT>(p, sF, pbar, &tmX, &tmS, &tmS2, first);
+  } else {
+    if (!(p.dbg & 2)) pair_pack<IoT>(p, reinterpret_cast<uint16_t*>(sF), true);
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      __threadfence();
+      atomicAdd(p.fcount, 1ull);
+      for (int u = blockIdx.x; u < p.nunits; u += gridDim.x)
+        asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p.bflag + u), "l"(p.epoch) : "memory");
     }
   }
   // the staging area is overwritten by TMA (async proxy) next
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
   __syncthreads();
-  if (threadIdx.x == 0) {
-    asm volatile("fence.proxy.async.global;" ::: "memory");  // TMA-stored A -> generic release
-    __threadfence();
-    atomicAdd(p.fcount, 1ull);
-  }
   if (trace && threadIdx.x == 0) tr[1] = global_ns();
   tc_fence_before();
   __syncthreads();
@@ -484,17 +530,8 @@ __global__ void __launch_bounds__(kPairThreads, 1)
     const uint32_t lead_ffull = mapa_rank0(smem_u32(ffull));
     const uint32_t sW0 = smem_u32(sWin), sF0 = smem_u32(sF);
     const int half = p.NN / 2;
-    if ((p.dbg & 1) && elect_one()) {  // timing experiment: filter loads before the pack is done (stale U)
-      for (int ch = 0; ch < p.nchunks; ++ch)
-        for (int tap = 0; tap < p.RS; ++tap) {
-          const int blk = ch * p.RS + tap;
-          if (rank == 0) mbar_arrive_expect_tx(ffull + blk, 2u * p.fbytes);
-          tma_load_2d_pair(sF0 + (uint32_t)blk * p.fbytes, &tmU, lead_ffull + 8u * (uint32_t)blk, ch * p.kc,
-                           tap * p.NN + (int)rank * half);
-        }
-    }
-    __syncwarp();
     if (lane == 0) {
+      // every CTA's slice of the packed filter is in global memory
       unsigned long long v;
       uint64_t t0 = 0;
       for (;;) {
@@ -506,15 +543,52 @@ __global__ void __launch_bounds__(kPairThreads, 1)
       }
       asm volatile("fence.proxy.async.global;" ::: "memory");  // generic writes -> TMA reads
       if (trace) tr[2] = global_ns();
+      // dbg&64: the whole filter half right away (default: each chunk's blocks after
+      // its first window, so that the window is not queued behind them)
+      if ((p.dbg & 64) && pair < p.num_tiles) {
+        for (int blk = 0; blk < p.nblk; ++blk) {
+          const int ch = blk / p.RS, tap = blk - ch * p.RS;
+          if (rank == 0) mbar_arrive_expect_tx(ffull + blk, 2u * p.fbytes);
+          tma_load_2d_pair(sF0 + (uint32_t)blk * p.fbytes, &tmU, lead_ffull + 8u * (uint32_t)blk, ch * p.kc,
+                           tap * p.NN + (int)rank * half);
+        }
+      }
     }
     __syncwarp();
     int wi = 0, lt = 0;
+    // padded rows one window covers
+    const int wrows_img = (p.nbox * p.box_rows + p.Wp - 1) / p.Wp + 1;
     for (int t = pair; t < p.num_tiles; t += p.num_pairs, ++lt) {
       // CTA tile 2t + rank = output rows [blk*tr, blk*tr + tr) of image n; its positions
       // start at coefficient n*L_A + blk*tr*sh*Wp (Eq. 12 base of output (blk*tr, 0))
       const int ct = 2 * t + (int)rank;
       const int tn = (int)p.ftpi.div((uint32_t)ct), tb = ct - tn * p.tpi;
       const int g0 = tn * (int)p.L_A + tb * p.tr * p.sh * p.Wp;
+      if (tn < p.N) {
+        // the bands of image tn this tile's windows read (rows past the image are junk);
+        // lane i polls band b_lo + i, so the flags' round trips overlap
+        const int r_lo = tb * p.tr * p.sh, r_hi = min(p.Hp - 1, r_lo + wrows_img);
+        const int b_lo = r_lo / p.rb, nbw = r_hi / p.rb - b_lo + 1;
+        uint64_t t0 = 0;
+        for (int b0 = 0; b0 < nbw; b0 += 32) {
+          bool done = b0 + lane >= nbw;
+          const unsigned long long* f = p.bflag + tn * p.nb + b_lo + b0 + lane;
+          while (!__all_sync(0xffffffffu, done)) {
+            if (!done) {
+              unsigned long long v;
+              asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(f) : "memory");
+              done = v >= p.epoch;
+            }
+            const uint64_t tt = global_ns();
+            if (t0 == 0) t0 = tt;
+            else if (tt - t0 > 500000000ull) __trap();
+          }
+        }
+        asm volatile("fence.acq_rel.gpu;" ::: "memory");   // acquire the bands' rows
+        asm volatile("fence.proxy.async.global;" ::: "memory");  // ... for the TMA reads
+        if (trace && lt == 0 && lane == 0) tr[14] = global_ns();
+      }
+      __syncwarp();
       for (int ci = 0; ci < p.nchunks; ++ci, ++wi) {
         // one fixed (chunk, tap) order everywhere: every output sees the same
         // accumulation order whatever tile or batch it is computed in (reading R12)
@@ -526,9 +600,8 @@ __global__ void __launch_bounds__(kPairThreads, 1)
           for (int b = 0; b < p.nbox; ++b)
             tma_load_2d_pair(sW0 + (uint32_t)slot * p.wbytes + (uint32_t)(b * p.box_rows * p.row_bytes), &tmA,
                              lead_wfull + 8u * (uint32_t)slot, ch * p.kc, g0 + b * p.box_rows);
-          if (lt == 0 && !(p.dbg & 1)) {  // the filter blocks of this chunk: loaded once, resident
-            for (int ti = 0; ti < p.RS; ++ti) {
-              const int tap = ti;
+          if (lt == 0 && !(p.dbg & 64)) {  // this chunk's filter blocks: loaded once, resident
+            for (int tap = 0; tap < p.RS; ++tap) {
               const int blk = ch * p.RS + tap;
               if (rank == 0) mbar_arrive_expect_tx(ffull + blk, 2u * p.fbytes);
               tma_load_2d_pair(sF0 + (uint32_t)blk * p.fbytes, &tmU, lead_ffull + 8u * (uint32_t)blk, ch * p.kc,
@@ -569,7 +642,7 @@ __global__ void __launch_bounds__(kPairThreads, 1)
           if (lt == 0 && !(p.dbg & 4)) {  // this chunk's filter blocks (first tile only; then resident)
             for (int tap = 0; tap < p.RS; ++tap) mbar_wait_cl(ffull + ch * p.RS + tap, 0u);
             tc_fence_after();
-            if (trace && lane == 0 && ci == p.nchunks - 1) tr[14] = global_ns();
+            if (trace && lane == 0 && ci == p.nchunks - 1) tr[12] = global_ns();
           }
           const uint64_t ad0 = make_sdesc(sW0 + (uint32_t)slot * p.wbytes, (uint32_t)p.row_bytes, 0);
           const uint64_t bd0 = make_sdesc(sF0 + (uint32_t)(ch * p.RS) * p.fbytes, (uint32_t)p.row_bytes, 0);
@@ -662,7 +735,7 @@ __global__ void __launch_bounds__(kPairThreads, 1)
           }
         }
       }
-      if (trace && threadIdx.x == kEpi0 * 32 && lt < 2) tr[10 + 2 * lt] = global_ns();
+      if (trace && threadIdx.x == kEpi0 * 32 && lt < 1) tr[10 + 2 * lt] = global_ns();
     }
     if (p.epi_tma && (e & 3) == 0 && lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
   }
@@ -799,12 +872,12 @@ PairTiling pair_tiling(const Geom& g, int fmt, bool io_bf16, int num_sms) {
     int rb2 = (int)cdivp(g.Hp, nb2);
     const int rb_cap = std::min(256 / g.Wp, 256 / g.W);
     if (rb2 > rb_cap) rb2 = rb_cap;
-    if (rb2 >= 1 && t.Cp % 64 == 0 && g.C <= 256 && ((long long)g.H * g.W * eb_in) % 16 == 0 &&
+    if (rb2 >= 1 && t.Cp % 64 == 0 && t.Cp <= 256 && ((long long)g.H * g.W * eb_in) % 16 == 0 &&
         !getenv("POLYCONV_PAIR_PACK_LD")) {
       const int nbb = (int)cdivp(g.Hp, rb2);
       const int last = g.Hp - (nbb - 1) * rb2;
       const int ne_box = (int)cdivp((long long)rb2 * g.W + ve - 1, ve) * ve;  // + the start's rounding
-      const long long in_b = cdivp((long long)g.C * ne_box * eb_in, 1024) * 1024;
+      const long long in_b = cdivp((long long)(t.Cp / 64) * 64 * ne_box * eb_in, 1024) * 1024;
       const long long ob = cdivp((long long)rb2 * g.Wp * 128, 1024) * 1024;
       const long long ob2 = cdivp((long long)last * g.Wp * 128, 1024) * 1024;
       if (ne_box <= 256 && in_b + (long long)(t.Cp / 64) * ob <= stage_cap) {
@@ -824,20 +897,33 @@ PairTiling pair_tiling(const Geom& g, int fmt, bool io_bf16, int num_sms) {
   return t;
 }
 
-cudaError_t launch_mac_pair(const Geom& g, const PairTiling& t, const void* x, const void* w, bool io_bf16,
-                            void* A, void* U, void* y, unsigned long long* fcount, unsigned long long ftarget,
-                            cudaStream_t st, char* err, size_t errlen) {
-  if (!t.ok) {
-    snprintf(err, errlen, "mac_pair: shape not supported");
-    return cudaErrorInvalidValue;
-  }
-  CUtensorMap tmA, tmU;
+namespace {
+// Everything a launch needs except the grid-counter target, built once per
+// (x, w, y, workspace) pointer set: the host path of a repeated forward is one
+// cudaLaunchKernelEx (tensor-map encoding and the co-residency check cost
+// microseconds that an idle stream would wait for).
+struct PairLaunchState {
+  const void *x = nullptr, *w = nullptr, *y = nullptr, *A = nullptr, *U = nullptr;
+  const unsigned long long* fcount = nullptr;
+  bool io_bf16 = false, valid = false;
+  CUtensorMap tmA, tmU, tmX, tmS, tmS2, tmY;
+  PairParams p;
+};
+
+cudaError_t prepare_mac_pair(PairLaunchState& S, const Geom& g, const PairTiling& t, const void* x, const void* w,
+                             bool io_bf16, void* A, void* U, void* y, unsigned long long* fcount, char* err,
+                             size_t errlen) {
+  S.valid = false;
+  CUtensorMap& tmA = S.tmA;
+  CUtensorMap& tmU = S.tmU;
   if (!encode_bf16(&tmA, A, (uint64_t)t.Cp, (uint64_t)g.N * g.L_A, (uint32_t)t.kc, (uint32_t)t.box_rows) ||
       !encode_bf16(&tmU, U, (uint64_t)t.Cp, (uint64_t)t.RS * t.NN, (uint32_t)t.kc, (uint32_t)(t.NN / 2))) {
     snprintf(err, errlen, "mac_pair: cuTensorMapEncodeTiled failed");
     return cudaErrorInvalidValue;
   }
-  CUtensorMap tmX, tmS, tmS2;
+  CUtensorMap& tmX = S.tmX;
+  CUtensorMap& tmS = S.tmS;
+  CUtensorMap& tmS2 = S.tmS2;
   memset(&tmX, 0, sizeof(tmX));
   memset(&tmS, 0, sizeof(tmS));
   memset(&tmS2, 0, sizeof(tmS2));
@@ -846,7 +932,7 @@ cudaError_t launch_mac_pair(const Geom& g, const PairTiling& t, const void* x, c
     const int eb_in = io_bf16 ? 2 : 4;
     cuuint64_t dims[2] = {(cuuint64_t)g.H * g.W, (cuuint64_t)g.N * g.C};
     cuuint64_t strides[1] = {(cuuint64_t)g.H * g.W * eb_in};
-    cuuint32_t box[2] = {(cuuint32_t)t.ne_box, (cuuint32_t)g.C};
+    cuuint32_t box[2] = {(cuuint32_t)t.ne_box, 64};
     cuuint32_t estr[2] = {1, 1};
     bool ok = enc && enc(&tmX, io_bf16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2,
                          const_cast<void*>(x), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
@@ -859,7 +945,7 @@ cudaError_t launch_mac_pair(const Geom& g, const PairTiling& t, const void* x, c
       return cudaErrorInvalidValue;
     }
   }
-  CUtensorMap tmY;
+  CUtensorMap& tmY = S.tmY;
   memset(&tmY, 0, sizeof(tmY));
   if (t.epi_tma) {
     EncodeTiledFnPair enc = get_encode_pair();
@@ -874,14 +960,15 @@ cudaError_t launch_mac_pair(const Geom& g, const PairTiling& t, const void* x, c
       return cudaErrorInvalidValue;
     }
   }
-  PairParams p{};
+  PairParams& p = S.p;
+  p = PairParams{};
   p.x = x; p.w = w; p.A = A; p.U = U; p.y = y;
   p.tr = t.tr; p.tpi = t.tpi; p.ntile = t.ntile; p.epi_tma = t.epi_tma;
   p.estage_bytes = (uint32_t)t.estage_bytes;
   p.ftpi.init((uint32_t)t.tpi);
   p.pack_tma = t.pack_tma; p.ne_box = t.ne_box; p.last_rows = t.last_rows;
   p.in_bytes = (uint32_t)t.in_bytes; p.obox_bytes = (uint32_t)t.obox_bytes; p.obox_bytes2 = (uint32_t)t.obox_bytes2;
-  p.fcount = fcount; p.ftarget = ftarget;
+  p.fcount = fcount; p.ftarget = 0;
   p.L_A = g.L_A;
   p.G = (long long)(g.N - 1) * g.L_A + g.M_ext;
   p.NLA = (long long)g.N * g.L_A;
@@ -900,8 +987,6 @@ cudaError_t launch_mac_pair(const Geom& g, const PairTiling& t, const void* x, c
   p.fWp.init((uint32_t)g.Wp);
   p.fsh.init((uint32_t)g.sh);
   p.fsw.init((uint32_t)g.sw);
-  const char* dbg = getenv("POLYCONV_PAIR_DEBUG");
-  p.dbg = dbg ? atoi(dbg) : 0;
   auto kern = io_bf16 ? mac_pair_kernel<__nv_bfloat16> : mac_pair_kernel<float>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, t.smem_bytes);
   if (e != cudaSuccess) return e;
@@ -909,7 +994,6 @@ cudaError_t launch_mac_pair(const Geom& g, const PairTiling& t, const void* x, c
   cfg.gridDim = dim3((unsigned)t.grid);
   cfg.blockDim = dim3(kPairThreads);
   cfg.dynamicSmemBytes = (size_t)t.smem_bytes;
-  cfg.stream = st;
   cudaLaunchAttribute attr[1];
   attr[0].id = cudaLaunchAttributeClusterDimension;
   attr[0].val.clusterDim.x = 2;
@@ -925,7 +1009,49 @@ cudaError_t launch_mac_pair(const Geom& g, const PairTiling& t, const void* x, c
     return cudaErrorInvalidConfiguration;
   }
   cudaGetLastError();
-  return cudaLaunchKernelEx(&cfg, kern, tmA, tmU, tmX, tmS, tmS2, tmY, p);
+  S.x = x; S.w = w; S.y = y; S.A = A; S.U = U; S.fcount = fcount; S.io_bf16 = io_bf16;
+  S.valid = true;
+  return cudaSuccess;
+}
+}  // namespace
+
+void* pair_state_new() { return new (std::nothrow) PairLaunchState(); }
+void pair_state_free(void* s) { delete static_cast<PairLaunchState*>(s); }
+
+cudaError_t launch_mac_pair(const Geom& g, const PairTiling& t, const void* x, const void* w, bool io_bf16,
+                            void* A, void* U, void* y, unsigned long long* fcount, unsigned long long ftarget,
+                            unsigned long long* bflag, unsigned long long epoch, cudaStream_t st, char* err,
+                            size_t errlen, void* state) {
+  if (!t.ok) {
+    snprintf(err, errlen, "mac_pair: shape not supported");
+    return cudaErrorInvalidValue;
+  }
+  PairLaunchState local;
+  PairLaunchState& S = state ? *static_cast<PairLaunchState*>(state) : local;
+  if (!S.valid || S.x != x || S.w != w || S.y != y || S.A != A || S.U != U || S.fcount != fcount ||
+      S.io_bf16 != io_bf16) {
+    cudaError_t e = prepare_mac_pair(S, g, t, x, w, io_bf16, A, U, y, fcount, err, errlen);
+    if (e != cudaSuccess) return e;
+  }
+  S.p.ftarget = ftarget;
+  S.p.bflag = bflag;
+  S.p.epoch = epoch;
+  const char* dbg = getenv("POLYCONV_PAIR_DEBUG");
+  S.p.dbg = dbg ? atoi(dbg) : 0;
+  auto kern = io_bf16 ? mac_pair_kernel<__nv_bfloat16> : mac_pair_kernel<float>;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)t.grid);
+  cfg.blockDim = dim3(kPairThreads);
+  cfg.dynamicSmemBytes = (size_t)t.smem_bytes;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = 2;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kern, S.tmA, S.tmU, S.tmX, S.tmS, S.tmS2, S.tmY, S.p);
 }
 
 }  // namespace polyconv

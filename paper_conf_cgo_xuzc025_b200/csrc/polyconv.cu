@@ -24,6 +24,8 @@ struct polyconv_plan_s {
   Tc2Tiling tc2;
   Fp32Tiling f32;
   PairTiling pair;
+  void* pair_state = nullptr;  // mac_pair launch cache
+  unsigned long long* bflag = nullptr;  // mac_pair band flags [N * pair.nb]
   // workspace (lazy)
   void* wsA = nullptr;
   size_t wsA_bytes = 0;
@@ -264,6 +266,7 @@ polyconv_status_t polyconv_plan_set_kernel(polyconv_plan_t p, polyconv_kernel_t 
   }
   // workspace sizes (and the grid the pack counter counts) may have changed
   if (p->fcount) { cudaFree(p->fcount); p->fcount = nullptr; }
+  if (p->pair_state) { pair_state_free(p->pair_state); p->pair_state = nullptr; }
   if (p->wsA) { cudaFree(p->wsA); p->wsA = nullptr; }
   if (p->wsU) { cudaFree(p->wsU); p->wsU = nullptr; }
   return POLYCONV_STATUS_SUCCESS;
@@ -326,22 +329,27 @@ polyconv_status_t polyconv_forward(polyconv_plan_t p, const void* x, const void*
     return finish(p, e, "mac_tc");
   }
   if (p->kernel == POLYCONV_KERNEL_TC_PAIR) {
-    // one launch: a3 + a2 into the workspace (every CTA a slice), grid counter,
-    // then a4 + a5 on CTA pairs.  All CTAs are co-resident (checked at launch).
+    // one launch: a3 (filter slices, every CTA; grid counter) + a2 (bands of A, each
+    // published on its own flag), then a4 + a5 on CTA pairs.  All CTAs are co-resident
+    // (checked when the launch is prepared).
     if (!p->fcount) {
-      if (cudaMalloc(&p->fcount, sizeof(unsigned long long)) != cudaSuccess ||
-          cudaMemsetAsync(p->fcount, 0, sizeof(unsigned long long), st) != cudaSuccess) {
+      const size_t nflag = 1 + (size_t)g.N * p->pair.nb;
+      if (cudaMalloc(&p->fcount, nflag * sizeof(unsigned long long)) != cudaSuccess ||
+          cudaMemsetAsync(p->fcount, 0, nflag * sizeof(unsigned long long), st) != cudaSuccess) {
         cudaGetLastError();
         p->fcount = nullptr;
-        set_err(p, "cudaMalloc of the %s failed", "pack counter");
+        set_err(p, "cudaMalloc of the %s failed", "pack counters");
         return POLYCONV_STATUS_ALLOC_FAILED;
       }
+      p->bflag = p->fcount + 1;
       p->fepoch = 0;
     }
     if (p->ev_start) cudaEventRecord(p->ev_start, st);
-    const unsigned long long target = (p->fepoch + 1) * (unsigned long long)p->pair.grid;
-    e = launch_mac_pair(g, p->pair, x, w, p->io_bf16, p->wsA, p->wsU, y, p->fcount, target, st, p->err,
-                        sizeof(p->err));
+    const unsigned long long epoch = p->fepoch + 1;
+    if (!p->pair_state) p->pair_state = pair_state_new();
+    e = launch_mac_pair(g, p->pair, x, w, p->io_bf16, p->wsA, p->wsU, y, p->fcount,
+                        epoch * (unsigned long long)p->pair.grid, p->bflag, epoch, st, p->err, sizeof(p->err),
+                        p->pair_state);
     if (e == cudaSuccess) ++p->fepoch;
     if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
     return finish(p, e, "mac_pair");
@@ -497,6 +505,7 @@ polyconv_status_t polyconv_destroy(polyconv_plan_t p) {
     if (p->hy) cudaFree(p->hy);
     if (p->fcount) cudaFree(p->fcount);
   }
+  if (p->pair_state) pair_state_free(p->pair_state);
   delete p;
   return s;
 }

@@ -19,7 +19,7 @@ fi
 if [[ $what == ncu || $what == all ]]; then
   timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 60 --csv --log-file gpurun_out/${tag}_launches.csv \
     python bench.py --steps 10 --warmup 3 --no-cpu-baseline --no-cudnn > gpurun_out/${tag}_ncu_bench.log 2>&1; echo "ncu launches rc=$?"
-  timeout 900 ncu --set full --clock-control none --import-source on -k regex:mac_tc2 -s 3 -c 2 -o gpurun_out/${tag}_mac_tc \
+  timeout 900 ncu --set full --clock-control none --import-source on -k regex:mac_pair -s 3 -c 1 -o gpurun_out/${tag}_mac_pair \
     python bench.py --steps 4 --warmup 3 --no-cpu-baseline --no-cudnn > gpurun_out/${tag}_ncu_full.log 2>&1; echo "ncu full rc=$?"
   timeout 600 ncu --set full --clock-control none -k regex:pack -s 3 -c 1 -o gpurun_out/${tag}_pack \
     python bench.py --steps 4 --warmup 3 --no-cpu-baseline --no-cudnn > gpurun_out/${tag}_ncu_pack.log 2>&1; echo "ncu pack rc=$?"

@@ -2,7 +2,7 @@
 (the bench's roofline.traffic comes from here) and print the key counters.
 
     python tools/ncu_summary.py gpurun_out/<rep>.ncu-rep <key> [launches.csv]
-key: e.g. mac_tc_bf16 (bench.py looks up "mac_tc_" + math)."""
+key: e.g. mac_tc_pair_bf16 (bench.py looks up "mac_<kernel>_<math>")."""
 import csv, io, json, os, subprocess, sys
 
 WANT = {

@@ -26,7 +26,7 @@ a = np.array(buf, dtype=np.float64).reshape(160, 16)
 a = a[a[:, 0] > 0]
 t0 = a[:, 0].min()
 names = ["start", "pack_done", "counter_passed", "win0", "win1", "win2", "win3", "tile0_issued", "tile1_issued",
-         "epi0_ready", "epi0_done", "epi1_ready", "epi1_done", "end", "filter_last", "prod_last_tma"]
+         "epi0_ready", "epi0_done", "epi1_ready", "filter_last", "end", "bands_ready0", "prod_last_tma"]
 print("CTAs", len(a))
 for k, nm in enumerate(names):
     col = a[:, k]
