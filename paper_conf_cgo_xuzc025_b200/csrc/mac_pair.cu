@@ -73,6 +73,7 @@ struct PairParams {
   int box_rows, nbox;
   uint32_t wbytes, wbytes_tx, fbytes;
   int ring, num_tiles, num_pairs;
+  int urep;  // filter copies in U; pair p reads copy p % urep (spreads the L2 lines all CTAs read)
   uint32_t idesc;
   int tmem_cols;
   int rb, nb, nunits, spitch;
@@ -192,7 +193,7 @@ __device__ __forceinline__ void pair_pack(const PairParams& p, uint16_t* stg, bo
   {
     const IoT* w = static_cast<const IoT*>(p.w);
     uint16_t* U = static_cast<uint16_t*>(p.U);
-    const int total = p.RS * p.NN * p.Cp;
+    const int total = p.RS * p.NN * p.Cp;  // one copy; urep copies are written
     const int stride = gridDim.x * nth;
     for (int base = blockIdx.x * nth + tid; base < total; base += 4 * stride) {
       uint16_t v[4];
@@ -206,10 +207,12 @@ __device__ __forceinline__ void pair_pack(const PairParams& p, uint16_t* stg, bo
           if (k < p.K && c < p.C) v[u] = to_bf16_bits<IoT>(w[((long long)k * p.C + c) * p.RS + tap]);
         }
       }
+      for (int rep = 0; rep < p.urep; ++rep) {
 #pragma unroll
-      for (int u = 0; u < 4; ++u) {
-        const int idx = base + u * stride;
-        if (idx < total) U[idx] = v[u];
+        for (int u = 0; u < 4; ++u) {
+          const int idx = base + u * stride;
+          if (idx < total) U[(long long)rep * total + idx] = v[u];
+        }
       }
     }
   }
@@ -550,7 +553,7 @@ __global__ void __launch_bounds__(kPairThreads, 1)
           const int ch = blk / p.RS, tap = blk - ch * p.RS;
           if (rank == 0) mbar_arrive_expect_tx(ffull + blk, 2u * p.fbytes);
           tma_load_2d_pair(sF0 + (uint32_t)blk * p.fbytes, &tmU, lead_ffull + 8u * (uint32_t)blk, ch * p.kc,
-                           tap * p.NN + (int)rank * half);
+                           tap * p.NN + (int)rank * half + (pair % p.urep) * p.RS * p.NN);
         }
       }
     }
@@ -605,7 +608,7 @@ __global__ void __launch_bounds__(kPairThreads, 1)
               const int blk = ch * p.RS + tap;
               if (rank == 0) mbar_arrive_expect_tx(ffull + blk, 2u * p.fbytes);
               tma_load_2d_pair(sF0 + (uint32_t)blk * p.fbytes, &tmU, lead_ffull + 8u * (uint32_t)blk, ch * p.kc,
-                               tap * p.NN + (int)rank * half);
+                               tap * p.NN + (int)rank * half + (pair % p.urep) * p.RS * p.NN);
             }
           }
         }
@@ -917,7 +920,7 @@ cudaError_t prepare_mac_pair(PairLaunchState& S, const Geom& g, const PairTiling
   CUtensorMap& tmA = S.tmA;
   CUtensorMap& tmU = S.tmU;
   if (!encode_bf16(&tmA, A, (uint64_t)t.Cp, (uint64_t)g.N * g.L_A, (uint32_t)t.kc, (uint32_t)t.box_rows) ||
-      !encode_bf16(&tmU, U, (uint64_t)t.Cp, (uint64_t)t.RS * t.NN, (uint32_t)t.kc, (uint32_t)(t.NN / 2))) {
+      !encode_bf16(&tmU, U, (uint64_t)t.Cp, (uint64_t)g.urep * t.RS * t.NN, (uint32_t)t.kc, (uint32_t)(t.NN / 2))) {
     snprintf(err, errlen, "mac_pair: cuTensorMapEncodeTiled failed");
     return cudaErrorInvalidValue;
   }
@@ -979,6 +982,7 @@ cudaError_t prepare_mac_pair(PairLaunchState& S, const Geom& g, const PairTiling
   p.nblk = t.nblk; p.box_rows = t.box_rows; p.nbox = t.nbox;
   p.wbytes = (uint32_t)t.wbytes; p.wbytes_tx = (uint32_t)t.wbytes_tx; p.fbytes = (uint32_t)t.fbytes;
   p.ring = t.ring; p.num_tiles = t.num_tiles; p.num_pairs = t.num_pairs;
+  p.urep = g.urep;
   // instruction descriptor: D=f32 @4, A/B = bf16 @7/@10, both K-major, N>>3 @17, M>>4 @24 (M = 256)
   p.idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(t.NN >> 3) << 17) | ((uint32_t)(256 >> 4) << 24);
   p.tmem_cols = t.tmem_cols;

@@ -109,9 +109,9 @@ polyconv_status_t resolve(polyconv_plan_t p) {
                                                                                        : (size_t)g.N * g.C * g.L_A;
   p->wsA_bytes = a_elems * eb;
   g.urep = 1;
-  if (k == POLYCONV_KERNEL_TC || k == POLYCONV_KERNEL_TC_FUSED) {
+  if (k == POLYCONV_KERNEL_TC || k == POLYCONV_KERNEL_TC_FUSED || k == POLYCONV_KERNEL_TC_PAIR) {
     const char* r = getenv("POLYCONV_FILTER_REP");  // experiments only
-    g.urep = r ? atoi(r) : 1;
+    g.urep = r ? atoi(r) : 1;  // tc_pair: replicas measured slower (more pack writes)
     if (g.urep < 1) g.urep = 1;
     if (g.urep > 64) g.urep = 64;
     if ((long long)g.urep * g.R * g.S * g.Kp >= (1LL << 31)) g.urep = 1;  // TMA row coordinate
