@@ -293,3 +293,34 @@ def test_errors_on_device():
     with pytest.raises(pc.PolyconvError) as e:
         plan.forward_ptr(x.data_ptr(), w.data_ptr(), x.data_ptr())       # y aliases x
     assert e.value.status == pc.BAD_PARAM
+
+
+def test_pair_repeated_launches_one_plan():
+    """tc_pair keeps per-plan state across launches (grid counter epochs, band flags,
+    cached tensor maps): consecutive forwards on one plan with new inputs and new
+    output buffers must each match the oracle bit for bit (integer data)."""
+    import torch
+    shape = ConvShape("pair_rep", 3, 64, 14, 14, 64, 3, 3, 1, 1, 1, 1)
+    plan = None
+    for it in range(4):
+        x, w = synth.make_inputs(shape, synth.seed_for(11, it), "int")
+        ref = bf16_round(oracle.conv2d(x, w, shape.stride, shape.padding))
+        y, plan = gpu_forward(shape, x, w, math="bf16", io="bf16", kernel="tc_pair", plan=plan)
+        assert plan.info()["kernel"] == "tc_pair"
+        assert np.array_equal(y, ref), it
+
+
+@pytest.mark.parametrize("shape", [ConvShape("pair_rows1", 2, 64, 9, 100, 64, 3, 3, 1, 1, 1, 1),   # tr = 1
+                                   ConvShape("pair_s2", 3, 64, 29, 29, 64, 3, 3, 2, 2, 1, 1),       # stride 2, odd P
+                                   ConvShape("pair_c192", 2, 192, 10, 10, 96, 3, 3, 1, 1, 1, 1),    # 3 chunks, K % 64
+                                   ConvShape("pair_k1", 4, 128, 14, 14, 128, 1, 1, 1, 1, 0, 0)],
+                         ids=lambda s: s.name)
+@pytest.mark.parametrize("io", ["bf16", "f32"])
+def test_pair_shapes(shape, io):
+    """tc_pair tilings off the bench shape: one output row per tile, stride 2 with a
+    ragged last row block, three channel chunks with K not a multiple of 64, 1x1."""
+    x, w = synth.make_inputs(shape, synth.seed_for(12, hash(shape.name) % 997), "int")
+    ref = oracle.conv2d(x, w, shape.stride, shape.padding)
+    y, plan = gpu_forward(shape, x, w, math="bf16", io=io, kernel="tc_pair")
+    assert plan.info()["kernel"] == "tc_pair"
+    assert np.array_equal(y, bf16_round(ref) if io == "bf16" else ref)
