@@ -312,7 +312,7 @@ def test_pair_repeated_launches_one_plan():
 
 @pytest.mark.parametrize("shape", [ConvShape("pair_rows1", 2, 64, 9, 100, 64, 3, 3, 1, 1, 1, 1),   # tr = 1
                                    ConvShape("pair_s2", 3, 64, 29, 29, 64, 3, 3, 2, 2, 1, 1),       # stride 2, odd P
-                                   ConvShape("pair_c192", 2, 192, 10, 10, 96, 3, 3, 1, 1, 1, 1),    # 3 chunks, K % 64
+                                   ConvShape("pair_c192", 2, 192, 10, 10, 48, 3, 3, 1, 1, 1, 1),    # 3 chunks, K % 64
                                    ConvShape("pair_k1", 4, 128, 14, 14, 128, 1, 1, 1, 1, 0, 0)],
                          ids=lambda s: s.name)
 @pytest.mark.parametrize("io", ["bf16", "f32"])
