@@ -88,6 +88,9 @@ struct PairParams {
   // ntile CTA tiles in all); epilogue by TMA stores of [32 channels][tr*Q pixels]
   // boxes staged in shared memory (epi_tma) or by direct stores
   int tr, tpi, ntile, epi_tma;
+  int fsmem;  // a3 straight into shared memory after the band packing (no global U, no counter):
+              // 1 = loads from w, 2 = bulk-copied slabs of frows rows of w
+  int frows;
   uint32_t estage_bytes;
   FastDiv ftpi;
 };
@@ -328,6 +331,151 @@ __device__ __forceinline__ void tma_store_2d(const void* tmap, uint32_t src, int
                : "memory");
 }
 
+// a3 straight into shared memory: CTA `rank` of the pair builds its NN/2 output
+// channels of every (channel chunk, tap) block of the tap-major filter -- the
+// nonzero coefficients of the reversed, gap-padded U_{k,c}(t) (Eq. 6), block
+// (ch, tap) row k = w[k][ch*kc .. ch*kc + kc)[tap] -- in the UMMA K-major layout
+// (rows of kc bf16 words, 32/64/128-byte swizzle).  One item = 8 channels of one
+// output channel: their R*S taps are contiguous in w (one 16-byte vector per tap
+// group when RS == 9 and C % 8 == 0), transposed in registers into one 16-byte
+// chunk per tap block.  Nothing goes to global memory.
+template <typename IoT>
+__device__ __forceinline__ void pair_filter_smem(const PairParams& p, uint8_t* sF, uint32_t rank) {
+  const int half = p.NN / 2, kb = (int)rank * half;
+  const int ncg = p.Cp / 8;
+  const int items = half * ncg;
+  const IoT* w = static_cast<const IoT*>(p.w);
+  const uint32_t M = (uint32_t)p.row_bytes / 16u - 1u;  // swizzle: 16-byte chunk ^= (row bits)
+  const bool vec9 = std::is_same<IoT, __nv_bfloat16>::value && p.RS == 9 && p.C % 8 == 0;
+  for (int it = threadIdx.x; it < items; it += blockDim.x) {
+    const int kl = it / ncg, cg = it - (it / ncg) * ncg;
+    const int k = kb + kl, c0 = cg * 8;
+    const int ch = c0 / p.kc, j = (c0 - ch * p.kc) >> 3;
+    const uint32_t o = (uint32_t)kl * (uint32_t)p.row_bytes + (uint32_t)j * 16u;
+    uint8_t* dst = sF + (size_t)(ch * p.RS) * p.fbytes + (o ^ (((o >> 7) & M) << 4));
+    if (vec9 && k < p.K && c0 + 8 <= p.C) {
+      // w[k][c0..c0+7][0..8]: 72 bf16 = 9 x 16 bytes, element c*9 + t
+      const uint4* src = reinterpret_cast<const uint4*>(w + ((long long)k * p.C + c0) * 9);
+      uint32_t e[36];
+#pragma unroll
+      for (int q = 0; q < 9; ++q) {
+        const uint4 v = __ldg(src + q);
+        e[4 * q] = v.x; e[4 * q + 1] = v.y; e[4 * q + 2] = v.z; e[4 * q + 3] = v.w;
+      }
+#pragma unroll
+      for (int t = 0; t < 9; ++t) {
+        uint32_t out[4];
+#pragma unroll
+        for (int m = 0; m < 4; ++m) {
+          const int i0 = (2 * m) * 9 + t, i1 = (2 * m + 1) * 9 + t;
+          const uint32_t lo = (e[i0 >> 1] >> ((i0 & 1) * 16)) & 0xFFFFu;
+          const uint32_t hi = (e[i1 >> 1] >> ((i1 & 1) * 16)) & 0xFFFFu;
+          out[m] = lo | (hi << 16);
+        }
+        *reinterpret_cast<uint4*>(dst + (size_t)t * p.fbytes) = make_uint4(out[0], out[1], out[2], out[3]);
+      }
+    } else {
+      for (int t = 0; t < p.RS; ++t) {
+        uint32_t out[4];
+#pragma unroll
+        for (int m = 0; m < 4; ++m) {
+          const int c = c0 + 2 * m;
+          const uint32_t lo =
+              (k < p.K && c < p.C) ? (uint32_t)to_bf16_bits<IoT>(w[((long long)k * p.C + c) * p.RS + t]) : 0u;
+          const uint32_t hi =
+              (k < p.K && c + 1 < p.C) ? (uint32_t)to_bf16_bits<IoT>(w[((long long)k * p.C + c + 1) * p.RS + t]) : 0u;
+          out[m] = lo | (hi << 16);
+        }
+        *reinterpret_cast<uint4*>(dst + (size_t)t * p.fbytes) = make_uint4(out[0], out[1], out[2], out[3]);
+      }
+    }
+  }
+}
+
+// a3 into shared memory from bulk-copied rows of w (fsmem == 2): slabs of `frows`
+// output-channel rows w[k][0..C*R*S) (contiguous in KCRS) land by cp.async.bulk in
+// a double-buffered staging area, and the warps transpose them into the resident
+// (chunk, tap) blocks: item (k, 8 channels) reads the 8*R*S contiguous coefficients
+// and writes one 16-byte chunk per tap block (same layout as pair_filter_smem).
+__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
+               "l"(src), "r"(bytes), "r"(smem_u32(bar))
+               : "memory");
+}
+
+__device__ __forceinline__ void pair_filter_bulk(const PairParams& p, uint8_t* sF, uint8_t* stage, uint64_t* fb,
+                                                 uint32_t rank) {
+  const int half = p.NN / 2, kb = (int)rank * half;
+  const int ncg = p.Cp / 8;
+  const uint32_t rowb = (uint32_t)p.C * p.RS * 2u;  // bytes of one w row (bf16)
+  const uint32_t slab = (uint32_t)p.frows * rowb;
+  const int nslab = (half + p.frows - 1) / p.frows;
+  const uint32_t M = (uint32_t)p.row_bytes / 16u - 1u;
+  const __nv_bfloat16* w = static_cast<const __nv_bfloat16*>(p.w);
+  auto issue = [&](int sl) {
+    const int k0 = kb + sl * p.frows;
+    const int nk = min(p.frows, p.K - k0);
+    if (nk <= 0) return;
+    uint8_t* dst = stage + (size_t)(sl & 1) * slab;
+    mbar_arrive_expect_tx(fb + (sl & 1), (uint32_t)nk * rowb);
+    for (int r = 0; r < nk; ++r)
+      bulk_g2s(smem_u32(dst + (size_t)r * rowb), w + (size_t)(k0 + r) * p.C * p.RS, rowb, fb + (sl & 1));
+  };
+  if (threadIdx.x == 0) {
+    issue(0);
+    if (nslab > 1) issue(1);
+  }
+  for (int sl = 0; sl < nslab; ++sl) {
+    const int k0 = kb + sl * p.frows;
+    const int nk_valid = max(0, min(p.frows, p.K - k0));
+    if (nk_valid > 0) mbar_wait(fb + (sl & 1), (uint32_t)((sl >> 1) & 1));
+    const uint8_t* src = stage + (size_t)(sl & 1) * slab;
+    const int rows = min(p.frows, half - sl * p.frows);
+    for (int it = threadIdx.x; it < rows * ncg; it += blockDim.x) {
+      const int r = it / ncg, cg = it - (it / ncg) * ncg;
+      const int kl = sl * p.frows + r, k = kb + kl, c0 = cg * 8;
+      const int ch = c0 / p.kc, j = (c0 - ch * p.kc) >> 3;
+      const uint32_t o = (uint32_t)kl * (uint32_t)p.row_bytes + (uint32_t)j * 16u;
+      uint8_t* dst = sF + (size_t)(ch * p.RS) * p.fbytes + (o ^ (((o >> 7) & M) << 4));
+      const uint16_t* row = reinterpret_cast<const uint16_t*>(src + (size_t)r * rowb);
+      if (p.RS == 9 && k < p.K && c0 + 8 <= p.C) {
+        const uint4* v4 = reinterpret_cast<const uint4*>(row + c0 * 9);
+        uint32_t e[36];
+#pragma unroll
+        for (int q = 0; q < 9; ++q) {
+          const uint4 v = v4[q];
+          e[4 * q] = v.x; e[4 * q + 1] = v.y; e[4 * q + 2] = v.z; e[4 * q + 3] = v.w;
+        }
+#pragma unroll
+        for (int t = 0; t < 9; ++t) {
+          uint32_t out[4];
+#pragma unroll
+          for (int m = 0; m < 4; ++m) {
+            const int i0 = (2 * m) * 9 + t, i1 = (2 * m + 1) * 9 + t;
+            out[m] = ((e[i0 >> 1] >> ((i0 & 1) * 16)) & 0xFFFFu) | (((e[i1 >> 1] >> ((i1 & 1) * 16)) & 0xFFFFu) << 16);
+          }
+          *reinterpret_cast<uint4*>(dst + (size_t)t * p.fbytes) = make_uint4(out[0], out[1], out[2], out[3]);
+        }
+      } else {
+        for (int t = 0; t < p.RS; ++t) {
+          uint32_t out[4];
+#pragma unroll
+          for (int m = 0; m < 4; ++m) {
+            const int c = c0 + 2 * m;
+            const uint32_t lo = (k < p.K && c < p.C) ? (uint32_t)row[c * p.RS + t] : 0u;
+            const uint32_t hi = (k < p.K && c + 1 < p.C) ? (uint32_t)row[(c + 1) * p.RS + t] : 0u;
+            out[m] = lo | (hi << 16);
+          }
+          *reinterpret_cast<uint4*>(dst + (size_t)t * p.fbytes) = make_uint4(out[0], out[1], out[2], out[3]);
+        }
+      }
+    }
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // staging reads -> next bulk copy
+    __syncthreads();
+    if (threadIdx.x == 0 && sl + 2 < nslab) issue(sl + 2);
+  }
+}
+
 // Publish band u of this launch (epoch): its A rows are in global memory.
 __device__ __forceinline__ void publish_band(const PairParams& p, int u) {
   asm volatile("fence.proxy.async.global;" ::: "memory");  // TMA-stored rows -> generic release
@@ -453,7 +601,7 @@ __global__ void __launch_bounds__(kPairThreads, 1)
   uint64_t* tempty = tfull + 2;           // [2] accumulator drained (leader: 16 epilogue warps)
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
   uint32_t* mtab = tmem_slot + 4;  // [kMaxBlk][2]: per tap, A shift and B offset (16-byte units)
-  uint64_t* pbar = reinterpret_cast<uint64_t*>(mtab + 2 * kMaxBlk);  // [4] pack: x box landed
+  uint64_t* pbar = reinterpret_cast<uint64_t*>(mtab + 2 * kMaxBlk);  // [6] pack: x boxes [0,4), w slabs [4,6)
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t rank = cluster_ctarank();
@@ -478,7 +626,7 @@ __global__ void __launch_bounds__(kPairThreads, 1)
       mbar_init(tfull + s, 1);
       mbar_init(tempty + s, 2 * 8);
     }
-    for (int i = 0; i < 4; ++i) mbar_init(pbar + i, 1);
+    for (int i = 0; i < 6; ++i) mbar_init(pbar + i, 1);
     fence_barrier_init();
   }
   if (warp == 1) tmem_alloc2(tmem_slot, (uint32_t)p.tmem_cols);
@@ -487,6 +635,17 @@ __global__ void __launch_bounds__(kPairThreads, 1)
   // phase 1: packing (all warps); the window ring and filter area are the staging buffer.
   // The filter slices meet on the grid counter *fcount; every band of A is published
   // on its own flag, so a tile's window waits only for the bands it reads.
+  if (p.fsmem == 2 && threadIdx.x == 0) {
+    // w (read by every CTA later) into L2 now: each CTA prefetches one slice
+    const size_t wb = (size_t)p.K * p.C * p.RS * 2;
+    const size_t per = ((wb + gridDim.x - 1) / gridDim.x + 15) & ~(size_t)15;
+    const size_t off = (size_t)blockIdx.x * per;
+    if (off < wb) {
+      const uint32_t n = (uint32_t)min(per, wb - off);
+      asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(static_cast<const char*>(p.w) + off), "r"(n)
+                   : "memory");
+    }
+  }
   if (p.pack_tma) {
     // the first band's input boxes fly while the filter is packed
     const bool first = (int)blockIdx.x < p.nunits;
@@ -500,13 +659,25 @@ __global__ void __launch_bounds__(kPairThreads, 1)
         for (int bx = 0; bx < p.Cp / 64; ++bx) pack_load<IoT>(p, &tmX, sF, pbar, u, bx);
       }
     }
-    if (!(p.dbg & 2)) pair_pack<IoT>(p, nullptr, false);  // dbg&2: no packing (timing experiments only)
-    __syncthreads();
-    if (threadIdx.x == 0) {
-      __threadfence();
-      atomicAdd(p.fcount, 1ull);
+    if (!p.fsmem) {
+      if (!(p.dbg & 2)) pair_pack<IoT>(p, nullptr, false);  // dbg&2: no packing (timing experiments only)
+      __syncthreads();
+      if (threadIdx.x == 0) {
+        __threadfence();
+        atomicAdd(p.fcount, 1ull);
+      }
     }
     pair_pack_x_tma<IoT>(p, sF, pbar, &tmX, &tmS, &tmS2, first);
+    if (p.fsmem) {
+      __syncthreads();  // the staging (filter area) is free: the bands' stores were read
+      if constexpr (std::is_same<IoT, __nv_bfloat16>::value) {
+        if (p.fsmem == 2) pair_filter_bulk(p, sF, sWin, pbar + 4, rank);
+        else pair_filter_smem<IoT>(p, sF, rank);
+      } else {
+        pair_filter_smem<IoT>(p, sF, rank);
+      }
+      if (trace && threadIdx.x == 0) g_pair_pk[blockIdx.x * 4] = global_ns();
+    }
   } else {
     if (!(p.dbg & 2)) pair_pack<IoT>(p, reinterpret_cast<uint16_t*>(sF), true);
     __syncthreads();
@@ -533,7 +704,7 @@ __global__ void __launch_bounds__(kPairThreads, 1)
     const uint32_t lead_ffull = mapa_rank0(smem_u32(ffull));
     const uint32_t sW0 = smem_u32(sWin), sF0 = smem_u32(sF);
     const int half = p.NN / 2;
-    if (lane == 0) {
+    if (lane == 0 && !p.fsmem) {
       // every CTA's slice of the packed filter is in global memory
       unsigned long long v;
       uint64_t t0 = 0;
@@ -603,7 +774,7 @@ __global__ void __launch_bounds__(kPairThreads, 1)
           for (int b = 0; b < p.nbox; ++b)
             tma_load_2d_pair(sW0 + (uint32_t)slot * p.wbytes + (uint32_t)(b * p.box_rows * p.row_bytes), &tmA,
                              lead_wfull + 8u * (uint32_t)slot, ch * p.kc, g0 + b * p.box_rows);
-          if (lt == 0 && !(p.dbg & 64)) {  // this chunk's filter blocks: loaded once, resident
+          if (lt == 0 && !(p.dbg & 64) && !p.fsmem) {  // this chunk's filter blocks: loaded once, resident
             for (int tap = 0; tap < p.RS; ++tap) {
               const int blk = ch * p.RS + tap;
               if (rank == 0) mbar_arrive_expect_tx(ffull + blk, 2u * p.fbytes);
@@ -642,7 +813,7 @@ __global__ void __launch_bounds__(kPairThreads, 1)
           if (!(p.dbg & 4)) mbar_wait_cl(wfull + slot, (uint32_t)((wi / p.ring) & 1));
           tc_fence_after();
           if (trace && lane == 0 && wi < 4) tr[3 + wi] = global_ns();
-          if (lt == 0 && !(p.dbg & 4)) {  // this chunk's filter blocks (first tile only; then resident)
+          if (lt == 0 && !(p.dbg & 4) && !p.fsmem) {  // this chunk's filter blocks (first tile only; then resident)
             for (int tap = 0; tap < p.RS; ++tap) mbar_wait_cl(ffull + ch * p.RS + tap, 0u);
             tc_fence_after();
             if (trace && lane == 0 && ci == p.nchunks - 1) tr[12] = global_ns();
@@ -967,6 +1138,14 @@ cudaError_t prepare_mac_pair(PairLaunchState& S, const Geom& g, const PairTiling
   p = PairParams{};
   p.x = x; p.w = w; p.A = A; p.U = U; p.y = y;
   p.tr = t.tr; p.tpi = t.tpi; p.ntile = t.ntile; p.epi_tma = t.epi_tma;
+  p.fsmem = (t.pack_tma && getenv("POLYCONV_PAIR_FSMEM")) ? atoi(getenv("POLYCONV_PAIR_FSMEM")) : 0;
+  {
+    // bulk-copied w slabs: two buffers of frows rows in the window ring + epilogue area
+    const long long rowb = (long long)g.C * g.R * g.S * 2;
+    const long long avail = (long long)t.ring * t.wbytes + t.estage_bytes;
+    p.frows = (int)std::min<long long>(32, avail / (2 * rowb));
+    if (p.fsmem == 2 && (!io_bf16 || p.frows < 1 || rowb % 16 != 0)) p.fsmem = 1;
+  }
   p.estage_bytes = (uint32_t)t.estage_bytes;
   p.ftpi.init((uint32_t)t.tpi);
   p.pack_tma = t.pack_tma; p.ne_box = t.ne_box; p.last_rows = t.last_rows;
