@@ -103,7 +103,8 @@ struct PairParams {
 constexpr int kTr = 16;
 __device__ unsigned long long g_pair_trace[160 * kTr];
 __device__ unsigned long long g_pair_clk[160 * 2];
-__device__ unsigned long long g_pair_pk[160 * 4];  // pack sub-phases: filter done, band staged, band written  // clock64 at tr[0] and tr[13]: SM clock = cycles / ns
+__device__ unsigned long long g_pair_pk[160 * 4];
+__device__ unsigned long long g_pair_iss[160 * 4];  // issuer, tile 0: chunk c filter ready [2c], MMAs issued [2c+1]  // pack sub-phases: filter done, band staged, band written  // clock64 at tr[0] and tr[13]: SM clock = cycles / ns
 
 // ---- pair-specific PTX ---------------------------------------------------------
 __device__ __forceinline__ uint32_t mapa_rank0(uint32_t local) {
@@ -777,6 +778,10 @@ __global__ void __launch_bounds__(kPairThreads, 1)
           if (lt == 0 && !(p.dbg & 64) && !p.fsmem) {  // this chunk's filter blocks: loaded once, resident
             for (int tap = 0; tap < p.RS; ++tap) {
               const int blk = ch * p.RS + tap;
+              if ((p.dbg & 256) && (blk & 1)) {  // timing experiment: half the filter traffic (wrong results)
+                if (rank == 0) mbar_arrive(ffull + blk);
+                continue;
+              }
               if (rank == 0) mbar_arrive_expect_tx(ffull + blk, 2u * p.fbytes);
               tma_load_2d_pair(sF0 + (uint32_t)blk * p.fbytes, &tmU, lead_ffull + 8u * (uint32_t)blk, ch * p.kc,
                                tap * p.NN + (int)rank * half + (pair % p.urep) * p.RS * p.NN);
@@ -818,6 +823,7 @@ __global__ void __launch_bounds__(kPairThreads, 1)
             tc_fence_after();
             if (trace && lane == 0 && ci == p.nchunks - 1) tr[12] = global_ns();
           }
+          if (trace && lane == 0 && lt == 0 && ci < 2) g_pair_iss[blockIdx.x * 4 + 2 * ci] = global_ns();
           const uint64_t ad0 = make_sdesc(sW0 + (uint32_t)slot * p.wbytes, (uint32_t)p.row_bytes, 0);
           const uint64_t bd0 = make_sdesc(sF0 + (uint32_t)(ch * p.RS) * p.fbytes, (uint32_t)p.row_bytes, 0);
           for (int ti = 0; ti < p.RS; ++ti) {
@@ -834,6 +840,7 @@ __global__ void __launch_bounds__(kPairThreads, 1)
             }
             __syncwarp();
           }
+          if (trace && lane == 0 && lt == 0 && ci < 2) g_pair_iss[blockIdx.x * 4 + 2 * ci + 1] = global_ns();
           if (elect_one()) umma2_commit_both(wempty + slot);  // window slot free in both CTAs
           __syncwarp();
         }
@@ -1241,6 +1248,9 @@ cudaError_t launch_mac_pair(const Geom& g, const PairTiling& t, const void* x, c
 
 // Debug only (not part of include/polyconv.h): the per-CTA phase trace of the
 // last POLYCONV_PAIR_DEBUG&8 launch (160 x 16 u64).
+extern "C" int polyconv_dbg_pair_iss(unsigned long long* host) {
+  return (int)cudaMemcpyFromSymbol(host, polyconv::g_pair_iss, sizeof(unsigned long long) * 160 * 4);
+}
 extern "C" int polyconv_dbg_pair_pk(unsigned long long* host) {
   return (int)cudaMemcpyFromSymbol(host, polyconv::g_pair_pk, sizeof(unsigned long long) * 160 * 4);
 }

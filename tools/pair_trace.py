@@ -12,12 +12,13 @@ plan = pc.Plan(x.shape, w.shape, shape.stride, shape.padding, math="bf16", io_dt
 print(plan.info())
 lib = pc.load_library()
 buf = (ctypes.c_ulonglong * (160 * 16))()
-flush = torch.empty(64 << 20, device="cuda")
-evict = torch.empty(64 << 20, device="cuda")
+flush = torch.empty(64 << 20, device="cuda")  # 256 MiB (float32), as bench.py
+evict = torch.empty(64 << 20, device="cuda")  # 256 MiB: no dirty flush lines remain
 os.environ["POLYCONV_PAIR_DEBUG"] = str(8 | (int(sys.argv[1]) if len(sys.argv) > 1 else 0))
 for it in range(3):
-    flush.zero_()
-    evict.sum()
+    if os.environ.get("FLUSH", "1") == "1":
+        flush.zero_()
+        evict.sum()
     y = plan.forward(x, w)
     torch.cuda.synchronize()
 os.environ["POLYCONV_PAIR_DEBUG"] = "0"
@@ -47,6 +48,16 @@ pk = (ctypes.c_ulonglong * (160 * 4))()
 lib.polyconv_dbg_pair_pk(pk)
 k = np.array(pk, dtype=np.float64).reshape(160, 4)[: len(a)]
 for col, nm in enumerate(["pk_filter_done", "pk_band_staged", "pk_band_written", "pk_band_gathered"]):
+    v = k[:, col]
+    v = v[v > 0]
+    if len(v):
+        rel = (v - t0) / 1e3
+        print("  %-16s n=%3d min %7.2f  med %7.2f  max %7.2f us" % (nm, len(v), rel.min(), np.median(rel), rel.max()))
+
+iss = (ctypes.c_ulonglong * (160 * 4))()
+lib.polyconv_dbg_pair_iss(iss)
+k = np.array(iss, dtype=np.float64).reshape(160, 4)[: len(a)]
+for col, nm in enumerate(["iss_c0_filter", "iss_c0_issued", "iss_c1_filter", "iss_c1_issued"]):
     v = k[:, col]
     v = v[v > 0]
     if len(v):
