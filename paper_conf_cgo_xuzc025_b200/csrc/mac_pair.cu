@@ -88,6 +88,7 @@ struct PairParams {
   // ntile CTA tiles in all); epilogue by TMA stores of [32 channels][tr*Q pixels]
   // boxes staged in shared memory (epi_tma) or by direct stores
   int tr, tpi, ntile, epi_tma;
+  int warm;   // warm-up MMA chunk at launch (code path + tensor pipe)
   int fsmem;  // a3 straight into shared memory after the band packing (no global U, no counter):
               // 1 = loads from w, 2 = bulk-copied slabs of frows rows of w
   int frows;
@@ -582,6 +583,28 @@ __device__ __forceinline__ void pair_pack_x_tma(const PairParams& p, uint8_t* st
   }
 }
 
+// One channel chunk's MMAs (all taps, all K-steps): the whole warp runs the loop,
+// one elected lane issues.  Out of line so that the warm-up issue at launch and
+// every later chunk execute the same instructions (after an L2 flush the first
+// execution of a code path otherwise waits for instruction fetches from DRAM).
+__device__ __noinline__ void issue_chunk(uint32_t d_tmem, uint64_t ad0, uint64_t bd0, const uint32_t* mtab, int RS,
+                                         int ksteps, uint32_t idesc, uint32_t acc_first) {
+  for (int ti = 0; ti < RS; ++ti) {
+    const uint64_t ad = ad0 + mtab[2 * ti], bd = bd0 + mtab[2 * ti + 1];
+    const uint32_t acc0 = (acc_first | (uint32_t)ti) != 0 ? 1u : 0u;
+    if (elect_one()) {
+      umma2_f16(d_tmem, ad, bd, idesc, acc0);
+      // K step = 32 bytes = +2 in the start field
+      if (ksteps > 1) umma2_f16(d_tmem, ad + 2, bd + 2, idesc, 1u);
+      if (ksteps > 2) {
+        umma2_f16(d_tmem, ad + 4, bd + 4, idesc, 1u);
+        umma2_f16(d_tmem, ad + 6, bd + 6, idesc, 1u);
+      }
+    }
+    __syncwarp();
+  }
+}
+
 template <typename IoT>
 __global__ void __launch_bounds__(kPairThreads, 1)
     mac_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmU,
@@ -630,8 +653,29 @@ __global__ void __launch_bounds__(kPairThreads, 1)
     for (int i = 0; i < 6; ++i) mbar_init(pbar + i, 1);
     fence_barrier_init();
   }
-  if (warp == 1) tmem_alloc2(tmem_slot, (uint32_t)p.tmem_cols);
+  if (warp == 1) {
+    tmem_alloc2(tmem_slot, (uint32_t)p.tmem_cols);
+    // descriptor offsets per tap, so that the issue loop is a few uniform adds per
+    // tap (divisions in it left the tensor pipe idle)
+    for (int ti = lane; ti < p.RS; ti += 32) {
+      const int i = ti / p.S, j = ti - (ti / p.S) * p.S;
+      mtab[2 * ti] = ((uint32_t)(p.Wp * i + j) * (uint32_t)p.row_bytes) >> 4;
+      mtab[2 * ti + 1] = ((uint32_t)ti * p.fbytes) >> 4;
+    }
+  }
   __syncthreads();  // pbar initialised
+  if (p.warm) {
+    // Warm-up: one chunk of MMAs on whatever shared memory holds, into accumulator 1
+    // (the first tile that uses it starts with accumulate = 0), so the issue path is
+    // fetched and the tensor pipe started while the packing runs.  The pair's TMEM
+    // must be allocated in both CTAs first.
+    tc_fence_before();
+    cluster_sync();
+    tc_fence_after();
+    if (warp == 1 && rank == 0)
+      issue_chunk(*tmem_slot + (uint32_t)p.NN, make_sdesc(smem_u32(sWin), (uint32_t)p.row_bytes, 0),
+                  make_sdesc(smem_u32(sF), (uint32_t)p.row_bytes, 0), mtab, p.RS, p.row_bytes / 32, p.idesc, 0u);
+  }
 
   // phase 1: packing (all warps); the window ring and filter area are the staging buffer.
   // The filter slices meet on the grid counter *fcount; every band of A is published
@@ -797,21 +841,19 @@ __global__ void __launch_bounds__(kPairThreads, 1)
     if (rank == 0) {
       const uint32_t sW0 = smem_u32(sWin), sF0 = smem_u32(sF);
       const int ksteps = p.row_bytes / 32;
-      // descriptor offsets per tap, so that the issue loop is a few uniform adds
-      // per tap (divisions in it left the tensor pipe idle)
-      for (int ti = lane; ti < p.RS; ti += 32) {
-        const int tap = ti;
-        const int i = tap / p.S, j = tap - (tap / p.S) * p.S;
-        mtab[2 * ti] = ((uint32_t)(p.Wp * i + j) * (uint32_t)p.row_bytes) >> 4;
-        mtab[2 * ti + 1] = ((uint32_t)tap * p.fbytes) >> 4;
-      }
-      __syncwarp();
       int wi = 0, lt = 0;
       for (int t = pair; t < p.num_tiles; t += p.num_pairs, ++lt) {
         const int a = lt & 1;
         if (!(p.dbg & 4)) mbar_wait_cl(tempty + a, (uint32_t)((lt >> 1) & 1) ^ 1u);  // dbg&4: no waits (timing)
         tc_fence_after();
         const uint32_t d_tmem = tmem_base + (uint32_t)(a * p.NN);
+        if (lt == 0 && (p.dbg & 1024) && !p.fsmem) {
+          // timing experiment: the whole first tile's operands resident before any MMA
+          // (TMA writes into shared memory are starved while the MMAs read it)
+          for (int b = 0; b < p.nblk; ++b) mbar_wait_cl(ffull + b, 0u);
+          for (int c = 0; c < p.nchunks && c < p.ring; ++c) mbar_wait_cl(wfull + c, 0u);
+          tc_fence_after();
+        }
         for (int ci = 0; ci < p.nchunks; ++ci, ++wi) {
           const int ch = ci;  // the producer's order
           const int slot = wi % p.ring;
@@ -826,20 +868,7 @@ __global__ void __launch_bounds__(kPairThreads, 1)
           if (trace && lane == 0 && lt == 0 && ci < 2) g_pair_iss[blockIdx.x * 4 + 2 * ci] = global_ns();
           const uint64_t ad0 = make_sdesc(sW0 + (uint32_t)slot * p.wbytes, (uint32_t)p.row_bytes, 0);
           const uint64_t bd0 = make_sdesc(sF0 + (uint32_t)(ch * p.RS) * p.fbytes, (uint32_t)p.row_bytes, 0);
-          for (int ti = 0; ti < p.RS; ++ti) {
-            const uint64_t ad = ad0 + mtab[2 * ti], bd = bd0 + mtab[2 * ti + 1];
-            const uint32_t acc0 = (ci | ti) != 0 ? 1u : 0u;
-            if (elect_one()) {
-              umma2_f16(d_tmem, ad, bd, p.idesc, acc0);
-              // K step = 32 bytes = +2 in the start field
-              if (ksteps > 1) umma2_f16(d_tmem, ad + 2, bd + 2, p.idesc, 1u);
-              if (ksteps > 2) {
-                umma2_f16(d_tmem, ad + 4, bd + 4, p.idesc, 1u);
-                umma2_f16(d_tmem, ad + 6, bd + 6, p.idesc, 1u);
-              }
-            }
-            __syncwarp();
-          }
+          issue_chunk(d_tmem, ad0, bd0, mtab, p.RS, ksteps, p.idesc, (uint32_t)ci);
           if (trace && lane == 0 && lt == 0 && ci < 2) g_pair_iss[blockIdx.x * 4 + 2 * ci + 1] = global_ns();
           if (elect_one()) umma2_commit_both(wempty + slot);  // window slot free in both CTAs
           __syncwarp();
@@ -1145,6 +1174,7 @@ cudaError_t prepare_mac_pair(PairLaunchState& S, const Geom& g, const PairTiling
   p = PairParams{};
   p.x = x; p.w = w; p.A = A; p.U = U; p.y = y;
   p.tr = t.tr; p.tpi = t.tpi; p.ntile = t.ntile; p.epi_tma = t.epi_tma;
+  p.warm = getenv("POLYCONV_PAIR_WARM") ? atoi(getenv("POLYCONV_PAIR_WARM")) : 0;
   p.fsmem = (t.pack_tma && getenv("POLYCONV_PAIR_FSMEM")) ? atoi(getenv("POLYCONV_PAIR_FSMEM")) : 0;
   {
     // bulk-copied w slabs: two buffers of frows rows in the window ring + epilogue area
