@@ -7,7 +7,8 @@
 //   p[base + L_U - 1] = sum_c sum_{i,j} A_{n,c}[base + Wp*i + j] * U_{k,c}[e(i,j)]
 // and stores the ones on the extraction lattice (Eq. 12 + R4) into NCHW y.
 //
-// CTA tile: 64 output channels x 256 consecutive degrees; 8 warps, warp w owns
+// CTA tile: 64 output channels x 256 consecutive degrees (two CTAs per SM: one
+// stages while the other computes); 8 warps, warp w owns
 // 8 channels, lane l owns 8 consecutive degrees (64 fp32 accumulators/thread).
 // Per channel chunk (8 channels) the CTA stages R windows of A (one per kernel
 // row i, starting at degree m0 + Wp*i) and the 8 x R*S x 64 filter
@@ -30,7 +31,7 @@ __host__ __device__ constexpr int phys(int q) { return q + (q >> 5) * 4; }  // b
 __host__ __device__ constexpr int winp_phys(int smax) { return phys(winp_for(smax) - 1) + 1; }
 
 template <int SMAX>
-__global__ void __launch_bounds__(NT, 1) mac_fp32_kernel(Geom g, const float* __restrict__ A,
+__global__ void __launch_bounds__(NT, 2) mac_fp32_kernel(Geom g, const float* __restrict__ A,
                                                          const float* __restrict__ U, int Kp, int Cp,
                                                          float* __restrict__ y) {
   constexpr int NV = nv_for(SMAX);
