@@ -83,7 +83,13 @@ typedef enum {
  * output channels per pair tile) with the filter resident in shared memory
  * and the extraction (a5) fused into its epilogue (bf16 math, K <= 256 and a
  * filter half that fits shared memory; polyconv_plan_set_kernel returns
- * POLYCONV_STATUS_BAD_PARAM otherwise);
+ * POLYCONV_STATUS_BAD_PARAM otherwise).  Its CTAs meet on plan-owned counters
+ * and flags, so the whole grid (one CTA per SM) must be co-resident: the launch
+ * checks the co-resident cluster capacity, and a grid that cannot make progress
+ * (SMs held by other work for > 0.5 s) traps and forward returns
+ * POLYCONV_STATUS_EXECUTION_FAILED instead of hanging.  One plan must not run
+ * two TC_PAIR forwards concurrently on different streams (the counters are
+ * per plan);
  * FP32 = SIMT register-blocked FFMA; THIN = warp-per-output with shuffle
  * reduction over C*R*S (tiny channel counts). */
 typedef enum {
