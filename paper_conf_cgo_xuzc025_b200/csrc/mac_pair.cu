@@ -89,6 +89,11 @@ struct PairParams {
   // boxes staged in shared memory (epi_tma) or by direct stores
   int tr, tpi, ntile, epi_tma;
   int warm;   // warm-up MMA chunk at launch (code path + tensor pipe)
+  // direct0: every CTA builds its FIRST tile's windows in shared memory straight from x
+  // (one TMA box of ne_w plane elements x 64 channels per chunk, staged at sF + w0_off);
+  // the packed input A (bands) is written only for the images of later tiles, from u_img0 on
+  int direct0, ne_w, u_img0;
+  uint32_t w0_off;
   int fsmem;  // a3 straight into shared memory after the band packing (no global U, no counter):
               // 1 = loads from w, 2 = bulk-copied slabs of frows rows of w
   int frows;
@@ -489,7 +494,7 @@ __device__ __forceinline__ void publish_band(const PairParams& p, int u) {
 template <typename IoT>
 __device__ __forceinline__ void pack_load(const PairParams& p, const CUtensorMap* tmX, uint8_t* stage,
                                           uint64_t* pbar, int u, int bx) {
-  const int n = u / p.nb, b = u - (u / p.nb) * p.nb;
+  const int n = p.u_img0 + u / p.nb, b = u - (u / p.nb) * p.nb;
   const int r0 = b * p.rb;
   const int h0 = min(max(r0 - p.ph, 0), p.H);
   const uint32_t bytes = 64u * p.ne_box * (uint32_t)sizeof(IoT);
@@ -513,7 +518,7 @@ __device__ __forceinline__ void pair_pack_x_tma(const PairParams& p, uint8_t* st
   uint8_t* out = stage + p.in_bytes;
   int it = 0;
   for (int u = blockIdx.x; u < p.nunits; u += gridDim.x, ++it) {
-    const int n = u / p.nb, b = u - (u / p.nb) * p.nb;
+    const int n = p.u_img0 + u / p.nb, b = u - (u / p.nb) * p.nb;
     const int r0 = b * p.rb, r1 = min(p.Hp, r0 + p.rb);
     const int h0 = min(max(r0 - p.ph, 0), p.H), h1 = min(max(r1 - p.ph, 0), p.H);
     const bool any = h1 > h0 && !(p.dbg & 2);
@@ -583,6 +588,55 @@ __device__ __forceinline__ void pair_pack_x_tma(const PairParams& p, uint8_t* st
   }
 }
 
+// direct0: the x rows of this CTA's first tile, one TMA box per 64-channel chunk
+// (start rounded down to 16 bytes), into the staging at sF + w0_off
+template <typename IoT>
+__device__ __forceinline__ void w0_load(const PairParams& p, const CUtensorMap* tmX0, uint8_t* stage,
+                                        uint64_t* bar, int tn, int h0w, int c) {
+  const uint32_t bytes = 64u * p.ne_w * (uint32_t)sizeof(IoT);
+  mbar_arrive_expect_tx(bar, bytes);
+  tma_load_2d(stage + (size_t)c * bytes, tmX0, bar, (h0w * p.W) & ~(16 / (int)sizeof(IoT) - 1), tn * p.C + c * 64);
+}
+
+// direct0: window slot c of the first tile = rows m of the interleaved input polynomial
+// from coefficient g0 = tn*L_A + r_lo*Wp on (Eq. 10: coefficient r*Wp + s of A_{n,c}(t)
+// is xpad[n][c][r][s]), 64 channel words per row, 128-byte swizzled exactly as the TMA
+// writes a window; rows past the image (junk positions) are zero.
+template <typename IoT>
+__device__ __forceinline__ void w0_gather(const PairParams& p, const uint8_t* stage, uint8_t* slot, int r_lo, int h0w,
+                                          int c) {
+  const IoT* in = reinterpret_cast<const IoT*>(stage + (size_t)c * 64u * p.ne_w * sizeof(IoT));
+  const int eoff = (h0w * p.W) & (16 / (int)sizeof(IoT) - 1);
+  const int rows = p.nbox * p.box_rows;
+  const int cbase = c * 64;
+  for (int m = threadIdx.x; m < rows; m += blockDim.x) {
+    const int rr = (int)p.fWp.div((uint32_t)m);
+    const int r = r_lo + rr, h = r - p.ph, ww = m - rr * p.Wp - p.pw;
+    uint8_t* drow = slot + (size_t)m * 128;
+    const uint32_t sw = (uint32_t)(m & 7);
+    if (r < p.Hp && h >= 0 && h < p.H && ww >= 0 && ww < p.W) {
+      const IoT* src = in + (h - h0w) * p.W + ww + eoff;
+#pragma unroll
+      for (int q8 = 0; q8 < 8; ++q8) {
+        const int c0 = cbase + q8 * 8;
+        uint32_t v[4];
+#pragma unroll
+        for (int mm = 0; mm < 4; ++mm) {
+          const int cc = c0 + 2 * mm;
+          const uint32_t lo = cc < p.C ? (uint32_t)to_bf16_bits<IoT>(src[(q8 * 8 + 2 * mm) * p.ne_w]) : 0u;
+          const uint32_t hi = cc + 1 < p.C ? (uint32_t)to_bf16_bits<IoT>(src[(q8 * 8 + 2 * mm + 1) * p.ne_w]) : 0u;
+          v[mm] = lo | (hi << 16);
+        }
+        *reinterpret_cast<uint4*>(drow + (((uint32_t)q8 ^ sw) << 4)) = make_uint4(v[0], v[1], v[2], v[3]);
+      }
+    } else {
+#pragma unroll
+      for (int q8 = 0; q8 < 8; ++q8)
+        *reinterpret_cast<uint4*>(drow + (((uint32_t)q8 ^ sw) << 4)) = make_uint4(0u, 0u, 0u, 0u);
+    }
+  }
+}
+
 // One channel chunk's MMAs (all taps, all K-steps): the whole warp runs the loop,
 // one elected lane issues.  Out of line so that the warm-up issue at launch and
 // every later chunk execute the same instructions (after an L2 flush the first
@@ -610,7 +664,7 @@ __global__ void __launch_bounds__(kPairThreads, 1)
     mac_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmU,
                     const __grid_constant__ CUtensorMap tmX, const __grid_constant__ CUtensorMap tmS,
                     const __grid_constant__ CUtensorMap tmS2, const __grid_constant__ CUtensorMap tmY,
-                    const PairParams p) {
+                    const __grid_constant__ CUtensorMap tmX0, const PairParams p) {
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw = smem_u32(smem_raw);
   uint8_t* smem = smem_raw + (((raw + 1023u) & ~1023u) - raw);
@@ -691,12 +745,21 @@ __global__ void __launch_bounds__(kPairThreads, 1)
                    : "memory");
     }
   }
+  // direct0: this CTA's first tile (CTA tile blockIdx.x) and the padded rows its windows read
+  const int w0_tn = (int)p.ftpi.div((uint32_t)blockIdx.x);
+  const int w0_rlo = ((int)blockIdx.x - w0_tn * p.tpi) * p.tr * p.sh;
+  const int w0_h0 = min(max(w0_rlo - p.ph, 0), p.H);
+  const bool w0_any = p.direct0 && (int)blockIdx.x < p.ntile && !(p.dbg & 2);
+  if (w0_any && threadIdx.x == 0) {
+    prefetch_tmap(&tmX0);
+    for (int c = 0; c < p.nchunks; ++c) w0_load<IoT>(p, &tmX0, sF + p.w0_off, pbar + 2 + c, w0_tn, w0_h0, c);
+  }
   if (p.pack_tma) {
     // the first band's input boxes fly while the filter is packed
     const bool first = (int)blockIdx.x < p.nunits;
     if (threadIdx.x == 0 && first && !(p.dbg & 2)) {
       const int u = (int)blockIdx.x;
-      const int n = u / p.nb, b = u - n * p.nb;
+      const int n = p.u_img0 + u / p.nb, b = u - (u / p.nb) * p.nb;
       const int r0 = b * p.rb, r1 = min(p.Hp, r0 + p.rb);
       const int h0 = min(max(r0 - p.ph, 0), p.H), h1 = min(max(r1 - p.ph, 0), p.H);
       if (h1 > h0) {
@@ -711,6 +774,14 @@ __global__ void __launch_bounds__(kPairThreads, 1)
         __threadfence();
         atomicAdd(p.fcount, 1ull);
       }
+    }
+    if (p.direct0) {
+      // the first tile's windows, straight into window slots 0 .. nchunks-1
+      for (int c = 0; c < p.nchunks; ++c) {
+        if (w0_any) mbar_wait(pbar + 2 + c, 0u);
+        w0_gather<IoT>(p, sF + p.w0_off, sWin + (size_t)c * p.wbytes, w0_any ? w0_rlo : p.Hp, w0_h0, c);
+      }
+      if (trace && threadIdx.x == 0) g_pair_pk[blockIdx.x * 4 + 3] = global_ns();
     }
     pair_pack_x_tma<IoT>(p, sF, pbar, &tmX, &tmS, &tmS2, first);
     if (p.fsmem) {
@@ -783,7 +854,8 @@ __global__ void __launch_bounds__(kPairThreads, 1)
       const int ct = 2 * t + (int)rank;
       const int tn = (int)p.ftpi.div((uint32_t)ct), tb = ct - tn * p.tpi;
       const int g0 = tn * (int)p.L_A + tb * p.tr * p.sh * p.Wp;
-      if (tn < p.N) {
+      const bool direct = p.direct0 && lt == 0;  // windows already in shared memory (phase 1)
+      if (tn < p.N && !direct) {
         // the bands of image tn this tile's windows read (rows past the image are junk);
         // lane i polls band b_lo + i, so the flags' round trips overlap
         const int r_lo = tb * p.tr * p.sh, r_hi = min(p.Hp - 1, r_lo + wrows_img);
@@ -791,7 +863,7 @@ __global__ void __launch_bounds__(kPairThreads, 1)
         uint64_t t0 = 0;
         for (int b0 = 0; b0 < nbw; b0 += 32) {
           bool done = b0 + lane >= nbw;
-          const unsigned long long* f = p.bflag + tn * p.nb + b_lo + b0 + lane;
+          const unsigned long long* f = p.bflag + (tn - p.u_img0) * p.nb + b_lo + b0 + lane;
           while (!__all_sync(0xffffffffu, done)) {
             if (!done) {
               unsigned long long v;
@@ -814,11 +886,16 @@ __global__ void __launch_bounds__(kPairThreads, 1)
         const int ch = ci;
         const int slot = wi % p.ring;
         mbar_wait_cl(wempty + slot, (uint32_t)((wi / p.ring) & 1) ^ 1u, (p.dbg & 16) ? 500u : 0u);
-        if (elect_one()) {
+        if (direct) {
+          if (elect_one() && rank == 0) mbar_arrive(wfull + slot);  // built in phase 1 (cluster barrier since)
+        } else if (elect_one()) {
           if (rank == 0) mbar_arrive_expect_tx(wfull + slot, 2u * p.wbytes_tx);
           for (int b = 0; b < p.nbox; ++b)
             tma_load_2d_pair(sW0 + (uint32_t)slot * p.wbytes + (uint32_t)(b * p.box_rows * p.row_bytes), &tmA,
                              lead_wfull + 8u * (uint32_t)slot, ch * p.kc, g0 + b * p.box_rows);
+        }
+        __syncwarp();
+        if (elect_one()) {
           if (lt == 0 && !(p.dbg & 64) && !p.fsmem) {  // this chunk's filter blocks: loaded once, resident
             for (int tap = 0; tap < p.RS; ++tap) {
               const int blk = ch * p.RS + tap;
@@ -1072,35 +1149,59 @@ PairTiling pair_tiling(const Geom& g, int fmt, bool io_bf16, int num_sms) {
   if ((long long)t.Cp * t.spitch * 2 > stage_cap) return t;
   t.nb = (int)cdivp(g.Hp, t.rb);
   t.nunits = g.N * t.nb;
-  // TMA pack path: x band by one TMA box, A rows out by TMA stores (64-channel SW128 boxes)
+  // TMA pack path: x band by one TMA box, A rows out by TMA stores (64-channel SW128 boxes).
+  // direct0: the first round of tiles builds its windows in shared memory from x, so A is
+  // packed only for the images of later tiles (from u_img0 on), and the band staging
+  // shares the filter area with the first tile's x boxes.
   t.pack_tma = 0;
+  t.direct0 = 0;
+  t.u_img0 = 0;
   {
     const int eb_in = io_bf16 ? 2 : 4;
     const int ve = 16 / eb_in;
-    int nb2 = std::max(1, t.grid / g.N);
-    if (nb2 > g.Hp) nb2 = g.Hp;
-    int rb2 = (int)cdivp(g.Hp, nb2);
     const int rb_cap = std::min(256 / g.Wp, 256 / g.W);
-    if (rb2 > rb_cap) rb2 = rb_cap;
-    if (rb2 >= 1 && t.Cp % 64 == 0 && t.Cp <= 256 && ((long long)g.H * g.W * eb_in) % 16 == 0 &&
-        !getenv("POLYCONV_PAIR_PACK_LD")) {
+    const bool tma_ok = t.Cp % 64 == 0 && t.Cp <= 256 && ((long long)g.H * g.W * eb_in) % 16 == 0 &&
+                        !getenv("POLYCONV_PAIR_PACK_LD");
+    // the first tile's x rows: padded rows [r_lo, r_lo + rows_w) -> one box of ne_w elements
+    const int rows_w = (int)cdivp((long long)t.nbox * t.box_rows, g.Wp) + 1;
+    const int ne_w = (int)cdivp((long long)rows_w * g.W + ve - 1, ve) * ve;
+    const long long w0_b = (long long)t.nchunks * 64 * ne_w * eb_in;
+    const bool want_d0 = tma_ok && t.nchunks <= 2 && t.ring >= t.nchunks && ne_w <= 256 &&
+                         getenv("POLYCONV_PAIR_DIRECT0");  // measured no faster (filter waits for phase 1)
+    for (int d0 = want_d0 ? 1 : 0; d0 >= 0 && !t.pack_tma; --d0) {
+      const int img0 = d0 ? std::min(g.N, (2 * t.num_pairs) / t.tpi) : 0;
+      const int nimg = g.N - img0;
+      int nb2 = std::max(1, nimg > 0 ? t.grid / nimg : 1);
+      if (nb2 > g.Hp) nb2 = g.Hp;
+      int rb2 = (int)cdivp(g.Hp, nb2);
+      if (rb2 > rb_cap) rb2 = rb_cap;
+      if (rb2 < 1 || !tma_ok) continue;
       const int nbb = (int)cdivp(g.Hp, rb2);
       const int last = g.Hp - (nbb - 1) * rb2;
       const int ne_box = (int)cdivp((long long)rb2 * g.W + ve - 1, ve) * ve;  // + the start's rounding
       const long long in_b = cdivp((long long)(t.Cp / 64) * 64 * ne_box * eb_in, 1024) * 1024;
       const long long ob = cdivp((long long)rb2 * g.Wp * 128, 1024) * 1024;
       const long long ob2 = cdivp((long long)last * g.Wp * 128, 1024) * 1024;
-      if (ne_box <= 256 && in_b + (long long)(t.Cp / 64) * ob <= stage_cap) {
-        t.pack_tma = 1;
-        t.rb = rb2;
-        t.nb = nbb;
-        t.nunits = g.N * nbb;
-        t.last_rows = last;
-        t.ne_box = ne_box;
-        t.in_bytes = (int)in_b;
-        t.obox_bytes = (int)ob;
-        t.obox_bytes2 = (int)ob2;
+      const long long band_b = in_b + (long long)(t.Cp / 64) * std::max(ob, ob2);
+      if (ne_box > 256) continue;
+      if (d0) {
+        if (band_b + w0_b > fil) continue;  // both in the filter area (free during packing)
+      } else if (band_b > stage_cap) {
+        continue;
       }
+      t.pack_tma = 1;
+      t.direct0 = d0;
+      t.u_img0 = img0;
+      t.ne_w = ne_w;
+      t.w0_off = (int)band_b;
+      t.rb = rb2;
+      t.nb = nbb;
+      t.nunits = nimg * nbb;
+      t.last_rows = last;
+      t.ne_box = ne_box;
+      t.in_bytes = (int)in_b;
+      t.obox_bytes = (int)ob;
+      t.obox_bytes2 = (int)ob2;
     }
   }
   t.ok = true;
@@ -1116,7 +1217,7 @@ struct PairLaunchState {
   const void *x = nullptr, *w = nullptr, *y = nullptr, *A = nullptr, *U = nullptr;
   const unsigned long long* fcount = nullptr;
   bool io_bf16 = false, valid = false;
-  CUtensorMap tmA, tmU, tmX, tmS, tmS2, tmY;
+  CUtensorMap tmA, tmU, tmX, tmS, tmS2, tmY, tmX0;
   PairParams p;
 };
 
@@ -1170,11 +1271,29 @@ cudaError_t prepare_mac_pair(PairLaunchState& S, const Geom& g, const PairTiling
       return cudaErrorInvalidValue;
     }
   }
+  CUtensorMap& tmX0 = S.tmX0;
+  memset(&tmX0, 0, sizeof(tmX0));
+  if (t.direct0) {
+    EncodeTiledFnPair enc = get_encode_pair();
+    const int eb_in = io_bf16 ? 2 : 4;
+    cuuint64_t dims[2] = {(cuuint64_t)g.H * g.W, (cuuint64_t)g.N * g.C};
+    cuuint64_t strides[1] = {(cuuint64_t)g.H * g.W * eb_in};
+    cuuint32_t box[2] = {(cuuint32_t)t.ne_w, 64};
+    cuuint32_t estr[2] = {1, 1};
+    if (!enc || enc(&tmX0, io_bf16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2,
+                    const_cast<void*>(x), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                    CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS) {
+      snprintf(err, errlen, "mac_pair: cuTensorMapEncodeTiled (first-tile input) failed");
+      return cudaErrorInvalidValue;
+    }
+  }
   PairParams& p = S.p;
   p = PairParams{};
   p.x = x; p.w = w; p.A = A; p.U = U; p.y = y;
   p.tr = t.tr; p.tpi = t.tpi; p.ntile = t.ntile; p.epi_tma = t.epi_tma;
   p.warm = getenv("POLYCONV_PAIR_WARM") ? atoi(getenv("POLYCONV_PAIR_WARM")) : 0;
+  p.direct0 = t.direct0; p.ne_w = t.ne_w; p.u_img0 = t.u_img0; p.w0_off = (uint32_t)t.w0_off;
   p.fsmem = (t.pack_tma && getenv("POLYCONV_PAIR_FSMEM")) ? atoi(getenv("POLYCONV_PAIR_FSMEM")) : 0;
   {
     // bulk-copied w slabs: two buffers of frows rows in the window ring + epilogue area
@@ -1271,7 +1390,7 @@ cudaError_t launch_mac_pair(const Geom& g, const PairTiling& t, const void* x, c
   attr[0].val.clusterDim.z = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  return cudaLaunchKernelEx(&cfg, kern, S.tmA, S.tmU, S.tmX, S.tmS, S.tmS2, S.tmY, S.p);
+  return cudaLaunchKernelEx(&cfg, kern, S.tmA, S.tmU, S.tmX, S.tmS, S.tmS2, S.tmY, S.tmX0, S.p);
 }
 
 }  // namespace polyconv
