@@ -126,6 +126,7 @@ struct PairTiling {
   int tr, tpi, ntile;          // row-aligned CTA tiles: tr output rows of one image each
   int epi_tma, estage_bytes;   // epilogue staged in shared memory and written by TMA stores
   int direct0, ne_w, u_img0, w0_off;  // first tile's windows from x in shared memory; A from image u_img0
+  int split, pack_grid, pack_smem;    // packing in its own grid, the pair kernel its programmatic dependent
 };
 PairTiling pair_tiling(const Geom& g, int fmt, bool io_bf16, int num_sms);
 // One launch: packs w -> U [R*S][NN][Cp] and x -> A [N*L_A][Cp] (bf16, plan workspace),

@@ -94,6 +94,9 @@ struct PairParams {
   // the packed input A (bands) is written only for the images of later tiles, from u_img0 on
   int direct0, ne_w, u_img0;
   uint32_t w0_off;
+  // split: a2 + a3 run in a separate pack kernel (pair_pack_kernel) that this kernel
+  // follows as a programmatic dependent launch: no grid counter, no band flags
+  int split;
   int fsmem;  // a3 straight into shared memory after the band packing (no global U, no counter):
               // 1 = loads from w, 2 = bulk-copied slabs of frows rows of w
   int frows;
@@ -581,7 +584,7 @@ __device__ __forceinline__ void pair_pack_x_tma(const PairParams& p, uint8_t* st
     }
     if (tid == 0) {
       asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");  // written (before publishing / reuse)
-      publish_band(p, u);
+      if (!p.split) publish_band(p, u);
       if (ptr) g_pair_pk[blockIdx.x * 4 + 2] = global_ns();
     }
     __syncthreads();
@@ -635,6 +638,39 @@ __device__ __forceinline__ void w0_gather(const PairParams& p, const uint8_t* st
         *reinterpret_cast<uint4*>(drow + (((uint32_t)q8 ^ sw) << 4)) = make_uint4(0u, 0u, 0u, 0u);
     }
   }
+}
+
+// a2 + a3 as their own grid (split mode): every CTA packs a slice of the tap-major
+// filter U and one band of A (TMA in, transpose, TMA store); the pair kernel is its
+// programmatic dependent and starts its prologue as soon as every CTA here has begun.
+template <typename IoT>
+__global__ void __launch_bounds__(256) pair_pack_kernel(const __grid_constant__ CUtensorMap tmX,
+                                                        const __grid_constant__ CUtensorMap tmS,
+                                                        const __grid_constant__ CUtensorMap tmS2,
+                                                        const PairParams p) {
+  extern __shared__ uint8_t smem_raw[];
+  const uint32_t raw = smem_u32(smem_raw);
+  uint8_t* stage = smem_raw + (((raw + 1023u) & ~1023u) - raw);
+  __shared__ uint64_t pbar[4];
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < 4; ++i) mbar_init(pbar + i, 1);
+    fence_barrier_init();
+  }
+  __syncthreads();
+  const bool first = (int)blockIdx.x < p.nunits;
+  if (threadIdx.x == 0 && first) {
+    const int u = (int)blockIdx.x;
+    const int b = u - (u / p.nb) * p.nb;
+    const int r0 = b * p.rb, r1 = min(p.Hp, r0 + p.rb);
+    const int h0 = min(max(r0 - p.ph, 0), p.H), h1 = min(max(r1 - p.ph, 0), p.H);
+    if (h1 > h0) {
+      prefetch_tmap(&tmX);
+      for (int bx = 0; bx < p.Cp / 64; ++bx) pack_load<IoT>(p, &tmX, stage, pbar, u, bx);
+    }
+  }
+  pair_pack<IoT>(p, nullptr, false);
+  pair_pack_x_tma<IoT>(p, stage, pbar, &tmX, &tmS, &tmS2, first);
 }
 
 // One channel chunk's MMAs (all taps, all K-steps): the whole warp runs the loop,
@@ -745,6 +781,7 @@ __global__ void __launch_bounds__(kPairThreads, 1)
                    : "memory");
     }
   }
+  if (!p.split) {
   // direct0: this CTA's first tile (CTA tile blockIdx.x) and the padded rows its windows read
   const int w0_tn = (int)p.ftpi.div((uint32_t)blockIdx.x);
   const int w0_rlo = ((int)blockIdx.x - w0_tn * p.tpi) * p.tr * p.sh;
@@ -804,6 +841,7 @@ __global__ void __launch_bounds__(kPairThreads, 1)
         asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p.bflag + u), "l"(p.epoch) : "memory");
     }
   }
+  }  // !split
   // the staging area is overwritten by TMA (async proxy) next
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
   __syncthreads();
@@ -820,7 +858,13 @@ __global__ void __launch_bounds__(kPairThreads, 1)
     const uint32_t lead_ffull = mapa_rank0(smem_u32(ffull));
     const uint32_t sW0 = smem_u32(sWin), sF0 = smem_u32(sF);
     const int half = p.NN / 2;
-    if (lane == 0 && !p.fsmem) {
+    if (p.split) {
+      // the pack kernel (the programmatic-launch primary) has written A and U
+      asm volatile("griddepcontrol.wait;" ::: "memory");
+      asm volatile("fence.proxy.async.global;" ::: "memory");
+      if (trace && lane == 0) tr[2] = global_ns();
+    }
+    if (lane == 0 && !p.fsmem && !p.split) {
       // every CTA's slice of the packed filter is in global memory
       unsigned long long v;
       uint64_t t0 = 0;
@@ -855,7 +899,7 @@ __global__ void __launch_bounds__(kPairThreads, 1)
       const int tn = (int)p.ftpi.div((uint32_t)ct), tb = ct - tn * p.tpi;
       const int g0 = tn * (int)p.L_A + tb * p.tr * p.sh * p.Wp;
       const bool direct = p.direct0 && lt == 0;  // windows already in shared memory (phase 1)
-      if (tn < p.N && !direct) {
+      if (tn < p.N && !direct && !p.split) {
         // the bands of image tn this tile's windows read (rows past the image are junk);
         // lane i polls band b_lo + i, so the flags' round trips overlap
         const int r_lo = tb * p.tr * p.sh, r_hi = min(p.Hp - 1, r_lo + wrows_img);
@@ -1204,6 +1248,38 @@ PairTiling pair_tiling(const Geom& g, int fmt, bool io_bf16, int num_sms) {
       t.obox_bytes2 = (int)ob2;
     }
   }
+  // split: the packing runs as its own grid (pair_pack_kernel, several CTAs per SM,
+  // small bands), the pair kernel follows it as a programmatic dependent launch
+  t.split = 0;
+  if (t.pack_tma && !t.direct0 && getenv("POLYCONV_PAIR_SPLIT")) {  // measured no faster: off by default
+    const int eb_in = io_bf16 ? 2 : 4;
+    const int ve = 16 / eb_in;
+    const int rb_cap = std::min(256 / g.Wp, 256 / g.W);
+    int nb2 = std::max(1, (4 * num_sms) / g.N);
+    if (nb2 > g.Hp) nb2 = g.Hp;
+    int rb2 = std::max(1, std::min((int)cdivp(g.Hp, nb2), rb_cap));
+    const int nbb = (int)cdivp(g.Hp, rb2);
+    const int last = g.Hp - (nbb - 1) * rb2;
+    const int ne_box = (int)cdivp((long long)rb2 * g.W + ve - 1, ve) * ve;
+    const long long in_b = cdivp((long long)(t.Cp / 64) * 64 * ne_box * eb_in, 1024) * 1024;
+    const long long ob = cdivp((long long)rb2 * g.Wp * 128, 1024) * 1024;
+    const long long ob2 = cdivp((long long)last * g.Wp * 128, 1024) * 1024;
+    const long long band_b = in_b + (long long)(t.Cp / 64) * std::max(ob, ob2);
+    if (ne_box <= 256 && band_b + 1024 <= 100 * 1024 && (long long)g.N * nbb < (1LL << 30)) {
+      t.split = 1;
+      t.u_img0 = 0;
+      t.rb = rb2;
+      t.nb = nbb;
+      t.nunits = g.N * nbb;
+      t.last_rows = last;
+      t.ne_box = ne_box;
+      t.in_bytes = (int)in_b;
+      t.obox_bytes = (int)ob;
+      t.obox_bytes2 = (int)ob2;
+      t.pack_smem = (int)(band_b + 1024);
+      t.pack_grid = std::max(t.nunits, num_sms);
+    }
+  }
   t.ok = true;
   return t;
 }
@@ -1294,6 +1370,7 @@ cudaError_t prepare_mac_pair(PairLaunchState& S, const Geom& g, const PairTiling
   p.tr = t.tr; p.tpi = t.tpi; p.ntile = t.ntile; p.epi_tma = t.epi_tma;
   p.warm = getenv("POLYCONV_PAIR_WARM") ? atoi(getenv("POLYCONV_PAIR_WARM")) : 0;
   p.direct0 = t.direct0; p.ne_w = t.ne_w; p.u_img0 = t.u_img0; p.w0_off = (uint32_t)t.w0_off;
+  p.split = t.split;
   p.fsmem = (t.pack_tma && getenv("POLYCONV_PAIR_FSMEM")) ? atoi(getenv("POLYCONV_PAIR_FSMEM")) : 0;
   {
     // bulk-copied w slabs: two buffers of frows rows in the window ring + epilogue area
@@ -1329,6 +1406,11 @@ cudaError_t prepare_mac_pair(PairLaunchState& S, const Geom& g, const PairTiling
   auto kern = io_bf16 ? mac_pair_kernel<__nv_bfloat16> : mac_pair_kernel<float>;
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, t.smem_bytes);
   if (e != cudaSuccess) return e;
+  if (t.split) {
+    auto pk = io_bf16 ? pair_pack_kernel<__nv_bfloat16> : pair_pack_kernel<float>;
+    e = cudaFuncSetAttribute(pk, cudaFuncAttributeMaxDynamicSharedMemorySize, t.pack_smem);
+    if (e != cudaSuccess) return e;
+  }
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)t.grid);
   cfg.blockDim = dim3(kPairThreads);
@@ -1377,19 +1459,31 @@ cudaError_t launch_mac_pair(const Geom& g, const PairTiling& t, const void* x, c
   S.p.epoch = epoch;
   const char* dbg = getenv("POLYCONV_PAIR_DEBUG");
   S.p.dbg = dbg ? atoi(dbg) : 0;
+  if (t.split) {
+    auto pk = io_bf16 ? pair_pack_kernel<__nv_bfloat16> : pair_pack_kernel<float>;
+    cudaLaunchConfig_t pc = {};
+    pc.gridDim = dim3((unsigned)t.pack_grid);
+    pc.blockDim = dim3(256);
+    pc.dynamicSmemBytes = (size_t)t.pack_smem;
+    pc.stream = st;
+    cudaError_t e = cudaLaunchKernelEx(&pc, pk, S.tmX, S.tmS, S.tmS2, S.p);
+    if (e != cudaSuccess) return e;
+  }
   auto kern = io_bf16 ? mac_pair_kernel<__nv_bfloat16> : mac_pair_kernel<float>;
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)t.grid);
   cfg.blockDim = dim3(kPairThreads);
   cfg.dynamicSmemBytes = (size_t)t.smem_bytes;
   cfg.stream = st;
-  cudaLaunchAttribute attr[1];
+  cudaLaunchAttribute attr[2];
   attr[0].id = cudaLaunchAttributeClusterDimension;
   attr[0].val.clusterDim.x = 2;
   attr[0].val.clusterDim.y = 1;
   attr[0].val.clusterDim.z = 1;
+  attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[1].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
-  cfg.numAttrs = 1;
+  cfg.numAttrs = t.split ? 2 : 1;
   return cudaLaunchKernelEx(&cfg, kern, S.tmA, S.tmU, S.tmX, S.tmS, S.tmS2, S.tmY, S.tmX0, S.p);
 }
 

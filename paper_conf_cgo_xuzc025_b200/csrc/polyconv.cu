@@ -293,7 +293,8 @@ polyconv_status_t polyconv_plan_info(polyconv_plan_t p, polyconv_info_t* info) {
       info->tile_m = p->tc2.nt; info->tile_n = 128; info->stages = p->tc2.a_stages;
       info->launches = p->kernel == POLYCONV_KERNEL_TC_FUSED ? 1 : 2; break;
     case POLYCONV_KERNEL_TC_PAIR:  // pair tile = 256 positions x NN output channels
-      info->tile_m = 256; info->tile_n = p->pair.NN; info->stages = p->pair.ring; info->launches = 1; break;
+      info->tile_m = 256; info->tile_n = p->pair.NN; info->stages = p->pair.ring;
+      info->launches = p->pair.split ? 2 : 1; break;
     case POLYCONV_KERNEL_TC_PERTAP:
       info->tile_m = p->tc.bm; info->tile_n = p->tc.bn; info->stages = p->tc.stages; info->launches = 2; break;
     case POLYCONV_KERNEL_FP32:
