@@ -396,6 +396,7 @@ def bench_cudnn(torch, x, w, shape, math, flush, K, world, dist):
     torch.backends.cudnn.benchmark = True
     torch.backends.cudnn.allow_tf32 = math == "tf32"
     best = None
+    by_layout = {}
     for layout in ("nchw", "channels_last"):
         xx, ww = (x, w) if layout == "nchw" else (x.contiguous(memory_format=torch.channels_last),
                                                    w.contiguous(memory_format=torch.channels_last))
@@ -413,10 +414,14 @@ def bench_cudnn(torch, x, w, shape, math, flush, K, world, dist):
         if world > 1:
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
         v = shape.flops() * world / (float(t) * 1e-3) / 1e12
+        by_layout[layout] = {"value": v, "ms_per_step": float(t)}
         if best is None or v > best["value"]:
             best = {"value": v, "unit": UNIT, "ms_per_step": float(t), "layout": layout,
                     "library": "cuDNN %s via torch.nn.functional.conv2d (benchmark=True)" %
                     torch.backends.cudnn.version()}
+    # nchw = the same NCHW tensors this library takes; channels_last = cuDNN's preferred
+    # layout (input converted outside the timed region)
+    best["by_layout"] = by_layout
     return best
 
 
