@@ -1068,7 +1068,8 @@ __global__ void __launch_bounds__(kPairThreads, 1)
       }
       if (trace && threadIdx.x == kEpi0 * 32 && lt < 1) tr[10 + 2 * lt] = global_ns();
     }
-    if (p.epi_tma && (e & 3) == 0 && lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+    // the staging must outlive the stores' reads; the writes themselves complete with the grid
+    if (p.epi_tma && (e & 3) == 0 && lane == 0) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
   }
 
   tc_fence_before();
