@@ -120,7 +120,11 @@ int main() {
     }
   };
   struct Var { const char* name; int box_e, box_c, swz, bulk, ring; };
-  std::vector<Var> vars = {{"mx: box 64el x 64ch sw128 ring6", 64, 64, 1, 0, 6},
+  const bool noflush = getenv("NOFLUSH") != nullptr;  // x L2-warm
+  printf("L2 %s between reps\n", noflush ? "NOT flushed" : "flushed");
+  std::vector<Var> vars = {{"box 232el x 64ch noswz ring2 (mac_pair)", 232, 64, 0, 0, 2},
+                           {"box 256el x 64ch noswz ring2 line-aligned", 256, 64, 0, 0, 2},
+                           {"mx: box 64el x 64ch sw128 ring6", 64, 64, 1, 0, 6},
                            {"mx: box 64el x 64ch sw128 ring12", 64, 64, 1, 0, 12},
                            {"box 256el x 32ch noswz ring8", 256, 32, 0, 0, 8},
                            {"box 256el x 16ch noswz ring12", 256, 16, 0, 0, 12},
@@ -150,7 +154,8 @@ int main() {
               }
             } else {
               for (int cc = 0; cc < 64; cc += v.box_c)
-                for (int e = elo; e < ehi; e += v.box_e) items.push_back({e, n * C + ch * 64 + cc});
+                for (int e = (v.box_e == 256 && v.box_c == 64) ? (elo & ~63) : elo; e < ehi; e += v.box_e)
+                  items.push_back({e, n * C + ch * 64 + cc});
             }
           }
       }
@@ -175,7 +180,7 @@ int main() {
     std::vector<float> ts;
     double spread = 0, medend = 0;
     for (int rep = 0; rep < 12; ++rep) {
-      flush_kernel<<<1184, 256>>>(fl, fn, sink);
+      if (!noflush) flush_kernel<<<1184, 256>>>(fl, fn, sink);
       cudaEventRecord(e0);
       ring_load<<<nsm, 64, v.ring * slot + 2048>>>(tm, x, ditems, dstart, v.ring, slot, box_bytes, v.bulk ? 1 : 0,
                                                    tout);
