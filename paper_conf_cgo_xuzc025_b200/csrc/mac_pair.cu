@@ -12,30 +12,36 @@
 // Design (DESIGN.md §4 "mac_pair"):
 //  * Phase 1 (every CTA, all warps): pack a slice of the filter into the
 //    tap-major layout U[R*S][NN][Cp] (a3: the nonzero coefficients of the
-//    reversed, gap-padded U_{k,c}(t), Eq. 6, grouped by degree e(i,j)) and a
-//    band of images rows into the channel-interleaved input polynomial
-//    A[N*L_A][Cp] (a2: coefficient r*Wp + s of A_{n,c}(t) = xpad[n][c][r][s],
-//    Eq. 10 + zero padding P.1353-1356), converted to BF16 (RNE, reading R11).
-//    The packed copies are written to the plan workspace (they stay in L2);
-//    the CTAs then meet on a grid counter (all CTAs are co-resident: one per
-//    SM, grid <= the co-resident cluster count).
-//  * Phase 2 (CTA pairs): UMMA M = 256 positions (128 per CTA: A operand =
-//    a window of the interleaved input, K-major, loaded by TMA), N = NN output
-//    channels (B operand = the filter, each CTA holding NN/2 rows of every
-//    (tap, channel chunk) block -- RESIDENT in shared memory for the whole
-//    kernel: loaded once, reused by every tile).  One window of
-//    128 + (R-1)*Wp + S-1 positions per channel chunk serves all R*S taps: each
-//    tap's MMA reads it through a descriptor whose start is shifted by
-//    (Wp*i + j) rows (tools/umma_probe.cu).  The leader CTA issues
-//    tcgen05.mma.cta_group::2; accumulators (fp32) live in TMEM, double
-//    buffered, so the epilogue of tile t overlaps the MMAs of tile t+1.
-//  * Epilogue (a5, fused): positions are TMEM lanes, so every warp-wide store
-//    of one output channel writes 32 consecutive output pixels (Eq. 12 /
-//    reading R4 extraction: y[n][k][oh][ow] = p[Wp*sh*oh + sw*ow + L_U - 1];
-//    positions off the lattice are junk and dropped).
+//    reversed, gap-padded U_{k,c}(t), Eq. 6, grouped by degree e(i,j)); the
+//    slices meet on a grid counter.  Then one band of rb padded rows of one
+//    image of the channel-interleaved input polynomial A[N*L_A][Cp] (a2:
+//    coefficient r*Wp + s of A_{n,c}(t) = xpad[n][c][r][s], Eq. 10 + zero
+//    padding P.1353-1356, BF16 RNE, reading R11): TMA boxes of the band's x
+//    rows (64 channel planes each), a shared-memory transpose into 128-byte
+//    swizzled rows, TMA stores, then the band is published on its own flag.
+//    The packed copies stay in L2.  All CTAs are co-resident (one per SM,
+//    checked when the launch is prepared).
+//  * Phase 2 (CTA pairs): UMMA M = 256 positions (128 per CTA = the TMEM lanes:
+//    a window of the interleaved input, K-major, TMA), N = NN output channels
+//    (B operand = the filter, each CTA holding NN/2 rows of every (chunk, tap)
+//    block -- RESIDENT in shared memory: loaded once, reused by every tile).
+//    One window of 128 + (R-1)*Wp + S-1 positions per channel chunk serves all
+//    R*S taps through descriptors shifted by (Wp*i + j) rows
+//    (tools/umma_probe.cu).  A window waits only for the bands it reads.  The
+//    leader CTA issues tcgen05.mma.cta_group::2 from a per-tap descriptor table;
+//    accumulators (fp32) live in TMEM, double buffered, so the epilogue of tile
+//    t overlaps the MMAs of tile t+1.  A CTA tile = tr output rows of one image.
+//  * Epilogue (a5, fused): positions are TMEM lanes; the Eq. 12 / reading R4
+//    extraction y[n][k][oh][ow] = p[Wp*sh*oh + sw*ow + L_U - 1] is a per-lane
+//    predicate; bf16 outputs are staged per channel half in shared memory and
+//    TMA-stored as [32 channels][tr*Q pixels] boxes of y viewed as [N*K][P*Q]
+//    (direct stores for f32 outputs or K % 32 != 0).
 //  * Warp roles: warp 0 = TMA producer, warp 1 = TMEM allocator + MMA issuer
 //    (leader CTA), warps 2..9 = epilogue (2 per TMEM lane quadrant, each half
 //    of the channels).  All ten warps pack in phase 1.
+//  * Experiment switches (DESIGN.md §4 table; off by default): split packing
+//    grid, direct first-tile windows, filter built in shared memory, warm-up
+//    MMA chunk, per-CTA phase trace.
 #include <cuda.h>
 #include <cstdio>
 #include <cstdlib>
