@@ -63,8 +63,12 @@ polyconv_status_t resolve(polyconv_plan_t p) {
   const bool tc_math = p->math != POLYCONV_MATH_FP32_FMA;
   if (k == POLYCONV_KERNEL_AUTO || k == POLYCONV_KERNEL_TC_PAIR) p->pair = pair_tiling(g, p->fmt, p->io_bf16, p->num_sms);
   if (k == POLYCONV_KERNEL_AUTO) {
-    if (tc_math && g.K >= 16 && p->pair.ok && !getenv("POLYCONV_NO_PAIR_DEFAULT"))
-      k = POLYCONV_KERNEL_TC_PAIR;  // bf16: one launch, CTA pairs, resident filter
+    // bf16, at most two rounds of pair tiles: one launch on CTA pairs with a resident filter
+    // (its fixed startup wins on small problems); larger problems pipeline better in mac_tc2
+    // (measured per layer: tools/layer_sweep.py)
+    if (tc_math && g.K >= 16 && p->pair.ok && p->pair.num_tiles <= 2 * p->pair.num_pairs &&
+        !getenv("POLYCONV_NO_PAIR_DEFAULT"))
+      k = POLYCONV_KERNEL_TC_PAIR;
     else if (tc_math && g.K >= 16 && tc2_supported(g, p->fmt) && p->io_bf16 && !getenv("POLYCONV_NO_FUSED_DEFAULT") &&
         tc2_is_mx(tc2_tiling(g, p->fmt, p->io_bf16, p->num_sms, true, p->io_bf16)))
       k = POLYCONV_KERNEL_TC_FUSED;  // bf16 in/out: one launch, input packed in-kernel
