@@ -40,6 +40,11 @@ cudaError_t launch_pack_filter_tapmajor(const Geom& g, const void* w, bool w_bf1
 cudaError_t launch_pack_both_interleaved(const Geom& g, const void* x, const void* w, bool io_bf16,
                                          void* xdst, void* wdst, int fmt, cudaStream_t st);
 
+// ---- polyphase.cu (stride s: phases of the padded input as channels, reading R4b) ----
+// xq [N][s*s*C][Hq][Wq] and wq [K][s*s*C][Rq][Sq] in the io dtype
+cudaError_t launch_polyphase(const Geom& g, int Hq, int Wq, int Rq, int Sq, const void* x, const void* w, void* xq,
+                             void* wq, bool io_bf16, cudaStream_t st);
+
 // ---- extract.cu -----------------------------------------------------------
 cudaError_t launch_extract(const Geom& g, const float* coeffs, void* y, bool y_bf16,
                            cudaStream_t st);

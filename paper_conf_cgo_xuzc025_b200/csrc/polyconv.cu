@@ -26,6 +26,12 @@ struct polyconv_plan_s {
   PairTiling pair;
   void* pair_state = nullptr;  // mac_pair launch cache
   unsigned long long* bflag = nullptr;  // mac_pair band flags [N * pair.nb]
+  // stride s >= 2 (reading R4b): the stride-1 inner plan over the input's s*s phases
+  polyconv_plan_s* inner = nullptr;
+  int Hq = 0, Wq = 0, Rq = 0, Sq = 0;
+  void* xq = nullptr;
+  void* wq = nullptr;
+  size_t xq_bytes = 0, wq_bytes = 0;
   // workspace (lazy)
   void* wsA = nullptr;
   size_t wsA_bytes = 0;
@@ -254,12 +260,49 @@ polyconv_status_t polyconv_plan(polyconv_plan_t* plan, int N, int C, int H, int 
     delete p;
     return POLYCONV_STATUS_BAD_PARAM;
   }
+  // stride s >= 2 with large kernels: the s*s phases of the padded input become channels
+  // and the convolution a stride-1 one of ceil(R/s) x ceil(S/s) kernels (polyphase.cu,
+  // reading R4b), so only the stride lattice is computed.  Measured per layer
+  // (tools/layer_sweep.py): the ResNet-50 7x7/s2 stem 14 -> 73 TFLOP/s; 3x3/s2 layers ran
+  // slower through their inner plans (phase planes of odd width have no TMA view), so the
+  // rule is R, S >= 5 (POLYCONV_POLYPHASE=1 forces it for any R, S >= 2, =0 disables it).
+  const char* pp_env = getenv("POLYCONV_POLYPHASE");
+  const int pp_min = pp_env ? (atoi(pp_env) == 0 ? 1 << 30 : 2) : 5;
+  if (sh == sw && sh >= 2 && R >= pp_min && S >= pp_min) {
+    const int s = sh;
+    const int Rq = (R + s - 1) / s, Sq = (S + s - 1) / s;
+    const long long Hq = P + Rq - 1, Wq = Q + Sq - 1;
+    const long long Cq = (long long)s * s * C;
+    polyconv_plan_t in = nullptr;
+    if (Cq <= kMaxElems && (long long)N * Cq * Hq * Wq <= kMaxElems &&
+        polyconv_plan(&in, N, (int)Cq, (int)Hq, (int)Wq, K, Rq, Sq, 1, 1, 0, 0, io_dtype, math, device) ==
+            POLYCONV_STATUS_SUCCESS) {
+      p->inner = in;
+      p->Hq = (int)Hq; p->Wq = (int)Wq; p->Rq = Rq; p->Sq = Sq;
+      const size_t eb = p->io_bf16 ? 2 : 4;
+      p->xq_bytes = eb * (size_t)N * Cq * Hq * Wq;
+      p->wq_bytes = eb * (size_t)K * Cq * Rq * Sq;
+    }
+  }
   *plan = p;
   return POLYCONV_STATUS_SUCCESS;
 }
 
 polyconv_status_t polyconv_plan_set_kernel(polyconv_plan_t p, polyconv_kernel_t kernel) {
   if (!p) return POLYCONV_STATUS_BAD_PARAM;
+  if (p->inner) {
+    // the forward runs the inner (phase) plan; this plan keeps the same choice for its
+    // polyconv_pack_* layouts.  Both must accept the kernel.
+    const int old_inner = p->inner->forced;
+    polyconv_status_t si = polyconv_plan_set_kernel(p->inner, kernel);
+    if (si != POLYCONV_STATUS_SUCCESS) return si;
+    polyconv_plan_s* in = p->inner;
+    p->inner = nullptr;
+    polyconv_status_t so = polyconv_plan_set_kernel(p, kernel);
+    p->inner = in;
+    if (so != POLYCONV_STATUS_SUCCESS) polyconv_plan_set_kernel(in, (polyconv_kernel_t)old_inner);
+    return so;
+  }
   if (kernel < POLYCONV_KERNEL_AUTO || kernel > POLYCONV_KERNEL_TC_PAIR) return POLYCONV_STATUS_BAD_PARAM;
   const int old = p->forced;
   p->forced = kernel;
@@ -307,6 +350,14 @@ polyconv_status_t polyconv_plan_info(polyconv_plan_t p, polyconv_info_t* info) {
       info->tile_m = 1; info->tile_n = 1; info->stages = 1; info->launches = 3; break;
   }
   info->workspace_bytes = p->wsA_bytes + p->wsU_bytes;
+  if (p->inner) {  // the forward runs the inner (stride-1, phase) plan: its kernel and tiling;
+                   // Cp/Kp stay this plan's (they describe the polyconv_pack_* layouts)
+    polyconv_info_t ii;
+    polyconv_plan_info(p->inner, &ii);
+    info->kernel = ii.kernel; info->tile_m = ii.tile_m; info->tile_n = ii.tile_n; info->stages = ii.stages;
+    info->launches = ii.launches + 2;
+    info->workspace_bytes = ii.workspace_bytes + p->xq_bytes + p->wq_bytes;
+  }
   return POLYCONV_STATUS_SUCCESS;
 }
 
@@ -315,13 +366,32 @@ polyconv_status_t polyconv_forward(polyconv_plan_t p, const void* x, const void*
   if (!x || !w || !y || x == y || w == y) return POLYCONV_STATUS_BAD_PARAM;
   if (!aligned(x, 16) || !aligned(w, 16) || !aligned(y, 16)) return POLYCONV_STATUS_NOT_SUPPORTED;
   PC_BEGIN(p);
-  polyconv_status_t s = ensure_workspace(p);
+  polyconv_status_t s = p->inner ? POLYCONV_STATUS_SUCCESS : ensure_workspace(p);  // phase plans: inner's
   if (s != POLYCONV_STATUS_SUCCESS) return s;
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   p->last_stream = st;
   p->used = true;
   const Geom& g = p->g;
   cudaError_t e;
+  if (p->inner) {
+    // stride s: phase split of x and w (polyphase.cu), then the stride-1 inner plan
+    if ((!p->xq && cudaMalloc(&p->xq, p->xq_bytes) != cudaSuccess) ||
+        (!p->wq && cudaMalloc(&p->wq, p->wq_bytes) != cudaSuccess)) {
+      cudaGetLastError();
+      set_err(p, "cudaMalloc of the %s failed", "phase buffers");
+      return POLYCONV_STATUS_ALLOC_FAILED;
+    }
+    if (p->ev_start) cudaEventRecord(p->ev_start, st);
+    e = launch_polyphase(g, p->Hq, p->Wq, p->Rq, p->Sq, x, w, p->xq, p->wq, p->io_bf16, st);
+    if (e != cudaSuccess) return finish(p, e, "polyphase");
+    polyconv_status_t si = polyconv_forward(p->inner, p->xq, p->wq, y, stream);
+    if (si != POLYCONV_STATUS_SUCCESS) {
+      snprintf(p->err, sizeof(p->err), "inner (phase) plan: %s", polyconv_last_error(p->inner));
+      return si;
+    }
+    if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
+    return POLYCONV_STATUS_SUCCESS;
+  }
   if (p->kernel == POLYCONV_KERNEL_TC) {
     // a2 + a3 in one pack launch (interleaved input rows, tap-major filter), then the
     // windowed tensor-core MAC (a4+a5) as its programmatic dependent
@@ -511,6 +581,12 @@ polyconv_status_t polyconv_destroy(polyconv_plan_t p) {
     if (p->fcount) cudaFree(p->fcount);
   }
   if (p->pair_state) pair_state_free(p->pair_state);
+  if (p->inner) {
+    if (polyconv_destroy(p->inner) != POLYCONV_STATUS_SUCCESS) s = POLYCONV_STATUS_EXECUTION_FAILED;
+    DeviceGuard guard(p->device);
+    if (p->xq) cudaFree(p->xq);
+    if (p->wq) cudaFree(p->wq);
+  }
   delete p;
   return s;
 }

@@ -324,3 +324,21 @@ def test_pair_shapes(shape, io):
     y, plan = gpu_forward(shape, x, w, math="bf16", io=io, kernel="tc_pair")
     assert plan.info()["kernel"] == "tc_pair"
     assert np.array_equal(y, bf16_round(ref) if io == "bf16" else ref)
+
+
+@pytest.mark.parametrize("shape", [ConvShape("pp_3x3s2", 2, 32, 15, 14, 64, 3, 3, 2, 2, 1, 1),
+                                   ConvShape("pp_5x5s2", 2, 16, 17, 17, 48, 5, 5, 2, 2, 2, 2),
+                                   ConvShape("pp_7x7s2_c3", 2, 3, 30, 30, 64, 7, 7, 2, 2, 3, 3),
+                                   ConvShape("pp_3x3s3", 1, 8, 16, 16, 16, 3, 3, 3, 3, 1, 1),
+                                   ConvShape("pp_4x2s2", 2, 8, 11, 9, 16, 4, 2, 2, 2, 1, 0)],
+                         ids=lambda s: s.name)
+@pytest.mark.parametrize("math,io", [("bf16", "bf16"), ("fp32", "f32"), ("tf32", "f32")])
+def test_polyphase_stride(shape, math, io, monkeypatch):
+    """Stride s as a stride-1 convolution of the s*s input phases (reading R4b), forced on
+    for every kernel size: integer data bit-exact against the oracle."""
+    monkeypatch.setenv("POLYCONV_POLYPHASE", "1")
+    x, w = synth.make_inputs(shape, synth.seed_for(13, hash(shape.name) % 997), "int")
+    ref = oracle.conv2d(x, w, shape.stride, shape.padding)
+    y, plan = gpu_forward(shape, x, w, math=math, io=io)
+    assert plan.info()["launches"] >= 3  # phase split + the inner plan's launches
+    assert np.array_equal(y, bf16_round(ref) if io == "bf16" else ref)
