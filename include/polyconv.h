@@ -89,7 +89,9 @@ typedef enum {
  * (SMs held by other work for > 0.5 s) traps and forward returns
  * POLYCONV_STATUS_EXECUTION_FAILED instead of hanging.  One plan must not run
  * two TC_PAIR forwards concurrently on different streams (the counters are
- * per plan);
+ * per plan); TC_1X1 = 1x1, stride-1, unpadded BF16 layers: the input polynomials are
+ * the NCHW planes themselves, read by the tensor cores as the MN-major operand
+ * (no packed input copy);
  * FP32 = SIMT register-blocked FFMA; THIN = warp-per-output with shuffle
  * reduction over C*R*S (tiny channel counts). */
 typedef enum {
@@ -99,7 +101,8 @@ typedef enum {
     POLYCONV_KERNEL_THIN = 3,
     POLYCONV_KERNEL_TC_PERTAP = 4,
     POLYCONV_KERNEL_TC_FUSED = 5,
-    POLYCONV_KERNEL_TC_PAIR = 6
+    POLYCONV_KERNEL_TC_PAIR = 6,
+    POLYCONV_KERNEL_TC_1X1 = 7
 } polyconv_kernel_t;
 
 /* Packed-operand layouts exposed for bit-exact tests (a2/a3):

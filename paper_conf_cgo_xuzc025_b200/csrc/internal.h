@@ -40,6 +40,13 @@ cudaError_t launch_pack_filter_tapmajor(const Geom& g, const void* w, bool w_bf1
 cudaError_t launch_pack_both_interleaved(const Geom& g, const void* x, const void* w, bool io_bf16,
                                          void* xdst, void* wdst, int fmt, cudaStream_t st);
 
+// ---- mac_1x1.cu (1x1 stride-1 unpadded, BF16: x read as the MN-major operand) ----
+bool mac1x1_supported(const Geom& g, int fmt, bool io_bf16);
+// U: tap-major packed filter [1][Kp][Cp], Kp % 128 == 0, Cp % 64 == 0; launched as a
+// programmatic dependent of the filter pack
+cudaError_t launch_mac_1x1(const Geom& g, const void* x, const void* U, int Kp, int Cp, void* y, int num_sms,
+                           cudaStream_t st, char* err, size_t errlen);
+
 // ---- polyphase.cu (stride s: phases of the padded input as channels, reading R4b) ----
 // xq [N][s*s*C][Hq][Wq] and wq [K][s*s*C][Rq][Sq] in the io dtype
 cudaError_t launch_polyphase(const Geom& g, int Hq, int Wq, int Rq, int Sq, const void* x, const void* w, void* xq,

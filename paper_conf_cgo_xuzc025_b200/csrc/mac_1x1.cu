@@ -1,0 +1,269 @@
+// mac_1x1.cu — 1x1, stride-1, unpadded layers (BF16): a4 + a5 with the input
+// polynomials read straight from NCHW x.
+//
+// For R = S = 1 the kernel polynomial U_{k,c}(t) is the constant w[k][c] (Eq. 6
+// with L_U = 1), the input polynomial A_{n,c}(t) is the plane x[n][c] itself
+// (Eq. 10 with no padding: Wp = W), and the product coefficients are
+//   p_{n,k}[m] = sum_c A_{n,c}[m] * w[k][c]          (P.965, P.1350-1352)
+// with every coefficient an output pixel (Eq. 12: L_U - 1 = 0, m = oh*W + ow).
+// That is one GEMM per image, D[k][m] = sum_c W[k][c] * X_n[c][m], whose position
+// operand is already laid out by NCHW: x viewed as [N*C][H*W] has positions
+// contiguous, i.e. the MN-major B operand of tcgen05.mma (tools/mn_probe.cu:
+// SW128, LBO = the next 64-position box, SBO = the next 8 channels).  No packed
+// copy of x is made.  The A operand is the tap-major packed filter [1][Kp][Cp]
+// (a3, channels past C zero, so the rows a box reads past an image's last channel
+// contribute nothing).
+//
+// Tiles: (image, block of NT positions, 128 output channels); K-chunks of 64
+// channels through a ring of stages (TMA); fp32 accumulators in TMEM, double
+// buffered; the epilogue holds one output channel per TMEM lane, so each thread
+// stores runs of consecutive pixels of its channel as 16-byte vectors.
+// Warps: 0 TMA producer, 1 TMEM allocator + MMA issuer, 2..5 epilogue.
+#include <cuda.h>
+#include <cstdio>
+#include <cstring>
+#include <cstdlib>
+#include <algorithm>
+#include "common.cuh"
+#include "sm100.cuh"
+
+namespace polyconv {
+
+namespace {
+
+using namespace sm100;
+
+constexpr int k1Threads = 192;
+constexpr int k1MaxStages = 8;
+
+struct P1x1 {
+  void* y;
+  int N, C, K, HW;
+  int NT, nbox, kchunks, num_pb, num_kt, num_tiles;
+  int stages;
+  uint32_t a_bytes, b_bytes;  // per stage
+  uint32_t idesc;
+  int tmem_cols;
+};
+
+__device__ __forceinline__ uint64_t desc_mn(uint32_t saddr) {
+  // MN-major, 128-byte swizzle: LBO = 8192 (next 64-position box), SBO = 1024 (next 8 k-rows)
+  uint64_t d = 0;
+  d |= (uint64_t)((saddr & 0x3FFFFu) >> 4);
+  d |= (uint64_t)(8192u >> 4) << 16;
+  d |= (uint64_t)(1024u >> 4) << 32;
+  d |= (uint64_t)1u << 46;
+  d |= (uint64_t)2u << 61;
+  return d;
+}
+
+__global__ void __launch_bounds__(k1Threads, 1)
+    mac_1x1_kernel(const __grid_constant__ CUtensorMap tmU, const __grid_constant__ CUtensorMap tmX, const P1x1 p) {
+  extern __shared__ uint8_t smem_raw[];
+  const uint32_t raw = smem_u32(smem_raw);
+  uint8_t* smem = smem_raw + (((raw + 1023u) & ~1023u) - raw);
+  uint8_t* sA = smem;                                      // [stages][128 rows][128 B]
+  uint8_t* sB = sA + (size_t)p.stages * p.a_bytes;         // [stages][nbox][64 ch][128 B]
+  uint64_t* full = reinterpret_cast<uint64_t*>(sB + (size_t)p.stages * p.b_bytes);
+  uint64_t* empty = full + k1MaxStages;
+  uint64_t* tfull = empty + k1MaxStages;
+  uint64_t* tempty = tfull + 2;
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(tempty + 2);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    prefetch_tmap(&tmU);
+    prefetch_tmap(&tmX);
+    for (int s = 0; s < p.stages; ++s) {
+      mbar_init(full + s, 1);
+      mbar_init(empty + s, 1);
+    }
+    for (int a = 0; a < 2; ++a) {
+      mbar_init(tfull + a, 1);
+      mbar_init(tempty + a, 4);
+    }
+    fence_barrier_init();
+  }
+  if (warp == 1) tmem_alloc(tslot, (uint32_t)p.tmem_cols);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tslot;
+  // the packed filter comes from the preceding pack launch (programmatic dependent launch)
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+
+  if (warp == 0) {
+    int st = 0;
+    uint32_t ph = 0;
+    for (int t = blockIdx.x; t < p.num_tiles; t += gridDim.x) {
+      const int kt = t % p.num_kt, rest = t / p.num_kt;
+      const int pb = rest % p.num_pb, n = rest / p.num_pb;
+      for (int kc = 0; kc < p.kchunks; ++kc) {
+        mbar_wait(empty + st, ph ^ 1u);
+        if (elect_one()) {
+          mbar_arrive_expect_tx(full + st, p.a_bytes + (uint32_t)p.nbox * 8192u);
+          tma_load_2d(sA + (size_t)st * p.a_bytes, &tmU, full + st, kc * 64, kt * 128);
+          for (int b = 0; b < p.nbox; ++b)
+            tma_load_2d(sB + (size_t)st * p.b_bytes + (size_t)b * 8192, &tmX, full + st, pb * p.NT + b * 64,
+                        n * p.C + kc * 64);
+        }
+        __syncwarp();
+        if (++st == p.stages) { st = 0; ph ^= 1u; }
+      }
+    }
+  } else if (warp == 1) {
+    int st = 0, lt = 0;
+    uint32_t ph = 0;
+    for (int t = blockIdx.x; t < p.num_tiles; t += gridDim.x, ++lt) {
+      const int a = lt & 1;
+      mbar_wait(tempty + a, (uint32_t)((lt >> 1) & 1) ^ 1u);
+      tc_fence_after();
+      const uint32_t d = tmem + (uint32_t)(a * p.NT);
+      for (int kc = 0; kc < p.kchunks; ++kc) {
+        mbar_wait(full + st, ph);
+        tc_fence_after();
+        const uint64_t ad = make_sdesc(smem_u32(sA + (size_t)st * p.a_bytes), 128, 0);
+        const uint64_t bd = desc_mn(smem_u32(sB + (size_t)st * p.b_bytes));
+        if (elect_one()) {
+#pragma unroll
+          for (int ks = 0; ks < 4; ++ks)  // K step: +32 B (K-major A), +2048 B (MN-major B)
+            umma<false>(d, ad + 2 * ks, bd + 128 * ks, p.idesc, (kc | ks) != 0 ? 1u : 0u);
+          umma_commit(empty + st);
+        }
+        __syncwarp();
+        if (++st == p.stages) { st = 0; ph ^= 1u; }
+      }
+      if (elect_one()) umma_commit(tfull + a);
+      __syncwarp();
+    }
+  } else {
+    // epilogue: lane = output channel (quadrant warp % 4), 32 positions per TMEM load
+    const int q = warp & 3;
+    __nv_bfloat16* y = static_cast<__nv_bfloat16*>(p.y);
+    int lt = 0;
+    for (int t = blockIdx.x; t < p.num_tiles; t += gridDim.x, ++lt) {
+      const int kt = t % p.num_kt, rest = t / p.num_kt;
+      const int pb = rest % p.num_pb, n = rest / p.num_pb;
+      const int a = lt & 1;
+      mbar_wait_sleep(tfull + a, (uint32_t)((lt >> 1) & 1), 64);
+      tc_fence_after();
+      const int k = kt * 128 + q * 32 + lane;
+      __nv_bfloat16* yrow = y + ((long long)n * p.K + k) * p.HW + (long long)pb * p.NT;
+      const int nvalid = min(p.NT, p.HW - pb * p.NT);
+      for (int c = 0; c < p.NT; c += 32) {
+        uint32_t v[32];
+        tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(a * p.NT + c), v);
+        tmem_ld_wait();
+        if (k < p.K && c < nvalid) {
+#pragma unroll
+          for (int g8 = 0; g8 < 4; ++g8) {
+            if (c + g8 * 8 < nvalid) {  // HW is a multiple of 8: whole 8-pixel groups
+              uint32_t w4[4];
+#pragma unroll
+              for (int m = 0; m < 4; ++m) {
+                const __nv_bfloat162 h2 = __floats2bfloat162_rn(__uint_as_float(v[g8 * 8 + 2 * m]),
+                                                                __uint_as_float(v[g8 * 8 + 2 * m + 1]));
+                w4[m] = *reinterpret_cast<const uint32_t*>(&h2);
+              }
+              *reinterpret_cast<uint4*>(yrow + c + g8 * 8) = make_uint4(w4[0], w4[1], w4[2], w4[3]);
+            }
+          }
+        }
+      }
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(tempty + a);
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    tc_fence_after();
+    tmem_dealloc(tmem, (uint32_t)p.tmem_cols);
+  }
+}
+
+typedef CUresult (*EncFn1)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                           const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                           CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+EncFn1 get_enc1() {
+  static EncFn1 fn = nullptr;
+  if (!fn) {
+    void* f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<EncFn1>(f);
+  }
+  return fn;
+}
+
+bool enc2(CUtensorMap* m, const void* base, uint64_t cols, uint64_t rows, uint32_t bc, uint32_t br) {
+  EncFn1 enc = get_enc1();
+  if (!enc) return false;
+  cuuint64_t dims[2] = {cols, rows};
+  cuuint64_t strides[1] = {cols * 2};
+  cuuint32_t box[2] = {bc, br};
+  cuuint32_t es[2] = {1, 1};
+  return enc(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box, es,
+             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+
+}  // namespace
+
+bool mac1x1_supported(const Geom& g, int fmt, bool io_bf16) {
+  return fmt == FMT_BF16 && io_bf16 && g.R == 1 && g.S == 1 && g.sh == 1 && g.sw == 1 && g.ph == 0 && g.pw == 0 &&
+         ((long long)g.H * g.W) % 8 == 0 && (long long)g.N * g.C < (1LL << 31) && (long long)g.H * g.W >= 64;
+}
+
+cudaError_t launch_mac_1x1(const Geom& g, const void* x, const void* U, int Kp, int Cp, void* y, int num_sms,
+                           cudaStream_t st, char* err, size_t errlen) {
+  P1x1 p{};
+  p.y = y;
+  p.N = g.N; p.C = g.C; p.K = g.K; p.HW = g.H * g.W;
+  p.NT = p.HW >= 256 ? 256 : (p.HW + 63) / 64 * 64;
+  p.nbox = p.NT / 64;
+  p.kchunks = Cp / 64;
+  p.num_pb = (p.HW + p.NT - 1) / p.NT;
+  p.num_kt = Kp / 128;
+  const long long tiles = (long long)g.N * p.num_pb * p.num_kt;
+  if (tiles >= (1LL << 31) || p.kchunks < 1) {
+    snprintf(err, errlen, "mac_1x1: unsupported shape");
+    return cudaErrorInvalidValue;
+  }
+  p.num_tiles = (int)tiles;
+  p.a_bytes = 128 * 128;
+  p.b_bytes = (uint32_t)p.nbox * 8192;
+  const int per = (int)(p.a_bytes + p.b_bytes);
+  p.stages = std::min(k1MaxStages, (227 * 1024 - 2048) / per);
+  if (p.stages < 2) {
+    snprintf(err, errlen, "mac_1x1: shared memory");
+    return cudaErrorInvalidValue;
+  }
+  // D f32 @4, A/B bf16 @7/@10, B MN-major (bit 16), N >> 3 @17, M = 128 >> 4 @24
+  p.idesc = (1u << 4) | (1u << 7) | (1u << 10) | (1u << 16) | ((uint32_t)(p.NT >> 3) << 17) | ((128u >> 4) << 24);
+  p.tmem_cols = 2 * p.NT <= 32 ? 32 : (2 * p.NT <= 64 ? 64 : (2 * p.NT <= 128 ? 128 : (2 * p.NT <= 256 ? 256 : 512)));
+  CUtensorMap tmU, tmX;
+  if (!enc2(&tmU, U, (uint64_t)Cp, (uint64_t)Kp, 64, 128) ||
+      !enc2(&tmX, x, (uint64_t)p.HW, (uint64_t)g.N * g.C, 64, 64)) {
+    snprintf(err, errlen, "mac_1x1: cuTensorMapEncodeTiled failed");
+    return cudaErrorInvalidValue;
+  }
+  const int smem = 1024 + p.stages * per + 1024;
+  cudaError_t e = cudaFuncSetAttribute(mac_1x1_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e != cudaSuccess) return e;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)std::min(p.num_tiles, num_sms));
+  cfg.blockDim = dim3(k1Threads);
+  cfg.dynamicSmemBytes = (size_t)smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, mac_1x1_kernel, tmU, tmX, p);
+}
+
+}  // namespace polyconv

@@ -68,6 +68,8 @@ polyconv_status_t resolve(polyconv_plan_t p) {
   int k = p->forced;
   const bool tc_math = p->math != POLYCONV_MATH_FP32_FMA;
   if (k == POLYCONV_KERNEL_AUTO || k == POLYCONV_KERNEL_TC_PAIR) p->pair = pair_tiling(g, p->fmt, p->io_bf16, p->num_sms);
+  if (k == POLYCONV_KERNEL_AUTO && mac1x1_supported(g, p->fmt, p->io_bf16) && !getenv("POLYCONV_NO_1X1"))
+    k = POLYCONV_KERNEL_TC_1X1;  // 1x1 stride 1: x is already the (MN-major) position operand
   if (k == POLYCONV_KERNEL_AUTO) {
     // bf16, at most two rounds of pair tiles: one launch on CTA pairs with a resident filter
     // (its fixed startup wins on small problems); larger problems pipeline better in mac_tc2
@@ -89,12 +91,16 @@ polyconv_status_t resolve(polyconv_plan_t p) {
   if ((k == POLYCONV_KERNEL_TC || k == POLYCONV_KERNEL_TC_FUSED) && (!tc_math || !tc2_supported(g, p->fmt)))
     return POLYCONV_STATUS_BAD_PARAM;
   if (k == POLYCONV_KERNEL_TC_PAIR && (!tc_math || !p->pair.ok)) return POLYCONV_STATUS_BAD_PARAM;
+  if (k == POLYCONV_KERNEL_TC_1X1 && !mac1x1_supported(g, p->fmt, p->io_bf16)) return POLYCONV_STATUS_BAD_PARAM;
   if (k == POLYCONV_KERNEL_TC_PERTAP && (!tc_math || !tc_supported(g, p->fmt))) return POLYCONV_STATUS_BAD_PARAM;
   if (k == POLYCONV_KERNEL_FP32 && (tc_math || fp32_tiling(g).smax == 0)) return POLYCONV_STATUS_BAD_PARAM;
   p->kernel = k;
   if (k == POLYCONV_KERNEL_TC_PAIR) {
     g.Cp = p->pair.Cp;
     g.Kp = p->pair.NN;
+  } else if (k == POLYCONV_KERNEL_TC_1X1) {
+    g.Cp = (g.C + 63) / 64 * 64;
+    g.Kp = (g.K + 127) / 128 * 128;
   } else if (k == POLYCONV_KERNEL_TC || k == POLYCONV_KERNEL_TC_FUSED) {
     p->tc2 = tc2_tiling(g, p->fmt, p->io_bf16, p->num_sms, k == POLYCONV_KERNEL_TC_FUSED, p->io_bf16);
     g.Cp = (g.C + p->tc2.kc - 1) / p->tc2.kc * p->tc2.kc;
@@ -114,7 +120,7 @@ polyconv_status_t resolve(polyconv_plan_t p) {
   const int eb = fmt_bytes(p->fmt);
   // TC packs the input on the fly (no input workspace); TC_PERTAP needs the
   // interleaved copy, FP32/THIN the planar one
-  const size_t a_elems = k == POLYCONV_KERNEL_TC_FUSED ? 0
+  const size_t a_elems = (k == POLYCONV_KERNEL_TC_FUSED || k == POLYCONV_KERNEL_TC_1X1) ? 0
                          : (k == POLYCONV_KERNEL_TC || k == POLYCONV_KERNEL_TC_PERTAP || k == POLYCONV_KERNEL_TC_PAIR) ? (size_t)g.N * g.L_A * g.Cp
                                                                                        : (size_t)g.N * g.C * g.L_A;
   p->wsA_bytes = a_elems * eb;
@@ -303,7 +309,7 @@ polyconv_status_t polyconv_plan_set_kernel(polyconv_plan_t p, polyconv_kernel_t 
     if (so != POLYCONV_STATUS_SUCCESS) polyconv_plan_set_kernel(in, (polyconv_kernel_t)old_inner);
     return so;
   }
-  if (kernel < POLYCONV_KERNEL_AUTO || kernel > POLYCONV_KERNEL_TC_PAIR) return POLYCONV_STATUS_BAD_PARAM;
+  if (kernel < POLYCONV_KERNEL_AUTO || kernel > POLYCONV_KERNEL_TC_1X1) return POLYCONV_STATUS_BAD_PARAM;
   const int old = p->forced;
   p->forced = kernel;
   if (resolve(p) != POLYCONV_STATUS_SUCCESS) {
@@ -342,6 +348,9 @@ polyconv_status_t polyconv_plan_info(polyconv_plan_t p, polyconv_info_t* info) {
     case POLYCONV_KERNEL_TC_PAIR:  // pair tile = 256 positions x NN output channels
       info->tile_m = 256; info->tile_n = p->pair.NN; info->stages = p->pair.ring;
       info->launches = p->pair.split ? 2 : 1; break;
+    case POLYCONV_KERNEL_TC_1X1:  // tile = 128 output channels x up to 256 positions
+      info->tile_m = 128; info->tile_n = g.H * g.W >= 256 ? 256 : (g.H * g.W + 63) / 64 * 64; info->stages = 0;
+      info->launches = 2; break;
     case POLYCONV_KERNEL_TC_PERTAP:
       info->tile_m = p->tc.bm; info->tile_n = p->tc.bn; info->stages = p->tc.stages; info->launches = 2; break;
     case POLYCONV_KERNEL_FP32:
@@ -402,6 +411,15 @@ polyconv_status_t polyconv_forward(polyconv_plan_t p, const void* x, const void*
                        sizeof(p->err));
     if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
     return finish(p, e, "mac_tc");
+  }
+  if (p->kernel == POLYCONV_KERNEL_TC_1X1) {
+    // a3 (the [1][Kp][Cp] filter), then the GEMM over the NCHW planes as its programmatic dependent
+    if (p->ev_start) cudaEventRecord(p->ev_start, st);
+    e = launch_pack_filter_tapmajor(g, w, p->io_bf16, p->wsU, p->fmt, g.Kp, g.Cp, st);
+    if (e != cudaSuccess) return finish(p, e, "pack_filter");
+    e = launch_mac_1x1(g, x, p->wsU, g.Kp, g.Cp, y, p->num_sms, st, p->err, sizeof(p->err));
+    if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
+    return finish(p, e, "mac_1x1");
   }
   if (p->kernel == POLYCONV_KERNEL_TC_PAIR) {
     // one launch: a3 (filter slices, every CTA; grid counter) + a2 (bands of A, each

@@ -342,3 +342,21 @@ def test_polyphase_stride(shape, math, io, monkeypatch):
     y, plan = gpu_forward(shape, x, w, math=math, io=io)
     assert plan.info()["launches"] >= 3  # phase split + the inner plan's launches
     assert np.array_equal(y, bf16_round(ref) if io == "bf16" else ref)
+
+
+@pytest.mark.parametrize("shape", [ConvShape("k1_a", 2, 64, 8, 8, 96, 1, 1),          # one partial block
+                                   ConvShape("k1_b", 3, 130, 16, 16, 200, 1, 1),      # 3 chunks, 2 k-tiles
+                                   ConvShape("k1_c", 2, 48, 28, 28, 64, 1, 1),        # ragged last block, C < 64
+                                   ConvShape("k1_d", 1, 256, 56, 56, 64, 1, 1)],      # 13 blocks
+                         ids=lambda s: s.name)
+def test_1x1_planes_as_operand(shape):
+    """1x1 stride-1 layers read the NCHW planes directly as the MN-major operand (mac_1x1):
+    integer data bit-exact against round_bf16(oracle); AUTO picks it for bf16 in/out."""
+    x, w = synth.make_inputs(shape, synth.seed_for(14, hash(shape.name) % 997), "int")
+    ref = oracle.conv2d(x, w, shape.stride, shape.padding)
+    y, plan = gpu_forward(shape, x, w, math="bf16", io="bf16")
+    assert plan.info()["kernel"] == "tc_1x1"
+    assert np.array_equal(y, bf16_round(ref))
+    x, w = synth.make_inputs(shape, synth.seed_for(15, hash(shape.name) % 997), "uniform")
+    y, _ = gpu_forward(shape, x, w, math="bf16", io="bf16", plan=plan)
+    assert normwise(y, oracle.conv2d(x, w, shape.stride, shape.padding)) <= GATE["bf16"]
