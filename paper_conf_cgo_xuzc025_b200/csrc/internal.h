@@ -42,8 +42,11 @@ cudaError_t launch_pack_both_interleaved(const Geom& g, const void* x, const voi
 
 // ---- mac_1x1.cu (1x1 stride-1 unpadded, BF16: x read as the MN-major operand) ----
 bool mac1x1_supported(const Geom& g, int fmt, bool io_bf16);
-// U: tap-major packed filter [1][Kp][Cp], Kp % 128 == 0, Cp % 64 == 0; launched as a
-// programmatic dependent of the filter pack
+// 0: x is read in place; else the pitch of the gathered position operand [N*C][pitch]
+int mac1x1_pitch(const Geom& g);
+cudaError_t launch_gather1x1(const Geom& g, const void* x, void* xq, cudaStream_t st);
+// x: NCHW input (pitch 0) or the gathered copy; U: tap-major packed filter [1][Kp][Cp],
+// Kp % 128 == 0, Cp % 64 == 0; launched as a programmatic dependent of the filter pack
 cudaError_t launch_mac_1x1(const Geom& g, const void* x, const void* U, int Kp, int Cp, void* y, int num_sms,
                            cudaStream_t st, char* err, size_t errlen);
 

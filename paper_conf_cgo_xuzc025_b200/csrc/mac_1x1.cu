@@ -1,5 +1,6 @@
-// mac_1x1.cu — 1x1, stride-1, unpadded layers (BF16): a4 + a5 with the input
-// polynomials read straight from NCHW x.
+// mac_1x1.cu — 1x1 unpadded layers (BF16): a4 + a5 with the input polynomials
+// read straight from NCHW x (stride 1, planes of a multiple of 8 pixels), or from a
+// gathered copy of the output-lattice pixels (stride > 1, or other plane sizes).
 //
 // For R = S = 1 the kernel polynomial U_{k,c}(t) is the constant w[k][c] (Eq. 6
 // with L_U = 1), the input polynomial A_{n,c}(t) is the plane x[n][c] itself
@@ -38,7 +39,8 @@ constexpr int k1MaxStages = 8;
 
 struct P1x1 {
   void* y;
-  int N, C, K, HW;
+  int N, C, K, HW;   // HW: the operand's plane pitch (positions per [n][c] row of x or of the gathered copy)
+  int HWo;           // output pixels per plane (P*Q) <= HW
   int NT, nbox, kchunks, num_pb, num_kt, num_tiles;
   int stages;
   uint32_t a_bytes, b_bytes;  // per stage
@@ -147,16 +149,29 @@ __global__ void __launch_bounds__(k1Threads, 1)
       mbar_wait_sleep(tfull + a, (uint32_t)((lt >> 1) & 1), 64);
       tc_fence_after();
       const int k = kt * 128 + q * 32 + lane;
-      __nv_bfloat16* yrow = y + ((long long)n * p.K + k) * p.HW + (long long)pb * p.NT;
-      const int nvalid = min(p.NT, p.HW - pb * p.NT);
+      __nv_bfloat16* yrow = y + ((long long)n * p.K + k) * p.HWo + (long long)pb * p.NT;
+      const int nvalid = min(p.NT, p.HWo - pb * p.NT);
+      const bool vec = (p.HWo & 7) == 0;  // 16-byte aligned 8-pixel groups
       for (int c = 0; c < p.NT; c += 32) {
         uint32_t v[32];
         tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(a * p.NT + c), v);
         tmem_ld_wait();
-        if (k < p.K && c < nvalid) {
+        if (k < p.K && c < nvalid && !vec) {
+          // HWo a multiple of 4 (mac1x1_supported): 8-byte groups of 4 pixels
+#pragma unroll
+          for (int g4 = 0; g4 < 8; ++g4) {
+            if (c + g4 * 4 < nvalid) {
+              const __nv_bfloat162 h0 = __floats2bfloat162_rn(__uint_as_float(v[g4 * 4]), __uint_as_float(v[g4 * 4 + 1]));
+              const __nv_bfloat162 h1 =
+                  __floats2bfloat162_rn(__uint_as_float(v[g4 * 4 + 2]), __uint_as_float(v[g4 * 4 + 3]));
+              *reinterpret_cast<uint2*>(yrow + c + g4 * 4) =
+                  make_uint2(*reinterpret_cast<const uint32_t*>(&h0), *reinterpret_cast<const uint32_t*>(&h1));
+            }
+          }
+        } else if (k < p.K && c < nvalid) {
 #pragma unroll
           for (int g8 = 0; g8 < 4; ++g8) {
-            if (c + g8 * 8 < nvalid) {  // HW is a multiple of 8: whole 8-pixel groups
+            if (c + g8 * 8 < nvalid) {  // HWo is a multiple of 8: whole 8-pixel groups
               uint32_t w4[4];
 #pragma unroll
               for (int m = 0; m < 4; ++m) {
@@ -179,6 +194,27 @@ __global__ void __launch_bounds__(k1Threads, 1)
   if (warp == 1) {
     tc_fence_after();
     tmem_dealloc(tmem, (uint32_t)p.tmem_cols);
+  }
+}
+
+// The position operand when the planes cannot be read in place (stride > 1, or a plane
+// size that is not a multiple of 8 pixels, i.e. no 16-byte TMA row pitch): the output
+// lattice pixels of every plane, xq[n*C + c][m] = x[n][c][oh*sh][ow*sw] for m = oh*Q + ow
+// < P*Q, zero up to the pitch (Eq. 12 with R = S = 1: the coefficients that become outputs).
+__global__ void __launch_bounds__(256) gather1x1_kernel(const __nv_bfloat16* __restrict__ x,
+                                                        __nv_bfloat16* __restrict__ xq, long long rows, int H, int W,
+                                                        int Q, int PQ, int pitch, int sh, int sw) {
+  const long long total = rows * pitch;
+  for (long long idx = blockIdx.x * (long long)blockDim.x + threadIdx.x; idx < total;
+       idx += (long long)gridDim.x * blockDim.x) {
+    const long long r = idx / pitch;
+    const int m = (int)(idx - r * pitch);
+    __nv_bfloat16 v = __float2bfloat16(0.f);
+    if (m < PQ) {
+      const int oh = m / Q, ow = m - (m / Q) * Q;
+      v = x[(r * H + (long long)oh * sh) * W + (long long)ow * sw];
+    }
+    xq[idx] = v;
   }
 }
 
@@ -213,19 +249,40 @@ bool enc2(CUtensorMap* m, const void* base, uint64_t cols, uint64_t rows, uint32
 }  // namespace
 
 bool mac1x1_supported(const Geom& g, int fmt, bool io_bf16) {
-  return fmt == FMT_BF16 && io_bf16 && g.R == 1 && g.S == 1 && g.sh == 1 && g.sw == 1 && g.ph == 0 && g.pw == 0 &&
-         ((long long)g.H * g.W) % 8 == 0 && (long long)g.N * g.C < (1LL << 31) && (long long)g.H * g.W >= 64;
+  // output planes of a multiple of 4 pixels: the epilogue stores 8- or 16-byte groups
+  return fmt == FMT_BF16 && io_bf16 && g.R == 1 && g.S == 1 && g.ph == 0 && g.pw == 0 &&
+         (long long)g.N * g.C < (1LL << 31) && (long long)g.P * g.Q >= 16 && ((long long)g.P * g.Q) % 4 == 0;
+}
+
+int mac1x1_pitch(const Geom& g) {
+  const bool direct = g.sh == 1 && g.sw == 1 && ((long long)g.H * g.W) % 8 == 0;
+  return direct ? 0 : (g.P * g.Q + 7) / 8 * 8;
+}
+
+cudaError_t launch_gather1x1(const Geom& g, const void* x, void* xq, cudaStream_t st) {
+  const int pitch = mac1x1_pitch(g);
+  const long long rows = (long long)g.N * g.C;
+  const long long total = rows * pitch;
+  long long blocks = (total + 255) / 256;
+  if (blocks > 148LL * 32) blocks = 148LL * 32;
+  gather1x1_kernel<<<(unsigned)blocks, 256, 0, st>>>(static_cast<const __nv_bfloat16*>(x),
+                                                     static_cast<__nv_bfloat16*>(xq), rows, g.H, g.W, g.Q,
+                                                     g.P * g.Q, pitch, g.sh, g.sw);
+  return cudaGetLastError();
 }
 
 cudaError_t launch_mac_1x1(const Geom& g, const void* x, const void* U, int Kp, int Cp, void* y, int num_sms,
                            cudaStream_t st, char* err, size_t errlen) {
   P1x1 p{};
   p.y = y;
-  p.N = g.N; p.C = g.C; p.K = g.K; p.HW = g.H * g.W;
-  p.NT = p.HW >= 256 ? 256 : (p.HW + 63) / 64 * 64;
+  const int pitch = mac1x1_pitch(g);
+  p.N = g.N; p.C = g.C; p.K = g.K;
+  p.HW = pitch ? pitch : g.H * g.W;  // x (direct) or the gathered copy
+  p.HWo = g.P * g.Q;
+  p.NT = p.HWo >= 256 ? 256 : (p.HWo + 63) / 64 * 64;
   p.nbox = p.NT / 64;
   p.kchunks = Cp / 64;
-  p.num_pb = (p.HW + p.NT - 1) / p.NT;
+  p.num_pb = (p.HWo + p.NT - 1) / p.NT;
   p.num_kt = Kp / 128;
   const long long tiles = (long long)g.N * p.num_pb * p.num_kt;
   if (tiles >= (1LL << 31) || p.kchunks < 1) {

@@ -68,8 +68,12 @@ polyconv_status_t resolve(polyconv_plan_t p) {
   int k = p->forced;
   const bool tc_math = p->math != POLYCONV_MATH_FP32_FMA;
   if (k == POLYCONV_KERNEL_AUTO || k == POLYCONV_KERNEL_TC_PAIR) p->pair = pair_tiling(g, p->fmt, p->io_bf16, p->num_sms);
-  if (k == POLYCONV_KERNEL_AUTO && mac1x1_supported(g, p->fmt, p->io_bf16) && !getenv("POLYCONV_NO_1X1"))
-    k = POLYCONV_KERNEL_TC_1X1;  // 1x1 stride 1: x is already the (MN-major) position operand
+  // 1x1: x is already the (MN-major) position operand when its planes have a 16-byte pitch;
+  // strided 1x1 layers gather their output lattice first.  Stride-1 layers on other plane
+  // sizes measured faster on the packed path (tools/layer_sweep.py)
+  if (k == POLYCONV_KERNEL_AUTO && mac1x1_supported(g, p->fmt, p->io_bf16) && !getenv("POLYCONV_NO_1X1") &&
+      (mac1x1_pitch(g) == 0 || g.sh > 1 || g.sw > 1))
+    k = POLYCONV_KERNEL_TC_1X1;
   if (k == POLYCONV_KERNEL_AUTO) {
     // bf16, at most two rounds of pair tiles: one launch on CTA pairs with a resident filter
     // (its fixed startup wins on small problems); larger problems pipeline better in mac_tc2
@@ -120,7 +124,8 @@ polyconv_status_t resolve(polyconv_plan_t p) {
   const int eb = fmt_bytes(p->fmt);
   // TC packs the input on the fly (no input workspace); TC_PERTAP needs the
   // interleaved copy, FP32/THIN the planar one
-  const size_t a_elems = (k == POLYCONV_KERNEL_TC_FUSED || k == POLYCONV_KERNEL_TC_1X1) ? 0
+  const size_t a_elems = k == POLYCONV_KERNEL_TC_1X1 ? (size_t)g.N * g.C * mac1x1_pitch(g)
+                         : k == POLYCONV_KERNEL_TC_FUSED ? 0
                          : (k == POLYCONV_KERNEL_TC || k == POLYCONV_KERNEL_TC_PERTAP || k == POLYCONV_KERNEL_TC_PAIR) ? (size_t)g.N * g.L_A * g.Cp
                                                                                        : (size_t)g.N * g.C * g.L_A;
   p->wsA_bytes = a_elems * eb;
@@ -349,8 +354,8 @@ polyconv_status_t polyconv_plan_info(polyconv_plan_t p, polyconv_info_t* info) {
       info->tile_m = 256; info->tile_n = p->pair.NN; info->stages = p->pair.ring;
       info->launches = p->pair.split ? 2 : 1; break;
     case POLYCONV_KERNEL_TC_1X1:  // tile = 128 output channels x up to 256 positions
-      info->tile_m = 128; info->tile_n = g.H * g.W >= 256 ? 256 : (g.H * g.W + 63) / 64 * 64; info->stages = 0;
-      info->launches = 2; break;
+      info->tile_m = 128; info->tile_n = g.P * g.Q >= 256 ? 256 : (g.P * g.Q + 63) / 64 * 64; info->stages = 0;
+      info->launches = mac1x1_pitch(g) ? 3 : 2; break;
     case POLYCONV_KERNEL_TC_PERTAP:
       info->tile_m = p->tc.bm; info->tile_n = p->tc.bn; info->stages = p->tc.stages; info->launches = 2; break;
     case POLYCONV_KERNEL_FP32:
@@ -415,9 +420,14 @@ polyconv_status_t polyconv_forward(polyconv_plan_t p, const void* x, const void*
   if (p->kernel == POLYCONV_KERNEL_TC_1X1) {
     // a3 (the [1][Kp][Cp] filter), then the GEMM over the NCHW planes as its programmatic dependent
     if (p->ev_start) cudaEventRecord(p->ev_start, st);
+    const bool gather = mac1x1_pitch(g) != 0;  // stride or plane size: gather the output lattice first
+    if (gather) {
+      e = launch_gather1x1(g, x, p->wsA, st);
+      if (e != cudaSuccess) return finish(p, e, "gather1x1");
+    }
     e = launch_pack_filter_tapmajor(g, w, p->io_bf16, p->wsU, p->fmt, g.Kp, g.Cp, st);
     if (e != cudaSuccess) return finish(p, e, "pack_filter");
-    e = launch_mac_1x1(g, x, p->wsU, g.Kp, g.Cp, y, p->num_sms, st, p->err, sizeof(p->err));
+    e = launch_mac_1x1(g, gather ? p->wsA : x, p->wsU, g.Kp, g.Cp, y, p->num_sms, st, p->err, sizeof(p->err));
     if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
     return finish(p, e, "mac_1x1");
   }

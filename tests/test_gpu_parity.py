@@ -360,3 +360,19 @@ def test_1x1_planes_as_operand(shape):
     x, w = synth.make_inputs(shape, synth.seed_for(15, hash(shape.name) % 997), "uniform")
     y, _ = gpu_forward(shape, x, w, math="bf16", io="bf16", plan=plan)
     assert normwise(y, oracle.conv2d(x, w, shape.stride, shape.padding)) <= GATE["bf16"]
+
+
+@pytest.mark.parametrize("shape", [ConvShape("k1g_6x6", 3, 96, 6, 6, 130, 1, 1),              # 36 px: gathered
+                                   ConvShape("k1g_14", 2, 72, 14, 14, 64, 1, 1),              # 196 px
+                                   ConvShape("k1g_s2", 2, 64, 28, 28, 128, 1, 1, 2, 2, 0, 0),  # stride 2
+                                   ConvShape("k1g_s2_odd", 2, 32, 15, 13, 48, 1, 1, 2, 2, 0, 0)],
+                         ids=lambda s: s.name)
+def test_1x1_gathered(shape):
+    """1x1 layers whose planes cannot be read in place (stride > 1, or a plane size that is
+    not a multiple of 8 pixels): the output-lattice pixels are gathered first, then the same
+    MN-major GEMM; bit-exact on integer data."""
+    x, w = synth.make_inputs(shape, synth.seed_for(16, hash(shape.name) % 997), "int")
+    ref = oracle.conv2d(x, w, shape.stride, shape.padding)
+    y, plan = gpu_forward(shape, x, w, math="bf16", io="bf16", kernel="tc_1x1")
+    assert plan.info()["kernel"] == "tc_1x1" and plan.info()["launches"] == 3
+    assert np.array_equal(y, bf16_round(ref))
