@@ -46,6 +46,9 @@ struct P1x1 {
   uint32_t a_bytes, b_bytes;  // per stage
   uint32_t idesc;
   int tmem_cols;
+  int epi_tma;  // 1: stage each warp's 32 channels x NT pixels (SW128) and TMA-store them;
+                // 2: whole planes (one position block): stage the warp's 32 channel planes densely
+                //    (a contiguous run of y) and write them with one bulk copy
 };
 
 __device__ __forceinline__ uint64_t desc_mn(uint32_t saddr) {
@@ -59,14 +62,23 @@ __device__ __forceinline__ uint64_t desc_mn(uint32_t saddr) {
   return d;
 }
 
+__device__ __forceinline__ void tma_store_2d(const void* tmap, uint32_t src, int c0, int c1) {
+  asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
+                   reinterpret_cast<uint64_t>(tmap)),
+               "r"(src), "r"(c0), "r"(c1)
+               : "memory");
+}
+
 __global__ void __launch_bounds__(k1Threads, 1)
-    mac_1x1_kernel(const __grid_constant__ CUtensorMap tmU, const __grid_constant__ CUtensorMap tmX, const P1x1 p) {
+    mac_1x1_kernel(const __grid_constant__ CUtensorMap tmU, const __grid_constant__ CUtensorMap tmX,
+                   const __grid_constant__ CUtensorMap tmY, const P1x1 p) {
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw = smem_u32(smem_raw);
   uint8_t* smem = smem_raw + (((raw + 1023u) & ~1023u) - raw);
   uint8_t* sA = smem;                                      // [stages][128 rows][128 B]
   uint8_t* sB = sA + (size_t)p.stages * p.a_bytes;         // [stages][nbox][64 ch][128 B]
-  uint64_t* full = reinterpret_cast<uint64_t*>(sB + (size_t)p.stages * p.b_bytes);
+  uint8_t* sE = sB + (size_t)p.stages * p.b_bytes;          // epi_tma: [4 warps][nbox][32 ch][128 B]
+  uint64_t* full = reinterpret_cast<uint64_t*>(sE + (p.epi_tma ? (size_t)p.nbox * 16384 : 0));
   uint64_t* empty = full + k1MaxStages;
   uint64_t* tfull = empty + k1MaxStages;
   uint64_t* tempty = tfull + 2;
@@ -75,6 +87,7 @@ __global__ void __launch_bounds__(k1Threads, 1)
   if (threadIdx.x == 0) {
     prefetch_tmap(&tmU);
     prefetch_tmap(&tmX);
+    if (p.epi_tma == 1) prefetch_tmap(&tmY);
     for (int s = 0; s < p.stages; ++s) {
       mbar_init(full + s, 1);
       mbar_init(empty + s, 1);
@@ -152,12 +165,79 @@ __global__ void __launch_bounds__(k1Threads, 1)
       __nv_bfloat16* yrow = y + ((long long)n * p.K + k) * p.HWo + (long long)pb * p.NT;
       const int nvalid = min(p.NT, p.HWo - pb * p.NT);
       const bool vec = (p.HWo & 7) == 0;  // 16-byte aligned 8-pixel groups
+      // epi_tma (K % 32 == 0): the warp's 32 channels are all valid or all past K
+      const bool wvalid = kt * 128 + q * 32 < p.K;
+      uint8_t* stg = sE + (size_t)q * p.nbox * 4096;
+      if (p.epi_tma) {
+        if (lane == 0) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");  // staging free
+        __syncwarp();
+      }
       for (int c = 0; c < p.NT; c += 32) {
         uint32_t v[32];
         tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(a * p.NT + c), v);
         tmem_ld_wait();
-        if (k < p.K && c < nvalid && !vec) {
-          // HWo a multiple of 4 (mac1x1_supported): 8-byte groups of 4 pixels
+        if (p.epi_tma == 2) {
+          // plane `lane` of the warp's dense [32][HWo] run; positions past HWo are not stored
+          if (wvalid) {
+            uint8_t* row = stg + (size_t)lane * p.HWo * 2;
+            if ((p.HWo & 1) == 0) {
+#pragma unroll
+              for (int j = 0; j < 32; j += 2)
+                if (c + j < p.HWo) {
+                  const __nv_bfloat162 h2 = __floats2bfloat162_rn(__uint_as_float(v[j]), __uint_as_float(v[j + 1]));
+                  *reinterpret_cast<__nv_bfloat162*>(row + (c + j) * 2) = h2;
+                }
+            } else {
+#pragma unroll
+              for (int j = 0; j < 32; ++j)
+                if (c + j < p.HWo)
+                  *reinterpret_cast<__nv_bfloat16*>(row + (c + j) * 2) = __float2bfloat16_rn(__uint_as_float(v[j]));
+            }
+          }
+          if (c + 32 >= p.NT) {
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            __syncwarp();
+            if (lane == 0 && wvalid) {
+              const uint32_t bytes = 64u * (uint32_t)p.HWo;  // 32 planes x HWo x 2 B, a multiple of 16
+              __nv_bfloat16* dst = y + ((long long)n * p.K + kt * 128 + q * 32) * p.HWo;
+              asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst),
+                           "r"(smem_u32(stg)), "r"(bytes)
+                           : "memory");
+              asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+            }
+          }
+        } else if (p.epi_tma) {
+          // row `lane` of box c/64 (SW128: 16-byte chunk j at j ^ (lane & 7)); conflict-free
+          if (wvalid && c < nvalid) {
+            uint8_t* row = stg + (size_t)(c >> 6) * 4096 + lane * 128;
+#pragma unroll
+            for (int g8 = 0; g8 < 4; ++g8) {
+              uint32_t w4[4];
+#pragma unroll
+              for (int m = 0; m < 4; ++m) {
+                const __nv_bfloat162 h2 = __floats2bfloat162_rn(__uint_as_float(v[g8 * 8 + 2 * m]),
+                                                                __uint_as_float(v[g8 * 8 + 2 * m + 1]));
+                w4[m] = *reinterpret_cast<const uint32_t*>(&h2);
+              }
+              const int j = (((c & 63) >> 3) + g8) ^ (lane & 7);
+              *reinterpret_cast<uint4*>(row + j * 16) = make_uint4(w4[0], w4[1], w4[2], w4[3]);
+            }
+          }
+          if ((c & 63) == 32 || c + 32 >= p.NT) {  // a 64-pixel box is complete
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            __syncwarp();
+            const int b = c >> 6;
+            if (lane == 0 && wvalid && b * 64 < nvalid) {
+              tma_store_2d(&tmY, smem_u32(stg + (size_t)b * 4096), pb * p.NT + b * 64, n * p.K + kt * 128 + q * 32);
+              asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+            }
+          }
+        } else if (k < p.K && c < nvalid && (p.HWo & 3) != 0) {
+#pragma unroll
+          for (int j = 0; j < 32; ++j)
+            if (c + j < nvalid) yrow[c + j] = __float2bfloat16_rn(__uint_as_float(v[j]));
+        } else if (k < p.K && c < nvalid && !vec) {
+          // HWo a multiple of 4: 8-byte groups of 4 pixels
 #pragma unroll
           for (int g4 = 0; g4 < 8; ++g4) {
             if (c + g4 * 4 < nvalid) {
@@ -188,6 +268,7 @@ __global__ void __launch_bounds__(k1Threads, 1)
       __syncwarp();
       if (lane == 0) mbar_arrive(tempty + a);
     }
+    if (p.epi_tma && lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
   }
   tc_fence_before();
   __syncthreads();
@@ -249,9 +330,8 @@ bool enc2(CUtensorMap* m, const void* base, uint64_t cols, uint64_t rows, uint32
 }  // namespace
 
 bool mac1x1_supported(const Geom& g, int fmt, bool io_bf16) {
-  // output planes of a multiple of 4 pixels: the epilogue stores 8- or 16-byte groups
   return fmt == FMT_BF16 && io_bf16 && g.R == 1 && g.S == 1 && g.ph == 0 && g.pw == 0 &&
-         (long long)g.N * g.C < (1LL << 31) && (long long)g.P * g.Q >= 16 && ((long long)g.P * g.Q) % 4 == 0;
+         (long long)g.N * g.C < (1LL << 31) && (long long)g.P * g.Q >= 16;
 }
 
 int mac1x1_pitch(const Geom& g) {
@@ -293,7 +373,12 @@ cudaError_t launch_mac_1x1(const Geom& g, const void* x, const void* U, int Kp, 
   p.a_bytes = 128 * 128;
   p.b_bytes = (uint32_t)p.nbox * 8192;
   const int per = (int)(p.a_bytes + p.b_bytes);
-  p.stages = std::min(k1MaxStages, (227 * 1024 - 2048) / per);
+  // TMA-stored epilogue: whole 32-channel row blocks, 16-byte output row pitch and base
+  const char* ev = getenv("POLYCONV_1X1_EPI_TMA");
+  const bool ep_ok = g.K % 32 == 0 && (reinterpret_cast<uintptr_t>(y) & 15) == 0 && (ev == nullptr || ev[0] != '0');
+  p.epi_tma = !ep_ok ? 0 : (p.num_pb == 1 && g.K % 8 == 0) ? 2 : (p.HWo % 8 == 0 ? 1 : 0);
+  const int estage = p.epi_tma ? p.nbox * 16384 : 0;
+  p.stages = std::min(k1MaxStages, (227 * 1024 - 2048 - estage) / per);
   if (p.stages < 2) {
     snprintf(err, errlen, "mac_1x1: shared memory");
     return cudaErrorInvalidValue;
@@ -301,13 +386,15 @@ cudaError_t launch_mac_1x1(const Geom& g, const void* x, const void* U, int Kp, 
   // D f32 @4, A/B bf16 @7/@10, B MN-major (bit 16), N >> 3 @17, M = 128 >> 4 @24
   p.idesc = (1u << 4) | (1u << 7) | (1u << 10) | (1u << 16) | ((uint32_t)(p.NT >> 3) << 17) | ((128u >> 4) << 24);
   p.tmem_cols = 2 * p.NT <= 32 ? 32 : (2 * p.NT <= 64 ? 64 : (2 * p.NT <= 128 ? 128 : (2 * p.NT <= 256 ? 256 : 512)));
-  CUtensorMap tmU, tmX;
+  CUtensorMap tmU, tmX, tmY;
+  memset(&tmY, 0, sizeof(tmY));
   if (!enc2(&tmU, U, (uint64_t)Cp, (uint64_t)Kp, 64, 128) ||
-      !enc2(&tmX, x, (uint64_t)p.HW, (uint64_t)g.N * g.C, 64, 64)) {
+      !enc2(&tmX, x, (uint64_t)p.HW, (uint64_t)g.N * g.C, 64, 64) ||
+      (p.epi_tma == 1 && !enc2(&tmY, y, (uint64_t)p.HWo, (uint64_t)g.N * g.K, 64, 32))) {
     snprintf(err, errlen, "mac_1x1: cuTensorMapEncodeTiled failed");
     return cudaErrorInvalidValue;
   }
-  const int smem = 1024 + p.stages * per + 1024;
+  const int smem = 1024 + p.stages * per + estage + 1024;
   cudaError_t e = cudaFuncSetAttribute(mac_1x1_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e != cudaSuccess) return e;
   cudaLaunchConfig_t cfg = {};
@@ -320,7 +407,7 @@ cudaError_t launch_mac_1x1(const Geom& g, const void* x, const void* U, int Kp, 
   attr[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  return cudaLaunchKernelEx(&cfg, mac_1x1_kernel, tmU, tmX, p);
+  return cudaLaunchKernelEx(&cfg, mac_1x1_kernel, tmU, tmX, tmY, p);
 }
 
 }  // namespace polyconv

@@ -72,7 +72,7 @@ polyconv_status_t resolve(polyconv_plan_t p) {
   // strided 1x1 layers gather their output lattice first.  Stride-1 layers on other plane
   // sizes measured faster on the packed path (tools/layer_sweep.py)
   if (k == POLYCONV_KERNEL_AUTO && mac1x1_supported(g, p->fmt, p->io_bf16) && !getenv("POLYCONV_NO_1X1") &&
-      (mac1x1_pitch(g) == 0 || g.sh > 1 || g.sw > 1))
+      (mac1x1_pitch(g) == 0 || g.sh > 1 || g.sw > 1 || getenv("POLYCONV_1X1_SMALL")))
     k = POLYCONV_KERNEL_TC_1X1;
   if (k == POLYCONV_KERNEL_AUTO) {
     // bf16, at most two rounds of pair tiles: one launch on CTA pairs with a resident filter

@@ -349,9 +349,13 @@ def test_polyphase_stride(shape, math, io, monkeypatch):
                                    ConvShape("k1_c", 2, 48, 28, 28, 64, 1, 1),        # ragged last block, C < 64
                                    ConvShape("k1_d", 1, 256, 56, 56, 64, 1, 1)],      # 13 blocks
                          ids=lambda s: s.name)
-def test_1x1_planes_as_operand(shape):
+@pytest.mark.parametrize("epi", ["auto", "direct"])
+def test_1x1_planes_as_operand(shape, epi, monkeypatch):
     """1x1 stride-1 layers read the NCHW planes directly as the MN-major operand (mac_1x1):
-    integer data bit-exact against round_bf16(oracle); AUTO picks it for bf16 in/out."""
+    integer data bit-exact against round_bf16(oracle); AUTO picks it for bf16 in/out.
+    epi: the staged bulk/TMA-stored epilogue (auto) or per-thread stores (direct)."""
+    if epi == "direct":
+        monkeypatch.setenv("POLYCONV_1X1_EPI_TMA", "0")
     x, w = synth.make_inputs(shape, synth.seed_for(14, hash(shape.name) % 997), "int")
     ref = oracle.conv2d(x, w, shape.stride, shape.padding)
     y, plan = gpu_forward(shape, x, w, math="bf16", io="bf16")
@@ -365,7 +369,11 @@ def test_1x1_planes_as_operand(shape):
 @pytest.mark.parametrize("shape", [ConvShape("k1g_6x6", 3, 96, 6, 6, 130, 1, 1),              # 36 px: gathered
                                    ConvShape("k1g_14", 2, 72, 14, 14, 64, 1, 1),              # 196 px
                                    ConvShape("k1g_s2", 2, 64, 28, 28, 128, 1, 1, 2, 2, 0, 0),  # stride 2
-                                   ConvShape("k1g_s2_odd", 2, 32, 15, 13, 48, 1, 1, 2, 2, 0, 0)],
+                                   ConvShape("k1g_s2_odd", 2, 32, 15, 13, 48, 1, 1, 2, 2, 0, 0),
+                                   ConvShape("k1g_7", 2, 64, 7, 7, 96, 1, 1),                  # 49 px, odd
+                                   ConvShape("k1g_7_k40", 2, 32, 7, 7, 40, 1, 1),              # K % 32 != 0
+                                   ConvShape("k1g_s2_14", 3, 64, 14, 14, 64, 1, 1, 2, 2, 0, 0),  # 7x7 out
+                                   ConvShape("k1g_10x9", 2, 130, 10, 9, 160, 1, 1)],           # 90 px, 3 chunks
                          ids=lambda s: s.name)
 def test_1x1_gathered(shape):
     """1x1 layers whose planes cannot be read in place (stride > 1, or a plane size that is
