@@ -285,17 +285,26 @@ __global__ void __launch_bounds__(k1Threads, 1)
 __global__ void __launch_bounds__(256) gather1x1_kernel(const __nv_bfloat16* __restrict__ x,
                                                         __nv_bfloat16* __restrict__ xq, long long rows, int H, int W,
                                                         int Q, int PQ, int pitch, int sh, int sw) {
-  const long long total = rows * pitch;
-  for (long long idx = blockIdx.x * (long long)blockDim.x + threadIdx.x; idx < total;
-       idx += (long long)gridDim.x * blockDim.x) {
-    const long long r = idx / pitch;
-    const int m = (int)(idx - r * pitch);
-    __nv_bfloat16 v = __float2bfloat16(0.f);
-    if (m < PQ) {
-      const int oh = m / Q, ow = m - (m / Q) * Q;
-      v = x[(r * H + (long long)oh * sh) * W + (long long)ow * sw];
+  // one warp per plane row r = n*C + c, lanes over pixel pairs (pitch is even); the plane
+  // index math is 32-bit and per row, the contiguous case (stride 1) needs none
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const bool contiguous = sh == 1 && sw == 1 && Q == W;
+  for (long long r = (long long)blockIdx.x * 8 + warp; r < rows; r += (long long)gridDim.x * 8) {
+    const __nv_bfloat16* src = x + r * H * W;
+    __nv_bfloat162* dst = reinterpret_cast<__nv_bfloat162*>(xq + r * pitch);
+    for (int m = 2 * lane; m < pitch; m += 64) {
+      float v[2];
+#pragma unroll
+      for (int e = 0; e < 2; ++e) {
+        const int mm = m + e;
+        v[e] = 0.f;
+        if (mm < PQ) {
+          const int oh = contiguous ? 0 : mm / Q, ow = contiguous ? mm : mm - oh * Q;
+          v[e] = __bfloat162float(src[oh * sh * W + ow * sw]);
+        }
+      }
+      dst[m >> 1] = __floats2bfloat162_rn(v[0], v[1]);
     }
-    xq[idx] = v;
   }
 }
 
@@ -342,8 +351,7 @@ int mac1x1_pitch(const Geom& g) {
 cudaError_t launch_gather1x1(const Geom& g, const void* x, void* xq, cudaStream_t st) {
   const int pitch = mac1x1_pitch(g);
   const long long rows = (long long)g.N * g.C;
-  const long long total = rows * pitch;
-  long long blocks = (total + 255) / 256;
+  long long blocks = (rows + 7) / 8;
   if (blocks > 148LL * 32) blocks = 148LL * 32;
   gather1x1_kernel<<<(unsigned)blocks, 256, 0, st>>>(static_cast<const __nv_bfloat16*>(x),
                                                      static_cast<__nv_bfloat16*>(xq), rows, g.H, g.W, g.Q,

@@ -62,6 +62,18 @@ void set_err(polyconv_plan_t p, const char* fmt_, const char* a = "", long long 
   if (p) snprintf(p->err, sizeof(p->err), fmt_, a, b);
 }
 
+// AUTO for 1x1 layers (tools/layer_sweep.py, ResNet-50 at N=256): in place when the planes can be
+// read by TMA; gathered for strided layers and for stride-1 planes that are not a multiple of 8
+// pixels, except expansion layers (K > C) on planes under 64 pixels, where the 64-position tiles
+// lose to mac_tc2 (7x7, 512 -> 2048: 282 vs 317 TFLOP/s).  POLYCONV_1X1_SMALL=0/1 forces the
+// stride-1 gathered choice off/on.
+bool mac1x1_auto(const Geom& g) {
+  if (mac1x1_pitch(g) == 0 || g.sh > 1 || g.sw > 1) return true;
+  const char* ev = getenv("POLYCONV_1X1_SMALL");
+  if (ev) return ev[0] != '0';
+  return !((long long)g.P * g.Q < 64 && g.K > g.C);
+}
+
 // Resolve the MAC variant and fill the kernel-specific padded sizes.
 polyconv_status_t resolve(polyconv_plan_t p) {
   Geom& g = p->g;
@@ -69,10 +81,9 @@ polyconv_status_t resolve(polyconv_plan_t p) {
   const bool tc_math = p->math != POLYCONV_MATH_FP32_FMA;
   if (k == POLYCONV_KERNEL_AUTO || k == POLYCONV_KERNEL_TC_PAIR) p->pair = pair_tiling(g, p->fmt, p->io_bf16, p->num_sms);
   // 1x1: x is already the (MN-major) position operand when its planes have a 16-byte pitch;
-  // strided 1x1 layers gather their output lattice first.  Stride-1 layers on other plane
-  // sizes measured faster on the packed path (tools/layer_sweep.py)
+  // other 1x1 layers gather their output lattice first (mac1x1_auto)
   if (k == POLYCONV_KERNEL_AUTO && mac1x1_supported(g, p->fmt, p->io_bf16) && !getenv("POLYCONV_NO_1X1") &&
-      (mac1x1_pitch(g) == 0 || g.sh > 1 || g.sw > 1 || getenv("POLYCONV_1X1_SMALL")))
+      mac1x1_auto(g))
     k = POLYCONV_KERNEL_TC_1X1;
   if (k == POLYCONV_KERNEL_AUTO) {
     // bf16, at most two rounds of pair tiles: one launch on CTA pairs with a resident filter

@@ -77,6 +77,16 @@ def test_kernel_selection_and_forcing():
         pc.Plan((1, 4, 8, 8), (16, 4, 3, 3), math="bf16", kernel="fp32")
     p = pc.Plan((1, 4, 8, 8), (16, 4, 3, 3), math="bf16", kernel="thin")
     assert p.info()["kernel"] == "thin"
+    # 1x1 (bf16 in/out): in place on 56x56, gathered on 14x14 / strided, mac_tc2 for an
+    # expansion layer on 7x7 planes (mac1x1_auto)
+    k1 = lambda xs, ws, s=1: pc.Plan(xs, ws, (s, s), math="bf16", io_dtype="bf16").info()
+    assert (k1((4, 64, 56, 56), (256, 64, 1, 1))["kernel"], k1((4, 64, 56, 56), (256, 64, 1, 1))["launches"]) == \
+        ("tc_1x1", 2)
+    assert (k1((4, 1024, 14, 14), (256, 1024, 1, 1))["kernel"], k1((4, 1024, 14, 14), (256, 1024, 1, 1))["launches"]) \
+        == ("tc_1x1", 3)
+    assert k1((4, 256, 28, 28), (512, 256, 1, 1), 2)["kernel"] == "tc_1x1"
+    assert k1((4, 1024, 7, 7), (512, 1024, 1, 1))["kernel"] == "tc_1x1"
+    assert k1((4, 512, 7, 7), (2048, 512, 1, 1))["kernel"] == "tc"
 
 
 def test_tc_tiling_choices():
