@@ -11,8 +11,9 @@
 // (i = i'*s + a, j = j'*s + b), so the polynomial method of the inner plan runs
 // on s^2*C channels of ceil(R/s) x ceil(S/s) kernels and computes only the
 // lattice.  xq is cropped to exactly P + Rq - 1 rows and Q + Sq - 1 columns.
-// Both transforms are copies (HBM-bound), one thread per output element,
-// consecutive threads along the contiguous output dimension.
+// Both transforms are copies (HBM-bound): x one warp per output row (lanes along the
+// contiguous output dimension), w one thread per output element.
+#include <algorithm>
 #include "common.cuh"
 
 namespace polyconv {
@@ -22,21 +23,25 @@ namespace {
 template <typename T>
 __global__ void __launch_bounds__(256) s2d_kernel(const T* __restrict__ x, T* __restrict__ xq, int N, int C, int H,
                                                   int W, int s, int ph, int pw, int Hq, int Wq) {
-  const long long total = (long long)N * s * s * C * Hq * Wq;
-  for (long long idx = blockIdx.x * (long long)blockDim.x + threadIdx.x; idx < total;
-       idx += (long long)gridDim.x * blockDim.x) {
-    const int v = (int)(idx % Wq);
-    long long r = idx / Wq;
+  // one warp per output row (n, (a, b, c), u), lanes along v: the row's index math is done
+  // once and in 32 bits; reads are strided by s, writes contiguous
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const long long rows = (long long)N * s * s * C * Hq;
+  for (long long r = (long long)blockIdx.x * 8 + warp; r < rows; r += (long long)gridDim.x * 8) {
     const int u = (int)(r % Hq);
-    r /= Hq;
-    const int cq = (int)(r % ((long long)s * s * C));
-    const int n = (int)(r / ((long long)s * s * C));
+    const long long nq = r / Hq;
+    const int cq = (int)(nq % ((long long)s * s * C));
+    const int n = (int)(nq / ((long long)s * s * C));
     const int ab = cq / C, c = cq - ab * C;
     const int a = ab / s, b = ab - a * s;
-    const int h = u * s + a - ph, w = v * s + b - pw;
-    T val = T(0.f);
-    if (h >= 0 && h < H && w >= 0 && w < W) val = x[(((long long)n * C + c) * H + h) * W + w];
-    xq[idx] = val;
+    const int h = u * s + a - ph;
+    T* dst = xq + r * Wq;
+    const bool hin = h >= 0 && h < H;
+    const T* src = x + (((long long)n * C + c) * H + (hin ? h : 0)) * W;
+    for (int v = lane; v < Wq; v += 32) {
+      const int w = v * s + b - pw;
+      dst[v] = (hin && w >= 0 && w < W) ? src[w] : T(0.f);
+    }
   }
 }
 
@@ -71,17 +76,18 @@ inline unsigned blocks_for(long long n) {
 cudaError_t launch_polyphase(const Geom& g, int Hq, int Wq, int Rq, int Sq, const void* x, const void* w, void* xq,
                              void* wq, bool io_bf16, cudaStream_t st) {
   const int s = g.sh;
-  const long long nx = (long long)g.N * s * s * g.C * Hq * Wq;
   const long long nw = (long long)g.K * s * s * g.C * Rq * Sq;
+  const long long xrows = (long long)g.N * s * s * g.C * Hq;
+  const unsigned xblocks = (unsigned)std::min<long long>(std::max<long long>((xrows + 7) / 8, 1), 148LL * 32);
   if (io_bf16) {
-    s2d_kernel<__nv_bfloat16><<<blocks_for(nx), 256, 0, st>>>(static_cast<const __nv_bfloat16*>(x),
+    s2d_kernel<__nv_bfloat16><<<xblocks, 256, 0, st>>>(static_cast<const __nv_bfloat16*>(x),
                                                                static_cast<__nv_bfloat16*>(xq), g.N, g.C, g.H, g.W,
                                                                s, g.ph, g.pw, Hq, Wq);
     wphase_kernel<__nv_bfloat16><<<blocks_for(nw), 256, 0, st>>>(static_cast<const __nv_bfloat16*>(w),
                                                                   static_cast<__nv_bfloat16*>(wq), g.K, g.C, g.R,
                                                                   g.S, s, Rq, Sq);
   } else {
-    s2d_kernel<float><<<blocks_for(nx), 256, 0, st>>>(static_cast<const float*>(x), static_cast<float*>(xq), g.N,
+    s2d_kernel<float><<<xblocks, 256, 0, st>>>(static_cast<const float*>(x), static_cast<float*>(xq), g.N,
                                                        g.C, g.H, g.W, s, g.ph, g.pw, Hq, Wq);
     wphase_kernel<float><<<blocks_for(nw), 256, 0, st>>>(static_cast<const float*>(w), static_cast<float*>(wq),
                                                           g.K, g.C, g.R, g.S, s, Rq, Sq);
