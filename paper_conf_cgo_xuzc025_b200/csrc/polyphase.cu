@@ -11,8 +11,8 @@
 // (i = i'*s + a, j = j'*s + b), so the polynomial method of the inner plan runs
 // on s^2*C channels of ceil(R/s) x ceil(S/s) kernels and computes only the
 // lattice.  xq is cropped to exactly P + Rq - 1 rows and Q + Sq - 1 columns.
-// Both transforms are copies (HBM-bound): x one warp per output row (lanes along the
-// contiguous output dimension), w one thread per output element.
+// Both transforms are copies (HBM-bound): x one block per output plane (warps over rows,
+// lanes along the contiguous output dimension), w one thread per output element.
 #include <algorithm>
 #include "common.cuh"
 
@@ -23,24 +23,25 @@ namespace {
 template <typename T>
 __global__ void __launch_bounds__(256) s2d_kernel(const T* __restrict__ x, T* __restrict__ xq, int N, int C, int H,
                                                   int W, int s, int ph, int pw, int Hq, int Wq) {
-  // one warp per output row (n, (a, b, c), u), lanes along v: the row's index math is done
-  // once and in 32 bits; reads are strided by s, writes contiguous
+  // one block per output plane (n, (a, b), c), decoded once; warps over its rows u, lanes
+  // along v (contiguous writes; reads strided by s, the other phases hit the same sectors)
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const long long rows = (long long)N * s * s * C * Hq;
-  for (long long r = (long long)blockIdx.x * 8 + warp; r < rows; r += (long long)gridDim.x * 8) {
-    const int u = (int)(r % Hq);
-    const long long nq = r / Hq;
-    const int cq = (int)(nq % ((long long)s * s * C));
-    const int n = (int)(nq / ((long long)s * s * C));
+  const int planes = N * s * s * C;
+  for (int pl = blockIdx.x; pl < planes; pl += gridDim.x) {
+    const int n = pl / (s * s * C), cq = pl - n * (s * s * C);
     const int ab = cq / C, c = cq - ab * C;
     const int a = ab / s, b = ab - a * s;
-    const int h = u * s + a - ph;
-    T* dst = xq + r * Wq;
-    const bool hin = h >= 0 && h < H;
-    const T* src = x + (((long long)n * C + c) * H + (hin ? h : 0)) * W;
-    for (int v = lane; v < Wq; v += 32) {
-      const int w = v * s + b - pw;
-      dst[v] = (hin && w >= 0 && w < W) ? src[w] : T(0.f);
+    const T* xp = x + ((long long)n * C + c) * H * W;
+    T* dp = xq + (long long)pl * Hq * Wq;
+    for (int u = warp; u < Hq; u += 8) {
+      const int h = u * s + a - ph;
+      const bool hin = h >= 0 && h < H;
+      const T* src = xp + (long long)(hin ? h : 0) * W;
+      T* dst = dp + (long long)u * Wq;
+      for (int v = lane; v < Wq; v += 32) {
+        const int w = v * s + b - pw;
+        dst[v] = (hin && w >= 0 && w < W) ? src[w] : T(0.f);
+      }
     }
   }
 }
@@ -77,8 +78,8 @@ cudaError_t launch_polyphase(const Geom& g, int Hq, int Wq, int Rq, int Sq, cons
                              void* wq, bool io_bf16, cudaStream_t st) {
   const int s = g.sh;
   const long long nw = (long long)g.K * s * s * g.C * Rq * Sq;
-  const long long xrows = (long long)g.N * s * s * g.C * Hq;
-  const unsigned xblocks = (unsigned)std::min<long long>(std::max<long long>((xrows + 7) / 8, 1), 148LL * 32);
+  const long long planes = (long long)g.N * s * s * g.C;  // < 2^31: the plan's element limits
+  const unsigned xblocks = (unsigned)std::min<long long>(std::max<long long>(planes, 1), 148LL * 16);
   if (io_bf16) {
     s2d_kernel<__nv_bfloat16><<<xblocks, 256, 0, st>>>(static_cast<const __nv_bfloat16*>(x),
                                                                static_cast<__nv_bfloat16*>(xq), g.N, g.C, g.H, g.W,
