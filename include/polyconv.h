@@ -158,8 +158,14 @@ polyconv_status_t polyconv_forward(polyconv_plan_t plan, const void *x, const vo
  * pointers (pinned for asynchronous copies; pageable works but serialises).
  * Enqueues on `stream`: H2D copy of x and w into plan-owned device buffers
  * (allocated at first use, freed by polyconv_destroy), polyconv_forward, D2H
- * copy of y.  Does not synchronise: x, w, y must stay valid until `stream`
- * is synchronised.  Errors as polyconv_forward (ALLOC_FAILED if the device
+ * copy of y.  For N >= 2 the batch is pipelined in chunks (environment
+ * POLYCONV_HOST_CHUNKS, default 4, 1 = off): chunk copies run on two
+ * plan-owned copy streams ordered by events after the work already on
+ * `stream`, each chunk's forward (a plan-owned sub-plan with this plan's
+ * kernel: the same bytes as one polyconv_forward) on `stream`, and `stream`
+ * waits for the last copy.  Not pipelined for stride >= 2 polyphase plans or
+ * while timing events are set.  Does not synchronise: x, w, y must stay valid
+ * until `stream` is synchronised.  Errors as polyconv_forward (ALLOC_FAILED if the device
  * buffers cannot be allocated). */
 polyconv_status_t polyconv_forward_host(polyconv_plan_t plan, const void *x, const void *w,
                                         void *y, void *stream);

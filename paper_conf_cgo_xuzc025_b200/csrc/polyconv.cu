@@ -45,6 +45,13 @@ struct polyconv_plan_s {
   void* hx = nullptr;
   void* hw = nullptr;
   void* hy = nullptr;
+  // ... and its copy/compute pipeline over batch chunks: sub-plans of nc and of the tail
+  // images (same kernel), two copy streams, per-chunk events
+  int hchunks = 0, hnc = 0;
+  polyconv_plan_s* hsub = nullptr;
+  polyconv_plan_s* hsub_tail = nullptr;
+  cudaStream_t hs_in = nullptr, hs_out = nullptr;
+  cudaEvent_t hev[3 * 16 + 2] = {};
   // polyconv_plan_set_timing_events: recorded around the MAC launch
   cudaEvent_t ev_start = nullptr;
   cudaEvent_t ev_stop = nullptr;
@@ -338,6 +345,10 @@ polyconv_status_t polyconv_plan_set_kernel(polyconv_plan_t p, polyconv_kernel_t 
   if (p->pair_state) { pair_state_free(p->pair_state); p->pair_state = nullptr; }
   if (p->wsA) { cudaFree(p->wsA); p->wsA = nullptr; }
   if (p->wsU) { cudaFree(p->wsU); p->wsU = nullptr; }
+  // the forward_host pipeline's sub-plans carry the old kernel: rebuilt on the next call
+  if (p->hsub) { polyconv_destroy(p->hsub); p->hsub = nullptr; }
+  if (p->hsub_tail) { polyconv_destroy(p->hsub_tail); p->hsub_tail = nullptr; }
+  p->hchunks = 0;
   return POLYCONV_STATUS_SUCCESS;
 }
 
@@ -518,6 +529,45 @@ polyconv_status_t polyconv_forward(polyconv_plan_t p, const void* x, const void*
   return finish(p, e, "mac_thin");
 }
 
+// forward_host pipeline setup (lazy): G = POLYCONV_HOST_CHUNKS (default 4, 1 = off) chunks of
+// ceil(N/G) images, each a forward of a sub-plan forced to this plan's kernel, so every image
+// gets the arithmetic of a plain forward (the kernels are batch-shard invariant).  Not for
+// polyphase plans or when the timing hook is set; false = the unpipelined path.
+static bool host_pipeline(polyconv_plan_t p) {
+  if (p->hchunks < 0) return false;
+  if (p->hchunks > 0) return true;
+  p->hchunks = -1;
+  const char* ev = getenv("POLYCONV_HOST_CHUNKS");
+  int G = ev ? atoi(ev) : 4;
+  G = std::min(std::min(G, 16), p->g.N);
+  if (G < 2 || p->inner || p->ev_start) return false;
+  const int nc = (p->g.N + G - 1) / G;
+  G = (p->g.N + nc - 1) / nc;
+  const int tail = p->g.N - (G - 1) * nc;
+  const Geom& g = p->g;
+  const polyconv_dtype_t io = p->io_bf16 ? POLYCONV_BF16 : POLYCONV_F32;
+  const polyconv_math_t m = static_cast<polyconv_math_t>(p->math);
+  auto make = [&](int n, polyconv_plan_s** out) {
+    if (polyconv_plan(out, n, g.C, g.H, g.W, g.K, g.R, g.S, g.sh, g.sw, g.ph, g.pw, io, m, p->device) !=
+        POLYCONV_STATUS_SUCCESS)
+      return false;
+    return polyconv_plan_set_kernel(*out, static_cast<polyconv_kernel_t>(p->kernel)) == POLYCONV_STATUS_SUCCESS;
+  };
+  bool ok = make(nc, &p->hsub) && (tail == nc || make(tail, &p->hsub_tail));
+  DeviceGuard guard(p->device);
+  ok = ok && (p->hs_in || cudaStreamCreateWithFlags(&p->hs_in, cudaStreamNonBlocking) == cudaSuccess) &&
+       (p->hs_out || cudaStreamCreateWithFlags(&p->hs_out, cudaStreamNonBlocking) == cudaSuccess);
+  for (int i = 0; ok && i < 2 + 3 * G; ++i)
+    ok = p->hev[i] || cudaEventCreateWithFlags(&p->hev[i], cudaEventDisableTiming) == cudaSuccess;
+  if (!ok) {
+    cudaGetLastError();
+    return false;  // resources stay owned by the plan and are freed by polyconv_destroy
+  }
+  p->hchunks = G;
+  p->hnc = nc;
+  return true;
+}
+
 polyconv_status_t polyconv_forward_host(polyconv_plan_t p, const void* x, const void* w, void* y, void* stream) {
   if (!p) return POLYCONV_STATUS_BAD_PARAM;
   if (!x || !w || !y || x == y || w == y) return POLYCONV_STATUS_BAD_PARAM;
@@ -534,6 +584,45 @@ polyconv_status_t polyconv_forward_host(polyconv_plan_t p, const void* x, const 
     }
   }
   cudaStream_t st = static_cast<cudaStream_t>(stream);
+  if (host_pipeline(p)) {
+    // chunk i: H2D of its images on hs_in -> forward on `stream` -> D2H on hs_out, so the two
+    // copy directions and the MAC of neighbouring chunks overlap; `stream` waits for the last
+    // D2H, so synchronising it covers the whole call
+    const int G = p->hchunks, nc = p->hnc;
+    const size_t xi = xb / g.N, yi = yb / g.N;
+    cudaEvent_t* ev = p->hev;  // [0] entry, [1] done, [2 + 3i] in, [3 + 3i] computed
+    cudaError_t e = cudaEventRecord(ev[0], st);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(p->hs_in, ev[0], 0);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(p->hs_out, ev[0], 0);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(p->hw, w, wb, cudaMemcpyHostToDevice, p->hs_in);
+    for (int i = 0; i < G && e == cudaSuccess; ++i) {
+      const int n0 = i * nc, n = std::min(nc, g.N - n0);
+      e = cudaMemcpyAsync(static_cast<char*>(p->hx) + n0 * xi, static_cast<const char*>(x) + n0 * xi, n * xi,
+                          cudaMemcpyHostToDevice, p->hs_in);
+      if (e == cudaSuccess) e = cudaEventRecord(ev[2 + 3 * i], p->hs_in);
+    }
+    if (e != cudaSuccess) return finish(p, e, "forward_host H2D");
+    for (int i = 0; i < G; ++i) {
+      const int n0 = i * nc, n = std::min(nc, g.N - n0);
+      if ((e = cudaStreamWaitEvent(st, ev[2 + 3 * i], 0)) != cudaSuccess) return finish(p, e, "forward_host wait");
+      polyconv_plan_s* sp = n == nc ? p->hsub : p->hsub_tail;
+      polyconv_status_t s = polyconv_forward(sp, static_cast<char*>(p->hx) + n0 * xi, p->hw,
+                                             static_cast<char*>(p->hy) + n0 * yi, stream);
+      if (s != POLYCONV_STATUS_SUCCESS) {
+        snprintf(p->err, sizeof(p->err), "forward_host chunk %d: %s", i, sp->err);
+        return s;
+      }
+      e = cudaEventRecord(ev[3 + 3 * i], st);
+      if (e == cudaSuccess) e = cudaStreamWaitEvent(p->hs_out, ev[3 + 3 * i], 0);
+      if (e == cudaSuccess)
+        e = cudaMemcpyAsync(static_cast<char*>(y) + n0 * yi, static_cast<char*>(p->hy) + n0 * yi, n * yi,
+                            cudaMemcpyDeviceToHost, p->hs_out);
+      if (e != cudaSuccess) return finish(p, e, "forward_host D2H");
+    }
+    e = cudaEventRecord(ev[1], p->hs_out);
+    if (e == cudaSuccess) e = cudaStreamWaitEvent(st, ev[1], 0);
+    return finish(p, e, "forward_host join");
+  }
   cudaError_t e = cudaMemcpyAsync(p->hx, x, xb, cudaMemcpyHostToDevice, st);
   if (e == cudaSuccess) e = cudaMemcpyAsync(p->hw, w, wb, cudaMemcpyHostToDevice, st);
   if (e != cudaSuccess) return finish(p, e, "forward_host H2D");
@@ -620,6 +709,15 @@ polyconv_status_t polyconv_destroy(polyconv_plan_t p) {
     if (p->fcount) cudaFree(p->fcount);
   }
   if (p->pair_state) pair_state_free(p->pair_state);
+  if (p->hsub && polyconv_destroy(p->hsub) != POLYCONV_STATUS_SUCCESS) s = POLYCONV_STATUS_EXECUTION_FAILED;
+  if (p->hsub_tail && polyconv_destroy(p->hsub_tail) != POLYCONV_STATUS_SUCCESS) s = POLYCONV_STATUS_EXECUTION_FAILED;
+  if (p->hs_in || p->hs_out || p->hev[0]) {
+    DeviceGuard guard(p->device);
+    for (cudaEvent_t e : p->hev)
+      if (e) cudaEventDestroy(e);
+    if (p->hs_in) cudaStreamDestroy(p->hs_in);
+    if (p->hs_out) cudaStreamDestroy(p->hs_out);
+  }
   if (p->inner) {
     if (polyconv_destroy(p->inner) != POLYCONV_STATUS_SUCCESS) s = POLYCONV_STATUS_EXECUTION_FAILED;
     DeviceGuard guard(p->device);

@@ -384,3 +384,35 @@ def test_1x1_gathered(shape):
     y, plan = gpu_forward(shape, x, w, math="bf16", io="bf16", kernel="tc_1x1")
     assert plan.info()["kernel"] == "tc_1x1" and plan.info()["launches"] == 3
     assert np.array_equal(y, bf16_round(ref))
+
+
+@pytest.mark.parametrize("shape,math,io", [
+    (ConvShape("host_pair", 7, 64, 28, 28, 64, 3, 3, 1, 1, 1, 1), "bf16", "bf16"),   # 4 chunks, tail of 1
+    (ConvShape("host_1x1", 6, 64, 16, 16, 128, 1, 1), "bf16", "bf16"),              # 3 chunks of 2
+    (ConvShape("host_fp32", 5, 16, 12, 12, 32, 3, 3, 1, 1, 1, 1), "fp32", "f32"),  # 3 chunks, tail 1
+    (ConvShape("host_s2", 4, 16, 15, 15, 32, 7, 7, 2, 2, 3, 3), "bf16", "bf16")],    # polyphase: one piece
+    ids=lambda v: v.name if isinstance(v, ConvShape) else str(v))
+@pytest.mark.parametrize("chunks", ["default", "1"])
+def test_forward_host_pipeline(shape, math, io, chunks, monkeypatch):
+    """polyconv_forward_host (pinned host buffers): the chunked copy/compute pipeline gives the
+    bytes of a device forward of the whole batch (same kernel per chunk), repeated calls too,
+    and integer data equals round(oracle)."""
+    import torch
+    import paper_conf_cgo_xuzc025_b200 as pc
+    if chunks != "default":
+        monkeypatch.setenv("POLYCONV_HOST_CHUNKS", chunks)
+    x, w = synth.make_inputs(shape, synth.seed_for(17, hash(shape.name) % 997), "int")
+    dt = torch.bfloat16 if io == "bf16" else torch.float32
+    xh = torch.from_numpy(x).to(dt).contiguous().pin_memory()
+    wh = torch.from_numpy(w).to(dt).contiguous().pin_memory()
+    plan = pc.Plan(xh.shape, wh.shape, shape.stride, shape.padding, math=math, io_dtype=io)
+    yh = torch.empty(plan.output_shape, dtype=dt).pin_memory()
+    for _ in range(3):
+        yh.zero_()
+        plan.forward_host(xh, wh, yh)
+        torch.cuda.synchronize()
+        yd = plan.forward(xh.cuda(), wh.cuda())
+        torch.cuda.synchronize()
+        assert torch.equal(yh, yd.cpu())
+    ref = oracle.conv2d(x, w, shape.stride, shape.padding)
+    assert np.array_equal(yh.float().numpy(), bf16_round(ref) if io == "bf16" else ref)
