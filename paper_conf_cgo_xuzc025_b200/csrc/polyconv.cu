@@ -81,6 +81,17 @@ bool mac1x1_auto(const Geom& g) {
   return !((long long)g.P * g.Q < 64 && g.K > g.C);
 }
 
+// mac_tc2 packing in-kernel (TC_FUSED) or by a pack launch (TC), measured per layer
+// (tools/kernel_cmp.py, ResNet-50 N=256 and VGG-16 N=64): the fused packers rebuild each
+// window once per 128-channel output tile and transpose nt + (R-1)*Wp positions per tile, so
+// fusing pays only for one output tile and narrow planes (l2_3x3_128 699 vs 584 TFLOP/s,
+// Wp = 30) and loses otherwise (VGG conv2_1, Wp = 114: 274 vs 605; conv4_2, K = 512: 818 vs
+// 1019).  POLYCONV_FUSED_ANY restores the earlier rule (every bf16-io shape the tiling takes).
+bool fused_pays(const Geom& g) {
+  if (getenv("POLYCONV_FUSED_ANY")) return true;
+  return g.K <= 128 && g.Wp <= 64;
+}
+
 // Resolve the MAC variant and fill the kernel-specific padded sizes.
 polyconv_status_t resolve(polyconv_plan_t p) {
   Geom& g = p->g;
@@ -100,7 +111,7 @@ polyconv_status_t resolve(polyconv_plan_t p) {
         !getenv("POLYCONV_NO_PAIR_DEFAULT"))
       k = POLYCONV_KERNEL_TC_PAIR;
     else if (tc_math && g.K >= 16 && tc2_supported(g, p->fmt) && p->io_bf16 && !getenv("POLYCONV_NO_FUSED_DEFAULT") &&
-        tc2_is_mx(tc2_tiling(g, p->fmt, p->io_bf16, p->num_sms, true, p->io_bf16)))
+             fused_pays(g) && tc2_is_mx(tc2_tiling(g, p->fmt, p->io_bf16, p->num_sms, true, p->io_bf16)))
       k = POLYCONV_KERNEL_TC_FUSED;  // bf16 in/out: one launch, input packed in-kernel
     else if (tc_math)
       k = (g.K >= 16 && tc2_supported(g, p->fmt))  ? POLYCONV_KERNEL_TC
