@@ -106,12 +106,18 @@ polyconv_status_t resolve(polyconv_plan_t p) {
   if (k == POLYCONV_KERNEL_AUTO) {
     // bf16, at most two rounds of pair tiles: one launch on CTA pairs with a resident filter
     // (its fixed startup wins on small problems); larger problems pipeline better in mac_tc2
-    // (measured per layer: tools/layer_sweep.py)
+    // (measured per layer: tools/layer_sweep.py). Below one full round of pair
+    // tiles the one-launch TC_FUSED kernel starts faster where it applies (tools/kernel_cmp.py
+    // synthnet: 14x14 C=64 K=64 N=32, 32 pair tiles on 74 pairs, 19.7 vs 14.6 TFLOP/s).
+    const bool fused_any = tc_math && g.K >= 16 && tc2_supported(g, p->fmt) && p->io_bf16 &&
+                           !getenv("POLYCONV_NO_FUSED_DEFAULT") && fused_pays(g);
+    const bool fused_ok =
+        fused_any && tc2_is_mx(tc2_tiling(g, p->fmt, p->io_bf16, p->num_sms, true, p->io_bf16));
+    const bool under_one_round = p->pair.ok && p->pair.num_tiles < p->num_sms / 2;
     if (tc_math && g.K >= 16 && p->pair.ok && p->pair.num_tiles <= 2 * p->pair.num_pairs &&
-        !getenv("POLYCONV_NO_PAIR_DEFAULT"))
+        !(under_one_round && fused_any) && !getenv("POLYCONV_NO_PAIR_DEFAULT"))
       k = POLYCONV_KERNEL_TC_PAIR;
-    else if (tc_math && g.K >= 16 && tc2_supported(g, p->fmt) && p->io_bf16 && !getenv("POLYCONV_NO_FUSED_DEFAULT") &&
-             fused_pays(g) && tc2_is_mx(tc2_tiling(g, p->fmt, p->io_bf16, p->num_sms, true, p->io_bf16)))
+    else if (fused_ok || (under_one_round && fused_any))
       k = POLYCONV_KERNEL_TC_FUSED;  // bf16 in/out: one launch, input packed in-kernel
     else if (tc_math)
       k = (g.K >= 16 && tc2_supported(g, p->fmt))  ? POLYCONV_KERNEL_TC

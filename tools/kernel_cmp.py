@@ -16,7 +16,12 @@ import synth  # noqa: E402
 
 which = sys.argv[1] if len(sys.argv) > 1 else "all"
 reps = int(sys.argv[2]) if len(sys.argv) > 2 else 10
-layers = {"resnet50": synth.RESNET50, "vgg16": synth.VGG16}.get(which, synth.RESNET50 + synth.VGG16)
+# the unique layers of the synthetic 20-layer nets (torch_integration.SyntheticNet, batch 32, width 64)
+SYNTHNET = [synth.ConvShape("syn_%d_%d_%d_r%d" % (H, C, K, R), 32, C, H, H, K, R, R, 1, 1, R // 2, R // 2)
+            for H in (4, 8, 14, 28, 56) for (C, K, R) in ((64, 64, 3), (64, 128, 5), (128, 64, 1), (64, 128, 7),
+                                                         (128, 64, 3))]
+layers = {"resnet50": synth.RESNET50, "vgg16": synth.VGG16, "synthnet": SYNTHNET}.get(
+    which, synth.RESNET50 + synth.VGG16)
 flush = torch.empty(64 << 20, device="cuda")
 
 
