@@ -86,10 +86,12 @@ bool mac1x1_auto(const Geom& g) {
 // window once per 128-channel output tile and transpose nt + (R-1)*Wp positions per tile, so
 // fusing pays only for one output tile and narrow planes (l2_3x3_128 699 vs 584 TFLOP/s,
 // Wp = 30) and loses otherwise (VGG conv2_1, Wp = 114: 274 vs 605; conv4_2, K = 512: 818 vs
-// 1019).  POLYCONV_FUSED_ANY restores the earlier rule (every bf16-io shape the tiling takes).
+// 1019).  Kernels larger than 3x3 lose too (synthetic nets, N=32: 5x5 / 7x7, C=64 -> K=128 on
+// 56x56 planes 565 vs 637 and 651 vs 779; on 8x8 planes 32.7 vs 35.6 and 41.3 vs 45.8).
+// POLYCONV_FUSED_ANY restores the earlier rule (every bf16-io shape the tiling takes).
 bool fused_pays(const Geom& g) {
   if (getenv("POLYCONV_FUSED_ANY")) return true;
-  return g.K <= 128 && g.Wp <= 64;
+  return g.K <= 128 && g.Wp <= 64 && g.R * g.S <= 9;
 }
 
 // Resolve the MAC variant and fill the kernel-specific padded sizes.
@@ -107,17 +109,20 @@ polyconv_status_t resolve(polyconv_plan_t p) {
     // bf16, at most two rounds of pair tiles: one launch on CTA pairs with a resident filter
     // (its fixed startup wins on small problems); larger problems pipeline better in mac_tc2
     // (measured per layer: tools/layer_sweep.py). Below one full round of pair
-    // tiles the one-launch TC_FUSED kernel starts faster where it applies (tools/kernel_cmp.py
-    // synthnet: 14x14 C=64 K=64 N=32, 32 pair tiles on 74 pairs, 19.7 vs 14.6 TFLOP/s).
-    const bool fused_any = tc_math && g.K >= 16 && tc2_supported(g, p->fmt) && p->io_bf16 &&
-                           !getenv("POLYCONV_NO_FUSED_DEFAULT") && fused_pays(g);
-    const bool fused_ok =
-        fused_any && tc2_is_mx(tc2_tiling(g, p->fmt, p->io_bf16, p->num_sms, true, p->io_bf16));
-    const bool under_one_round = p->pair.ok && p->pair.num_tiles < p->num_sms / 2;
-    if (tc_math && g.K >= 16 && p->pair.ok && p->pair.num_tiles <= 2 * p->pair.num_pairs &&
-        !(under_one_round && fused_any) && !getenv("POLYCONV_NO_PAIR_DEFAULT"))
+    // tiles with bf16 I/O, the pack launch + mac_tc2 pipeline starts faster than either one-launch
+    // kernel (tools/kernel_cmp.py synthnet, N=32, 3x3, TFLOP/s tc / pair / fused: 8x8 C=K=64
+    // 9.8 / 7.8 / 8.7, 14x14 C=128 K=64 33.5 / 25.7 / 29.1; 5 of 6 such layers).
+    const bool fused_ok = tc_math && g.K >= 16 && tc2_supported(g, p->fmt) && p->io_bf16 &&
+                          !getenv("POLYCONV_NO_FUSED_DEFAULT") && fused_pays(g) &&
+                          tc2_is_mx(tc2_tiling(g, p->fmt, p->io_bf16, p->num_sms, true, p->io_bf16));
+    const bool small_tc = p->pair.ok && p->pair.num_tiles < p->num_sms / 2 && p->io_bf16 && tc_math &&
+                          g.K >= 16 && tc2_supported(g, p->fmt) && !getenv("POLYCONV_SMALL_PAIR");
+    if (tc_math && g.K >= 16 && p->pair.ok && p->pair.num_tiles <= 2 * p->pair.num_pairs && !small_tc &&
+        !getenv("POLYCONV_NO_PAIR_DEFAULT"))
       k = POLYCONV_KERNEL_TC_PAIR;
-    else if (fused_ok || (under_one_round && fused_any))
+    else if (small_tc)
+      k = POLYCONV_KERNEL_TC;
+    else if (fused_ok)
       k = POLYCONV_KERNEL_TC_FUSED;  // bf16 in/out: one launch, input packed in-kernel
     else if (tc_math)
       k = (g.K >= 16 && tc2_supported(g, p->fmt))  ? POLYCONV_KERNEL_TC

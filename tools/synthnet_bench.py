@@ -4,7 +4,7 @@ once with PyTorch's own conv2d (cuDNN, NCHW, benchmark=True) and once after `rep
 (every convolution through libpolyconv.so, AUTO kernel). Same weights, same seeded input, bf16.
 
 Per conv layer, CUDA events recorded by forward hooks on the current stream bracket the operator;
-the sum over the 20 layers is averaged over --iters passes after --warmup passes.
+the sum over the 20 layers is the median of --iters passes after --warmup passes.
 Usage: python tools/synthnet_bench.py [--batch 32] [--width 64] [--sizes 4,8,...] > out.jsonl
 """
 from __future__ import annotations
@@ -53,7 +53,9 @@ def timed_conv_ms(net, x, warmup, iters):
         torch.cuda.synchronize()
     for h in hs:
         h.remove()
-    return sum(a.elapsed_time(b) for a, b in pairs) / iters
+    per_pass = sorted(sum(a.elapsed_time(b) for a, b in pairs[i * ti.N_LAYERS:(i + 1) * ti.N_LAYERS])
+                      for i in range(iters))
+    return per_pass[iters // 2]  # median pass (host hiccups land in single passes)
 
 
 def main():
