@@ -87,6 +87,18 @@ def test_kernel_selection_and_forcing():
     assert k1((4, 256, 28, 28), (512, 256, 1, 1), 2)["kernel"] == "tc_1x1"
     assert k1((4, 1024, 7, 7), (512, 1024, 1, 1))["kernel"] == "tc_1x1"
     assert k1((4, 512, 7, 7), (2048, 512, 1, 1))["kernel"] == "tc"
+    # bf16 in/out (synthetic-net kernel comparison): mac_pair from one full round of
+    # pair tiles (conv3_x: 112 on 74 pairs), pack + mac_tc2 below it; in-kernel packing
+    # (TC_FUSED) for 3x3 on narrow planes only, a pack launch for 5x5 / 7x7
+    k3 = lambda xs, ws: pc.Plan(xs, ws, (1, 1), (ws[2] // 2, ws[3] // 2), math="bf16", io_dtype="bf16").info()["kernel"]
+    assert k3((32, 128, 28, 28), (128, 128, 3, 3)) == "tc_pair"
+    assert k3((32, 64, 8, 8), (64, 64, 3, 3)) == "tc"
+    assert k3((32, 128, 14, 14), (64, 128, 3, 3)) == "tc"
+    assert k3((32, 64, 56, 56), (64, 64, 3, 3)) == "tc_fused"
+    assert k3((32, 64, 56, 56), (128, 64, 5, 5)) == "tc"
+    assert k3((32, 64, 56, 56), (128, 64, 7, 7)) == "tc"
+    # f32 I/O keeps mac_pair on small problems (the sub-round rule was measured for bf16 I/O)
+    assert pc.Plan((32, 64, 8, 8), (64, 64, 3, 3), (1, 1), (1, 1), math="bf16").info()["kernel"] == "tc_pair"
 
 
 def test_tc_tiling_choices():
