@@ -197,6 +197,24 @@ polyconv_status_t polyconv_packed_bytes(polyconv_plan_t plan, int which,
 polyconv_status_t polyconv_extract(polyconv_plan_t plan, const float *coeffs, void *y,
                                    void *stream);
 
+/* --- Gradients (an extension, the paper is forward-only) -------------
+ * For a stride-1 convolution y = conv(x, w) with padding (ph, pw) both gradients are
+ * forward convolutions (cross-correlation, P.138-150) on re-laid-out operands:
+ *   dx   = conv(dy, wt),   wt = polyconv_flip_filter(w),  padding (R-1-ph, S-1-pw)
+ *   dw^T = conv(x^T, dy^T) with padding (ph, pw),  ^T = polyconv_swap_nc
+ * so a forward plan of the transformed shapes computes them.  Both calls are plain
+ * stream-ordered device copies (bit-exact), allocate nothing, and return BAD_PARAM for
+ * NULL/aliased pointers, dims < 1 or a bad dtype, NOT_SUPPORTED past 2^31 (flip) or 2^40 (swap)
+ * elements, EXECUTION_FAILED if the launch fails.  Device pointers, caller-owned. */
+
+/* wt[c][k][R-1-i][S-1-j] = w[k][c][i][j]; w is [K][C][R][S], wt is [C][K][R][S]. */
+polyconv_status_t polyconv_flip_filter(const void *w, void *wt, int K, int C, int R, int S,
+                                       polyconv_dtype_t dtype, void *stream);
+
+/* xt[c][n][e] = x[n][c][e] for e < HW; x is [N][C][HW], xt is [C][N][HW]. */
+polyconv_status_t polyconv_swap_nc(const void *x, void *xt, int N, int C, long long HW,
+                                   polyconv_dtype_t dtype, void *stream);
+
 /* Synchronise the last stream used by the plan, free its workspace and the plan.
  * NULL is accepted (no-op). */
 polyconv_status_t polyconv_destroy(polyconv_plan_t plan);

@@ -47,7 +47,7 @@ class Info(ctypes.Structure):
 EXPORTS = ["polyconv_plan", "polyconv_plan_set_kernel", "polyconv_output_dims", "polyconv_plan_info",
            "polyconv_forward", "polyconv_forward_host", "polyconv_plan_set_timing_events", "polyconv_pack_input", "polyconv_pack_filter", "polyconv_packed_bytes",
            "polyconv_extract", "polyconv_destroy", "polyconv_status_string", "polyconv_last_error",
-           "polyconv_abi_version"]
+           "polyconv_abi_version", "polyconv_flip_filter", "polyconv_swap_nc"]
 
 _lib = None
 
@@ -80,6 +80,8 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
     lib.polyconv_last_error.argtypes = [vp]
     lib.polyconv_last_error.restype = ctypes.c_char_p
     lib.polyconv_abi_version.argtypes = []
+    lib.polyconv_flip_filter.argtypes = [vp, vp, i, i, i, i, i, vp]
+    lib.polyconv_swap_nc.argtypes = [vp, vp, i, i, ctypes.c_longlong, i, vp]
     for name in EXPORTS:
         if name not in ("polyconv_status_string", "polyconv_last_error"):
             getattr(lib, name).restype = ctypes.c_int
@@ -254,6 +256,44 @@ class Plan:
             self.close()
         except Exception:
             pass
+
+
+def _dtype_code(t):
+    import torch
+    if t.dtype == torch.bfloat16:
+        return BF16
+    if t.dtype == torch.float32:
+        return F32
+    raise PolyconvError(BAD_PARAM, "dtype %s (float32 or bfloat16)" % t.dtype)
+
+
+def flip_filter(w, stream=None):
+    """f4 layout step (include/polyconv.h): wt[c][k][R-1-i][S-1-j] = w[k][c][i][j]."""
+    import torch
+    if not w.is_cuda or not w.is_contiguous() or w.dim() != 4:
+        raise PolyconvError(BAD_PARAM, "w must be a contiguous 4-D CUDA tensor")
+    K, C, R, S = w.shape
+    wt = torch.empty((C, K, R, S), dtype=w.dtype, device=w.device)
+    st = load_library().polyconv_flip_filter(ctypes.c_void_p(w.data_ptr()), ctypes.c_void_p(wt.data_ptr()), K, C, R,
+                                            S, _dtype_code(w), _stream_ptr(stream))
+    if st != SUCCESS:
+        raise PolyconvError(st, "polyconv_flip_filter: %s" % status_string(st))
+    return wt
+
+
+def swap_nc(x, stream=None):
+    """f4 layout step (include/polyconv.h): xt[c][n][...] = x[n][c][...]."""
+    import torch
+    if not x.is_cuda or not x.is_contiguous() or x.dim() < 2:
+        raise PolyconvError(BAD_PARAM, "x must be a contiguous CUDA tensor of rank >= 2")
+    N, C = x.shape[:2]
+    hw = x.numel() // (N * C) if x.numel() else 0
+    xt = torch.empty((C, N) + tuple(x.shape[2:]), dtype=x.dtype, device=x.device)
+    st = load_library().polyconv_swap_nc(ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(xt.data_ptr()), N, C, hw,
+                                        _dtype_code(x), _stream_ptr(stream))
+    if st != SUCCESS:
+        raise PolyconvError(st, "polyconv_swap_nc: %s" % status_string(st))
+    return xt
 
 
 def conv2d(x, w, stride=(1, 1), padding=(0, 0), math="bf16", kernel="auto"):

@@ -120,3 +120,49 @@ def test_synthetic_net_cuda_graph_replay_bit_identical():
         graph.replay()
     torch.cuda.synchronize()
     assert torch.equal(out, eager)
+
+
+# --- f4: gradients through the forward library (include/polyconv.h, "Gradients") ---------------
+@pytest.mark.gpu
+@pytest.mark.parametrize("dtype", [torch.float32, torch.bfloat16])
+def test_flip_and_swap_bit_exact(dtype):
+    import paper_conf_cgo_xuzc025_b200 as pc
+    w = torch.randn(5, 3, 4, 7).to(dtype)
+    wt = pc.flip_filter(w.cuda()).cpu()
+    assert torch.equal(wt, w.permute(1, 0, 2, 3).flip(2, 3))  # wt[c][k][R-1-i][S-1-j] = w[k][c][i][j]
+    for shape in [(3, 4, 5, 7), (2, 6, 8, 8), (1, 1, 1, 1)]:   # odd rows (element loop) and 16-B rows (vector)
+        x = torch.randn(*shape).to(dtype)
+        assert torch.equal(pc.swap_nc(x.cuda()).cpu(), x.transpose(0, 1))
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("shape", [(2, 5, 9, 11, 7, 3, 3, 1, 1), (3, 4, 8, 8, 6, 5, 3, 2, 0), (2, 3, 6, 7, 4, 1, 1, 0, 0)],
+                         ids=lambda s: "x".join(map(str, s)))
+@pytest.mark.parametrize("dtype,math,gate", [(torch.float32, "fp32", 1e-5), (torch.bfloat16, "bf16", 2e-2)])
+def test_polyconv2d_gradients(shape, dtype, math, gate):
+    """dx and dw of PolyConv2d against torch's fp64 CPU autograd of the same convolution (a
+    library routine, independent of this path), normwise as the forward gates (reading R14)."""
+    N, C, H, W, K, R, S, ph, pw = shape
+    g = torch.Generator().manual_seed(sum(shape))
+    x = (torch.rand(N, C, H, W, generator=g) * 2 - 1).to(dtype)
+    w = (torch.rand(K, C, R, S, generator=g) * 2 - 1).to(dtype)
+    P, Q = H + 2 * ph - R + 1, W + 2 * pw - S + 1
+    dy = (torch.rand(N, K, P, Q, generator=g) * 2 - 1).to(dtype)
+    x64, w64 = x.double().requires_grad_(), w.double().requires_grad_()
+    torch.nn.functional.conv2d(x64, w64, padding=(ph, pw)).backward(dy.double())
+    mod = ti.PolyConv2d(C, K, (R, S), padding=(ph, pw), math=math,
+                        weight=torch.nn.Parameter(w.cuda()))
+    xc = x.cuda().requires_grad_()
+    y = mod(xc)
+    assert tuple(y.shape) == (N, K, P, Q)
+    y.backward(dy.cuda())
+    assert normwise(xc.grad.float().cpu().numpy(), x64.grad.numpy()) <= gate
+    assert normwise(mod.weight.grad.float().cpu().numpy(), w64.grad.numpy()) <= gate
+
+
+@pytest.mark.gpu
+def test_polyconv2d_backward_rejects_stride():
+    mod = ti.PolyConv2d(2, 2, 3, stride=2, padding=1, math="fp32", weight=torch.nn.Parameter(torch.randn(2, 2, 3, 3).cuda()))
+    y = mod(torch.randn(1, 2, 8, 8, device="cuda", requires_grad=True))
+    with pytest.raises(NotImplementedError):
+        y.sum().backward()
