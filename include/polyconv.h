@@ -202,7 +202,9 @@ polyconv_status_t polyconv_extract(polyconv_plan_t plan, const float *coeffs, vo
  * forward convolutions (cross-correlation, P.138-150) on re-laid-out operands:
  *   dx   = conv(dy, wt),   wt = polyconv_flip_filter(w),  padding (R-1-ph, S-1-pw)
  *   dw^T = conv(x^T, dy^T) with padding (ph, pw),  ^T = polyconv_swap_nc
- * so a forward plan of the transformed shapes computes them.  Both calls are plain
+ * so a forward plan of the transformed shapes computes them.  Stride (sh, sw) >= 2: dy is first
+ * spread onto the stride lattice (polyconv_dilate, eh/ew = (H+2ph-R) mod sh, (W+2pw-S) mod sw);
+ * dx is then the stride-1 formula on the dilated dy, and dw^T the first R x S outputs of it.  Both calls are plain
  * stream-ordered device copies (bit-exact), allocate nothing, and return BAD_PARAM for
  * NULL/aliased pointers, dims < 1 or a bad dtype, NOT_SUPPORTED past 2^31 (flip) or 2^40 (swap)
  * elements, EXECUTION_FAILED if the launch fails.  Device pointers, caller-owned. */
@@ -210,6 +212,11 @@ polyconv_status_t polyconv_extract(polyconv_plan_t plan, const float *coeffs, vo
 /* wt[c][k][R-1-i][S-1-j] = w[k][c][i][j]; w is [K][C][R][S], wt is [C][K][R][S]. */
 polyconv_status_t polyconv_flip_filter(const void *w, void *wt, int K, int C, int R, int S,
                                        polyconv_dtype_t dtype, void *stream);
+
+/* xd[n][c][sh*h][sw*w] = x[n][c][h][w], every other element 0; x is [N][C][H][W], xd is
+ * [N][C][(H-1)*sh+1+eh][(W-1)*sw+1+ew]. */
+polyconv_status_t polyconv_dilate(const void *x, void *xd, int N, int C, int H, int W, int sh, int sw,
+                                  int eh, int ew, polyconv_dtype_t dtype, void *stream);
 
 /* xt[c][n][e] = x[n][c][e] for e < HW; x is [N][C][HW], xt is [C][N][HW]. */
 polyconv_status_t polyconv_swap_nc(const void *x, void *xt, int N, int C, long long HW,

@@ -47,7 +47,8 @@ class Info(ctypes.Structure):
 EXPORTS = ["polyconv_plan", "polyconv_plan_set_kernel", "polyconv_output_dims", "polyconv_plan_info",
            "polyconv_forward", "polyconv_forward_host", "polyconv_plan_set_timing_events", "polyconv_pack_input", "polyconv_pack_filter", "polyconv_packed_bytes",
            "polyconv_extract", "polyconv_destroy", "polyconv_status_string", "polyconv_last_error",
-           "polyconv_abi_version", "polyconv_flip_filter", "polyconv_swap_nc"]
+           "polyconv_abi_version", "polyconv_flip_filter", "polyconv_swap_nc",
+           "polyconv_dilate"]
 
 _lib = None
 
@@ -82,6 +83,7 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
     lib.polyconv_abi_version.argtypes = []
     lib.polyconv_flip_filter.argtypes = [vp, vp, i, i, i, i, i, vp]
     lib.polyconv_swap_nc.argtypes = [vp, vp, i, i, ctypes.c_longlong, i, vp]
+    lib.polyconv_dilate.argtypes = [vp, vp] + [i] * 8 + [i, vp]
     for name in EXPORTS:
         if name not in ("polyconv_status_string", "polyconv_last_error"):
             getattr(lib, name).restype = ctypes.c_int
@@ -294,6 +296,22 @@ def swap_nc(x, stream=None):
     if st != SUCCESS:
         raise PolyconvError(st, "polyconv_swap_nc: %s" % status_string(st))
     return xt
+
+
+def dilate(x, stride, extra=(0, 0), stream=None):
+    """f4 layout step (include/polyconv.h): x on the stride lattice of a zero plane, plus
+    `extra` zero rows / columns at the bottom / right."""
+    import torch
+    if not x.is_cuda or not x.is_contiguous() or x.dim() != 4:
+        raise PolyconvError(BAD_PARAM, "x must be a contiguous 4-D CUDA tensor")
+    N, C, H, W = x.shape
+    (sh, sw), (eh, ew) = stride, extra
+    xd = torch.empty((N, C, (H - 1) * sh + 1 + eh, (W - 1) * sw + 1 + ew), dtype=x.dtype, device=x.device)
+    st = load_library().polyconv_dilate(ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(xd.data_ptr()), N, C, H, W,
+                                       sh, sw, eh, ew, _dtype_code(x), _stream_ptr(stream))
+    if st != SUCCESS:
+        raise PolyconvError(st, "polyconv_dilate: %s" % status_string(st))
+    return xd
 
 
 def conv2d(x, w, stride=(1, 1), padding=(0, 0), math="bf16", kernel="auto"):

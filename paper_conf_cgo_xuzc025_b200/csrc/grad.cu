@@ -5,6 +5,8 @@
 //          wt[c][k][R-1-i][S-1-j] = w[k][c][i][j]
 //   wgrad: dw^T = conv(x^T, dy^T) with padding p          -> polyconv_swap_nc (x, dy, and back)
 //          xt[c][n][:] = x[n][c][:]
+// Stride s >= 2: dx = conv(dilate(dy), flip(w)^T) and dw^T = conv(x^T, dilate(dy)^T), cropped,
+// where dilate puts dy on the stride lattice of a zero plane      -> polyconv_dilate
 // swap_nc: one block per destination row (c, n); the row is a contiguous run of HW elements in
 // both layouts, copied with 16-byte vectors when both ends are 16-byte aligned.
 #include <cuda_runtime.h>
@@ -46,6 +48,22 @@ __global__ void __launch_bounds__(256) swap_nc_kernel(const T* __restrict__ x, T
   }
 }
 
+template <typename T>
+__global__ void __launch_bounds__(256) dilate_kernel(const T* __restrict__ x, T* __restrict__ xd, long long NC, int H,
+                                                    int W, int sh, int sw, int Hd, int Wd) {
+  const long long total = NC * Hd * Wd;
+  for (long long idx = blockIdx.x * 256LL + threadIdx.x; idx < total; idx += (long long)gridDim.x * 256) {
+    // idx enumerates the destination xd[nc][hd][wd]: coalesced stores, zeros off the lattice
+    const long long nc = idx / ((long long)Hd * Wd);
+    const int t = (int)(idx - nc * Hd * Wd);
+    const int hd = t / Wd, wd = t - hd * Wd;
+    const int h = hd / sh, w = wd / sw;
+    T v = T(0);
+    if (hd == h * sh && wd == w * sw && h < H && w < W) v = x[(nc * H + h) * W + w];
+    xd[idx] = v;
+  }
+}
+
 int grid_for(long long work, int per_block) {
   long long b = (work + per_block - 1) / per_block;
   return (int)(b < 1 ? 1 : (b > 148 * 16 ? 148 * 16 : b));
@@ -72,6 +90,26 @@ extern "C" polyconv_status_t polyconv_flip_filter(const void* w, void* wt, int K
   else
     flip_filter_kernel<uint16_t><<<grid_for(total, 256), 256, 0, st>>>(
         static_cast<const uint16_t*>(w), static_cast<uint16_t*>(wt), K, C, R, S);
+  return status_of(cudaGetLastError());
+}
+
+extern "C" polyconv_status_t polyconv_dilate(const void* x, void* xd, int N, int C, int H, int W, int sh, int sw,
+                                             int eh, int ew, polyconv_dtype_t dtype, void* stream) {
+  if (!x || !xd || x == xd || N < 1 || C < 1 || H < 1 || W < 1 || sh < 1 || sw < 1 || eh < 0 || ew < 0 ||
+      (dtype != POLYCONV_F32 && dtype != POLYCONV_BF16))
+    return POLYCONV_STATUS_BAD_PARAM;
+  const long long Hd = (long long)(H - 1) * sh + 1 + eh, Wd = (long long)(W - 1) * sw + 1 + ew;
+  if (Hd * Wd >= (1LL << 31) || (long long)N * C * Hd * Wd >= (1LL << 40)) return POLYCONV_STATUS_NOT_SUPPORTED;
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  const long long total = (long long)N * C * Hd * Wd;
+  if (dtype == POLYCONV_F32)
+    dilate_kernel<uint32_t><<<grid_for(total, 256), 256, 0, st>>>(static_cast<const uint32_t*>(x),
+                                                                  static_cast<uint32_t*>(xd), (long long)N * C, H, W,
+                                                                  sh, sw, (int)Hd, (int)Wd);
+  else
+    dilate_kernel<uint16_t><<<grid_for(total, 256), 256, 0, st>>>(static_cast<const uint16_t*>(x),
+                                                                  static_cast<uint16_t*>(xd), (long long)N * C, H, W,
+                                                                  sh, sw, (int)Hd, (int)Wd);
   return status_of(cudaGetLastError());
 }
 

@@ -161,8 +161,45 @@ def test_polyconv2d_gradients(shape, dtype, math, gate):
 
 
 @pytest.mark.gpu
-def test_polyconv2d_backward_rejects_stride():
-    mod = ti.PolyConv2d(2, 2, 3, stride=2, padding=1, math="fp32", weight=torch.nn.Parameter(torch.randn(2, 2, 3, 3).cuda()))
+def test_polyconv2d_backward_rejects_wide_padding():
+    mod = ti.PolyConv2d(2, 2, 3, padding=3, math="fp32", weight=torch.nn.Parameter(torch.randn(2, 2, 3, 3).cuda()))
     y = mod(torch.randn(1, 2, 8, 8, device="cuda", requires_grad=True))
     with pytest.raises(NotImplementedError):
         y.sum().backward()
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("dtype", [torch.float32, torch.bfloat16])
+def test_dilate_bit_exact(dtype):
+    import paper_conf_cgo_xuzc025_b200 as pc
+    x = torch.randn(2, 3, 5, 4).to(dtype)
+    xd = pc.dilate(x.cuda(), (2, 3), (1, 2)).cpu()
+    ref = torch.zeros(2, 3, 4 * 2 + 1 + 1, 3 * 3 + 1 + 2, dtype=dtype)
+    ref[:, :, 0:9:2, 0:10:3] = x
+    assert torch.equal(xd, ref)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("shape", [(2, 5, 9, 11, 7, 3, 3, 1, 1, 2, 2), (3, 4, 10, 9, 6, 1, 1, 0, 0, 2, 2),
+                                   (2, 3, 15, 13, 4, 7, 7, 3, 3, 2, 2), (2, 4, 11, 10, 5, 3, 2, 1, 0, 3, 2)],
+                         ids=lambda s: "x".join(map(str, s)))
+@pytest.mark.parametrize("dtype,math,gate", [(torch.float32, "fp32", 1e-5), (torch.bfloat16, "bf16", 2e-2)])
+def test_polyconv2d_gradients_strided(shape, dtype, math, gate):
+    """Strided layers (ResNet's 3x3 / 1x1 / 7x7 stride-2 shapes, ragged and stride 3): dx and dw
+    against torch's fp64 CPU autograd."""
+    N, C, H, W, K, R, S, ph, pw, sh, sw = shape
+    g = torch.Generator().manual_seed(sum(shape))
+    x = (torch.rand(N, C, H, W, generator=g) * 2 - 1).to(dtype)
+    w = (torch.rand(K, C, R, S, generator=g) * 2 - 1).to(dtype)
+    x64, w64 = x.double().requires_grad_(), w.double().requires_grad_()
+    y64 = torch.nn.functional.conv2d(x64, w64, stride=(sh, sw), padding=(ph, pw))
+    dy = (torch.rand(y64.shape, generator=g) * 2 - 1).to(dtype)
+    y64.backward(dy.double())
+    mod = ti.PolyConv2d(C, K, (R, S), stride=(sh, sw), padding=(ph, pw), math=math,
+                        weight=torch.nn.Parameter(w.cuda()))
+    xc = x.cuda().requires_grad_()
+    y = mod(xc)
+    assert tuple(y.shape) == tuple(y64.shape)
+    y.backward(dy.cuda())
+    assert normwise(xc.grad.float().cpu().numpy(), x64.grad.numpy()) <= gate
+    assert normwise(mod.weight.grad.float().cpu().numpy(), w64.grad.numpy()) <= gate
