@@ -218,6 +218,15 @@ polyconv_status_t polyconv_flip_filter(const void *w, void *wt, int K, int C, in
 polyconv_status_t polyconv_dilate(const void *x, void *xd, int N, int C, int H, int W, int sh, int sw,
                                   int eh, int ew, polyconv_dtype_t dtype, void *stream);
 
+/* wgrad as its own split-K contraction (any stride / padding):
+ *   dw[k][c][i][j] = sum_n sum_oh sum_ow dy[n][k][oh][ow] * xpad[n][c][sh*oh+i][sw*ow+j]
+ * x [N][C][H][W], dy [N][K][P][Q] (P, Q as for the forward), dw [K][C][R][S], all in `dtype`;
+ * ws: caller-owned fp32 device workspace of K*C*R*S floats (zeroed and accumulated here with
+ * atomics, so the summation order is not fixed).  dw is written from ws (bf16: RNE). */
+polyconv_status_t polyconv_wgrad(const void *x, const void *dy, void *dw, float *ws, int N, int C,
+                                 int H, int W, int K, int R, int S, int sh, int sw, int ph, int pw,
+                                 polyconv_dtype_t dtype, void *stream);
+
 /* xt[c][n][e] = x[n][c][e] for e < HW; x is [N][C][HW], xt is [C][N][HW]. */
 polyconv_status_t polyconv_swap_nc(const void *x, void *xt, int N, int C, long long HW,
                                    polyconv_dtype_t dtype, void *stream);

@@ -48,7 +48,7 @@ EXPORTS = ["polyconv_plan", "polyconv_plan_set_kernel", "polyconv_output_dims", 
            "polyconv_forward", "polyconv_forward_host", "polyconv_plan_set_timing_events", "polyconv_pack_input", "polyconv_pack_filter", "polyconv_packed_bytes",
            "polyconv_extract", "polyconv_destroy", "polyconv_status_string", "polyconv_last_error",
            "polyconv_abi_version", "polyconv_flip_filter", "polyconv_swap_nc",
-           "polyconv_dilate"]
+           "polyconv_dilate", "polyconv_wgrad"]
 
 _lib = None
 
@@ -84,6 +84,7 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
     lib.polyconv_flip_filter.argtypes = [vp, vp, i, i, i, i, i, vp]
     lib.polyconv_swap_nc.argtypes = [vp, vp, i, i, ctypes.c_longlong, i, vp]
     lib.polyconv_dilate.argtypes = [vp, vp] + [i] * 8 + [i, vp]
+    lib.polyconv_wgrad.argtypes = [vp, vp, vp, vp] + [i] * 11 + [i, vp]
     for name in EXPORTS:
         if name not in ("polyconv_status_string", "polyconv_last_error"):
             getattr(lib, name).restype = ctypes.c_int
@@ -312,6 +313,27 @@ def dilate(x, stride, extra=(0, 0), stream=None):
     if st != SUCCESS:
         raise PolyconvError(st, "polyconv_dilate: %s" % status_string(st))
     return xd
+
+
+def wgrad(x, dy, w_shape, stride=(1, 1), padding=(0, 0), stream=None):
+    """f4 (include/polyconv.h): dw[k][c][i][j] = sum dy[n][k][oh][ow] * xpad[n][c][sh*oh+i][sw*ow+j]."""
+    import torch
+    for t, nm in ((x, "x"), (dy, "dy")):
+        if not t.is_cuda or not t.is_contiguous() or t.dim() != 4:
+            raise PolyconvError(BAD_PARAM, "%s must be a contiguous 4-D CUDA tensor" % nm)
+    if x.dtype != dy.dtype:
+        raise PolyconvError(BAD_PARAM, "x and dy must share a dtype")
+    N, C, H, W = x.shape
+    K, _, R, S = w_shape
+    dw = torch.empty((K, C, R, S), dtype=x.dtype, device=x.device)
+    ws = torch.empty(K * C * R * S, dtype=torch.float32, device=x.device)
+    st = load_library().polyconv_wgrad(ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(dy.data_ptr()),
+                                      ctypes.c_void_p(dw.data_ptr()), ctypes.c_void_p(ws.data_ptr()), N, C, H, W, K,
+                                      R, S, stride[0], stride[1], padding[0], padding[1], _dtype_code(x),
+                                      _stream_ptr(stream))
+    if st != SUCCESS:
+        raise PolyconvError(st, "polyconv_wgrad: %s" % status_string(st))
+    return dw
 
 
 def conv2d(x, w, stride=(1, 1), padding=(0, 0), math="bf16", kernel="auto"):

@@ -10,6 +10,7 @@
 // swap_nc: one block per destination row (c, n); the row is a contiguous run of HW elements in
 // both layouts, copied with 16-byte vectors when both ends are 16-byte aligned.
 #include <cuda_runtime.h>
+#include <algorithm>
 #include <cstdint>
 #include "../../include/polyconv.h"
 
@@ -129,5 +130,123 @@ extern "C" polyconv_status_t polyconv_swap_nc(const void* x, void* xt, int N, in
   else
     swap_nc_kernel<uint16_t><<<grid, 256, 0, st>>>(static_cast<const uint16_t*>(x), static_cast<uint16_t*>(xt), N,
                                                    C, HW, vec);
+  return status_of(cudaGetLastError());
+}
+
+// ---------------------------------------------------------------------------------------------
+// wgrad as its own contraction (the forward-conv mapping leaves R*S positions per plane, see
+// DESIGN.md "Backward"): per tap (i, j), dw[:, :, i, j] = DY[K x NPQ] . X_ij[NPQ x C], the NPQ
+// sum split across blocks.  Block = one tap, a 32 (k) x 32 (c) tile and a slice of the NPQ
+// positions; 32-position chunks of dy and of the tap-shifted x are staged in shared memory
+// (coalesced along positions), each thread accumulates 2 x 2 outputs in fp32 and adds them
+// into an fp32 workspace with atomics; a second pass converts to the io dtype.
+namespace {
+
+__device__ __forceinline__ float ld_as_float(const uint32_t* p, long long i) { return __uint_as_float(p[i]); }
+__device__ __forceinline__ float ld_as_float(const uint16_t* p, long long i) {
+  return __uint_as_float((uint32_t)p[i] << 16);
+}
+
+template <typename T>
+__global__ void __launch_bounds__(256) wgrad_kernel(const T* __restrict__ x, const T* __restrict__ dy,
+                                                    float* __restrict__ ws, int N, int C, int H, int W, int K, int R,
+                                                    int S, int sh, int sw, int ph, int pw, int P, int Q, int splits,
+                                                    long long per_split) {
+  __shared__ float sdy[32][33];
+  __shared__ float sx[32][33];
+  const int tap = blockIdx.z / splits, split = blockIdx.z - tap * splits;
+  const int ti = tap / S, tj = tap - ti * S;
+  const int k0 = blockIdx.x * 32, c0 = blockIdx.y * 32;
+  const long long PQ = (long long)P * Q, NPQ = (long long)N * PQ;
+  const long long p_begin = split * per_split, p_end = min(NPQ, p_begin + per_split);
+  const int tid = threadIdx.x;
+  const int tk = (tid / 16) * 2, tc = (tid % 16) * 2;
+  float acc00 = 0.f, acc01 = 0.f, acc10 = 0.f, acc11 = 0.f;
+  for (long long p0 = p_begin; p0 < p_end; p0 += 32) {
+    // stage 32 rows (k or c) x 32 positions; element e = row * 32 + pos, 4 per thread
+    for (int e = tid; e < 1024; e += 256) {
+      const int row = e >> 5, q = e & 31;
+      const long long p = p0 + q;
+      float vdy = 0.f, vx = 0.f;
+      if (p < p_end) {
+        const long long n = p / PQ;
+        const int r = (int)(p - n * PQ);
+        const int oh = r / Q, ow = r - oh * Q;
+        if (k0 + row < K) vdy = ld_as_float(dy, ((n * K + k0 + row) * P + oh) * (long long)Q + ow);
+        const int h = sh * oh + ti - ph, w = sw * ow + tj - pw;
+        if (c0 + row < C && h >= 0 && h < H && w >= 0 && w < W)
+          vx = ld_as_float(x, ((n * C + c0 + row) * H + h) * (long long)W + w);
+      }
+      sdy[row][q] = vdy;
+      sx[row][q] = vx;
+    }
+    __syncthreads();
+#pragma unroll 8
+    for (int q = 0; q < 32; ++q) {
+      const float a0 = sdy[tk][q], a1 = sdy[tk + 1][q], b0 = sx[tc][q], b1 = sx[tc + 1][q];
+      acc00 = fmaf(a0, b0, acc00);
+      acc01 = fmaf(a0, b1, acc01);
+      acc10 = fmaf(a1, b0, acc10);
+      acc11 = fmaf(a1, b1, acc11);
+    }
+    __syncthreads();
+  }
+  const long long RS = (long long)R * S;
+  auto add = [&](int k, int c, float v) {
+    if (k < K && c < C) atomicAdd(ws + ((long long)k * C + c) * RS + tap, v);
+  };
+  add(k0 + tk, c0 + tc, acc00);
+  add(k0 + tk, c0 + tc + 1, acc01);
+  add(k0 + tk + 1, c0 + tc, acc10);
+  add(k0 + tk + 1, c0 + tc + 1, acc11);
+}
+
+__global__ void __launch_bounds__(256) f32_to_out(const float* __restrict__ ws, void* __restrict__ out, long long n,
+                                                  bool bf16) {
+  for (long long i = blockIdx.x * 256LL + threadIdx.x; i < n; i += (long long)gridDim.x * 256) {
+    const float v = ws[i];
+    if (bf16) {
+      uint32_t u = __float_as_uint(v);
+      u = (u + 0x7FFFu + ((u >> 16) & 1u)) >> 16;  // round to nearest even (finite values)
+      static_cast<uint16_t*>(out)[i] = (uint16_t)u;
+    } else {
+      static_cast<float*>(out)[i] = v;
+    }
+  }
+}
+
+}  // namespace
+
+extern "C" polyconv_status_t polyconv_wgrad(const void* x, const void* dy, void* dw, float* ws, int N, int C, int H,
+                                            int W, int K, int R, int S, int sh, int sw, int ph, int pw,
+                                            polyconv_dtype_t dtype, void* stream) {
+  if (!x || !dy || !dw || !ws || N < 1 || C < 1 || H < 1 || W < 1 || K < 1 || R < 1 || S < 1 || sh < 1 || sw < 1 ||
+      ph < 0 || pw < 0 || (dtype != POLYCONV_F32 && dtype != POLYCONV_BF16))
+    return POLYCONV_STATUS_BAD_PARAM;
+  const int P = (H + 2 * ph - R) / sh + 1, Q = (W + 2 * pw - S) / sw + 1;
+  if (H + 2 * ph < R || W + 2 * pw < S || P < 1 || Q < 1) return POLYCONV_STATUS_BAD_PARAM;
+  const long long NPQ = (long long)N * P * Q, RS = (long long)R * S;
+  if ((long long)N * C * H * W >= (1LL << 40) || (long long)K * C * RS >= (1LL << 31) || RS > 65535)
+    return POLYCONV_STATUS_NOT_SUPPORTED;
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  const long long nout = (long long)K * C * RS;
+  cudaError_t e = cudaMemsetAsync(ws, 0, nout * sizeof(float), st);
+  if (e != cudaSuccess) return status_of(e);
+  const int kt = (K + 31) / 32, ct = (C + 31) / 32;
+  // about 4 blocks per SM in total, each with at least 1024 positions
+  long long splits = (148LL * 4 + kt * ct * RS - 1) / (kt * ct * RS);
+  splits = std::max(1LL, std::min(splits, (NPQ + 1023) / 1024));
+  while (splits * RS > 65535) --splits;
+  const long long per_split = ((NPQ + splits - 1) / splits + 31) / 32 * 32;
+  splits = (NPQ + per_split - 1) / per_split;
+  dim3 grid(kt, ct, (unsigned)(splits * RS));
+  if (dtype == POLYCONV_F32)
+    wgrad_kernel<uint32_t><<<grid, 256, 0, st>>>(static_cast<const uint32_t*>(x), static_cast<const uint32_t*>(dy), ws,
+                                                 N, C, H, W, K, R, S, sh, sw, ph, pw, P, Q, (int)splits, per_split);
+  else
+    wgrad_kernel<uint16_t><<<grid, 256, 0, st>>>(static_cast<const uint16_t*>(x), static_cast<const uint16_t*>(dy), ws,
+                                                 N, C, H, W, K, R, S, sh, sw, ph, pw, P, Q, (int)splits, per_split);
+  if ((e = cudaGetLastError()) != cudaSuccess) return status_of(e);
+  f32_to_out<<<grid_for(nout, 256), 256, 0, st>>>(ws, dw, nout, dtype == POLYCONV_BF16);
   return status_of(cudaGetLastError());
 }
