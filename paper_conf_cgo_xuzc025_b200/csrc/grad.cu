@@ -136,9 +136,9 @@ extern "C" polyconv_status_t polyconv_swap_nc(const void* x, void* xt, int N, in
 // ---------------------------------------------------------------------------------------------
 // wgrad as its own contraction (the forward-conv mapping leaves R*S positions per plane, see
 // DESIGN.md "Backward"): per tap (i, j), dw[:, :, i, j] = DY[K x NPQ] . X_ij[NPQ x C], the NPQ
-// sum split across blocks.  Block = one tap, a 32 (k) x 32 (c) tile and a slice of the NPQ
+// sum split across blocks.  Block = one tap, a 64 (k) x 64 (c) tile and a slice of the NPQ
 // positions; 32-position chunks of dy and of the tap-shifted x are staged in shared memory
-// (coalesced along positions), each thread accumulates 2 x 2 outputs in fp32 and adds them
+// (coalesced along positions), each thread accumulates 4 x 4 outputs in fp32 and adds them
 // into an fp32 workspace with atomics; a second pass converts to the io dtype.
 namespace {
 
@@ -152,20 +152,22 @@ __global__ void __launch_bounds__(256) wgrad_kernel(const T* __restrict__ x, con
                                                     float* __restrict__ ws, int N, int C, int H, int W, int K, int R,
                                                     int S, int sh, int sw, int ph, int pw, int P, int Q, int splits,
                                                     long long per_split) {
-  __shared__ float sdy[32][33];
-  __shared__ float sx[32][33];
+  constexpr int TM = 64, TP = 32;  // 64 (k) x 64 (c) tile, 32 positions per staged chunk
+  __shared__ __align__(16) float sdy[TP][TM + 4];
+  __shared__ __align__(16) float sx[TP][TM + 4];
   const int tap = blockIdx.z / splits, split = blockIdx.z - tap * splits;
   const int ti = tap / S, tj = tap - ti * S;
-  const int k0 = blockIdx.x * 32, c0 = blockIdx.y * 32;
+  const int k0 = blockIdx.x * TM, c0 = blockIdx.y * TM;
   const long long PQ = (long long)P * Q, NPQ = (long long)N * PQ;
   const long long p_begin = split * per_split, p_end = min(NPQ, p_begin + per_split);
   const int tid = threadIdx.x;
-  const int tk = (tid / 16) * 2, tc = (tid % 16) * 2;
-  float acc00 = 0.f, acc01 = 0.f, acc10 = 0.f, acc11 = 0.f;
-  for (long long p0 = p_begin; p0 < p_end; p0 += 32) {
-    // stage 32 rows (k or c) x 32 positions; element e = row * 32 + pos, 4 per thread
-    for (int e = tid; e < 1024; e += 256) {
-      const int row = e >> 5, q = e & 31;
+  const int tk = (tid / 16) * 4, tc = (tid % 16) * 4;
+  float acc[4][4] = {};
+  for (long long p0 = p_begin; p0 < p_end; p0 += TP) {
+    // stage [position][row] so each thread's 4 consecutive rows are one 16-byte shared load;
+    // element e = row * TP + pos: consecutive threads -> consecutive positions (coalesced)
+    for (int e = tid; e < TM * TP; e += 256) {
+      const int row = e / TP, q = e % TP;
       const long long p = p0 + q;
       float vdy = 0.f, vx = 0.f;
       if (p < p_end) {
@@ -177,28 +179,30 @@ __global__ void __launch_bounds__(256) wgrad_kernel(const T* __restrict__ x, con
         if (c0 + row < C && h >= 0 && h < H && w >= 0 && w < W)
           vx = ld_as_float(x, ((n * C + c0 + row) * H + h) * (long long)W + w);
       }
-      sdy[row][q] = vdy;
-      sx[row][q] = vx;
+      sdy[q][row] = vdy;
+      sx[q][row] = vx;
     }
     __syncthreads();
-#pragma unroll 8
-    for (int q = 0; q < 32; ++q) {
-      const float a0 = sdy[tk][q], a1 = sdy[tk + 1][q], b0 = sx[tc][q], b1 = sx[tc + 1][q];
-      acc00 = fmaf(a0, b0, acc00);
-      acc01 = fmaf(a0, b1, acc01);
-      acc10 = fmaf(a1, b0, acc10);
-      acc11 = fmaf(a1, b1, acc11);
+#pragma unroll 4
+    for (int q = 0; q < TP; ++q) {
+      const float4 a = *reinterpret_cast<const float4*>(&sdy[q][tk]);
+      const float4 b = *reinterpret_cast<const float4*>(&sx[q][tc]);
+      const float av[4] = {a.x, a.y, a.z, a.w}, bv[4] = {b.x, b.y, b.z, b.w};
+#pragma unroll
+      for (int u = 0; u < 4; ++u)
+#pragma unroll
+        for (int v = 0; v < 4; ++v) acc[u][v] = fmaf(av[u], bv[v], acc[u][v]);
     }
     __syncthreads();
   }
   const long long RS = (long long)R * S;
-  auto add = [&](int k, int c, float v) {
-    if (k < K && c < C) atomicAdd(ws + ((long long)k * C + c) * RS + tap, v);
-  };
-  add(k0 + tk, c0 + tc, acc00);
-  add(k0 + tk, c0 + tc + 1, acc01);
-  add(k0 + tk + 1, c0 + tc, acc10);
-  add(k0 + tk + 1, c0 + tc + 1, acc11);
+#pragma unroll
+  for (int u = 0; u < 4; ++u)
+#pragma unroll
+    for (int v = 0; v < 4; ++v) {
+      const int k = k0 + tk + u, c = c0 + tc + v;
+      if (k < K && c < C) atomicAdd(ws + ((long long)k * C + c) * RS + tap, acc[u][v]);
+    }
 }
 
 __global__ void __launch_bounds__(256) f32_to_out(const float* __restrict__ ws, void* __restrict__ out, long long n,
@@ -232,10 +236,10 @@ extern "C" polyconv_status_t polyconv_wgrad(const void* x, const void* dy, void*
   const long long nout = (long long)K * C * RS;
   cudaError_t e = cudaMemsetAsync(ws, 0, nout * sizeof(float), st);
   if (e != cudaSuccess) return status_of(e);
-  const int kt = (K + 31) / 32, ct = (C + 31) / 32;
-  // about 4 blocks per SM in total, each with at least 1024 positions
+  const int kt = (K + 63) / 64, ct = (C + 63) / 64;
+  // about 4 blocks per SM in total, each with at least 256 positions
   long long splits = (148LL * 4 + kt * ct * RS - 1) / (kt * ct * RS);
-  splits = std::max(1LL, std::min(splits, (NPQ + 1023) / 1024));
+  splits = std::max(1LL, std::min(splits, (NPQ + 255) / 256));
   while (splits * RS > 65535) --splits;
   const long long per_split = ((NPQ + splits - 1) / splits + 31) / 32 * 32;
   splits = (NPQ + per_split - 1) / per_split;
