@@ -165,20 +165,29 @@ __global__ void __launch_bounds__(256) wgrad_kernel(const T* __restrict__ x, con
   float acc[4][4] = {};
   for (long long p0 = p_begin; p0 < p_end; p0 += TP) {
     // stage [position][row] so each thread's 4 consecutive rows are one 16-byte shared load;
-    // element e = row * TP + pos: consecutive threads -> consecutive positions (coalesced)
-    for (int e = tid; e < TM * TP; e += 256) {
-      const int row = e / TP, q = e % TP;
-      const long long p = p0 + q;
+    // every element this thread stages has position q = tid % TP (256 is a multiple of TP), so
+    // the (n, oh, ow) decode and the tap shift are done once per chunk; consecutive threads read
+    // consecutive positions (coalesced)
+    const int q = tid % TP;
+    const long long p = p0 + q;
+    const bool live = p < p_end;
+    long long dy_base = 0, x_base = 0;
+    bool x_in = false;
+    if (live) {
+      const long long n = p / PQ;
+      const int r = (int)(p - n * PQ);
+      const int oh = r / Q, ow = r - oh * Q;
+      const int h = sh * oh + ti - ph, w = sw * ow + tj - pw;
+      dy_base = (n * K * P + oh) * (long long)Q + ow;      // + k * PQ
+      x_in = h >= 0 && h < H && w >= 0 && w < W;
+      x_base = (n * C * H + h) * (long long)W + w;          // + c * H * W
+    }
+    const long long HW = (long long)H * W;
+#pragma unroll
+    for (int row = tid / TP; row < TM; row += 256 / TP) {
       float vdy = 0.f, vx = 0.f;
-      if (p < p_end) {
-        const long long n = p / PQ;
-        const int r = (int)(p - n * PQ);
-        const int oh = r / Q, ow = r - oh * Q;
-        if (k0 + row < K) vdy = ld_as_float(dy, ((n * K + k0 + row) * P + oh) * (long long)Q + ow);
-        const int h = sh * oh + ti - ph, w = sw * ow + tj - pw;
-        if (c0 + row < C && h >= 0 && h < H && w >= 0 && w < W)
-          vx = ld_as_float(x, ((n * C + c0 + row) * H + h) * (long long)W + w);
-      }
+      if (live && k0 + row < K) vdy = ld_as_float(dy, dy_base + (long long)(k0 + row) * PQ);
+      if (x_in && c0 + row < C) vx = ld_as_float(x, x_base + (long long)(c0 + row) * HW);
       sdy[q][row] = vdy;
       sx[q][row] = vx;
     }
