@@ -156,4 +156,26 @@ cudaError_t launch_mac_pair(const Geom& g, const PairTiling& t, const void* x, c
 void* pair_state_new();
 void pair_state_free(void* s);
 
+// ---- mac_hankel.cu (persistent CTA-pair kernel fed from NCHW x; reading R16 layout) ----
+struct HankelTiling {
+  bool ok;
+  int pitch, HS, delta;    // input polynomial row pitch, image stride (rows), origin shift
+  int PT;                  // 256-position units
+  int Cp, nchunks;         // channels padded to whole 128-byte operand rows
+  int NN, NB, Kp;          // MMA N (output channels per block), blocks, padded K of U
+  int T;                   // 128-position tiles per CTA per item (accumulators share filter blocks)
+  int wrows, wslots;       // window rows per slot, window ring depth
+  int fslots, resident;    // filter blocks in shared memory; 1 = whole filter half resident
+  int aligned;             // every position pair is one aligned input pair (fast loader)
+  uint32_t wslot_bytes, fblk_bytes;
+  int smem_bytes, tmem_cols, npairs, grid;
+};
+HankelTiling hankel_tiling(const Geom& g, int fmt, int num_sms);
+// x: NCHW input (io dtype); U: tap-major packed filter [RS][Kp][Cp] (t.Kp, t.Cp), packed by
+// the preceding launch, which this one follows as a programmatic dependent
+// zero: device buffer of hankel_zero_bytes(g) zero bytes (read in place of padding)
+size_t hankel_zero_bytes(const Geom& g);
+cudaError_t launch_mac_hankel(const Geom& g, const HankelTiling& t, int fmt, const void* x, bool io_bf16,
+                              const void* U, void* y, const void* zero, cudaStream_t st, char* err, size_t errlen);
+
 }  // namespace polyconv

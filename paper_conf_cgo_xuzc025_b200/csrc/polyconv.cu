@@ -24,6 +24,8 @@ struct polyconv_plan_s {
   Tc2Tiling tc2;
   Fp32Tiling f32;
   PairTiling pair;
+  HankelTiling hk;
+  void* hkzero = nullptr;  // mac_hankel: zero words read in place of padding (hankel_zero_bytes)
   void* pair_state = nullptr;  // mac_pair launch cache
   unsigned long long* bflag = nullptr;  // mac_pair band flags [N * pair.nb]
   // stride s >= 2 (reading R4b): the stride-1 inner plan over the input's s*s phases
@@ -105,6 +107,17 @@ polyconv_status_t resolve(polyconv_plan_t p) {
   if (k == POLYCONV_KERNEL_AUTO && mac1x1_supported(g, p->fmt, p->io_bf16) && !getenv("POLYCONV_NO_1X1") &&
       mac1x1_auto(g))
     k = POLYCONV_KERNEL_TC_1X1;
+  // BF16 3x3 / 5x5 layers, stride 1 or 2, on even-width planes with C % 8 == 0 and at least one
+  // third of a round of pair units (24): the persistent pair kernel fed straight from NCHW x (mac_hankel.cu).
+  // Measured per layer against every other kernel (tools/kernel_cmp.py, profiles/r02_kcmp_*.jsonl):
+  // it wins on ResNet-50 l1-l3 3x3 (incl. stride 2), VGG-16 conv1_2..conv5_3, the sweep's 3x3 and
+  // 5x5 points; it loses on 7x7 kernels, odd-width planes (l4 7x7: general loader) and problems
+  // under a third of a round of units (the synthetic nets at 4x4 / 8x8: 1-11 units; 14x14: 30).
+  if (k == POLYCONV_KERNEL_AUTO && p->math == POLYCONV_MATH_BF16 && g.K >= 16 && g.sh == g.sw && g.sh <= 2 &&
+      g.R == g.S && (g.R == 3 || g.R == 5) && !getenv("POLYCONV_NO_HANKEL")) {
+    const HankelTiling h = hankel_tiling(g, p->fmt, p->num_sms);
+    if (h.ok && h.aligned && (long long)h.PT * h.NB >= 24) k = POLYCONV_KERNEL_TC_HANKEL;
+  }
   if (k == POLYCONV_KERNEL_AUTO) {
     // bf16, at most two rounds of pair tiles: one launch on CTA pairs with a resident filter
     // (its fixed startup wins on small problems); larger problems pipeline better in mac_tc2
@@ -136,12 +149,19 @@ polyconv_status_t resolve(polyconv_plan_t p) {
     return POLYCONV_STATUS_BAD_PARAM;
   if (k == POLYCONV_KERNEL_TC_PAIR && (!tc_math || !p->pair.ok)) return POLYCONV_STATUS_BAD_PARAM;
   if (k == POLYCONV_KERNEL_TC_1X1 && !mac1x1_supported(g, p->fmt, p->io_bf16)) return POLYCONV_STATUS_BAD_PARAM;
+  if (k == POLYCONV_KERNEL_TC_HANKEL) {
+    p->hk = hankel_tiling(g, p->fmt, p->num_sms);
+    if (!tc_math || !p->hk.ok) return POLYCONV_STATUS_BAD_PARAM;
+  }
   if (k == POLYCONV_KERNEL_TC_PERTAP && (!tc_math || !tc_supported(g, p->fmt))) return POLYCONV_STATUS_BAD_PARAM;
   if (k == POLYCONV_KERNEL_FP32 && (tc_math || fp32_tiling(g).smax == 0)) return POLYCONV_STATUS_BAD_PARAM;
   p->kernel = k;
   if (k == POLYCONV_KERNEL_TC_PAIR) {
     g.Cp = p->pair.Cp;
     g.Kp = p->pair.NN;
+  } else if (k == POLYCONV_KERNEL_TC_HANKEL) {
+    g.Cp = p->hk.Cp;
+    g.Kp = p->hk.Kp;
   } else if (k == POLYCONV_KERNEL_TC_1X1) {
     g.Cp = (g.C + 63) / 64 * 64;
     g.Kp = (g.K + 127) / 128 * 128;
@@ -165,7 +185,7 @@ polyconv_status_t resolve(polyconv_plan_t p) {
   // TC packs the input on the fly (no input workspace); TC_PERTAP needs the
   // interleaved copy, FP32/THIN the planar one
   const size_t a_elems = k == POLYCONV_KERNEL_TC_1X1 ? (size_t)g.N * g.C * mac1x1_pitch(g)
-                         : k == POLYCONV_KERNEL_TC_FUSED ? 0
+                         : (k == POLYCONV_KERNEL_TC_FUSED || k == POLYCONV_KERNEL_TC_HANKEL) ? 0
                          : (k == POLYCONV_KERNEL_TC || k == POLYCONV_KERNEL_TC_PERTAP || k == POLYCONV_KERNEL_TC_PAIR) ? (size_t)g.N * g.L_A * g.Cp
                                                                                        : (size_t)g.N * g.C * g.L_A;
   p->wsA_bytes = a_elems * eb;
@@ -319,7 +339,7 @@ polyconv_status_t polyconv_plan(polyconv_plan_t* plan, int N, int C, int H, int 
   // rule is R, S >= 5 (POLYCONV_POLYPHASE=1 forces it for any R, S >= 2, =0 disables it).
   const char* pp_env = getenv("POLYCONV_POLYPHASE");
   const int pp_min = pp_env ? (atoi(pp_env) == 0 ? 1 << 30 : 2) : 5;
-  if (sh == sw && sh >= 2 && R >= pp_min && S >= pp_min) {
+  if (sh == sw && sh >= 2 && R >= pp_min && S >= pp_min && p->kernel != POLYCONV_KERNEL_TC_HANKEL) {
     const int s = sh;
     const int Rq = (R + s - 1) / s, Sq = (S + s - 1) / s;
     const long long Hq = P + Rq - 1, Wq = Q + Sq - 1;
@@ -354,7 +374,7 @@ polyconv_status_t polyconv_plan_set_kernel(polyconv_plan_t p, polyconv_kernel_t 
     if (so != POLYCONV_STATUS_SUCCESS) polyconv_plan_set_kernel(in, (polyconv_kernel_t)old_inner);
     return so;
   }
-  if (kernel < POLYCONV_KERNEL_AUTO || kernel > POLYCONV_KERNEL_TC_1X1) return POLYCONV_STATUS_BAD_PARAM;
+  if (kernel < POLYCONV_KERNEL_AUTO || kernel > POLYCONV_KERNEL_TC_HANKEL) return POLYCONV_STATUS_BAD_PARAM;
   const int old = p->forced;
   p->forced = kernel;
   if (resolve(p) != POLYCONV_STATUS_SUCCESS) {
@@ -397,6 +417,9 @@ polyconv_status_t polyconv_plan_info(polyconv_plan_t p, polyconv_info_t* info) {
     case POLYCONV_KERNEL_TC_PAIR:  // pair tile = 256 positions x NN output channels
       info->tile_m = 256; info->tile_n = p->pair.NN; info->stages = p->pair.ring;
       info->launches = p->pair.split ? 2 : 1; break;
+    case POLYCONV_KERNEL_TC_HANKEL:  // pair item = 256*T positions x NN output channels
+      info->tile_m = 256 * p->hk.T; info->tile_n = p->hk.NN; info->stages = p->hk.wslots;
+      info->launches = 2; break;
     case POLYCONV_KERNEL_TC_1X1:  // tile = 128 output channels x up to 256 positions
       info->tile_m = 128; info->tile_n = g.P * g.Q >= 256 ? 256 : (g.P * g.Q + 63) / 64 * 64; info->stages = 0;
       info->launches = mac1x1_pitch(g) ? 3 : 2; break;
@@ -460,6 +483,26 @@ polyconv_status_t polyconv_forward(polyconv_plan_t p, const void* x, const void*
                        sizeof(p->err));
     if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
     return finish(p, e, "mac_tc");
+  }
+  if (p->kernel == POLYCONV_KERNEL_TC_HANKEL) {
+    // a3 (tap-major filter, one small launch), then a2 + a4 + a5 in the persistent pair
+    // kernel, which reads x directly and follows the pack as a programmatic dependent
+    if (!p->hkzero) {
+      const size_t zb = hankel_zero_bytes(g);
+      if (cudaMalloc(&p->hkzero, zb) != cudaSuccess || cudaMemsetAsync(p->hkzero, 0, zb, st) != cudaSuccess) {
+        cudaGetLastError();
+        if (p->hkzero) cudaFree(p->hkzero);
+        p->hkzero = nullptr;
+        set_err(p, "cudaMalloc of the %s failed", "zero buffer");
+        return POLYCONV_STATUS_ALLOC_FAILED;
+      }
+    }
+    if (p->ev_start) cudaEventRecord(p->ev_start, st);
+    e = launch_pack_filter_tapmajor(g, w, p->io_bf16, p->wsU, p->fmt, g.Kp, g.Cp, st);
+    if (e != cudaSuccess) return finish(p, e, "pack_filter");
+    e = launch_mac_hankel(g, p->hk, p->fmt, x, p->io_bf16, p->wsU, y, p->hkzero, st, p->err, sizeof(p->err));
+    if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
+    return finish(p, e, "mac_hankel");
   }
   if (p->kernel == POLYCONV_KERNEL_TC_1X1) {
     // a3 (the [1][Kp][Cp] filter), then the GEMM over the NCHW planes as its programmatic dependent
@@ -717,7 +760,7 @@ polyconv_status_t polyconv_extract(polyconv_plan_t p, const float* coeffs, void*
 polyconv_status_t polyconv_destroy(polyconv_plan_t p) {
   if (!p) return POLYCONV_STATUS_SUCCESS;
   polyconv_status_t s = POLYCONV_STATUS_SUCCESS;
-  if (p->used || p->wsA || p->wsU || p->hx || p->hw || p->hy || p->fcount) {
+  if (p->used || p->wsA || p->wsU || p->hx || p->hw || p->hy || p->fcount || p->hkzero) {
     DeviceGuard guard(p->device);
     if (p->used && cudaStreamSynchronize(p->last_stream) != cudaSuccess) {
       cudaGetLastError();
@@ -729,6 +772,7 @@ polyconv_status_t polyconv_destroy(polyconv_plan_t p) {
     if (p->hw) cudaFree(p->hw);
     if (p->hy) cudaFree(p->hy);
     if (p->fcount) cudaFree(p->fcount);
+    if (p->hkzero) cudaFree(p->hkzero);
   }
   if (p->pair_state) pair_state_free(p->pair_state);
   if (p->hsub && polyconv_destroy(p->hsub) != POLYCONV_STATUS_SUCCESS) s = POLYCONV_STATUS_EXECUTION_FAILED;

@@ -60,14 +60,19 @@ def test_plan_sizes_match_oracle(H, W, R, S, s, p):
 
 
 def test_kernel_selection_and_forcing():
-    assert pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="bf16").info()["kernel"] == "tc_pair"
-    # K > 256 (two output-channel tiles): the single-CTA tensor-core kernel
+    # bf16 3x3 / 5x5, stride <= 2, even width, C % 8 == 0, >= 24 pair units: mac_hankel
+    assert pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="bf16").info()["kernel"] == "tc_hankel"
+    # under 24 pair units (10x10, N=1): the single-CTA tensor-core kernel
     assert pc.Plan((1, 64, 10, 10), (320, 64, 3, 3), padding=(1, 1), math="bf16").info()["kernel"] == "tc"
     with pytest.raises(pc.PolyconvError):
         pc.Plan((1, 64, 10, 10), (320, 64, 3, 3), padding=(1, 1), math="bf16", kernel="tc_pair")
     with pytest.raises(pc.PolyconvError):
         pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="tf32", kernel="tc_pair")
+    with pytest.raises(pc.PolyconvError):
+        pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="fp32", kernel="tc_hankel")
     assert pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="tf32").info()["kernel"] == "tc"
+    assert pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="tf32",
+                   kernel="tc_hankel").info()["kernel"] == "tc_hankel"
     assert pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="fp32").info()["kernel"] == "fp32"
     assert pc.Plan((1, 1, 8, 8), (1, 1, 3, 3), math="fp32").info()["kernel"] == "thin"
     assert pc.Plan((1, 1, 8, 8), (1, 1, 3, 3), math="bf16").info()["kernel"] == "thin"
@@ -87,18 +92,23 @@ def test_kernel_selection_and_forcing():
     assert k1((4, 256, 28, 28), (512, 256, 1, 1), 2)["kernel"] == "tc_1x1"
     assert k1((4, 1024, 7, 7), (512, 1024, 1, 1))["kernel"] == "tc_1x1"
     assert k1((4, 512, 7, 7), (2048, 512, 1, 1))["kernel"] == "tc"
-    # bf16 in/out (synthetic-net kernel comparison): mac_pair from one full round of
-    # pair tiles (conv3_x: 112 on 74 pairs), pack + mac_tc2 below it; in-kernel packing
-    # (TC_FUSED) for 3x3 on narrow planes only, a pack launch for 5x5 / 7x7
-    k3 = lambda xs, ws: pc.Plan(xs, ws, (1, 1), (ws[2] // 2, ws[3] // 2), math="bf16", io_dtype="bf16").info()["kernel"]
-    assert k3((32, 128, 28, 28), (128, 128, 3, 3)) == "tc_pair"
-    assert k3((32, 64, 8, 8), (64, 64, 3, 3)) == "tc"
-    assert k3((32, 128, 14, 14), (64, 128, 3, 3)) == "tc"
-    assert k3((32, 64, 56, 56), (64, 64, 3, 3)) == "tc_fused"
-    assert k3((32, 64, 56, 56), (128, 64, 5, 5)) == "tc"
+    # bf16 in/out (profiles/r02_kcmp_*.jsonl): mac_hankel for 3x3 / 5x5 from 24 pair
+    # units, stride 1 or 2; odd plane widths, 7x7 kernels and sub-round problems keep the
+    # earlier rules (pack + mac_tc2 below one round of pair tiles, in-kernel packing for 3x3
+    # on narrow planes, a pack launch for 7x7)
+    k3 = lambda xs, ws, s=1: pc.Plan(xs, ws, (s, s), (ws[2] // 2, ws[3] // 2), math="bf16",
+                                     io_dtype="bf16").info()["kernel"]
+    assert k3((32, 128, 28, 28), (128, 128, 3, 3)) == "tc_hankel"
+    assert k3((256, 512, 7, 7), (512, 512, 3, 3)) == "tc"            # odd width
+    assert k3((256, 128, 56, 56), (128, 128, 3, 3), 2) == "tc_hankel"
+    assert k3((32, 64, 8, 8), (64, 64, 3, 3)) == "tc"                # 12 units < 24
+    assert k3((32, 128, 14, 14), (64, 128, 3, 3)) == "tc_hankel"
+    assert k3((32, 64, 56, 56), (64, 64, 3, 3)) == "tc_hankel"
+    assert k3((32, 64, 56, 56), (128, 64, 5, 5)) == "tc_hankel"
     assert k3((32, 64, 56, 56), (128, 64, 7, 7)) == "tc"
-    # f32 I/O keeps mac_pair on small problems (the sub-round rule was measured for bf16 I/O)
+    # f32 I/O, bf16 math: the same rule
     assert pc.Plan((32, 64, 8, 8), (64, 64, 3, 3), (1, 1), (1, 1), math="bf16").info()["kernel"] == "tc_pair"
+    assert pc.Plan((32, 64, 28, 28), (64, 64, 3, 3), (1, 1), (1, 1), math="bf16").info()["kernel"] == "tc_hankel"
 
 
 def test_tc_tiling_choices():
@@ -114,11 +124,22 @@ def test_tc_tiling_choices():
     assert inf["tile_n"] == 128 and inf["Kp"] == 384
     # TC_PAIR (bf16 default): pair tile = 256 positions x NN output channels (NN = K
     # rounded up to 64), channels in chunks of 64/32/16; one launch
-    inf = pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="bf16").info()
+    inf = pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="bf16", kernel="tc_pair").info()
     assert (inf["tile_m"], inf["tile_n"], inf["Cp"], inf["Kp"], inf["launches"]) == (256, 128, 128, 128, 1)
+    # TC_HANKEL: pair item = 256*T positions x NN output channels; NN = K (<= 256) else 128,
+    # T*NN <= 256; channels in chunks of 64 (bf16) / 32 (tf32); filter pack + one launch
+    hk = lambda xs, ws, m="bf16": pc.Plan(xs, ws, (1, 1), (1, 1), math=m, kernel="tc_hankel").info()
+    inf = hk((256, 64, 56, 56), (64, 64, 3, 3))
+    assert (inf["tile_m"], inf["tile_n"], inf["Cp"], inf["Kp"], inf["launches"]) == (1024, 64, 64, 64, 2)
+    inf = hk((256, 256, 14, 14), (256, 256, 3, 3))
+    assert (inf["tile_m"], inf["tile_n"], inf["Kp"]) == (256, 256, 256)
+    inf = hk((256, 512, 7, 7), (512, 512, 3, 3))
+    assert (inf["tile_m"], inf["tile_n"], inf["Kp"]) == (512, 128, 512)
+    inf = hk((2, 40, 9, 9), (72, 40, 3, 3), "tf32")
+    assert (inf["tile_n"], inf["Cp"], inf["Kp"]) == (80, 64, 80)
     inf = pc.Plan((2, 3, 30, 30), (64, 3, 7, 7), (2, 2), (3, 3), math="bf16").info()
     assert (inf["kernel"], inf["Cp"], inf["Kp"]) == ("tc_pair", 16, 64)
-    inf = pc.Plan((2, 40, 9, 9), (72, 40, 3, 3), (1, 1), (1, 1), math="bf16").info()
+    inf = pc.Plan((2, 40, 9, 9), (72, 40, 3, 3), (1, 1), (1, 1), math="bf16", kernel="tc_pair").info()
     assert (inf["kernel"], inf["Cp"], inf["Kp"]) == ("tc_pair", 64, 128)
     # TC_PERTAP (ablation): tile = 128 positions x bn output channels
     inf = pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="bf16", kernel="tc_pertap").info()

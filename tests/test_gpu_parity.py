@@ -18,7 +18,7 @@ pytestmark = pytest.mark.gpu
 
 MATH_KERNELS = [("fp32", "fp32"), ("fp32", "thin"), ("tf32", "tc"), ("bf16", "tc"), ("tf32", "tc_pertap"),
                 ("bf16", "tc_pertap"), ("tf32", "tc_fused"), ("bf16", "tc_fused"), ("tf32", "thin"),
-                ("bf16", "thin"), ("bf16", "tc_pair")]
+                ("bf16", "thin"), ("bf16", "tc_pair"), ("bf16", "tc_hankel"), ("tf32", "tc_hankel")]
 
 SHAPES = [
     ConvShape("tiny", 1, 1, 8, 8, 1, 3, 3),                      # BASELINE configs[0]
@@ -95,7 +95,7 @@ MX_SHAPES = [
 
 
 @pytest.mark.parametrize("shape", MX_SHAPES, ids=lambda s: s.name)
-@pytest.mark.parametrize("kernel", ["tc_fused", "tc", "tc_pair"])
+@pytest.mark.parametrize("kernel", ["tc_fused", "tc", "tc_pair", "tc_hankel"])
 def test_bf16_io_fused_packing(shape, kernel):
     """bf16 in/out, BF16 math: integer data bit-exact against round_bf16(O1);
     uniform data within the BF16 gate."""
@@ -108,7 +108,7 @@ def test_bf16_io_fused_packing(shape, kernel):
     assert normwise(y, oracle.conv2d(x, w, shape.stride, shape.padding)) <= GATE["bf16"]
 
 
-@pytest.mark.parametrize("kernel", ["tc_fused", "tc_pair"])
+@pytest.mark.parametrize("kernel", ["tc_fused", "tc_pair", "tc_hankel"])
 def test_conv3x_fused_bf16_io(kernel):
     """BASELINE configs[1] in full, bf16 in/out, the one-launch kernels."""
     shape = synth.CONV3X
@@ -119,7 +119,7 @@ def test_conv3x_fused_bf16_io(kernel):
 
 @pytest.mark.parametrize("math,kernel", [("fp32", "fp32"), ("bf16", "tc"), ("tf32", "tc"), ("fp32", "thin"),
                                          ("bf16", "tc_pertap"), ("bf16", "tc_fused"),
-                                         ("bf16", "tc_pair")])
+                                         ("bf16", "tc_pair"), ("bf16", "tc_hankel"), ("tf32", "tc_hankel")])
 def test_delta_filter_bit_exact(math, kernel):
     """w[k][c][i][j] = [c == k mod C][i == i0][j == j0] -> y = shifted xpad,
     bit-exact for every tap (checks each shift e(i,j) and the padding)."""
@@ -154,7 +154,7 @@ def test_conv3x_bench_launch_config():
     x, w = synth.make_inputs(shape, synth.seed_for(1), "uniform")
     ref = oracle.conv2d(x, w, shape.stride, shape.padding)
     y, plan = gpu_forward(shape, x, w, math="bf16", io="bf16")
-    assert plan.info()["kernel"] == "tc_pair"  # bf16: the one-launch CTA-pair kernel
+    assert plan.info()["kernel"] == "tc_hankel"  # bf16: the persistent pair kernel fed from NCHW x
     assert normwise(y, ref) <= GATE["bf16"]
     xi, wi = synth.make_inputs(shape, synth.seed_for(1), "int")
     y, _ = gpu_forward(shape, xi, wi, math="bf16", io="bf16", plan=plan)

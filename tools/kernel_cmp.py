@@ -20,7 +20,7 @@ reps = int(sys.argv[2]) if len(sys.argv) > 2 else 10
 SYNTHNET = [synth.ConvShape("syn_%d_%d_%d_r%d" % (H, C, K, R), 32, C, H, H, K, R, R, 1, 1, R // 2, R // 2)
             for H in (4, 8, 14, 28, 56) for (C, K, R) in ((64, 64, 3), (64, 128, 5), (128, 64, 1), (64, 128, 7),
                                                          (128, 64, 3))]
-layers = {"resnet50": synth.RESNET50, "vgg16": synth.VGG16, "synthnet": SYNTHNET}.get(
+layers = {"resnet50": synth.RESNET50, "vgg16": synth.VGG16, "synthnet": SYNTHNET, "sweep": synth.SWEEP}.get(
     which, synth.RESNET50 + synth.VGG16)
 flush = torch.empty(64 << 20, device="cuda")
 
@@ -49,7 +49,7 @@ for L in layers:
     rec = {"layer": L.name, "auto": auto}
     rec[auto] = round(L.flops() / timed(lambda: plan.forward(x, w, y)) / 1e9, 1)
     del plan
-    for k in ("tc_fused", "tc", "tc_pair", "tc_1x1"):
+    for k in ("tc_hankel", "tc_fused", "tc", "tc_pair", "tc_1x1"):
         if k == auto:
             continue
         try:
