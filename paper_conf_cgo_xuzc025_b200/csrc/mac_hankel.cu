@@ -60,25 +60,29 @@ namespace {
 
 using namespace sm100;
 
-constexpr int kHkLoadWarps = 8;
-constexpr int kHkEpiWarps = 8;
-constexpr int kHkThreads = 32 * 20;  // 20 warps, 5 per scheduler sub-partition (warp % 4)
+constexpr int kHkLoadWarps = 16;   // 8 16-byte channel groups x 2 halves of the window rows
+constexpr int kHkEpiWarps = 8;     // two per TMEM lane quadrant
+constexpr int kHkThreads = 32 * 28;  // 28 warps, 7 per scheduler sub-partition
 // Warp roles.  Warp w issues from sub-partition w % 4 and may read TMEM lanes 32*(w % 4)..+31.
-// The MMA issuer (warp 1) shares its sub-partition only with the filter producer and epilogue
-// warps, which mostly wait: with loaders beside it the issuer got a fraction of the issue
-// slots and the tensor pipe idled between MMAs (measured, tools/hk_trace.py).
-enum HkRole { kRoleIdle = 0, kRoleMma, kRoleProducer, kRoleLoader, kRoleEpi };
+// The MMA issuer (warp 1) shares its sub-partition only with the filter producer, the
+// forwarders and one epilogue warp, which mostly wait: with loaders beside it the issuer got a
+// fraction of the issue slots and the tensor pipe idled between MMAs (measured, tools/hk_trace.py).
+// Loaders: the window loads are latency-bound (ncu: long-scoreboard stalls), so 16 warps
+// split every window's rows in two halves to halve the round trips per window.
+enum HkRole { kRoleIdle = 0, kRoleMma, kRoleProducer, kRoleLoader, kRoleEpi, kRoleFwdW, kRoleFwdE };
 __device__ __forceinline__ int hk_role(int warp, int& idx) {
-  // loaders: 8 warps on sub-partitions 0, 2, 3; epilogue: two per TMEM lane quadrant
-  constexpr int kLoad[8] = {0, 12, 16, 2, 14, 18, 3, 15};
-  constexpr int kEpi[8] = {4, 8, 9, 13, 6, 10, 7, 11};  // (quadrant, half) = (w % 4, order)
+  constexpr int kLoad[16] = {0, 8, 12, 16, 20, 2, 10, 14, 18, 22, 3, 11, 15, 19, 23, 25};
+  constexpr int kEpi[8] = {4, 24, 9, 21, 6, 26, 7, 27};  // quadrant = w % 4, column half = order
   if (warp == 1) return kRoleMma;
   if (warp == 5) return kRoleProducer;
+  if (warp == 13) return kRoleFwdE;   // epilogue drained -> leader (one cluster arrive per CTA)
+  if (warp == 17) return kRoleFwdW;   // window stored -> leader
 #pragma unroll
-  for (int i = 0; i < 8; ++i) {
+  for (int i = 0; i < 16; ++i)
     if (warp == kLoad[i]) { idx = i; return kRoleLoader; }
+#pragma unroll
+  for (int i = 0; i < 8; ++i)
     if (warp == kEpi[i]) { idx = i; return kRoleEpi; }
-  }
   return kRoleIdle;
 }
 constexpr int kHkSmemMax = 232448;                         // 227 KB dynamic
@@ -244,16 +248,16 @@ __device__ __forceinline__ uint32_t hk_bf16(uint32_t raw) {
 // so the 8 lanes of each store phase hit 8 different 16-byte bank groups of the swizzle.
 template <typename IoT, bool kTf32>
 __device__ __forceinline__ void hk_load_window(const HkParams& p, uint32_t slot, long long q0, int c0, int lw,
-                                               int lane) {
+                                               int lane, int rp_lo, int rp_hi) {
   const uint32_t* xw = static_cast<const uint32_t*>(p.x);  // 32-bit words of x
   constexpr bool kBf16In = sizeof(IoT) == 2;
   constexpr int CPG = kTf32 ? 4 : 8;  // channels per 16-byte group
   const int cg = c0 + lw * CPG;
-  const int nrp = p.wrows >> 1;
+  const int nrp = rp_hi;
   const int odd_hw = p.HW & 1;
   const uint32_t sel = (uint32_t)(lane >> 2) & 1u;
   constexpr int B = 2;
-  for (int rp0 = 0; rp0 < nrp; rp0 += 32 * B) {
+  for (int rp0 = rp_lo; rp0 < nrp; rp0 += 32 * B) {
     uint32_t w0[B][CPG], w1[B][CPG];
     int s0[B], s1[B];
 #pragma unroll
@@ -331,17 +335,17 @@ __device__ __forceinline__ void hk_load_window(const HkParams& p, uint32_t slot,
 // the eight channel loads one base register plus immediate offsets.
 template <typename IoT, bool kTf32, int kHW2>
 __device__ __forceinline__ void hk_load_window_pairs(const HkParams& p, uint32_t slot, long long q0, int c0, int lw,
-                                                     int lane) {
+                                                     int lane, int rp_lo, int rp_hi) {
   constexpr bool kBf16In = sizeof(IoT) == 2;
   constexpr int CPG = kTf32 ? 4 : 8;          // channels per 16-byte group
   constexpr int B = kBf16In ? 4 : 2;          // position pairs per lane in flight
   const uint32_t hw2 = kHW2 ? (uint32_t)kHW2 : (uint32_t)p.HW >> 1;  // plane size in words / float2
   const int cg = c0 + lw * CPG;
-  const int nrp = p.wrows >> 1;
+  const int nrp = rp_hi;
   const uint32_t sel = (uint32_t)(lane >> 2) & 1u;
   const bool gz = cg >= p.C;  // group past C (warp-uniform); C % CPG == 0 for this loader
   const uint32_t cgo = gz ? 0u : (uint32_t)cg * hw2;
-  for (int rp0 = 0; rp0 < nrp; rp0 += 32 * B) {
+  for (int rp0 = rp_lo; rp0 < nrp; rp0 += 32 * B) {
     uint32_t lo[B][CPG], hi[B][kBf16In ? 1 : CPG];
 #pragma unroll
     for (int b = 0; b < B; ++b) {
@@ -351,7 +355,7 @@ __device__ __forceinline__ void hk_load_window_pairs(const HkParams& p, uint32_t
         const uint32_t* base = e >= 0 ? static_cast<const uint32_t*>(p.x) + (((uint32_t)e >> 1) + cgo)
                                       : static_cast<const uint32_t*>(p.zero);
 #pragma unroll
-        for (int c = 0; c < CPG; ++c) lo[b][c] = __ldg(base + c * hw2);
+        for (int c = 0; c < CPG; ++c) lo[b][c] = base[c * hw2];
       } else {
         const float2* base = e >= 0 ? static_cast<const float2*>(p.x) + (((uint32_t)e >> 1) + cgo)
                                     : static_cast<const float2*>(p.zero);
@@ -435,7 +439,13 @@ __global__ void __launch_bounds__(kHkThreads, 1)
   uint64_t* wempty = wfull + kHkMaxWSlots;   // [kHkMaxWSlots] both: MMAs done with the window
   uint64_t* tfull = wempty + kHkMaxWSlots;   // [2] both: accumulator ready
   uint64_t* tempty = tfull + 2;              // [2] leader: both CTAs' epilogues drained it
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+  // The 8 loader (epilogue) warps of a CTA arrive on a local barrier (CTA-scope release), and
+  // one forwarder warp per CTA passes it on to the leader with a single cluster-scope arrive:
+  // sixteen cluster-scope releases per window stalled every loader warp on a memory barrier
+  // (ncu: ERRBAR / membar was the loaders' largest stall after the loads themselves).
+  uint64_t* wloc = tempty + 2;               // [kHkMaxWSlots] this CTA's loaders done
+  uint64_t* eloc = wloc + kHkMaxWSlots;      // [2] this CTA's epilogue warps drained
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(eloc + 2);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t rank = cluster_ctarank();
@@ -453,12 +463,14 @@ __global__ void __launch_bounds__(kHkThreads, 1)
       mbar_init(fempty + i, 1);
     }
     for (int i = 0; i < kHkMaxWSlots; ++i) {
-      mbar_init(wfull + i, 2 * kHkLoadWarps);
+      mbar_init(wfull + i, 2);
       mbar_init(wempty + i, 1);
+      mbar_init(wloc + i, kHkLoadWarps);
     }
     for (int i = 0; i < 2; ++i) {
       mbar_init(tfull + i, 1);
-      mbar_init(tempty + i, 2 * kHkEpiWarps);
+      mbar_init(tempty + i, 2);
+      mbar_init(eloc + i, kHkEpiWarps);
     }
     fence_barrier_init();
   }
@@ -565,8 +577,11 @@ __global__ void __launch_bounds__(kHkThreads, 1)
     }
   } else if (role == kRoleLoader) {
     // ---- window loaders (a2) ----
-    const int lw = ridx;
-    const uint32_t wfull0 = hk_mapa0(smem_u32(wfull));
+    const int lw = ridx & 7;
+    // row-pair half of every window this warp converts (split on a multiple of 32 pairs)
+    const int nrp_all = p.wrows >> 1;
+    const int split = ((nrp_all / 2 + 31) / 32) * 32;
+    const int rp_lo = (ridx >> 3) ? min(split, nrp_all) : 0, rp_hi = (ridx >> 3) ? nrp_all : min(split, nrp_all);
     {
       long long u = u_lo;
       HkItem it;
@@ -576,28 +591,58 @@ __global__ void __launch_bounds__(kHkThreads, 1)
         for (int ch = 0; ch < p.nchunks; ++ch) {
           hk_wait(wempty + ws, (uint32_t)(wuse & 1) ^ 1u, 32);
           if constexpr (kHW2 >= 0)
-            hk_load_window_pairs<IoT, kTf32, kHW2>(p, sW + (uint32_t)ws * p.wslot_bytes, q0, ch * (kTf32 ? 32 : 64), lw, lane);
+            hk_load_window_pairs<IoT, kTf32, kHW2>(p, sW + (uint32_t)ws * p.wslot_bytes, q0, ch * (kTf32 ? 32 : 64), lw,
+                                                   lane, rp_lo, rp_hi);
           else
-            hk_load_window<IoT, kTf32>(p, sW + (uint32_t)ws * p.wslot_bytes, q0, ch * (kTf32 ? 32 : 64), lw, lane);
+            hk_load_window<IoT, kTf32>(p, sW + (uint32_t)ws * p.wslot_bytes, q0, ch * (kTf32 ? 32 : 64), lw, lane,
+                                       rp_lo, rp_hi);
           if (trace && lw == 0 && lane == 0 && u == u_lo + it.T && ch == 0) tr[2] = global_ns();
           asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> MMA reads
           __syncwarp();
           const int wi = (int)(wuse * p.wslots + ws);
           if ((p.dbg & 32) && blockIdx.x < 2 && lane == 0 && wi < 64) g_hk_ltrace[wi * 16 + rank * 8 + lw] = global_ns();
-          if (lane == 0) hk_arrive_cluster(wfull0 + (uint32_t)ws * 8u);
+          if (lane == 0) mbar_arrive(wloc + ws);
           if (++ws == p.wslots) { ws = 0; ++wuse; }
         }
       }
+    }
+  } else if (role == kRoleFwdW) {
+    // ---- forwarder: this CTA's window stored -> the leader's wfull ----
+    const uint32_t wfull0 = hk_mapa0(smem_u32(wfull));
+    long long u = u_lo;
+    HkItem it;
+    int ws = 0, wuse = 0;
+    while (hk_next(p, u, u_hi, it)) {
+      for (int ch = 0; ch < p.nchunks; ++ch) {
+        hk_wait(wloc + ws, (uint32_t)(wuse & 1));
+        if (lane == 0) hk_arrive_cluster(wfull0 + (uint32_t)ws * 8u);
+        __syncwarp();
+        if (++ws == p.wslots) { ws = 0; ++wuse; }
+      }
+    }
+  } else if (role == kRoleFwdE) {
+    // ---- forwarder: this CTA's epilogue drained an accumulator -> the leader's tempty ----
+    const uint32_t tempty0 = hk_mapa0(smem_u32(tempty));
+    long long u = u_lo;
+    HkItem it;
+    int item = 0;
+    while (hk_next(p, u, u_hi, it)) {
+      const int a = item & 1;
+      hk_wait(eloc + a, (uint32_t)((item >> 1) & 1), 64);
+      if (lane == 0) hk_arrive_cluster(tempty0 + (uint32_t)a * 8u);
+      __syncwarp();
+      ++item;
     }
   } else if (role == kRoleEpi) {
     // ---- epilogue (a5) ----
     const int e = ridx;
     const int quad = warp & 3;      // TMEM lane quadrant this warp may access
     const int half = e & 1;         // column groups half, half + 2, ...
-    const uint32_t tempty0 = hk_mapa0(smem_u32(tempty));
     const uint32_t tbase = *tmem_slot;
     IoT* y = static_cast<IoT*>(p.y);
     const long long PQ = (long long)p.P * p.Q;
+    // plane size of y as a compile-time constant when the output has the input's size
+    const bool pq_const = kHW2 > 0 && PQ == 2LL * kHW2;
     long long u = u_lo;
     HkItem it;
     int item = 0;
@@ -627,17 +672,24 @@ __global__ void __launch_bounds__(kHkThreads, 1)
           hk_tmem_ld16(trow + (uint32_t)(g * 16), v);
           tmem_ld_wait();
           if (ybase >= 0 && !(p.dbg & 2)) {
+            IoT* yp = y + ybase + (long long)(g * 16) * PQ;
+            const int kleft = p.K - (it.nb * p.NN + g * 16);  // output channels left (warp-uniform)
+            if (kHW2 > 0 && pq_const && kleft >= 16) {
+              // same-size output with a baked-in plane size: one base register, immediate offsets
 #pragma unroll
-            for (int c = 0; c < 16; ++c) {
-              const int k = it.nb * p.NN + g * 16 + c;
-              if (k < p.K) hk_store<IoT>(y, ybase + (long long)(g * 16 + c) * PQ, __uint_as_float(v[c]));
+              for (int c = 0; c < 16; ++c)
+                hk_store<IoT>(yp, (long long)c * (2 * (kHW2 > 0 ? kHW2 : 1)), __uint_as_float(v[c]));
+            } else {
+#pragma unroll
+              for (int c = 0; c < 16; ++c)
+                if (c < kleft) hk_store<IoT>(yp, (long long)c * PQ, __uint_as_float(v[c]));
             }
           }
         }
       }
       tc_fence_before();
       __syncwarp();
-      if (lane == 0) hk_arrive_cluster(tempty0 + (uint32_t)a * 8u);
+      if (lane == 0) mbar_arrive(eloc + a);
       if (trace && e == 0 && lane == 0) tr[item == 0 ? 5 : 7] = global_ns();
       ++item;
     }
@@ -680,10 +732,11 @@ int env_int(const char* name, int dflt) {
 size_t hankel_zero_bytes(const Geom& g) { return (size_t)32 * g.H * g.W + 256; }
 
 // Tiling.  NN (MMA N) = all output channels when K <= 256 (every window built once), else
-// blocks of 128; T = the most 128-position tiles per CTA whose accumulators fit TMEM twice
+// blocks of 256; T = the most 128-position tiles per CTA whose accumulators fit TMEM twice
 // (T*NN <= 256): the T tiles share each filter block and each window's halo rows.  Measured at
-// N=256 (tools/hk_check.py, tools/hk_sweep.sh; TFLOP/s): 256->256 14x14 NN=256/T=1 770 vs
-// NN=128/T=2 731; 512->512 7x7 NN=128/T=2 428 vs NN=64/T=4 203; 128->128 28x28 NN=128/T=2 792.
+// N=256 (tools/hk_trace.py with POLYCONV_HK_NN / POLYCONV_HK_T; TFLOP/s): 256->256 14x14
+// NN=256/T=1 750 vs NN=128/T=2 713; 512->512 7x7 NN=256/T=1 596 vs NN=128/T=2 416 (fewer
+// window rebuilds per output-channel block); 128->128 28x28 NN=128/T=2 862.
 // The filter is resident in shared memory when its (single) block fits beside two windows,
 // else streamed by TMA through a ring of (chunk, tap) blocks.
 HankelTiling hankel_tiling(const Geom& g, int fmt, int num_sms) {
@@ -713,7 +766,7 @@ HankelTiling hankel_tiling(const Geom& g, int fmt, int num_sms) {
   const bool no_res = env_int("POLYCONV_HK_STREAM", 0) != 0;
   const int max_pairs = std::max(1, num_sms / 2);
   const uint32_t fixed = 3072;  // alignment + barriers
-  int NN = forceNN ? forceNN : (K16 <= 256 ? K16 : 128);
+  int NN = forceNN ? forceNN : (K16 <= 256 ? K16 : 256);
   bool found = false;
   for (int T = 4; T >= 1 && !found; T >>= 1) {
     if ((forceT && T != forceT) || T * NN > 256) continue;
