@@ -234,10 +234,21 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-cudnn", action="store_true")
     ap.add_argument("--kernel", default="auto", help="force a MAC variant (ablation; default auto)")
+    ap.add_argument("--no-gate", action="store_true", help="skip the ResNet-50 N=256 3x3 gate records")
+    ap.add_argument("--no-by-math", action="store_true", help="skip the TF32 / FP32 conv3x records")
     args = ap.parse_args()
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    if "WORLD_SIZE" not in os.environ and args.gpus > 1:
+        # one process per GPU: re-launch this command under torch.distributed.run
+        import subprocess
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", str(args.gpus),
+               "--master-addr", "127.0.0.1", "--master-port", os.environ.get("MASTER_PORT", "29531"),
+               os.path.abspath(__file__)] + sys.argv[1:]
+        return subprocess.call(cmd)
+    if world != args.gpus:
+        raise SystemExit("--gpus %d but WORLD_SIZE=%d: launch one process per GPU" % (args.gpus, world))
     if args.impl == "reference":
         return run_reference(args, rank, world)
     if args.warmup < 3:
@@ -383,6 +394,10 @@ def main():
     if cudnn:
         line["cudnn"] = cudnn
         line["cudnn"]["ratio_ours_over_cudnn"] = value / cudnn["value"]
+    if world == 1 and not args.no_gate and args.math == "bf16" and args.workload == "conv3x":
+        line["gate"] = bench_gate(torch, pc, dev, flush_l2, peaks, 20, not args.no_cudnn)
+    if world == 1 and not args.no_by_math and args.math == "bf16" and args.workload == "conv3x":
+        line["by_math"] = bench_by_math(torch, pc, dev, shape, flush_l2, peaks, 20)
     if world == 1 and not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_baseline(shape)
     print(json.dumps(line), flush=True)
@@ -390,6 +405,93 @@ def main():
         dist.destroy_process_group()
     return 0
 
+
+
+# ------------------------------------------------------------ gate and by_math --
+
+GATE_LAYERS = [L for L in synth.RESNET50 if L.R == 3 and L.stride == (1, 1)]   # 13 convs, 4 shapes
+
+
+def _time_fn(torch, fn, flush, reps, warm=3):
+    for _ in range(warm):
+        flush()
+        fn()
+    torch.cuda.synchronize()
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(reps)]
+    for a, b in evs:
+        flush()
+        a.record()
+        fn()
+        b.record()
+    torch.cuda.synchronize()
+    ts = sorted(a.elapsed_time(b) for a, b in evs)
+    return ts[len(ts) // 2], sum(ts) / len(ts)
+
+
+def bench_gate(torch, pc, dev, flush, peaks, reps, with_cudnn):
+    """north_star gate: the 13 stride-1 3x3 convs of ResNet-50 at N=256 (BASELINE.json configs[4])
+    on one GPU, BF16 in/out and math, L2 flushed before every call.  Per layer: median time,
+    effective TFLOP/s, roofline time max(F/peak_bf16, B/HBM) and its fraction; aggregate
+    gate_frac = sum(count*roof) / sum(count*t)."""
+    import torch.nn.functional as Fn
+    recs = []
+    roof_sum = t_sum = 0.0
+    for li, L in enumerate(GATE_LAYERS):
+        g = torch.Generator(device=dev).manual_seed(synth.seed_for(4, li))
+        x = (torch.rand((L.N, L.C, L.H, L.W), device=dev, generator=g) * 2 - 1).bfloat16()
+        w = ((torch.rand((L.K, L.C, L.R, L.S), device=dev, generator=g) * 2 - 1) / (L.C * L.R * L.S) ** 0.5).bfloat16()
+        plan = pc.Plan(x.shape, w.shape, L.stride, L.padding, math="bf16", io_dtype="bf16", device=dev.index)
+        y = torch.empty(plan.output_shape, dtype=torch.bfloat16, device=dev)
+        t_med, t_mean = _time_fn(torch, lambda: plan.forward(x, w, y), flush, reps)
+        F = L.flops()
+        B = L.bytes(2, 2, 2)
+        roof_ms = max(F / (peaks["bf16_tflops"] * 1e12), B / (peaks["hbm_gbs"] * 1e9)) * 1e3
+        rec = {"layer": L.name, "count": L.count, "shape": [L.N, L.C, L.H, L.W, L.K, L.R, L.S],
+               "kernel": plan.info()["kernel"], "t_med_ms": t_med, "t_mean_ms": t_mean,
+               "tflops": F / (t_med * 1e-3) / 1e12, "roof_ms": roof_ms, "frac": roof_ms / t_med,
+               "bound": "tensor" if F / (peaks["bf16_tflops"] * 1e12) >= B / (peaks["hbm_gbs"] * 1e9) else "hbm"}
+        if with_cudnn:
+            torch.backends.cudnn.benchmark = True
+            best = None
+            for layout in ("nchw", "channels_last"):
+                xx, ww = (x, w) if layout == "nchw" else (x.contiguous(memory_format=torch.channels_last),
+                                                           w.contiguous(memory_format=torch.channels_last))
+                tc, _ = _time_fn(torch, lambda: Fn.conv2d(xx, ww, stride=L.stride, padding=L.padding), flush,
+                                 max(5, reps // 2))
+                v = F / (tc * 1e-3) / 1e12
+                rec["cudnn_%s_tflops" % layout] = v
+                if best is None or v > best[0]:
+                    best = (v, layout)
+            rec["cudnn_best_tflops"], rec["cudnn_best_layout"] = best
+        recs.append(rec)
+        roof_sum += L.count * roof_ms
+        t_sum += L.count * t_med
+        del plan, x, w, y
+    return {"layers": recs, "gate_frac": roof_sum / t_sum, "convs": sum(L.count for L in GATE_LAYERS),
+            "target": 0.60, "peak_tflops": peaks["bf16_tflops"], "hbm_gbs": peaks["hbm_gbs"],
+            "note": "ResNet-50 N=256 stride-1 3x3 convs on one GPU, BF16, L2 flushed, median of %d" % reps}
+
+
+def bench_by_math(torch, pc, dev, shape, flush, peaks, reps):
+    """conv3x (BASELINE configs[1]) in the other two maths (fp32 I/O): TF32 tensor cores and the
+    FP32 FFMA path (the paper's inferred precision), each against its own roofline."""
+    out = {}
+    x_np, w_np = synth.make_inputs(shape, synth.seed_for(1), "uniform")
+    x = torch.from_numpy(x_np).to(dev)
+    w = torch.from_numpy(w_np).to(dev)
+    for math in ("tf32", "fp32"):
+        plan = pc.Plan(x.shape, w.shape, shape.stride, shape.padding, math=math, io_dtype="f32", device=dev.index)
+        y = torch.empty(plan.output_shape, dtype=torch.float32, device=dev)
+        t_med, t_mean = _time_fn(torch, lambda: plan.forward(x, w, y), flush, reps)
+        bound, peak, note = _roofline_peak(math, peaks)
+        F = shape.flops()
+        B = shape.bytes(4, 4, 4)
+        roof_ms = max(F / (peak * 1e12), B / (peaks["hbm_gbs"] * 1e9)) * 1e3
+        out[math] = {"value": F / (t_mean * 1e-3) / 1e12, "unit": UNIT, "t_mean_ms": t_mean, "t_med_ms": t_med,
+                     "kernel": plan.info()["kernel"], "bound": bound, "peak": peak, "peak_source": note,
+                     "frac": roof_ms / t_mean, "io_dtype": "f32"}
+        del plan, y
+    return out
 
 def bench_cudnn(torch, x, w, shape, math, flush, K, world, dist):
     import torch.nn.functional as Fn

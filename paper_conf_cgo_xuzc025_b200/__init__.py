@@ -96,11 +96,20 @@ def status_string(status: int) -> str:
     return load_library().polyconv_status_string(status).decode()
 
 
-def _stream_ptr(stream):
+def _stream_ptr(stream, device=None):
+    """cudaStream_t of `stream`, else torch's current stream of `device` (the tensors'
+    device, not necessarily the current one)."""
     import torch
     if stream is None:
-        stream = torch.cuda.current_stream()
+        stream = torch.cuda.current_stream(device)
     return ctypes.c_void_p(stream.cuda_stream)
+
+
+def _on_device(t):
+    """Context making t's device current for a library call (the layout entry points take no
+    device argument and launch on the current device)."""
+    import torch
+    return torch.cuda.device(t.device)
 
 
 class Plan:
@@ -178,7 +187,7 @@ class Plan:
         else:
             self._check_tensor(y, self.output_shape, "y")
         self._check(self._lib.polyconv_forward(self._h, ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(w.data_ptr()),
-                                               ctypes.c_void_p(y.data_ptr()), _stream_ptr(stream)), "forward")
+                                               ctypes.c_void_p(y.data_ptr()), _stream_ptr(stream, self.device)), "forward")
         return y
 
     def forward_host(self, x, w, y, stream=None):
@@ -190,7 +199,7 @@ class Plan:
                 raise PolyconvError(BAD_PARAM, "%s must be a contiguous host tensor %s of %s" % (nm, shp, self.io_dtype))
         self._check(self._lib.polyconv_forward_host(self._h, ctypes.c_void_p(x.data_ptr()),
                                                     ctypes.c_void_p(w.data_ptr()), ctypes.c_void_p(y.data_ptr()),
-                                                    _stream_ptr(stream)), "forward_host")
+                                                    _stream_ptr(stream, self.device)), "forward_host")
         return y
 
     def set_timing_events(self, start, stop):
@@ -222,7 +231,7 @@ class Plan:
         out = torch.empty(self.packed_bytes("input", layout), dtype=torch.uint8, device=x.device)
         self._check(self._lib.polyconv_pack_input(self._h, ctypes.c_void_p(x.data_ptr()),
                                                   ctypes.c_void_p(out.data_ptr()), LAYOUT[layout],
-                                                  _stream_ptr(stream)), "pack_input")
+                                                  _stream_ptr(stream, self.device)), "pack_input")
         return out
 
     def pack_filter(self, w, layout="planar", stream=None):
@@ -232,7 +241,7 @@ class Plan:
         out = torch.empty(self.packed_bytes("filter", layout), dtype=torch.uint8, device=w.device)
         self._check(self._lib.polyconv_pack_filter(self._h, ctypes.c_void_p(w.data_ptr()),
                                                    ctypes.c_void_p(out.data_ptr()), LAYOUT[layout],
-                                                   _stream_ptr(stream)), "pack_filter")
+                                                   _stream_ptr(stream, self.device)), "pack_filter")
         return out
 
     def extract(self, coeffs, stream=None):
@@ -245,7 +254,7 @@ class Plan:
             raise PolyconvError(BAD_PARAM, "coeffs must be float32 CUDA [N][K][L_A+L_U-1]")
         y = torch.empty(self.output_shape, dtype=self._io_torch_dtype(), device=coeffs.device)
         self._check(self._lib.polyconv_extract(self._h, ctypes.c_void_p(coeffs.data_ptr()),
-                                               ctypes.c_void_p(y.data_ptr()), _stream_ptr(stream)), "extract")
+                                               ctypes.c_void_p(y.data_ptr()), _stream_ptr(stream, self.device)), "extract")
         return y
 
     def close(self):
@@ -277,8 +286,9 @@ def flip_filter(w, stream=None):
         raise PolyconvError(BAD_PARAM, "w must be a contiguous 4-D CUDA tensor")
     K, C, R, S = w.shape
     wt = torch.empty((C, K, R, S), dtype=w.dtype, device=w.device)
-    st = load_library().polyconv_flip_filter(ctypes.c_void_p(w.data_ptr()), ctypes.c_void_p(wt.data_ptr()), K, C, R,
-                                            S, _dtype_code(w), _stream_ptr(stream))
+    with _on_device(w):
+        st = load_library().polyconv_flip_filter(ctypes.c_void_p(w.data_ptr()), ctypes.c_void_p(wt.data_ptr()), K, C,
+                                                R, S, _dtype_code(w), _stream_ptr(stream, w.device))
     if st != SUCCESS:
         raise PolyconvError(st, "polyconv_flip_filter: %s" % status_string(st))
     return wt
@@ -292,8 +302,9 @@ def swap_nc(x, stream=None):
     N, C = x.shape[:2]
     hw = x.numel() // (N * C) if x.numel() else 0
     xt = torch.empty((C, N) + tuple(x.shape[2:]), dtype=x.dtype, device=x.device)
-    st = load_library().polyconv_swap_nc(ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(xt.data_ptr()), N, C, hw,
-                                        _dtype_code(x), _stream_ptr(stream))
+    with _on_device(x):
+        st = load_library().polyconv_swap_nc(ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(xt.data_ptr()), N, C, hw,
+                                            _dtype_code(x), _stream_ptr(stream, x.device))
     if st != SUCCESS:
         raise PolyconvError(st, "polyconv_swap_nc: %s" % status_string(st))
     return xt
@@ -308,8 +319,9 @@ def dilate(x, stride, extra=(0, 0), stream=None):
     N, C, H, W = x.shape
     (sh, sw), (eh, ew) = stride, extra
     xd = torch.empty((N, C, (H - 1) * sh + 1 + eh, (W - 1) * sw + 1 + ew), dtype=x.dtype, device=x.device)
-    st = load_library().polyconv_dilate(ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(xd.data_ptr()), N, C, H, W,
-                                       sh, sw, eh, ew, _dtype_code(x), _stream_ptr(stream))
+    with _on_device(x):
+        st = load_library().polyconv_dilate(ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(xd.data_ptr()), N, C, H,
+                                           W, sh, sw, eh, ew, _dtype_code(x), _stream_ptr(stream, x.device))
     if st != SUCCESS:
         raise PolyconvError(st, "polyconv_dilate: %s" % status_string(st))
     return xd
@@ -323,14 +335,23 @@ def wgrad(x, dy, w_shape, stride=(1, 1), padding=(0, 0), stream=None):
             raise PolyconvError(BAD_PARAM, "%s must be a contiguous 4-D CUDA tensor" % nm)
     if x.dtype != dy.dtype:
         raise PolyconvError(BAD_PARAM, "x and dy must share a dtype")
+    if x.device != dy.device:
+        raise PolyconvError(BAD_PARAM, "x and dy must be on one device")
     N, C, H, W = x.shape
-    K, _, R, S = w_shape
+    K, Cw, R, S = w_shape
+    if Cw != C:
+        raise PolyconvError(BAD_PARAM, "w_shape[1] = %d but x has %d channels" % (Cw, C))
+    P = (H + 2 * padding[0] - R) // stride[0] + 1
+    Q = (W + 2 * padding[1] - S) // stride[1] + 1
+    if tuple(dy.shape) != (N, K, P, Q):
+        raise PolyconvError(BAD_PARAM, "dy must be %s, got %s" % ((N, K, P, Q), tuple(dy.shape)))
     dw = torch.empty((K, C, R, S), dtype=x.dtype, device=x.device)
     ws = torch.empty(K * C * R * S, dtype=torch.float32, device=x.device)
-    st = load_library().polyconv_wgrad(ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(dy.data_ptr()),
-                                      ctypes.c_void_p(dw.data_ptr()), ctypes.c_void_p(ws.data_ptr()), N, C, H, W, K,
-                                      R, S, stride[0], stride[1], padding[0], padding[1], _dtype_code(x),
-                                      _stream_ptr(stream))
+    with _on_device(x):
+        st = load_library().polyconv_wgrad(ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(dy.data_ptr()),
+                                          ctypes.c_void_p(dw.data_ptr()), ctypes.c_void_p(ws.data_ptr()), N, C, H, W,
+                                          K, R, S, stride[0], stride[1], padding[0], padding[1], _dtype_code(x),
+                                          _stream_ptr(stream, x.device))
     if st != SUCCESS:
         raise PolyconvError(st, "polyconv_wgrad: %s" % status_string(st))
     return dw

@@ -67,7 +67,13 @@ def build(force: bool = False, verbose: bool = False) -> str:
             sys.stderr.write(log)
     objs = [o for o, _ in results]
     tmp = LIB + ".tmp%d" % os.getpid()
-    cmd = [NVCC] + ARCH + ["-shared", "-o", tmp] + objs
+    # export only the C-ABI: the static cudart stays internal (--exclude-libs) and a version
+    # script hides every other symbol of the objects
+    vmap = os.path.join(OUT_DIR, "obj", "exports.map")
+    with open(vmap, "w") as f:
+        f.write("{ global: polyconv_*; local: *; };\n")
+    cmd = [NVCC] + ARCH + ["-shared", "-Xlinker", "--exclude-libs,ALL", "-Xlinker", "--version-script=" + vmap,
+                           "-o", tmp] + objs
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError("link failed:\n%s\n%s" % (r.stdout, r.stderr))

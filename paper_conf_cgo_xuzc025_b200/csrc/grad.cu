@@ -10,6 +10,7 @@
 // swap_nc: one block per destination row (c, n); the row is a contiguous run of HW elements in
 // both layouts, copied with 16-byte vectors when both ends are 16-byte aligned.
 #include <cuda_runtime.h>
+#include <cuda_bf16.h>
 #include <algorithm>
 #include <cstdint>
 #include "../../include/polyconv.h"
@@ -219,9 +220,9 @@ __global__ void __launch_bounds__(256) f32_to_out(const float* __restrict__ ws, 
   for (long long i = blockIdx.x * 256LL + threadIdx.x; i < n; i += (long long)gridDim.x * 256) {
     const float v = ws[i];
     if (bf16) {
-      uint32_t u = __float_as_uint(v);
-      u = (u + 0x7FFFu + ((u >> 16) & 1u)) >> 16;  // round to nearest even (finite values)
-      static_cast<uint16_t*>(out)[i] = (uint16_t)u;
+      // round to nearest even; NaN stays NaN and Inf stays Inf (the integer
+      // rounding trick turned the canonical NaN into -0)
+      static_cast<__nv_bfloat16*>(out)[i] = __float2bfloat16_rn(v);
     } else {
       static_cast<float*>(out)[i] = v;
     }

@@ -545,28 +545,15 @@ polyconv_status_t polyconv_forward(polyconv_plan_t p, const void* x, const void*
     return finish(p, e, "mac_pair");
   }
   if (p->kernel == POLYCONV_KERNEL_TC_FUSED) {
-    // one launch: a3 (filter slices, every CTA), a2 (packer warps), a4, a5.  The
-    // grid is persistent (one CTA per SM at most), so all CTAs are co-resident
-    // and meet on the plan's counter before the first filter tile is loaded.
-    if (!p->fcount) {
-      if (cudaMalloc(&p->fcount, sizeof(unsigned long long)) != cudaSuccess ||
-          cudaMemsetAsync(p->fcount, 0, sizeof(unsigned long long), st) != cudaSuccess) {
-        cudaGetLastError();
-        p->fcount = nullptr;
-        set_err(p, "cudaMalloc of the %s failed", "filter-pack counter");
-        return POLYCONV_STATUS_ALLOC_FAILED;
-      }
-      p->fepoch = 0;
-    }
-    if (p->tc2.grid > p->num_sms) {
-      set_err(p, "mac_tc_fused: grid %s exceeds the SM count", "");
-      return POLYCONV_STATUS_NOT_SUPPORTED;
-    }
+    // a3 (tap-major filter, one small launch), then a2 (packer warps) + a4 + a5 in mac_tc2 as
+    // its programmatic dependent.  (The filter used to be packed inside the MAC grid, whose
+    // CTAs met on a plan-owned counter: that needed the whole grid co-resident and broke on
+    // CUDA-graph replay.)
     if (p->ev_start) cudaEventRecord(p->ev_start, st);
-    const unsigned long long target = (p->fepoch + 1) * (unsigned long long)p->tc2.grid;
-    e = launch_mac_tc2(g, p->tc2, p->fmt, x, p->io_bf16, nullptr, p->wsU, y, p->io_bf16, false, st, p->err,
-                       sizeof(p->err), w, p->fcount, target);
-    if (e == cudaSuccess) ++p->fepoch;
+    e = launch_pack_filter_tapmajor(g, w, p->io_bf16, p->wsU, p->fmt, g.Kp, g.Cp, st);
+    if (e != cudaSuccess) return finish(p, e, "pack_filter");
+    e = launch_mac_tc2(g, p->tc2, p->fmt, x, p->io_bf16, nullptr, p->wsU, y, p->io_bf16, true, st, p->err,
+                       sizeof(p->err));
     if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
     return finish(p, e, "mac_tc_fused");
   }

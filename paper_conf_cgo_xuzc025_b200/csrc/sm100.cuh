@@ -31,19 +31,13 @@ __device__ __forceinline__ uint64_t global_ns() {
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
   return t;
 }
+// Waits are plain polls: every mbarrier is signalled by work of the same CTA or CTA pair
+// (no grid-wide dependencies), so a wait cannot be starved by other work holding SMs; there
+// is no watchdog trap (a trap poisons the whole CUDA context).
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   const uint32_t a = smem_u32(bar);
   uint32_t done;
-  uint32_t spins = 0;
-  uint64_t t0 = 0;
   do {
-    // watchdog: a lost arrive traps (a launch error the host reports) after
-    // ~0.5 s instead of hanging the GPU
-    if ((++spins & 0xFFFu) == 0) {
-      const uint64_t t = global_ns();
-      if (t0 == 0) t0 = t;
-      else if (t - t0 > 500000000ull) __trap();
-    }
     asm volatile(
         "{\n\t.reg .pred p;\n\t"
         "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
@@ -59,9 +53,7 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
 __device__ __forceinline__ void mbar_wait_spin(uint64_t* bar, uint32_t parity) {
   const uint32_t a = smem_u32(bar);
   uint32_t done;
-  uint32_t spins = 0;
-  uint64_t t0 = 0;
-  for (;;) {
+  do {
     asm volatile(
         "{\n\t.reg .pred p;\n\t"
         "mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
@@ -69,13 +61,7 @@ __device__ __forceinline__ void mbar_wait_spin(uint64_t* bar, uint32_t parity) {
         : "=r"(done)
         : "r"(a), "r"(parity)
         : "memory");
-    if (done) return;
-    if ((++spins & 0xFFFu) == 0) {
-      const uint64_t t = global_ns();
-      if (t0 == 0) t0 = t;
-      else if (t - t0 > 500000000ull) __trap();
-    }
-  }
+  } while (!done);
 }
 
 // mbar_wait for roles that wait long (epilogue, packers): back off with
@@ -84,7 +70,6 @@ __device__ __forceinline__ void mbar_wait_spin(uint64_t* bar, uint32_t parity) {
 __device__ __forceinline__ void mbar_wait_sleep(uint64_t* bar, uint32_t parity, uint32_t ns) {
   const uint32_t a = smem_u32(bar);
   uint32_t done;
-  uint64_t t0 = 0;
   for (;;) {
     asm volatile(
         "{\n\t.reg .pred p;\n\t"
@@ -94,9 +79,6 @@ __device__ __forceinline__ void mbar_wait_sleep(uint64_t* bar, uint32_t parity, 
         : "r"(a), "r"(parity)
         : "memory");
     if (done) return;
-    const uint64_t t = global_ns();
-    if (t0 == 0) t0 = t;
-    else if (t - t0 > 500000000ull) __trap();
     __nanosleep(ns);
   }
 }

@@ -24,6 +24,16 @@ def test_exports_every_declared_symbol():
     assert lib.polyconv_abi_version() == 1
 
 
+def test_exports_only_the_c_abi():
+    """The shared library exports the polyconv_* C-ABI and nothing else: the static CUDA runtime
+    and the internal C++ symbols stay local (version script + --exclude-libs)."""
+    import subprocess
+    out = subprocess.run(["nm", "-D", "--defined-only", pc.LIB_PATH], capture_output=True, text=True).stdout
+    names = [l.split()[-1] for l in out.splitlines() if l.strip()]
+    assert names and all(n.startswith("polyconv_") for n in names), [n for n in names if not n.startswith("polyconv_")]
+    assert "cudaMemcpyAsync" not in names
+
+
 def test_status_strings():
     for s in range(5):
         assert pc.status_string(s).startswith("POLYCONV_STATUS_")
@@ -125,7 +135,7 @@ def test_tc_tiling_choices():
     # TC_PAIR (bf16 default): pair tile = 256 positions x NN output channels (NN = K
     # rounded up to 64), channels in chunks of 64/32/16; one launch
     inf = pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="bf16", kernel="tc_pair").info()
-    assert (inf["tile_m"], inf["tile_n"], inf["Cp"], inf["Kp"], inf["launches"]) == (256, 128, 128, 128, 1)
+    assert (inf["tile_m"], inf["tile_n"], inf["Cp"], inf["Kp"], inf["launches"]) == (256, 128, 128, 128, 2)
     # TC_HANKEL: pair item = 256*T positions x NN output channels; NN = K (<= 256) else 256,
     # T*NN <= 256; channels in chunks of 64 (bf16) / 32 (tf32); filter pack + one launch
     hk = lambda xs, ws, m="bf16": pc.Plan(xs, ws, (1, 1), (1, 1), math=m, kernel="tc_hankel").info()
@@ -137,10 +147,12 @@ def test_tc_tiling_choices():
     assert (inf["tile_m"], inf["tile_n"], inf["Kp"]) == (256, 256, 512)
     inf = hk((2, 40, 9, 9), (72, 40, 3, 3), "tf32")
     assert (inf["tile_n"], inf["Cp"], inf["Kp"]) == (80, 64, 80)
-    inf = pc.Plan((2, 3, 30, 30), (64, 3, 7, 7), (2, 2), (3, 3), math="bf16").info()
-    assert (inf["kernel"], inf["Cp"], inf["Kp"]) == ("tc_pair", 16, 64)
-    inf = pc.Plan((2, 40, 9, 9), (72, 40, 3, 3), (1, 1), (1, 1), math="bf16", kernel="tc_pair").info()
-    assert (inf["kernel"], inf["Cp"], inf["Kp"]) == ("tc_pair", 64, 128)
+    # TC_PAIR needs its separate packing grid (TMA views of x: H*W*elem % 16 == 0); the
+    # one-launch mode with a grid barrier is gone, so other shapes are not supported
+    with pytest.raises(pc.PolyconvError):
+        pc.Plan((2, 3, 30, 30), (64, 3, 7, 7), (2, 2), (3, 3), math="bf16", io_dtype="bf16", kernel="tc_pair")
+    inf = pc.Plan((2, 40, 8, 8), (72, 40, 3, 3), (1, 1), (1, 1), math="bf16", kernel="tc_pair").info()
+    assert (inf["kernel"], inf["Cp"], inf["Kp"], inf["launches"]) == ("tc_pair", 64, 128, 2)
     # TC_PERTAP (ablation): tile = 128 positions x bn output channels
     inf = pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="bf16", kernel="tc_pertap").info()
     assert (inf["tile_m"], inf["tile_n"], inf["Cp"], inf["Kp"]) == (128, 128, 128, 128)

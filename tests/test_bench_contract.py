@@ -8,13 +8,14 @@ import sys
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
-def _run(extra_env=None):
+def _run(extra_env=None, gpus=1):
     env = dict(os.environ)
     env.update({"POLYCONV_CPU_BASELINE_S": "0.5"})
     if extra_env:
         env.update(extra_env)
     return subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--impl", "reference", "--steps", "2",
-                           "--warmup", "0"], capture_output=True, text=True, env=env, timeout=600, cwd=ROOT)
+                           "--warmup", "0", "--gpus", str(gpus)], capture_output=True, text=True, env=env,
+                          timeout=600, cwd=ROOT)
 
 
 def test_reference_arm_line():
@@ -34,6 +35,13 @@ def test_reference_arm_line():
 
 
 def test_reference_arm_nonzero_rank_silent():
-    r = _run({"RANK": "1", "WORLD_SIZE": "2"})
+    r = _run({"RANK": "1", "WORLD_SIZE": "2"}, gpus=2)
     assert r.returncode == 0, r.stderr[-2000:]
     assert not [l for l in r.stdout.splitlines() if l.strip().startswith("{")]
+
+
+def test_gpus_must_match_world_size():
+    """--gpus N under a launcher with another WORLD_SIZE is an error, not a silent 1-GPU run."""
+    r = _run({"RANK": "0", "WORLD_SIZE": "2"}, gpus=4)
+    assert r.returncode != 0
+    assert "WORLD_SIZE" in (r.stderr + r.stdout)
