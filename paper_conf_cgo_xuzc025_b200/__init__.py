@@ -16,7 +16,7 @@ import ctypes
 import os
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "_lib", "libpolyconv.so")
+LIB_PATH = os.environ.get("POLYCONV_LIB") or os.path.join(_PKG, "_lib", "libpolyconv.so")  # override: A/B runs
 
 SUCCESS, BAD_PARAM, NOT_SUPPORTED, ALLOC_FAILED, EXECUTION_FAILED = range(5)
 F32, BF16 = 0, 1
