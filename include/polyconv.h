@@ -103,7 +103,8 @@ typedef enum {
     POLYCONV_KERNEL_TC_FUSED = 5,
     POLYCONV_KERNEL_TC_PAIR = 6,
     POLYCONV_KERNEL_TC_1X1 = 7,
-    POLYCONV_KERNEL_TC_HANKEL = 8
+    POLYCONV_KERNEL_TC_HANKEL = 8,
+    POLYCONV_KERNEL_FFT = 9
 } polyconv_kernel_t;
 
 /* Packed-operand layouts exposed for bit-exact tests (a2/a3):

@@ -21,7 +21,7 @@ LIB_PATH = os.environ.get("POLYCONV_LIB") or os.path.join(_PKG, "_lib", "libpoly
 SUCCESS, BAD_PARAM, NOT_SUPPORTED, ALLOC_FAILED, EXECUTION_FAILED = range(5)
 F32, BF16 = 0, 1
 MATH = {"fp32": 0, "tf32": 1, "bf16": 2}
-KERNEL = {"auto": 0, "tc": 1, "fp32": 2, "thin": 3, "tc_pertap": 4, "tc_fused": 5, "tc_pair": 6, "tc_1x1": 7, "tc_hankel": 8}
+KERNEL = {"auto": 0, "tc": 1, "fp32": 2, "thin": 3, "tc_pertap": 4, "tc_fused": 5, "tc_pair": 6, "tc_1x1": 7, "tc_hankel": 8, "fft": 9}
 KERNEL_NAME = {v: k for k, v in KERNEL.items()}
 LAYOUT = {"planar": 0, "interleaved": 1}
 

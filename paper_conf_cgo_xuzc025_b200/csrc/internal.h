@@ -178,4 +178,17 @@ size_t hankel_zero_bytes(const Geom& g);
 cudaError_t launch_mac_hankel(const Geom& g, const HankelTiling& t, int fmt, const void* x, bool io_bf16,
                               const void* U, void* y, const void* zero, cudaStream_t st, char* err, size_t errlen);
 
+// ---- fft.cu (R = IFFT(FFT(A) . FFT(U)) per channel, summed in frequency) ----
+struct FftTiling {
+  bool ok;
+  int L, logL, F;          // FFT length (power of two >= L_A + L_U - 1), bins kept (L/2 + 1)
+  int RB;                  // (n, k) rows per CTA of the inverse transform
+  size_t x_bytes, u_bytes, y_bytes, tw_bytes;  // spectra X^[F][N][C], U^[F][K][C], Y^[F][N][K]; twiddles
+};
+FftTiling fft_tiling(const Geom& g);
+cudaError_t launch_fft_twiddles(const FftTiling& t, void* tw, cudaStream_t st);
+// ws: x_bytes + u_bytes + y_bytes; tw: twiddles from launch_fft_twiddles
+cudaError_t launch_fft_conv(const Geom& g, const FftTiling& t, const void* x, const void* w, bool io_bf16, void* ws,
+                            const void* tw, void* y, cudaStream_t st);
+
 }  // namespace polyconv

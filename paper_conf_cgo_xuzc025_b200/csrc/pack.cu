@@ -220,10 +220,18 @@ __device__ __forceinline__ void pack_tapmajor_kc(const Geom& g, const InT* __res
   const bool in = k < g.K && c < g.C;
   const InT* src = w + ((long long)k * g.C + c) * RS;
   const long long rep_stride = (long long)RS * Kp * Cp;
-#pragma unroll 4
-  for (int tap = 0; tap < RS; ++tap) {
-    const auto v = Word<F>::enc(in ? load_io(src, tap) : 0.f);
-    for (int r = 0; r < g.urep; ++r) dst[r * rep_stride + ((long long)tap * Kp + k) * Cp + c] = v;
+  // eight taps' loads in flight before their stores (one dependent load per tap took ~4 us
+  // for the conv3_x filter, all of it latency)
+  for (int t0 = 0; t0 < RS; t0 += 8) {
+    float v[8];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) v[j] = (in && t0 + j < RS) ? load_io(src, t0 + j) : 0.f;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      if (t0 + j >= RS) break;
+      const auto e = Word<F>::enc(v[j]);
+      for (int r = 0; r < g.urep; ++r) dst[r * rep_stride + ((long long)(t0 + j) * Kp + k) * Cp + c] = e;
+    }
   }
 }
 

@@ -25,6 +25,8 @@ struct polyconv_plan_s {
   Fp32Tiling f32;
   PairTiling pair;
   HankelTiling hk;
+  FftTiling fft;
+  bool fft_tw_ready = false;  // twiddles computed into wsU
   void* hkzero = nullptr;  // mac_hankel: zero words read in place of padding (hankel_zero_bytes)
   void* pair_state = nullptr;  // mac_pair launch cache
   unsigned long long* bflag = nullptr;  // mac_pair band flags [N * pair.nb]
@@ -96,6 +98,23 @@ bool fused_pays(const Geom& g) {
   return g.K <= 128 && g.Wp <= 64 && g.R * g.S <= 9;
 }
 
+// FP32 math (method selection): the FFT solver (fft.cu, the paper's Eq. 13-15)
+// against the direct FFMA MAC, measured per layer (tools/fp32_cmp.py, profiles/r02_fp32_cmp.jsonl).
+// Direct work ~ R*S*P*Q per (n, k, c) against ~ L per (n, k, c) in the frequency domain, so the
+// FFT pays when R*S*P*Q / L is large; at L >= 2048 its transforms run one CTA per SM and need a
+// larger margin.  Wins: ResNet-50 l2/l3/l4 3x3 at N=256 (31/29/40 vs 26/26/7 TFLOP/s), VGG conv4-5
+// (56 vs 28), the 5x5/7x7 sweep points on 56x56 (31 vs 28); losses kept direct: l1 3x3 on 56x56
+// (12 vs 28), 1x1 layers on large planes.  POLYCONV_NO_FFT disables it.
+bool fft_pays(const Geom& g) {
+  if (getenv("POLYCONV_NO_FFT") || g.K < 16) return false;
+  const FftTiling t = fft_tiling(g);
+  if (!t.ok) return false;
+  const double work = (double)g.R * g.S * g.P * g.Q;
+  if (g.P * g.Q <= 64 && g.sh == 1 && (long long)g.C * g.K >= (1LL << 20)) return true;  // 1x1 on 7x7, C*K >= 1M
+  if (t.L <= 1024) return g.N >= 64 && work >= 0.8 * t.L;
+  return work >= 16.0 * t.L;
+}
+
 // Resolve the MAC variant and fill the kernel-specific padded sizes.
 polyconv_status_t resolve(polyconv_plan_t p) {
   Geom& g = p->g;
@@ -116,7 +135,10 @@ polyconv_status_t resolve(polyconv_plan_t p) {
   if (k == POLYCONV_KERNEL_AUTO && p->math == POLYCONV_MATH_BF16 && g.K >= 16 && g.sh == g.sw && g.sh <= 2 &&
       g.R == g.S && (g.R == 3 || g.R == 5) && !getenv("POLYCONV_NO_HANKEL")) {
     const HankelTiling h = hankel_tiling(g, p->fmt, p->num_sms);
-    if (h.ok && h.aligned && (long long)h.PT * h.NB >= 24) k = POLYCONV_KERNEL_TC_HANKEL;
+    // odd widths use the general (element-load) window loader: it still wins for wide 3x3
+    // layers (ResNet-50 l4 7x7, C = K = 512: 596 vs 572 TFLOP/s for mac_tc2)
+    const bool loader_ok = h.aligned || (g.R == 3 && g.C >= 256 && g.K >= 256);
+    if (h.ok && loader_ok && (long long)h.PT * h.NB >= 24) k = POLYCONV_KERNEL_TC_HANKEL;
   }
   if (k == POLYCONV_KERNEL_AUTO) {
     // bf16, at most two rounds of pair tiles: one launch on CTA pairs with a resident filter
@@ -141,6 +163,8 @@ polyconv_status_t resolve(polyconv_plan_t p) {
       k = (g.K >= 16 && tc2_supported(g, p->fmt))  ? POLYCONV_KERNEL_TC
           : (g.K >= 16 && tc_supported(g, p->fmt)) ? POLYCONV_KERNEL_TC_PERTAP
                                                    : POLYCONV_KERNEL_THIN;
+    else if (fft_pays(g))
+      k = POLYCONV_KERNEL_FFT;
     else
       k = (g.K >= 16 && g.C * g.R * g.S >= 16 && fp32_tiling(g).smax > 0) ? POLYCONV_KERNEL_FP32
                                                                           : POLYCONV_KERNEL_THIN;
@@ -153,6 +177,10 @@ polyconv_status_t resolve(polyconv_plan_t p) {
     p->hk = hankel_tiling(g, p->fmt, p->num_sms);
     if (!tc_math || !p->hk.ok) return POLYCONV_STATUS_BAD_PARAM;
   }
+  if (k == POLYCONV_KERNEL_FFT) {
+    p->fft = fft_tiling(g);
+    if (tc_math || !p->fft.ok) return POLYCONV_STATUS_BAD_PARAM;  // fp32 spectra: math FP32_FMA
+  }
   if (k == POLYCONV_KERNEL_TC_PERTAP && (!tc_math || !tc_supported(g, p->fmt))) return POLYCONV_STATUS_BAD_PARAM;
   if (k == POLYCONV_KERNEL_FP32 && (tc_math || fp32_tiling(g).smax == 0)) return POLYCONV_STATUS_BAD_PARAM;
   p->kernel = k;
@@ -162,6 +190,9 @@ polyconv_status_t resolve(polyconv_plan_t p) {
   } else if (k == POLYCONV_KERNEL_TC_HANKEL) {
     g.Cp = p->hk.Cp;
     g.Kp = p->hk.Kp;
+  } else if (k == POLYCONV_KERNEL_FFT) {
+    g.Cp = g.C;
+    g.Kp = g.K;
   } else if (k == POLYCONV_KERNEL_TC_1X1) {
     g.Cp = (g.C + 63) / 64 * 64;
     g.Kp = (g.K + 127) / 128 * 128;
@@ -198,6 +229,11 @@ polyconv_status_t resolve(polyconv_plan_t p) {
     if ((long long)g.urep * g.R * g.S * g.Kp >= (1LL << 31)) g.urep = 1;  // TMA row coordinate
   }
   p->wsU_bytes = (size_t)g.urep * g.R * g.S * g.Kp * g.Cp * eb;
+  if (k == POLYCONV_KERNEL_FFT) {
+    p->wsA_bytes = p->fft.x_bytes + p->fft.u_bytes + p->fft.y_bytes;
+    p->wsU_bytes = p->fft.tw_bytes;
+    p->fft_tw_ready = false;
+  }
   return POLYCONV_STATUS_SUCCESS;
 }
 
@@ -374,7 +410,7 @@ polyconv_status_t polyconv_plan_set_kernel(polyconv_plan_t p, polyconv_kernel_t 
     if (so != POLYCONV_STATUS_SUCCESS) polyconv_plan_set_kernel(in, (polyconv_kernel_t)old_inner);
     return so;
   }
-  if (kernel < POLYCONV_KERNEL_AUTO || kernel > POLYCONV_KERNEL_TC_HANKEL) return POLYCONV_STATUS_BAD_PARAM;
+  if (kernel < POLYCONV_KERNEL_AUTO || kernel > POLYCONV_KERNEL_FFT) return POLYCONV_STATUS_BAD_PARAM;
   const int old = p->forced;
   p->forced = kernel;
   if (resolve(p) != POLYCONV_STATUS_SUCCESS) {
@@ -417,6 +453,8 @@ polyconv_status_t polyconv_plan_info(polyconv_plan_t p, polyconv_info_t* info) {
     case POLYCONV_KERNEL_TC_PAIR:  // pair tile = 256 positions x NN output channels
       info->tile_m = 256; info->tile_n = p->pair.NN; info->stages = p->pair.ring;
       info->launches = p->pair.split ? 2 : 1; break;
+    case POLYCONV_KERNEL_FFT:  // one FFT length L per polynomial; tile = the contraction's 32 x 64
+      info->tile_m = p->fft.L; info->tile_n = 64; info->stages = p->fft.F; info->launches = 4; break;
     case POLYCONV_KERNEL_TC_HANKEL:  // pair item = 256*T positions x NN output channels
       info->tile_m = 256 * p->hk.T; info->tile_n = p->hk.NN; info->stages = p->hk.wslots;
       info->launches = 2; break;
@@ -483,6 +521,19 @@ polyconv_status_t polyconv_forward(polyconv_plan_t p, const void* x, const void*
                        sizeof(p->err));
     if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
     return finish(p, e, "mac_tc");
+  }
+  if (p->kernel == POLYCONV_KERNEL_FFT) {
+    // the paper's solver (Eq. 13-15): FFT of every A_{n,c} and U_{k,c}, per-frequency
+    // channel contraction, inverse FFT + Eq. 12 extraction (fft.cu)
+    if (!p->fft_tw_ready) {
+      e = launch_fft_twiddles(p->fft, p->wsU, st);
+      if (e != cudaSuccess) return finish(p, e, "fft_twiddles");
+      p->fft_tw_ready = true;
+    }
+    if (p->ev_start) cudaEventRecord(p->ev_start, st);
+    e = launch_fft_conv(g, p->fft, x, w, p->io_bf16, p->wsA, p->wsU, y, st);
+    if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
+    return finish(p, e, "fft_conv");
   }
   if (p->kernel == POLYCONV_KERNEL_TC_HANKEL) {
     // a3 (tap-major filter, one small launch), then a2 + a4 + a5 in the persistent pair

@@ -109,7 +109,8 @@ def test_kernel_selection_and_forcing():
     k3 = lambda xs, ws, s=1: pc.Plan(xs, ws, (s, s), (ws[2] // 2, ws[3] // 2), math="bf16",
                                      io_dtype="bf16").info()["kernel"]
     assert k3((32, 128, 28, 28), (128, 128, 3, 3)) == "tc_hankel"
-    assert k3((256, 512, 7, 7), (512, 512, 3, 3)) == "tc"            # odd width
+    assert k3((256, 512, 7, 7), (512, 512, 3, 3)) == "tc_hankel"     # odd width, wide layer
+    assert k3((256, 128, 7, 7), (128, 128, 3, 3)) == "tc"            # odd width, narrow
     assert k3((256, 128, 56, 56), (128, 128, 3, 3), 2) == "tc_hankel"
     assert k3((32, 64, 8, 8), (64, 64, 3, 3)) == "tc"                # 12 units < 24
     assert k3((32, 128, 14, 14), (64, 128, 3, 3)) == "tc_hankel"
@@ -119,6 +120,24 @@ def test_kernel_selection_and_forcing():
     # f32 I/O, bf16 math: the same rule
     assert pc.Plan((32, 64, 8, 8), (64, 64, 3, 3), (1, 1), (1, 1), math="bf16").info()["kernel"] == "tc_pair"
     assert pc.Plan((32, 64, 28, 28), (64, 64, 3, 3), (1, 1), (1, 1), math="bf16").info()["kernel"] == "tc_hankel"
+
+
+def test_fft_solver_planning():
+    """f1: the FFT length is the power of two >= L_A + L_U - 1 (Eq. 14, reading Z9); FP32 math
+    only; AUTO takes it for FP32 layers where the measured cost model favours it (fft_pays)."""
+    inf = pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="fp32", kernel="fft").info()
+    assert inf["kernel"] == "fft" and inf["tile_m"] == 1024 and inf["launches"] == 4   # 900 + 63 - 1 -> 1024
+    inf = pc.Plan((2, 8, 7, 7), (8, 8, 3, 3), padding=(1, 1), math="fp32", kernel="fft").info()
+    assert inf["tile_m"] == 128                                                          # 81 + 21 - 1 -> 128
+    with pytest.raises(pc.PolyconvError):
+        pc.Plan((1, 8, 100, 100), (8, 8, 3, 3), padding=(1, 1), math="fp32", kernel="fft")   # L > 8192
+    with pytest.raises(pc.PolyconvError):
+        pc.Plan((1, 8, 20, 20), (8, 8, 3, 3), padding=(1, 1), math="tf32", kernel="fft")
+    auto = lambda xs, ws, s=1: pc.Plan(xs, ws, (s, s), (ws[2] // 2, ws[3] // 2), math="fp32").info()["kernel"]
+    assert auto((256, 512, 7, 7), (512, 512, 3, 3)) == "fft"      # ResNet-50 l4 3x3: 40 vs 7 TFLOP/s
+    assert auto((256, 128, 28, 28), (128, 128, 3, 3)) == "fft"    # l2 3x3: 31 vs 26
+    assert auto((256, 64, 56, 56), (64, 64, 3, 3)) == "fp32"      # l1 3x3 (L = 4096): 12 vs 28
+    assert auto((32, 128, 28, 28), (128, 128, 3, 3)) == "fp32"    # conv3_x at N=32: 20 vs 22
 
 
 def test_tc_tiling_choices():

@@ -219,3 +219,42 @@ def test_forward_while_other_work_holds_sms(kernel, shape):
     torch.cuda.synchronize()
     assert np.array_equal(y.float().cpu().numpy(), bf16_round(oracle.conv2d(xi, wi, shape.stride, shape.padding)))
     assert torch.isfinite(a).all()
+
+
+# ---- f1: the FFT-domain solver (Eq. 13-15), FP32 -------------------------------------------
+FFT_SHAPES = [synth.TINY, synth.CONV3X,
+              ConvShape("fft_s2", 4, 32, 21, 19, 48, 3, 3, 2, 2, 1, 1),
+              ConvShape("fft_5x5", 8, 64, 28, 28, 64, 5, 5, 1, 1, 2, 2),
+              ConvShape("fft_7x7_nopad", 4, 16, 30, 26, 24, 7, 7, 1, 1, 0, 0),
+              ConvShape("fft_1x1", 4, 64, 14, 14, 96, 1, 1),
+              ConvShape("fft_rect", 3, 24, 9, 40, 40, 2, 4, 1, 1, 0, 1)] + \
+             [s for s in synth.SWEEP if s.name in ("A_h14_s1", "A_h28_s1", "A_h56_s1", "B_r7_s1", "B_r5_s2")] + \
+             [s for s in synth.RESNET50 if s.name in ("l3_3x3_256", "l4_3x3_512", "l4_3x3_512_s2")]
+
+
+@pytest.mark.parametrize("shape", FFT_SHAPES, ids=lambda s: s.name)
+@pytest.mark.parametrize("io", ["f32"])
+def test_fft_solver(shape, io):
+    """FFT of every A_{n,c}(t) and U_{k,c}(t), per-frequency channel sum, IFFT, Eq. 12
+    extraction (math FP32_FMA: fp32 spectra, f32 I/O): within the FP32 gate of O1."""
+    import torch
+    import paper_conf_cgo_xuzc025_b200 as pc
+    dt = torch.bfloat16 if io == "bf16" else torch.float32
+    gen = torch.Generator(device="cuda").manual_seed(51)
+    x = (torch.rand((shape.N, shape.C, shape.H, shape.W), generator=gen, device="cuda") * 2 - 1).to(dt)
+    w = ((torch.rand((shape.K, shape.C, shape.R, shape.S), generator=gen, device="cuda") * 2 - 1)
+         / np.sqrt(shape.C * shape.R * shape.S)).to(dt)
+    plan = pc.Plan(x.shape, w.shape, shape.stride, shape.padding, math="fp32", io_dtype=io, kernel="fft")
+    y = plan.forward(x, w).float().cpu().numpy()
+    images = sorted({0, shape.N - 1})
+    ref = oracle.conv2d(x[images].float().cpu().numpy(), w.float().cpu().numpy(), shape.stride, shape.padding)
+    gate = GATE["fp32"] if io == "f32" else 2 ** -8
+    assert normwise(y[images], ref) <= gate
+
+
+def test_fft_rejects_large_planes_and_tensor_math():
+    import paper_conf_cgo_xuzc025_b200 as pc
+    with pytest.raises(pc.PolyconvError):
+        pc.Plan((1, 8, 100, 100), (8, 8, 3, 3), padding=(1, 1), math="fp32", kernel="fft")   # L > 8192
+    with pytest.raises(pc.PolyconvError):
+        pc.Plan((1, 8, 20, 20), (8, 8, 3, 3), padding=(1, 1), math="bf16", kernel="fft")

@@ -18,7 +18,7 @@ pytestmark = pytest.mark.gpu
 
 MATH_KERNELS = [("fp32", "fp32"), ("fp32", "thin"), ("tf32", "tc"), ("bf16", "tc"), ("tf32", "tc_pertap"),
                 ("bf16", "tc_pertap"), ("tf32", "tc_fused"), ("bf16", "tc_fused"), ("tf32", "thin"),
-                ("bf16", "thin"), ("bf16", "tc_pair"), ("bf16", "tc_hankel"), ("tf32", "tc_hankel")]
+                ("bf16", "thin"), ("bf16", "tc_pair"), ("bf16", "tc_hankel"), ("tf32", "tc_hankel"), ("fp32", "fft")]
 
 SHAPES = [
     ConvShape("tiny", 1, 1, 8, 8, 1, 3, 3),                      # BASELINE configs[0]
@@ -71,7 +71,10 @@ def test_parity_uniform(shape, math, kernel):
 @pytest.mark.parametrize("math,kernel", MATH_KERNELS, ids=lambda v: str(v))
 def test_integer_exact(shape, math, kernel):
     """|x|<=8, |w|<=4: every product and partial sum is an integer < 2^24, so
-    every precision must reproduce the oracle bit for bit."""
+    every precision must reproduce the oracle bit for bit.  The FFT solver
+    (f1) rounds in its transforms: not an exact method, checked by the normwise gates."""
+    if kernel == "fft":
+        pytest.skip("FFT solver: fp32 transforms round (normwise gate in test_parity_uniform)")
     _skip_unsupported(shape, math, kernel)
     x, w = synth.make_inputs(shape, synth.seed_for(8, hash(shape.name) % 997), "int")
     ref = oracle.conv2d(x, w, shape.stride, shape.padding)
