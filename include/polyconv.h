@@ -70,30 +70,29 @@ typedef enum {
     POLYCONV_MATH_BF16 = 2
 } polyconv_math_t;
 
-/* MAC kernel variant.  AUTO picks by shape and math; the others force one
- * (ablations/tests).  TC = tcgen05/TMEM tensor-core contraction, filters as
- * the M=128 operand, one position window per channel chunk reused by every
- * tap (Hankel shift = descriptor offset), windows loaded by TMA from the
- * packed input; TC_FUSED = the same contraction with the input packing done
- * inside the kernel by packer warps (ablation); TC_PERTAP = the earlier
- * tensor-core variant with positions as M and one TMA window load per tap
- * (ablation); TC_PAIR = the BF16 default: ONE launch that packs the input
- * and filter polynomials (a2, a3) into the plan workspace, then runs the
- * contraction on CTA pairs (tcgen05 cta_group::2, 256 positions x up to 256
- * output channels per pair tile) with the filter resident in shared memory
- * and the extraction (a5) fused into its epilogue (bf16 math, K <= 256 and a
- * filter half that fits shared memory; polyconv_plan_set_kernel returns
- * POLYCONV_STATUS_BAD_PARAM otherwise).  Its CTAs meet on plan-owned counters
- * and flags, so the whole grid (one CTA per SM) must be co-resident: the launch
- * checks the co-resident cluster capacity, and a grid that cannot make progress
- * (SMs held by other work for > 0.5 s) traps and forward returns
- * POLYCONV_STATUS_EXECUTION_FAILED instead of hanging.  One plan must not run
- * two TC_PAIR forwards concurrently on different streams (the counters are
- * per plan); TC_1X1 = 1x1, stride-1, unpadded BF16 layers: the input polynomials are
- * the NCHW planes themselves, read by the tensor cores as the MN-major operand
- * (no packed input copy);
- * FP32 = SIMT register-blocked FFMA; THIN = warp-per-output with shuffle
- * reduction over C*R*S (tiny channel counts). */
+/* MAC kernel variant.  AUTO picks by shape and math (DESIGN.md §4.8); the others force one
+ * (ablations/tests; polyconv_plan_set_kernel returns POLYCONV_STATUS_BAD_PARAM when the shape or
+ * math does not fit the variant).
+ *  TC        tcgen05/TMEM contraction, filters as the M=128 operand, one position window per
+ *            channel chunk reused by every tap (Hankel shift = descriptor offset), windows by TMA
+ *            from a packed input (TF32 default).
+ *  TC_FUSED  the same contraction with the input packed inside the kernel (filter packed by its
+ *            own launch).
+ *  TC_PERTAP positions as M, one TMA window load per tap (ablation).
+ *  TC_PAIR   CTA pairs (cta_group::2) with the filter resident in shared memory, fed by a
+ *            separate packing grid (bf16 math, K <= 128, H*W*elem a multiple of 16 bytes).
+ *  TC_1X1    1x1 layers: the NCHW planes are the MN-major tensor-core operand.
+ *  TC_HANKEL the BF16 default for 3x3/5x5 layers: one persistent launch on CTA pairs that builds
+ *            the Hankel windows of the input polynomial in shared memory straight from NCHW x (the
+ *            batch as one polynomial whose images share padding rows, reading R16) and
+ *            runs tcgen05.mma cta_group::2 with the filter resident or streamed by TMA (bf16 or
+ *            tf32 math, any stride / padding / kernel size).
+ *  FFT       the paper's solver (Eq. 13-15): FFT of every A_{n,c}(t) and U_{k,c}(t), per-frequency
+ *            channel contraction, inverse FFT, Eq. 12 extraction (math FP32_FMA; FFT length
+ *            L = power of two >= L_A + L_U - 1 <= 8192).
+ *  FP32      SIMT register-blocked FFMA.   THIN  warp-per-output with shuffle reduction.
+ * No variant synchronises across CTAs outside a cluster: every launch is safe to capture into a
+ * CUDA graph and to run while other work holds SMs (it waits for them). */
 typedef enum {
     POLYCONV_KERNEL_AUTO = 0,
     POLYCONV_KERNEL_TC = 1,

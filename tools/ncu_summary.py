@@ -22,6 +22,10 @@ WANT = {
     "smsp__cycles_active.avg": "smsp_cycles_active",
     "sm__throughput.avg.pct_of_peak_sustained_elapsed": "sm_throughput_pct",
     "gpc__cycles_elapsed.avg.per_second": "gpc_hz",
+    "lts__t_sectors_srcunit_tex_op_write.sum": "l2_write_sectors",
+    "lts__t_sectors_srcunit_tex_op_read.sum": "l2_read_sectors",
+    "smsp__inst_executed.sum": "inst_executed",
+    "sm__warps_active.avg.pct_of_peak_sustained_active": "warps_active_pct",
 }
 UNIT = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "ns": 1, "us": 1e3, "ms": 1e6, "Ghz": 1e9, "Mhz": 1e6}
 
