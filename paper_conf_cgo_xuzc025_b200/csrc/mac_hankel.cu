@@ -787,6 +787,8 @@ HankelTiling hankel_tiling(const Geom& g, int fmt, int num_sms) {
       wslots = 2;
       fslots = (int)std::min<size_t>(kHkMaxFBlk, (kHkSmemMax - fixed - 2 * (size_t)wslot) / fblk);
       fslots = std::min(fslots, nblk);
+      const int fcap = env_int("POLYCONV_HK_FSLOTS", 0);  // experiment: cap the filter ring
+      if (fcap > 0) fslots = std::max(4, std::min(fslots, fcap));
     }
     if (wslots < 2) continue;
     found = true;
@@ -872,6 +874,15 @@ cudaError_t launch_mac_hankel(const Geom& g, const HankelTiling& t, int fmt, con
   }
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, t.smem_bytes);
   if (e != cudaSuccess) return e;
+  {
+    // shared-memory carveout: just what the kernel needs, the rest stays L1 (the window loaders'
+    // in-flight loads are tracked in L1: experiment POLYCONV_HK_CARVE=percent)
+    const int carve = env_int("POLYCONV_HK_CARVE", -1);
+    if (carve >= 0) {
+      e = cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, carve);
+      if (e != cudaSuccess) return e;
+    }
+  }
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)t.grid);
   cfg.blockDim = dim3(kHkThreads);
