@@ -50,7 +50,7 @@ import synth  # noqa: E402
 
 METRIC = "conv fwd effective TFLOP/s and % roofline per layer at 1/2/4/8 B200 vs cuDNN"
 UNIT = "TFLOP/s"
-WORKLOADS = {"conv3x": synth.CONV3X}
+WORKLOADS = {"conv3x": synth.CONV3X, "resnet50": None}   # resnet50: BASELINE configs[4], strong scaling
 L2_FLUSH_BYTES = 256 << 20
 PROFILES = os.path.join(ROOT, "profiles")
 
@@ -168,7 +168,8 @@ def run_reference(args, rank, world):
     if rank != 0:
         return 0
     import oracle
-    shape = WORKLOADS[args.workload]
+    # resnet50 (strong scaling): the oracle samples its l2 3x3 layer
+    shape = WORKLOADS[args.workload] or next(L for L in synth.RESNET50 if L.name == "l2_3x3_128")
     x, w = synth.make_inputs(shape, synth.seed_for(1), "uniform", batch=(0, 1))
     cores = oracle.max_threads()
     # calibrate: one image, all K output planes
@@ -203,6 +204,104 @@ def run_reference(args, rank, world):
     return 0
 
 
+
+# ------------------------------------------------------- config 4: strong scaling --
+
+def run_resnet50(args, torch, dist, pc, dev, rank, world, local):
+    """BASELINE configs[4]: all 53 forward convs of ResNet-50 v1.5 at N=256 (23 unique shapes,
+    synth.RESNET50 with counts), the batch split over the ranks (images [r*N/G, (r+1)*N/G)),
+    filters replicated; one step = every conv once on this rank's shard, L2 flushed before the
+    step.  value = FLOPs of the whole N=256 stack / max-rank step time (strong scaling)."""
+    io = "bf16" if args.math == "bf16" else "f32"
+    tdt = torch.bfloat16 if io == "bf16" else torch.float32
+    N = 256
+    lo, hi = N * rank // world, N * (rank + 1) // world
+    nb = hi - lo
+    layers = []
+    for li, L in enumerate(synth.RESNET50):
+        g = torch.Generator(device=dev).manual_seed(synth.seed_for(4, li) + rank)
+        x = (torch.rand((nb, L.C, L.H, L.W), device=dev, generator=g) * 2 - 1).to(tdt)
+        w = ((torch.rand((L.K, L.C, L.R, L.S), device=dev, generator=g) * 2 - 1) / (L.C * L.R * L.S) ** 0.5).to(tdt)
+        plan = pc.Plan(x.shape, w.shape, L.stride, L.padding, math=args.math, io_dtype=io, device=local)
+        y = torch.empty(plan.output_shape, dtype=tdt, device=dev)
+        layers.append((L, plan, x, w, y))
+    flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.float32, device=dev)
+
+    def step():
+        for L, plan, x, w, y in layers:
+            for _ in range(L.count):
+                plan.forward(x, w, y)
+
+    def barrier():
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    for _ in range(args.warmup):
+        flush.zero_()
+        step()
+    barrier()
+    stream = torch.cuda.current_stream()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    sampler = ClockSampler(local)
+    with sampler:
+        barrier()
+        for a, b in ev:
+            flush.zero_()
+            a.record(stream)
+            step()
+            b.record(stream)
+        barrier()
+    t = torch.tensor([sum(a.elapsed_time(b) for a, b in ev) / args.steps], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    F = sum(L.count * L.flops() for L in synth.RESNET50)   # whole N=256 stack
+    value = F / (float(t) * 1e-3) / 1e12
+    # end to end: the same step through polyconv_forward_host with pinned host buffers (one
+    # step: 11 GB of activations cross PCIe per pass, so a single timed pass)
+    hosts = [(L, plan, x.cpu().pin_memory(), w.cpu().pin_memory(),
+              torch.empty(plan.output_shape, dtype=tdt).pin_memory()) for L, plan, x, w, y in layers]
+    barrier()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    h2d = d2h = 0
+    for L, plan, xh, wh, yh in hosts:
+        for _ in range(L.count):
+            plan.forward_host(xh, wh, yh)
+            h2d += xh.numel() * xh.element_size() + wh.numel() * wh.element_size()
+            d2h += yh.numel() * yh.element_size()
+    e1.record(stream)
+    barrier()
+    te = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+    kernels = {}
+    for L, plan, *_ in layers:
+        k = plan.info()["kernel"]
+        kernels[k] = kernels.get(k, 0) + L.count
+    launches = sum(L.count * plan.info()["launches"] for L, plan, *_ in layers) * args.steps
+    if rank == 0:
+        peaks, src = _peaks()
+        line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": float(t), "higher_is_better": True, "scaling": "strong",
+                "vs_baseline": None, "dtype": args.math, "data": "synthetic",
+                "config": {"workload": "resnet50_n256_forward_convs", "N": N, "per_rank_batch": nb,
+                           "convs": sum(L.count for L in synth.RESNET50), "unique_shapes": len(synth.RESNET50),
+                           "io_dtype": io, "math": args.math, "kernels": kernels,
+                           "parallelism": "batch-sharded x%d (strong: N=256 split, no collective)" % world,
+                           "l2": "flushed before every step (256 MiB write)"},
+                "e2e": {"value": F / (float(te) * 1e-3) / 1e12, "unit": UNIT, "h2d_bytes_per_step": int(h2d),
+                        "d2h_bytes_per_step": int(d2h), "ms_per_step": float(te), "api": "polyconv_forward_host"},
+                "gpu_launches": int(launches), "clocks": sampler.summary(),
+                "roofline": {"bound": "tensor", "peak": peaks["bf16_tflops"], "unit": "TFLOP/s",
+                             "achieved": value / world, "frac": value / world / peaks["bf16_tflops"],
+                             "traffic": None, "note": "whole stack per GPU against the bf16 peak (%s)" % src}}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
 def cpu_baseline(shape):
     """Oracle timed on the host cores on a bounded sample (~10-20 s of CPU work)."""
     import oracle
@@ -229,7 +328,9 @@ def main():
     ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--workload", default="conv3x", choices=sorted(WORKLOADS))
+    ap.add_argument("--workload", default="conv3x", choices=sorted(WORKLOADS),
+                    help="conv3x: configs[1], weak scaling by batch; resnet50: configs[4], the 53 forward "
+                         "convs of ResNet-50 at N=256 split over the ranks (strong scaling)")
     ap.add_argument("--math", default="bf16", choices=["bf16", "tf32", "fp32"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-cudnn", action="store_true")
@@ -262,6 +363,8 @@ def main():
     dev = torch.device("cuda", local)
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
+    if args.workload == "resnet50":
+        return run_resnet50(args, torch, dist, pc, dev, rank, world, local)
     shape = WORKLOADS[args.workload]
     io = "bf16" if args.math == "bf16" else "f32"
     tdt = torch.bfloat16 if io == "bf16" else torch.float32
