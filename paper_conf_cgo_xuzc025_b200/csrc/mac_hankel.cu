@@ -778,17 +778,26 @@ HankelTiling hankel_tiling(const Geom& g, int fmt, int num_sms) {
     const uint32_t wslot = (uint32_t)wrows * 128u;
     bool resident = false;
     int wslots = 0, fslots = 0;
-    if (NB == 1 && nblk <= kHkMaxFBlk && !no_res && (size_t)nblk * fblk + 2 * wslot + fixed <= (size_t)kHkSmemMax) {
+    // Resident only when streaming would re-read more filter bytes per window than the window
+    // itself holds: otherwise a short filter ring leaves shared memory to L1, which the window
+    // loaders' global loads hit (tools/hk_slots.sh: 64->64 56x56 resident 583 vs streamed 650
+    // TFLOP/s; 128->128 28x28 resident 862 vs streamed 838).
+    const bool want_res = (size_t)nblk * fblk > wslot || env_int("POLYCONV_HK_RESIDENT", 0) != 0;
+    if (NB == 1 && nblk <= kHkMaxFBlk && !no_res && want_res &&
+        (size_t)nblk * fblk + 2 * wslot + fixed <= (size_t)kHkSmemMax) {
       resident = true;
       fslots = nblk;
       wslots = (int)std::min<size_t>(kHkMaxWSlots, (kHkSmemMax - fixed - (size_t)nblk * fblk) / wslot);
     } else {
       if (2 * wslot + fixed + (size_t)4 * fblk > (size_t)kHkSmemMax) continue;
-      wslots = 2;
-      fslots = (int)std::min<size_t>(kHkMaxFBlk, (kHkSmemMax - fixed - 2 * (size_t)wslot) / fblk);
+      // three window slots and a four-block filter ring (512->512 7x7: 596 -> 649 TFLOP/s,
+      // 256->256 14x14: 731 -> 770); POLYCONV_HK_WSLOTS / _FSLOTS override
+      wslots = std::max(2, std::min(kHkMaxWSlots, env_int("POLYCONV_HK_WSLOTS", 3)));
+      while (wslots > 2 && (size_t)wslots * wslot + fixed + (size_t)4 * fblk > (size_t)kHkSmemMax) --wslots;
+      fslots = (int)std::min<size_t>(kHkMaxFBlk, (kHkSmemMax - fixed - (size_t)wslots * wslot) / fblk);
       fslots = std::min(fslots, nblk);
-      const int fcap = env_int("POLYCONV_HK_FSLOTS", 0);  // experiment: cap the filter ring
-      if (fcap > 0) fslots = std::max(4, std::min(fslots, fcap));
+      const int fcap = env_int("POLYCONV_HK_FSLOTS", 4);
+      if (fcap > 0) fslots = std::max(std::min(4, fslots), std::min(fslots, fcap));
     }
     if (wslots < 2) continue;
     found = true;
@@ -807,6 +816,9 @@ HankelTiling hankel_tiling(const Geom& g, int fmt, int num_sms) {
   t.tmem_cols = tc <= 32 ? 32 : tc <= 64 ? 64 : tc <= 128 ? 128 : tc <= 256 ? 256 : 512;
   t.grid = 2 * t.npairs;
   t.ok = true;
+  if (env_int("POLYCONV_HK_VERBOSE", 0))
+    fprintf(stderr, "mac_hankel tiling: NN=%d NB=%d T=%d wrows=%d wslots=%d fslots=%d resident=%d smem=%d\n", t.NN,
+            t.NB, t.T, t.wrows, t.wslots, t.fslots, t.resident, t.smem_bytes);
   return t;
 }
 
