@@ -169,6 +169,7 @@ struct HankelTiling {
   int aligned;             // every position pair is one aligned input pair (fast loader)
   uint32_t wslot_bytes, fblk_bytes;
   int smem_bytes, tmem_cols, npairs, grid;
+  int nacc;  // TMEM accumulator buffers (1 or 2)
 };
 HankelTiling hankel_tiling(const Geom& g, int fmt, int num_sms);
 // x: NCHW input (io dtype); U: tap-major packed filter [RS][Kp][Cp] (t.Kp, t.Cp), packed by

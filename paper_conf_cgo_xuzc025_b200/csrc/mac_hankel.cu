@@ -108,6 +108,7 @@ struct HkParams {
   uint32_t wslot_bytes, fblk_bytes;
   uint32_t idesc;
   int tmem_cols;
+  int nacc;             // accumulator buffers in TMEM (2: the epilogue overlaps the next item's MMAs)
   FastDiv fpitch, fHS, fsh, fsw;
   int dbg;  // POLYCONV_HK_DEBUG (timing ablations, results wrong): 1 loaders store zeros without
             // loading, 2 epilogue skips stores, 4 no MMAs (commits only), 8 per-CTA trace
@@ -517,8 +518,8 @@ __global__ void __launch_bounds__(kHkThreads, 1)
       bool first = true;
       const uint32_t row16 = (uint32_t)p.pitch * 8u;  // one kernel row of taps = pitch window rows, 16-B units
       while (hk_next(p, u, u_hi, it)) {
-        const int a = item & 1;
-        hk_wait(tempty + a, (uint32_t)((item >> 1) & 1) ^ 1u);
+        const int a = p.nacc == 2 ? (item & 1) : 0;
+        hk_wait(tempty + a, (uint32_t)((item / p.nacc) & 1) ^ 1u);
         tc_fence_after();
         const uint32_t dacc = tbase + (uint32_t)(a * p.T * p.NN);
         int fb = 0;  // resident: block index
@@ -627,8 +628,8 @@ __global__ void __launch_bounds__(kHkThreads, 1)
     HkItem it;
     int item = 0;
     while (hk_next(p, u, u_hi, it)) {
-      const int a = item & 1;
-      hk_wait(eloc + a, (uint32_t)((item >> 1) & 1), 64);
+      const int a = p.nacc == 2 ? (item & 1) : 0;
+      hk_wait(eloc + a, (uint32_t)((item / p.nacc) & 1), 64);
       if (lane == 0) hk_arrive_cluster(tempty0 + (uint32_t)a * 8u);
       __syncwarp();
       ++item;
@@ -647,8 +648,8 @@ __global__ void __launch_bounds__(kHkThreads, 1)
     HkItem it;
     int item = 0;
     while (hk_next(p, u, u_hi, it)) {
-      const int a = item & 1;
-      hk_wait(tfull + a, (uint32_t)((item >> 1) & 1), 64);
+      const int a = p.nacc == 2 ? (item & 1) : 0;
+      hk_wait(tfull + a, (uint32_t)((item / p.nacc) & 1), 64);
       tc_fence_after();
       for (int t = 0; t < it.T; ++t) {
         // position of this lane -> output pixel (Eq. 12 / reading R4 / R16)
@@ -764,12 +765,19 @@ HankelTiling hankel_tiling(const Geom& g, int fmt, int num_sms) {
   const int K16 = (g.K + 15) / 16 * 16;
   const int forceT = env_int("POLYCONV_HK_T", 0), forceNN = env_int("POLYCONV_HK_NN", 0);
   const bool no_res = env_int("POLYCONV_HK_STREAM", 0) != 0;
+  const int acc1_mode = env_int("POLYCONV_HK_ACC1", -1);
   const int max_pairs = std::max(1, num_sms / 2);
   const uint32_t fixed = 3072;  // alignment + barriers
   int NN = forceNN ? forceNN : (K16 <= 256 ? K16 : 256);
   bool found = false;
   for (int T = 4; T >= 1 && !found; T >>= 1) {
-    if ((forceT && T != forceT) || T * NN > 256) continue;
+    // T*NN <= 256: two accumulator buffers, the epilogue overlapping the next item's MMAs.
+    // NN = 256 with a streamed filter: T = 2 in one buffer (all 512 TMEM columns) halves the
+    // filter blocks streamed per MAC, worth more than the overlap (256->256 14x14: 731 -> 792
+    // TFLOP/s; VGG 512->512 28x28 N=64: 1139 -> 1306; 512->512 7x7: 635 -> 649; tools/hk_acc1.sh).
+    // POLYCONV_HK_ACC1 = 0 / 1 forces it off / on.
+    const bool acc1 = acc1_mode == 1 || (acc1_mode < 0 && NN == 256);
+    if ((forceT && T != forceT) || T * NN > (acc1 ? 512 : 256)) continue;
     const int NB = (g.K + NN - 1) / NN;
     if ((long long)RS * NB * NN >= (1LL << 31)) break;
     const uint32_t fblk = (uint32_t)(NN / 2) * 128u;
@@ -812,7 +820,8 @@ HankelTiling hankel_tiling(const Geom& g, int fmt, int num_sms) {
                env_int("POLYCONV_HK_GENERAL", 0) == 0) ? 1 : 0;
   t.Kp = t.NB * t.NN;
   t.smem_bytes = (int)((size_t)t.fslots * t.fblk_bytes + (size_t)t.wslots * t.wslot_bytes + fixed);
-  const int tc = 2 * t.T * t.NN;
+  t.nacc = t.T * t.NN > 256 ? 1 : 2;
+  const int tc = t.nacc * t.T * t.NN;
   t.tmem_cols = tc <= 32 ? 32 : tc <= 64 ? 64 : tc <= 128 ? 128 : tc <= 256 ? 256 : 512;
   t.grid = 2 * t.npairs;
   t.ok = true;
@@ -862,6 +871,7 @@ cudaError_t launch_mac_hankel(const Geom& g, const HankelTiling& t, int fmt, con
   const uint32_t ab = tf32 ? 2u : 1u;
   p.idesc = (1u << 4) | (ab << 7) | (ab << 10) | ((uint32_t)(t.NN >> 3) << 17) | ((uint32_t)(256 >> 4) << 24);
   p.tmem_cols = t.tmem_cols;
+  p.nacc = t.nacc;
   p.fpitch.init((uint32_t)t.pitch);
   p.fHS.init((uint32_t)t.HS);
   p.fsh.init((uint32_t)g.sh);

@@ -156,14 +156,15 @@ def test_tc_tiling_choices():
     inf = pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="bf16", kernel="tc_pair").info()
     assert (inf["tile_m"], inf["tile_n"], inf["Cp"], inf["Kp"], inf["launches"]) == (256, 128, 128, 128, 2)
     # TC_HANKEL: pair item = 256*T positions x NN output channels; NN = K (<= 256) else 256,
-    # T*NN <= 256; channels in chunks of 64 (bf16) / 32 (tf32); filter pack + one launch
+    # T*NN <= 256 (two TMEM accumulators), NN = 256 streamed: T = 2 in one accumulator;
+    # channels in chunks of 64 (bf16) / 32 (tf32); filter pack + one launch
     hk = lambda xs, ws, m="bf16": pc.Plan(xs, ws, (1, 1), (1, 1), math=m, kernel="tc_hankel").info()
     inf = hk((256, 64, 56, 56), (64, 64, 3, 3))
     assert (inf["tile_m"], inf["tile_n"], inf["Cp"], inf["Kp"], inf["launches"]) == (1024, 64, 64, 64, 2)
     inf = hk((256, 256, 14, 14), (256, 256, 3, 3))
-    assert (inf["tile_m"], inf["tile_n"], inf["Kp"]) == (256, 256, 256)
+    assert (inf["tile_m"], inf["tile_n"], inf["Kp"]) == (512, 256, 256)
     inf = hk((256, 512, 7, 7), (512, 512, 3, 3))
-    assert (inf["tile_m"], inf["tile_n"], inf["Kp"]) == (256, 256, 512)
+    assert (inf["tile_m"], inf["tile_n"], inf["Kp"]) == (512, 256, 512)
     inf = hk((2, 40, 9, 9), (72, 40, 3, 3), "tf32")
     assert (inf["tile_n"], inf["Cp"], inf["Kp"]) == (80, 64, 80)
     # TC_PAIR needs its separate packing grid (TMA views of x: H*W*elem % 16 == 0); the

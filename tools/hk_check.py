@@ -86,6 +86,12 @@ if which in ("quick", "all"):
     for args in [(2, 64, 14, 14, 128, 3, 3, 1, 1), (2, 80, 13, 11, 48, 3, 3, 1, 1)]:
         run(*args, math="bf16", io="f32", name="quick_f32io")
         run(*args, math="tf32", io="f32", name="quick_tf32")
+if which in ("tail", "all"):
+    # unit counts just past a multiple of the pair count: tail units split into sub-units
+    for args in [(40, 128, 28, 28, 128, 3, 3, 1, 1), (100, 256, 14, 14, 256, 3, 3, 1, 1),
+                 (90, 512, 7, 7, 512, 3, 3, 1, 1), (70, 64, 28, 28, 96, 3, 3, 1, 1), (33, 96, 20, 21, 192, 3, 3, 1, 1)]:
+        run(*args, name="tail")
+        run(*args, math="tf32", io="f32", name="tail_tf32")
 if which in ("gate", "all"):
     for args, nm in [((32, 128, 28, 28, 128, 3, 3, 1, 1), "conv3x_n32"), ((256, 64, 56, 56, 64, 3, 3, 1, 1), "l1_3x3_64"),
                      ((256, 128, 28, 28, 128, 3, 3, 1, 1), "l2_3x3_128"), ((256, 256, 14, 14, 256, 3, 3, 1, 1), "l3_3x3_256"),
