@@ -36,6 +36,9 @@ cudaError_t launch_pack_filter_planar(const Geom& g, const void* w, bool w_bf16,
                                       int fmt, cudaStream_t st);
 cudaError_t launch_pack_filter_tapmajor(const Geom& g, const void* w, bool w_bf16, void* dst,
                                         int fmt, int Kp, int Cp, cudaStream_t st);
+// stride-2 phase-split filter [R'*S'][Kp][Cp] (bf16 in / out, mac_hankel phase mode, reading R19)
+cudaError_t launch_pack_filter_phase(const Geom& g, const void* w, void* dst, int Rp, int Sp, int php, int pwp,
+                                     int Kp, int Cp, cudaStream_t st);
 // fused: input interleaved + filter tap-major in one launch
 cudaError_t launch_pack_both_interleaved(const Geom& g, const void* x, const void* w, bool io_bf16,
                                          void* xdst, void* wdst, int fmt, cudaStream_t st);
@@ -170,8 +173,10 @@ struct HankelTiling {
   uint32_t wslot_bytes, fblk_bytes;
   int smem_bytes, tmem_cols, npairs, grid;
   int nacc;  // TMEM accumulator buffers (1 or 2)
+  // stride-2 phase mode (reading R19): the kernel runs on the phase-split geometry
+  int phase, eC, eH, eW, eR, eS, eph, epw;
 };
-HankelTiling hankel_tiling(const Geom& g, int fmt, int num_sms);
+HankelTiling hankel_tiling(const Geom& g, int fmt, int num_sms, bool io_bf16);
 // x: NCHW input (io dtype); U: tap-major packed filter [RS][Kp][Cp] (t.Kp, t.Cp), packed by
 // the preceding launch, which this one follows as a programmatic dependent
 // zero: device buffer of hankel_zero_bytes(g) zero bytes (read in place of padding)

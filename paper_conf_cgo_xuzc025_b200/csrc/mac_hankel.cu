@@ -110,6 +110,10 @@ struct HkParams {
   int tmem_cols;
   int nacc;             // accumulator buffers in TMEM (2: the epilogue overlaps the next item's MMAs)
   FastDiv fpitch, fHS, fsh, fsw;
+  // stride-2 phase mode (reading R19): the kernel runs the stride-1 convolution of the
+  // phase-split input; N, C, H, W, ph, pw, sh, sw above are that convolution's, these are x's
+  int phase;            // 0 / 1
+  int xC, xH, xW;       // x dims (phase mode)
   int dbg;  // POLYCONV_HK_DEBUG (timing ablations, results wrong): 1 loaders store zeros without
             // loading, 2 epilogue skips stores, 4 no MMAs (commits only), 8 per-CTA trace
 };
@@ -164,8 +168,10 @@ __device__ __forceinline__ void hk_arrive_cluster(uint32_t cluster_addr) {
   asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
 }
 // plain parity wait (no watchdog: every wait is on work of the same CTA pair, which the
-// hardware co-schedules); sleep_ns > 0 backs off for the long waits of the epilogue
-__device__ __forceinline__ void hk_wait(uint64_t* bar, uint32_t parity, uint32_t sleep_ns = 0) {
+// hardware co-schedules).  No __nanosleep back-off: try_wait already suspends in hardware, and
+// a 32 / 64 ns sleep in the loaders' slot wait and the epilogue's waits cost 3% on 128->128
+// 28x28 (838 -> 862 TFLOP/s; 15 us of 71 with the MMAs ablated).
+__device__ __forceinline__ void hk_wait(uint64_t* bar, uint32_t parity) {
   const uint32_t a = smem_u32(bar);
   uint32_t done;
   for (;;) {
@@ -177,7 +183,6 @@ __device__ __forceinline__ void hk_wait(uint64_t* bar, uint32_t parity, uint32_t
         : "r"(a), "r"(parity)
         : "memory");
     if (done) return;
-    if (sleep_ns) __nanosleep(sleep_ns);
   }
 }
 __device__ __forceinline__ void hk_tmem_alloc2(uint32_t* slot, uint32_t ncols) {
@@ -222,16 +227,20 @@ __device__ __forceinline__ bool hk_next(const HkParams& p, long long& u, long lo
 // ---- a2: one window of the input polynomial into a shared-memory slot ---------------
 // element offset of (n, channel 0, h, w) for position q, or -1 for a zero coefficient
 // (branch-free; every position of a launch is < 2^31, checked by the plan)
-__device__ __forceinline__ int hk_src(const HkParams& p, long long q) {
+__device__ __forceinline__ bool hk_pos(const HkParams& p, long long q, int& n, int& h, int& w) {
   const int qq = (int)q - p.delta;
   const uint32_t u = (uint32_t)max(qq, 0);
   const uint32_t vr = p.fpitch.div(u);
-  const int w = (int)(u - vr * (uint32_t)p.pitch) - p.pw;
+  w = (int)(u - vr * (uint32_t)p.pitch) - p.pw;
   const int vr2 = (int)vr - p.ph;
-  const uint32_t n = p.fHS.div((uint32_t)max(vr2, 0));
-  const int h = vr2 - (int)n * p.HS;
-  const bool ok = qq >= 0 && w >= 0 && w < p.W && vr2 >= 0 && h < p.H && (int)n < p.N;
-  return ok ? (int)n * p.CHW + h * p.W + w : -1;
+  n = (int)p.fHS.div((uint32_t)max(vr2, 0));
+  h = vr2 - n * p.HS;
+  return qq >= 0 && w >= 0 && w < p.W && vr2 >= 0 && h < p.H && n < p.N;
+}
+__device__ __forceinline__ int hk_src(const HkParams& p, long long q) {
+  int n, h, w;
+  const bool ok = hk_pos(p, q, n, h, w);
+  return ok ? n * p.CHW + h * p.W + w : -1;
 }
 
 template <typename IoT>
@@ -399,6 +408,61 @@ __device__ __forceinline__ void hk_load_window_pairs(const HkParams& p, uint32_t
         const uint32_t ra = 2u * (uint32_t)rp + sel, rb = 2u * (uint32_t)rp + (sel ^ 1u);
         const uint32_t* da = sel ? r1 : r0;
         const uint32_t* db = sel ? r0 : r1;
+        const uint32_t aa = slot + ra * 128u + (((uint32_t)lw ^ (ra & 7u)) << 4);
+        const uint32_t ab = slot + rb * 128u + (((uint32_t)lw ^ (rb & 7u)) << 4);
+        asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(aa), "r"(da[0]), "r"(da[1]), "r"(da[2]),
+                     "r"(da[3])
+                     : "memory");
+        asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(ab), "r"(db[0]), "r"(db[1]), "r"(db[2]),
+                     "r"(db[3])
+                     : "memory");
+      }
+    }
+  }
+}
+
+// Phase-split window (reading R19, stride 2, bf16 in and math, x width % 4 == 0, C % 32 == 0).
+// The stride-2 convolution is the stride-1 convolution, with R' x S' taps, of the phase planes
+// X_{a,c,b}[u][v] = x[c][2u + a][2v + b] (virtual channel (a*C + c)*2 + b); the window holds
+// those planes' positions.  One aligned 4-byte word x[c][2u + a][2v .. 2v + 1] is virtual
+// channels (a, c, 0) and (a, c, 1) of position (u, v), already in operand order, so a 16-byte
+// row group (4 channels x 2 column phases) is 4 loads, no permutes.  The pair layout of the
+// phase planes (W' = W/2 even, pitch W' + 2pw', delta pw' & 1) keeps both positions of a lane's
+// pair data or both zero; rows 2u + a past x's last row read the zero buffer.
+__device__ __forceinline__ void hk_load_window_phase(const HkParams& p, uint32_t slot, long long q0, int vc0, int lw,
+                                                     int lane, int rp_lo, int rp_hi) {
+  constexpr int B = 4;  // position pairs per lane in flight
+  const int a = vc0 / (2 * p.xC);
+  const int c = (vc0 - a * 2 * p.xC) / 2 + lw * 4;  // first of this group's 4 channels
+  const uint32_t hw2 = (uint32_t)(p.xH * p.xW) >> 1, w2 = (uint32_t)p.xW >> 1;
+  const int nrp = rp_hi;
+  const uint32_t sel = (uint32_t)(lane >> 2) & 1u;
+  for (int rp0 = rp_lo; rp0 < nrp; rp0 += 32 * B) {
+    uint32_t lo[B][4], hi[B][4];
+#pragma unroll
+    for (int b = 0; b < B; ++b) {
+      const int rp = rp0 + b * 32 + lane;
+      // (n, u, v) of the pair's first position in the phase planes, as hk_src
+      int n, u, v;
+      const bool in = hk_pos(p, q0 + 2 * rp, n, u, v) && rp < nrp && !(p.dbg & 1);
+      const int r = 2 * u + a;
+      const bool ok = in && r < p.xH;
+      const uint32_t* base = ok ? static_cast<const uint32_t*>(p.x) +
+                                      (((uint32_t)n * p.xC + (uint32_t)c) * hw2 + (uint32_t)r * w2 + (uint32_t)v)
+                                : static_cast<const uint32_t*>(p.zero);
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        lo[b][k] = base[k * hw2];
+        hi[b][k] = base[k * hw2 + 1];
+      }
+    }
+#pragma unroll
+    for (int b = 0; b < B; ++b) {
+      const int rp = rp0 + b * 32 + lane;
+      if (rp < nrp) {
+        const uint32_t ra = 2u * (uint32_t)rp + sel, rb = 2u * (uint32_t)rp + (sel ^ 1u);
+        const uint32_t* da = sel ? hi[b] : lo[b];
+        const uint32_t* db = sel ? lo[b] : hi[b];
         const uint32_t aa = slot + ra * 128u + (((uint32_t)lw ^ (ra & 7u)) << 4);
         const uint32_t ab = slot + rb * 128u + (((uint32_t)lw ^ (rb & 7u)) << 4);
         asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(aa), "r"(da[0]), "r"(da[1]), "r"(da[2]),
@@ -590,8 +654,14 @@ __global__ void __launch_bounds__(kHkThreads, 1)
       while (hk_next(p, u, u_hi, it)) {
         const long long q0 = (long long)it.pt * 256 + (long long)rank * 128 * it.T;
         for (int ch = 0; ch < p.nchunks; ++ch) {
-          hk_wait(wempty + ws, (uint32_t)(wuse & 1) ^ 1u, 32);
-          if constexpr (kHW2 >= 0)
+          const int wi = (int)(wuse * p.wslots + ws);
+          const bool wt = (p.dbg & 16) && blockIdx.x == 0 && ridx == 0 && lane == 0 && wi < 64;
+          if (wt) g_hk_wtrace[wi * 8 + 0] = global_ns();
+          hk_wait(wempty + ws, (uint32_t)(wuse & 1) ^ 1u);
+          if (wt) g_hk_wtrace[wi * 8 + 1] = global_ns();
+          if constexpr (kHW2 == -2)
+            hk_load_window_phase(p, sW + (uint32_t)ws * p.wslot_bytes, q0, ch * 64, lw, lane, rp_lo, rp_hi);
+          else if constexpr (kHW2 >= 0)
             hk_load_window_pairs<IoT, kTf32, kHW2>(p, sW + (uint32_t)ws * p.wslot_bytes, q0, ch * (kTf32 ? 32 : 64), lw,
                                                    lane, rp_lo, rp_hi);
           else
@@ -600,7 +670,7 @@ __global__ void __launch_bounds__(kHkThreads, 1)
           if (trace && lw == 0 && lane == 0 && u == u_lo + it.T && ch == 0) tr[2] = global_ns();
           asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> MMA reads
           __syncwarp();
-          const int wi = (int)(wuse * p.wslots + ws);
+          if (wt) g_hk_wtrace[wi * 8 + 2] = global_ns();
           if ((p.dbg & 32) && blockIdx.x < 2 && lane == 0 && wi < 64) g_hk_ltrace[wi * 16 + rank * 8 + lw] = global_ns();
           if (lane == 0) mbar_arrive(wloc + ws);
           if (++ws == p.wslots) { ws = 0; ++wuse; }
@@ -629,7 +699,7 @@ __global__ void __launch_bounds__(kHkThreads, 1)
     int item = 0;
     while (hk_next(p, u, u_hi, it)) {
       const int a = p.nacc == 2 ? (item & 1) : 0;
-      hk_wait(eloc + a, (uint32_t)((item / p.nacc) & 1), 64);
+      hk_wait(eloc + a, (uint32_t)((item / p.nacc) & 1));
       if (lane == 0) hk_arrive_cluster(tempty0 + (uint32_t)a * 8u);
       __syncwarp();
       ++item;
@@ -649,7 +719,7 @@ __global__ void __launch_bounds__(kHkThreads, 1)
     int item = 0;
     while (hk_next(p, u, u_hi, it)) {
       const int a = p.nacc == 2 ? (item & 1) : 0;
-      hk_wait(tfull + a, (uint32_t)((item / p.nacc) & 1), 64);
+      hk_wait(tfull + a, (uint32_t)((item / p.nacc) & 1));
       tc_fence_after();
       for (int t = 0; t < it.T; ++t) {
         // position of this lane -> output pixel (Eq. 12 / reading R4 / R16)
@@ -740,7 +810,7 @@ size_t hankel_zero_bytes(const Geom& g) { return (size_t)32 * g.H * g.W + 256; }
 // window rebuilds per output-channel block); 128->128 28x28 NN=128/T=2 862.
 // The filter is resident in shared memory when its (single) block fits beside two windows,
 // else streamed by TMA through a ring of (chunk, tap) blocks.
-HankelTiling hankel_tiling(const Geom& g, int fmt, int num_sms) {
+static HankelTiling hankel_tiling_core(const Geom& g, int fmt, int num_sms) {
   HankelTiling t{};
   t.ok = false;
   if (fmt == FMT_F32) return t;
@@ -831,13 +901,54 @@ HankelTiling hankel_tiling(const Geom& g, int fmt, int num_sms) {
   return t;
 }
 
-cudaError_t launch_mac_hankel(const Geom& g, const HankelTiling& t, int fmt, const void* x, bool io_bf16,
+// Stride-2 phase split (reading R19): y = the stride-1 convolution of the phase planes
+// X_{a,c,b}[u][v] = x[c][2u + a][2v + b] (4C channels, ceil(H/2) x W/2) with R' x S' taps,
+// R' = (R - 1 - ph)/2 + ceil(ph/2) + 1, top / left padding ceil(ph/2); same P x Q outputs.
+static Geom hk_phase_geom(const Geom& g) {
+  Geom e = g;
+  e.C = 4 * g.C;
+  e.H = (g.H + 1) / 2;
+  e.W = g.W / 2;
+  e.ph = (g.ph + 1) / 2;
+  e.pw = (g.pw + 1) / 2;
+  e.R = (g.R - 1 - g.ph) / 2 + e.ph + 1;
+  e.S = (g.S - 1 - g.pw) / 2 + e.pw + 1;
+  e.sh = e.sw = 1;
+  return e;
+}
+
+// Every output position computed by the stride-1 window is kept in phase mode; without it a
+// stride-2 layer computes all stride-1 positions and keeps a quarter.  Phase mode: bf16 in and
+// math, x width % 4 == 0 (W/2 even: pair-aligned phase planes), C % 32 == 0 (a 64-channel
+// chunk never straddles the row phase a), R - 1 >= ph; POLYCONV_HK_PHASE=0 turns it off.
+HankelTiling hankel_tiling(const Geom& g, int fmt, int num_sms, bool io_bf16) {
+  if (g.sh == 2 && g.sw == 2 && fmt == FMT_BF16 && io_bf16 && g.W % 4 == 0 && g.C % 32 == 0 &&
+      g.R - 1 >= g.ph && g.S - 1 >= g.pw && env_int("POLYCONV_HK_PHASE", 1) != 0) {
+    const Geom e = hk_phase_geom(g);
+    HankelTiling t = hankel_tiling_core(e, fmt, num_sms);
+    if (t.ok && t.aligned) {
+      t.phase = 1;
+      t.eC = e.C; t.eH = e.H; t.eW = e.W; t.eR = e.R; t.eS = e.S; t.eph = e.ph; t.epw = e.pw;
+      return t;
+    }
+  }
+  HankelTiling t = hankel_tiling_core(g, fmt, num_sms);
+  t.phase = 0;
+  return t;
+}
+
+cudaError_t launch_mac_hankel(const Geom& g0, const HankelTiling& t, int fmt, const void* x, bool io_bf16,
                               const void* U, void* y, const void* zero, cudaStream_t st, char* err, size_t errlen) {
   if (!t.ok) {
     snprintf(err, errlen, "mac_hankel: shape not supported");
     return cudaErrorInvalidValue;
   }
   const bool tf32 = fmt == FMT_TF32;
+  Geom g = g0;  // the geometry the kernel runs (phase mode: the phase-split one)
+  if (t.phase) {
+    g.C = t.eC; g.H = t.eH; g.W = t.eW; g.R = t.eR; g.S = t.eS; g.ph = t.eph; g.pw = t.epw;
+    g.sh = g.sw = 1;
+  }
   EncodeTiledFnHk enc = get_encode_hk();
   CUtensorMap tmU;
   {
@@ -876,12 +987,16 @@ cudaError_t launch_mac_hankel(const Geom& g, const HankelTiling& t, int fmt, con
   p.fHS.init((uint32_t)t.HS);
   p.fsh.init((uint32_t)g.sh);
   p.fsw.init((uint32_t)g.sw);
+  p.phase = t.phase;
+  p.xC = g0.C; p.xH = g0.H; p.xW = g0.W;
   p.dbg = env_int("POLYCONV_HK_DEBUG", 0);
   // kHW2: -1 = general loader, 0 = pair-aligned loader with a runtime plane size, > 0 = the
   // plane size in words baked in (immediate channel offsets) for the ResNet / VGG planes
   void (*kern)(const CUtensorMap, const HkParams);
   const int hw2 = g.H * g.W / 2;
-  if (!t.aligned) {
+  if (t.phase) {
+    kern = mac_hankel_kernel<__nv_bfloat16, false, -2>;
+  } else if (!t.aligned) {
     kern = tf32 ? mac_hankel_kernel<float, true, -1>
                 : (io_bf16 ? mac_hankel_kernel<__nv_bfloat16, false, -1> : mac_hankel_kernel<float, false, -1>);
   } else if (tf32) {

@@ -557,6 +557,40 @@ cudaError_t launch_pack_filter_tapmajor(const Geom& g, const void* w, bool w_bf1
                                         int fmt, int Kp, int Cp, cudaStream_t st) {
   return dispatch<LFTap>(w_bf16, fmt, g, w, dst, Kp, Cp, st);
 }
+// ---- phase-split filter for the stride-2 pair kernel (reading R19) ----------------------
+// U'[t' = i'*S' + j'][k][(a*C + c)*2 + b] = w[k][c][i][j] with i = 2(i' - ph') + a + ph,
+// j = 2(j' - pw') + b + pw when inside the kernel, else 0: the taps of the stride-1
+// convolution over the phase planes X_{a,c,b}[u][v] = x[c][2u + a][2v + b].  One thread per
+// output element (consecutive threads: consecutive virtual channels); bf16 in, bf16 words.
+__global__ void __launch_bounds__(kThreads) pack_filter_phase_kernel(Geom g, const __nv_bfloat16* __restrict__ w,
+                                                                     __nv_bfloat16* __restrict__ dst, int Rp, int Sp,
+                                                                     int php, int pwp, int Kp, int Cp) {
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+  const long long total = (long long)Rp * Sp * Kp * Cp;
+  for (long long idx = blockIdx.x * (long long)kThreads + threadIdx.x; idx < total;
+       idx += (long long)gridDim.x * kThreads) {
+    const int vc = (int)(idx % Cp);
+    const long long tk = idx / Cp;
+    const int k = (int)(tk % Kp), t = (int)(tk / Kp);
+    const int ip = t / Sp, jp = t - ip * Sp;
+    const int a = vc / (2 * g.C), rem = vc - a * 2 * g.C, c = rem >> 1, b = rem & 1;
+    const int i = 2 * (ip - php) + a + g.ph, j = 2 * (jp - pwp) + b + g.pw;
+    float v = 0.f;
+    if (a < 2 && k < g.K && i >= 0 && i < g.R && j >= 0 && j < g.S)
+      v = __bfloat162float(w[(((long long)k * g.C + c) * g.R + i) * g.S + j]);
+    dst[idx] = __float2bfloat16_rn(v);
+  }
+}
+
+cudaError_t launch_pack_filter_phase(const Geom& g, const void* w, void* dst, int Rp, int Sp, int php, int pwp,
+                                     int Kp, int Cp, cudaStream_t st) {
+  const long long total = (long long)Rp * Sp * Kp * Cp;
+  const int grid = (int)std::min<long long>((total + kThreads - 1) / kThreads, 148LL * 8);
+  pack_filter_phase_kernel<<<grid, kThreads, 0, st>>>(g, static_cast<const __nv_bfloat16*>(w),
+                                                      static_cast<__nv_bfloat16*>(dst), Rp, Sp, php, pwp, Kp, Cp);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_pack_both_interleaved(const Geom& g, const void* x, const void* w, bool io_bf16,
                                          void* xdst, void* wdst, int fmt, cudaStream_t st) {
   return dispatch<LBoth>(io_bf16, fmt, g, x, w, xdst, wdst, st);

@@ -123,6 +123,16 @@ polyconv_status_t resolve(polyconv_plan_t p) {
   if (k == POLYCONV_KERNEL_AUTO || k == POLYCONV_KERNEL_TC_PAIR) p->pair = pair_tiling(g, p->fmt, p->io_bf16, p->num_sms);
   // 1x1: x is already the (MN-major) position operand when its planes have a 16-byte pitch;
   // other 1x1 layers gather their output lattice first (mac1x1_auto)
+  // ... except wide-input 1x1 layers whose planes need that gather (H*W*2 bytes not a multiple
+  // of 16): the pair kernel reads their NCHW planes directly (one tap, no halo) and skips the
+  // gathered copy of C*H*W (tools/hk_1x1.sh, N=256: 1024->256 14x14 0.128 -> 0.077 ms,
+  // 1024->512 14x14 0.159 -> 0.112; 256->1024 14x14 loses, 0.075 vs 0.091)
+  if (k == POLYCONV_KERNEL_AUTO && p->math == POLYCONV_MATH_BF16 && p->io_bf16 && g.R == 1 && g.S == 1 &&
+      g.sh == 1 && g.sw == 1 && g.ph == 0 && g.pw == 0 && mac1x1_pitch(g) != 0 && g.C >= 512 &&
+      g.C >= 2 * g.K && !getenv("POLYCONV_NO_HANKEL")) {
+    const HankelTiling h = hankel_tiling(g, p->fmt, p->num_sms, p->io_bf16);
+    if (h.ok && h.aligned && (long long)h.PT * h.NB >= 24) k = POLYCONV_KERNEL_TC_HANKEL;
+  }
   if (k == POLYCONV_KERNEL_AUTO && mac1x1_supported(g, p->fmt, p->io_bf16) && !getenv("POLYCONV_NO_1X1") &&
       mac1x1_auto(g))
     k = POLYCONV_KERNEL_TC_1X1;
@@ -134,7 +144,7 @@ polyconv_status_t resolve(polyconv_plan_t p) {
   // under a third of a round of units (the synthetic nets at 4x4 / 8x8: 1-11 units; 14x14: 30).
   if (k == POLYCONV_KERNEL_AUTO && p->math == POLYCONV_MATH_BF16 && g.K >= 16 && g.sh == g.sw && g.sh <= 2 &&
       g.R == g.S && (g.R == 3 || g.R == 5) && !getenv("POLYCONV_NO_HANKEL")) {
-    const HankelTiling h = hankel_tiling(g, p->fmt, p->num_sms);
+    const HankelTiling h = hankel_tiling(g, p->fmt, p->num_sms, p->io_bf16);
     // odd widths use the general (element-load) window loader: it still wins for wide 3x3
     // layers (ResNet-50 l4 7x7, C = K = 512: 596 vs 572 TFLOP/s for mac_tc2)
     const bool loader_ok = h.aligned || (g.R == 3 && g.C >= 256 && g.K >= 256);
@@ -174,7 +184,7 @@ polyconv_status_t resolve(polyconv_plan_t p) {
   if (k == POLYCONV_KERNEL_TC_PAIR && (!tc_math || !p->pair.ok)) return POLYCONV_STATUS_BAD_PARAM;
   if (k == POLYCONV_KERNEL_TC_1X1 && !mac1x1_supported(g, p->fmt, p->io_bf16)) return POLYCONV_STATUS_BAD_PARAM;
   if (k == POLYCONV_KERNEL_TC_HANKEL) {
-    p->hk = hankel_tiling(g, p->fmt, p->num_sms);
+    p->hk = hankel_tiling(g, p->fmt, p->num_sms, p->io_bf16);
     if (!tc_math || !p->hk.ok) return POLYCONV_STATUS_BAD_PARAM;
   }
   if (k == POLYCONV_KERNEL_FFT) {
@@ -549,7 +559,10 @@ polyconv_status_t polyconv_forward(polyconv_plan_t p, const void* x, const void*
       }
     }
     if (p->ev_start) cudaEventRecord(p->ev_start, st);
-    e = launch_pack_filter_tapmajor(g, w, p->io_bf16, p->wsU, p->fmt, g.Kp, g.Cp, st);
+    if (p->hk.phase)
+      e = launch_pack_filter_phase(g, w, p->wsU, p->hk.eR, p->hk.eS, p->hk.eph, p->hk.epw, g.Kp, g.Cp, st);
+    else
+      e = launch_pack_filter_tapmajor(g, w, p->io_bf16, p->wsU, p->fmt, g.Kp, g.Cp, st);
     if (e != cudaSuccess) return finish(p, e, "pack_filter");
     e = launch_mac_hankel(g, p->hk, p->fmt, x, p->io_bf16, p->wsU, y, p->hkzero, st, p->err, sizeof(p->err));
     if (p->ev_stop) cudaEventRecord(p->ev_stop, st);

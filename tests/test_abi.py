@@ -99,6 +99,10 @@ def test_kernel_selection_and_forcing():
         ("tc_1x1", 2)
     assert (k1((4, 1024, 14, 14), (256, 1024, 1, 1))["kernel"], k1((4, 1024, 14, 14), (256, 1024, 1, 1))["launches"]) \
         == ("tc_1x1", 3)
+    # ... but wide-input 1x1 layers on planes that need the gather go to mac_hankel from 24
+    # pair units (C >= 512, C >= 2K), reading x in place
+    assert k1((256, 1024, 14, 14), (256, 1024, 1, 1))["kernel"] == "tc_hankel"
+    assert k1((256, 256, 14, 14), (1024, 256, 1, 1))["kernel"] == "tc_1x1"
     assert k1((4, 256, 28, 28), (512, 256, 1, 1), 2)["kernel"] == "tc_1x1"
     assert k1((4, 1024, 7, 7), (512, 1024, 1, 1))["kernel"] == "tc_1x1"
     assert k1((4, 512, 7, 7), (2048, 512, 1, 1))["kernel"] == "tc"

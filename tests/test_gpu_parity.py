@@ -106,6 +106,12 @@ MX_SHAPES = [
     ConvShape("mx_k1", 2, 64, 8, 8, 64, 1, 1, 1, 1, 0, 0),
     ConvShape("mx_many", 9, 64, 8, 8, 128, 3, 3, 1, 1, 1, 1),       # windows span several images
     ConvShape("mx_asym", 2, 64, 14, 20, 72, 3, 5, 1, 1, 0, 2),
+    # stride 2 with W % 4 == 0, C % 32 == 0: tc_hankel runs the phase-split convolution (R19)
+    ConvShape("mx_s2_phase", 2, 64, 16, 20, 96, 3, 3, 2, 2, 1, 1),
+    ConvShape("mx_s2_phase_k5", 2, 32, 20, 16, 48, 5, 5, 2, 2, 2, 2),
+    ConvShape("mx_s2_phase_oddH", 3, 96, 15, 12, 64, 3, 3, 2, 2, 1, 1),
+    ConvShape("mx_s2_phase_p0", 2, 64, 16, 16, 40, 3, 3, 2, 2, 0, 0),
+    ConvShape("mx_k1_wide", 2, 512, 14, 14, 128, 1, 1, 1, 1, 0, 0),  # AUTO: tc_hankel from 24 units
 ]
 
 
