@@ -426,9 +426,9 @@ __device__ __forceinline__ void hk_load_window_pairs(const HkParams& p, uint32_t
 // X_{a,c,b}[u][v] = x[c][2u + a][2v + b] (virtual channel (a*C + c)*2 + b); the window holds
 // those planes' positions.  One aligned 4-byte word x[c][2u + a][2v .. 2v + 1] is virtual
 // channels (a, c, 0) and (a, c, 1) of position (u, v), already in operand order, so a 16-byte
-// row group (4 channels x 2 column phases) is 4 loads, no permutes.  The pair layout of the
-// phase planes (W' = W/2 even, pitch W' + 2pw', delta pw' & 1) keeps both positions of a lane's
-// pair data or both zero; rows 2u + a past x's last row read the zero buffer.
+// row group (4 channels x 2 column phases) is 4 loads, no permutes.  Each position of a lane's
+// pair is decoded on its own (any W' = W/2); rows 2u + a past x's last row read the zero buffer.
+template <bool kAligned>
 __device__ __forceinline__ void hk_load_window_phase(const HkParams& p, uint32_t slot, long long q0, int vc0, int lw,
                                                      int lane, int rp_lo, int rp_hi) {
   constexpr int B = 4;  // position pairs per lane in flight
@@ -443,17 +443,23 @@ __device__ __forceinline__ void hk_load_window_phase(const HkParams& p, uint32_t
     for (int b = 0; b < B; ++b) {
       const int rp = rp0 + b * 32 + lane;
       // (n, u, v) of the pair's first position in the phase planes, as hk_src
-      int n, u, v;
-      const bool in = hk_pos(p, q0 + 2 * rp, n, u, v) && rp < nrp && !(p.dbg & 1);
-      const int r = 2 * u + a;
-      const bool ok = in && r < p.xH;
-      const uint32_t* base = ok ? static_cast<const uint32_t*>(p.x) +
-                                      (((uint32_t)n * p.xC + (uint32_t)c) * hw2 + (uint32_t)r * w2 + (uint32_t)v)
-                                : static_cast<const uint32_t*>(p.zero);
+      // kAligned (W' even, pitch W' + 2pw', delta pw' & 1): both positions of a pair are data of
+      // one row or both zero, one decode; else each position is decoded on its own
+      const uint32_t* base[2];
+#pragma unroll
+      for (int s2 = 0; s2 < (kAligned ? 1 : 2); ++s2) {
+        int n, u, v;
+        const bool in = hk_pos(p, q0 + 2 * rp + s2, n, u, v) && rp < nrp && !(p.dbg & 1);
+        const int r = 2 * u + a;
+        base[s2] = (in && r < p.xH) ? static_cast<const uint32_t*>(p.x) +
+                                          (((uint32_t)n * p.xC + (uint32_t)c) * hw2 + (uint32_t)r * w2 + (uint32_t)v)
+                                    : static_cast<const uint32_t*>(p.zero);
+      }
+      if (kAligned) base[1] = base[0] + 1;
 #pragma unroll
       for (int k = 0; k < 4; ++k) {
-        lo[b][k] = base[k * hw2];
-        hi[b][k] = base[k * hw2 + 1];
+        lo[b][k] = base[0][k * hw2];
+        hi[b][k] = base[1][k * hw2];
       }
     }
 #pragma unroll
@@ -659,8 +665,9 @@ __global__ void __launch_bounds__(kHkThreads, 1)
           if (wt) g_hk_wtrace[wi * 8 + 0] = global_ns();
           hk_wait(wempty + ws, (uint32_t)(wuse & 1) ^ 1u);
           if (wt) g_hk_wtrace[wi * 8 + 1] = global_ns();
-          if constexpr (kHW2 == -2)
-            hk_load_window_phase(p, sW + (uint32_t)ws * p.wslot_bytes, q0, ch * 64, lw, lane, rp_lo, rp_hi);
+          if constexpr (kHW2 == -2 || kHW2 == -4)
+            hk_load_window_phase<kHW2 == -2>(p, sW + (uint32_t)ws * p.wslot_bytes, q0, ch * 64, lw, lane, rp_lo,
+                                             rp_hi);
           else if constexpr (kHW2 >= 0)
             hk_load_window_pairs<IoT, kTf32, kHW2>(p, sW + (uint32_t)ws * p.wslot_bytes, q0, ch * (kTf32 ? 32 : 64), lw,
                                                    lane, rp_lo, rp_hi);
@@ -919,14 +926,14 @@ static Geom hk_phase_geom(const Geom& g) {
 
 // Every output position computed by the stride-1 window is kept in phase mode; without it a
 // stride-2 layer computes all stride-1 positions and keeps a quarter.  Phase mode: bf16 in and
-// math, x width % 4 == 0 (W/2 even: pair-aligned phase planes), C % 32 == 0 (a 64-channel
-// chunk never straddles the row phase a), R - 1 >= ph; POLYCONV_HK_PHASE=0 turns it off.
+// math, even x width (x[2v], x[2v+1] one aligned word), C % 32 == 0 (a 64-channel chunk never
+// straddles the row phase a), R - 1 >= ph; POLYCONV_HK_PHASE=0 turns it off.
 HankelTiling hankel_tiling(const Geom& g, int fmt, int num_sms, bool io_bf16) {
-  if (g.sh == 2 && g.sw == 2 && fmt == FMT_BF16 && io_bf16 && g.W % 4 == 0 && g.C % 32 == 0 &&
+  if (g.sh == 2 && g.sw == 2 && fmt == FMT_BF16 && io_bf16 && g.W % 2 == 0 && g.C % 32 == 0 &&
       g.R - 1 >= g.ph && g.S - 1 >= g.pw && env_int("POLYCONV_HK_PHASE", 1) != 0) {
     const Geom e = hk_phase_geom(g);
     HankelTiling t = hankel_tiling_core(e, fmt, num_sms);
-    if (t.ok && t.aligned) {
+    if (t.ok) {
       t.phase = 1;
       t.eC = e.C; t.eH = e.H; t.eW = e.W; t.eR = e.R; t.eS = e.S; t.eph = e.ph; t.epw = e.pw;
       return t;
@@ -995,7 +1002,7 @@ cudaError_t launch_mac_hankel(const Geom& g0, const HankelTiling& t, int fmt, co
   void (*kern)(const CUtensorMap, const HkParams);
   const int hw2 = g.H * g.W / 2;
   if (t.phase) {
-    kern = mac_hankel_kernel<__nv_bfloat16, false, -2>;
+    kern = t.aligned ? mac_hankel_kernel<__nv_bfloat16, false, -2> : mac_hankel_kernel<__nv_bfloat16, false, -4>;
   } else if (!t.aligned) {
     kern = tf32 ? mac_hankel_kernel<float, true, -1>
                 : (io_bf16 ? mac_hankel_kernel<__nv_bfloat16, false, -1> : mac_hankel_kernel<float, false, -1>);

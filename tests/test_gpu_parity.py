@@ -111,6 +111,7 @@ MX_SHAPES = [
     ConvShape("mx_s2_phase_k5", 2, 32, 20, 16, 48, 5, 5, 2, 2, 2, 2),
     ConvShape("mx_s2_phase_oddH", 3, 96, 15, 12, 64, 3, 3, 2, 2, 1, 1),
     ConvShape("mx_s2_phase_p0", 2, 64, 16, 16, 40, 3, 3, 2, 2, 0, 0),
+    ConvShape("mx_s2_phase_w14", 3, 64, 14, 14, 96, 3, 3, 2, 2, 1, 1),   # W/2 odd: per-position decode
     ConvShape("mx_k1_wide", 2, 512, 14, 14, 128, 1, 1, 1, 1, 0, 0),  # AUTO: tc_hankel from 24 units
 ]
 

@@ -96,9 +96,11 @@ if which in ("s2", "all"):
     # stride 2: phase-split mode (reading R19) where W % 4 == 0 and C % 32 == 0
     for args in [(2, 64, 16, 16, 64, 3, 3, 2, 1), (3, 128, 56, 56, 128, 3, 3, 2, 1), (2, 256, 28, 28, 256, 3, 3, 2, 1),
                  (2, 32, 12, 20, 48, 3, 3, 2, 1), (2, 64, 24, 24, 64, 5, 5, 2, 2), (2, 64, 15, 16, 64, 3, 3, 2, 1),
-                 (2, 64, 16, 16, 64, 3, 3, 2, 0), (40, 128, 56, 56, 128, 3, 3, 2, 1), (2, 96, 20, 12, 80, 5, 5, 2, 1)]:
+                 (2, 64, 16, 16, 64, 3, 3, 2, 0), (40, 128, 56, 56, 128, 3, 3, 2, 1), (2, 96, 20, 12, 80, 5, 5, 2, 1),
+                 (3, 64, 14, 14, 96, 3, 3, 2, 1), (2, 32, 10, 18, 64, 5, 5, 2, 2), (20, 512, 14, 14, 512, 3, 3, 2, 1)]:
         run(*args, name="s2")
-    for args, nm in [((256, 128, 56, 56, 128, 3, 3, 2, 1), "l2_3x3_128_s2"), ((256, 256, 28, 28, 256, 3, 3, 2, 1), "l3_3x3_256_s2")]:
+    for args, nm in [((256, 128, 56, 56, 128, 3, 3, 2, 1), "l2_3x3_128_s2"), ((256, 256, 28, 28, 256, 3, 3, 2, 1), "l3_3x3_256_s2"),
+                     ((256, 512, 14, 14, 512, 3, 3, 2, 1), "l4_3x3_512_s2")]:
         run(*args, time_it=True, name=nm)
 if which in ("gate", "all"):
     for args, nm in [((32, 128, 28, 28, 128, 3, 3, 1, 1), "conv3x_n32"), ((256, 64, 56, 56, 64, 3, 3, 1, 1), "l1_3x3_64"),
