@@ -175,6 +175,7 @@ struct HankelTiling {
   int nacc;  // TMEM accumulator buffers (1 or 2)
   // stride-2 phase mode (reading R19): the kernel runs on the phase-split geometry
   int phase, eC, eH, eW, eR, eS, eph, epw;
+  int kc;  // channels per window row: 64 bf16 / 32 tf32 (128 B), 16 bf16 (32 B, small-C phase mode)
 };
 HankelTiling hankel_tiling(const Geom& g, int fmt, int num_sms, bool io_bf16);
 // x: NCHW input (io dtype); U: tap-major packed filter [RS][Kp][Cp] (t.Kp, t.Cp), packed by

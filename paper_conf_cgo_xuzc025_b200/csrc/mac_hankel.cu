@@ -428,13 +428,22 @@ __device__ __forceinline__ void hk_load_window_pairs(const HkParams& p, uint32_t
 // channels (a, c, 0) and (a, c, 1) of position (u, v), already in operand order, so a 16-byte
 // row group (4 channels x 2 column phases) is 4 loads, no permutes.  Each position of a lane's
 // pair is decoded on its own (any W' = W/2); rows 2u + a past x's last row read the zero buffer.
-template <bool kAligned>
+template <bool kAligned, uint32_t kRowB>
 __device__ __forceinline__ void hk_load_window_phase(const HkParams& p, uint32_t slot, long long q0, int vc0, int lw,
                                                      int lane, int rp_lo, int rp_hi) {
   constexpr int B = 4;  // position pairs per lane in flight
-  const int a = vc0 / (2 * p.xC);
-  const int c = (vc0 - a * 2 * p.xC) / 2 + lw * 4;  // first of this group's 4 channels
   const uint32_t hw2 = (uint32_t)(p.xH * p.xW) >> 1, w2 = (uint32_t)p.xW >> 1;
+  // this group's 4 (a, c) slots: virtual channels vc0 + 8 lw + 2k + {0, 1}; C % 32 == 0 keeps
+  // a (and so the row offset) one per chunk, else (the stem, 4C <= 16) per slot, a >= 2 zero
+  int sa[4], sc[4];
+#pragma unroll
+  for (int k = 0; k < 4; ++k) {
+    const int s2 = vc0 / 2 + lw * 4 + k;
+    sa[k] = s2 / p.xC;
+    sc[k] = s2 - sa[k] * p.xC;
+  }
+  const bool small_c = p.xC % 32 != 0;
+  const int a = sa[0], c = sc[0];
   const int nrp = rp_hi;
   const uint32_t sel = (uint32_t)(lane >> 2) & 1u;
   for (int rp0 = rp_lo; rp0 < nrp; rp0 += 32 * B) {
@@ -446,6 +455,22 @@ __device__ __forceinline__ void hk_load_window_phase(const HkParams& p, uint32_t
       // kAligned (W' even, pitch W' + 2pw', delta pw' & 1): both positions of a pair are data of
       // one row or both zero, one decode; else each position is decoded on its own
       const uint32_t* base[2];
+      if (small_c) {
+        // (the stem) every slot its own row phase and channel; W' even (aligned) assumed
+        int n, u, v;
+        const bool in = hk_pos(p, q0 + 2 * rp, n, u, v) && rp < nrp && !(p.dbg & 1);
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          const int r = 2 * u + sa[k];
+          const uint32_t* bk = (in && sa[k] < 2 && r < p.xH)
+                                   ? static_cast<const uint32_t*>(p.x) + (((uint32_t)n * p.xC + (uint32_t)sc[k]) * hw2 +
+                                                                          (uint32_t)r * w2 + (uint32_t)v)
+                                   : static_cast<const uint32_t*>(p.zero);
+          lo[b][k] = bk[0];
+          hi[b][k] = bk[1];
+        }
+        continue;
+      }
 #pragma unroll
       for (int s2 = 0; s2 < (kAligned ? 1 : 2); ++s2) {
         int n, u, v;
@@ -469,8 +494,12 @@ __device__ __forceinline__ void hk_load_window_phase(const HkParams& p, uint32_t
         const uint32_t ra = 2u * (uint32_t)rp + sel, rb = 2u * (uint32_t)rp + (sel ^ 1u);
         const uint32_t* da = sel ? hi[b] : lo[b];
         const uint32_t* db = sel ? lo[b] : hi[b];
-        const uint32_t aa = slot + ra * 128u + (((uint32_t)lw ^ (ra & 7u)) << 4);
-        const uint32_t ab = slot + rb * 128u + (((uint32_t)lw ^ (rb & 7u)) << 4);
+        // 16-B chunk ^= byte-address bits [7, 10) of the row: SW128 row & 7, SW64 (row >> 1) & 3,
+        // SW32 (row >> 2) & 1
+        const uint32_t xa = kRowB == 128 ? (ra & 7u) : kRowB == 64 ? ((ra >> 1) & 3u) : ((ra >> 2) & 1u);
+        const uint32_t xb = kRowB == 128 ? (rb & 7u) : kRowB == 64 ? ((rb >> 1) & 3u) : ((rb >> 2) & 1u);
+        const uint32_t aa = slot + ra * kRowB + (((uint32_t)lw ^ xa) << 4);
+        const uint32_t ab = slot + rb * kRowB + (((uint32_t)lw ^ xb) << 4);
         asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(aa), "r"(da[0]), "r"(da[1]), "r"(da[2]),
                      "r"(da[3])
                      : "memory");
@@ -494,7 +523,7 @@ __device__ __forceinline__ void hk_store<__nv_bfloat16>(__nv_bfloat16* y, long l
   y[i] = __float2bfloat16_rn(v);
 }
 
-template <typename IoT, bool kTf32, int kHW2>
+template <typename IoT, bool kTf32, int kHW2, int kKC = (kTf32 ? 32 : 64)>
 __global__ void __launch_bounds__(kHkThreads, 1)
     mac_hankel_kernel(const __grid_constant__ CUtensorMap tmU, const HkParams p) {
   extern __shared__ uint8_t smem_raw[];
@@ -519,6 +548,11 @@ __global__ void __launch_bounds__(kHkThreads, 1)
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(eloc + 2);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  // window / filter rows: kKC channels of 128 B (SW128) or, for the small-C phase convolution
+  // (the stem, 4C <= 16 virtual channels), 16 bf16 channels of 32 B (SW32)
+  constexpr uint32_t kRowB = kTf32 ? 4u * kKC : 2u * kKC;
+  constexpr uint32_t kRow16 = kRowB / 16u;  // 16-byte units per row
+  constexpr int kKSteps = (int)kRowB / 32;   // MMA K steps (32 bytes each) per row
   const uint32_t rank = cluster_ctarank();
   const int pair = (int)(blockIdx.x >> 1);
   const long long U = (long long)p.PT * p.NB;
@@ -570,7 +604,7 @@ __global__ void __launch_bounds__(kHkThreads, 1)
               const uint32_t bar = ffull0 + (uint32_t)fs * 8u;
               if (rank == 0) mbar_arrive_expect_tx(ffull + fs, 2u * p.fblk_bytes);
               const int row = tap * p.Kp + it.nb * p.NN + (int)rank * (p.NN / 2);
-              hk_tma_pair(sF + (uint32_t)fs * p.fblk_bytes, &tmU, bar, ch * (kTf32 ? 32 : 64), row);
+              hk_tma_pair(sF + (uint32_t)fs * p.fblk_bytes, &tmU, bar, ch * kKC, row);
             }
             __syncwarp();
             if (++fs == p.fslots) { fs = 0; ++fuse; }
@@ -586,7 +620,7 @@ __global__ void __launch_bounds__(kHkThreads, 1)
       HkItem it;
       int fs = 0, fuse = 0, ws = 0, wuse = 0, item = 0;
       bool first = true;
-      const uint32_t row16 = (uint32_t)p.pitch * 8u;  // one kernel row of taps = pitch window rows, 16-B units
+      const uint32_t row16 = (uint32_t)p.pitch * kRow16;  // one kernel row of taps = pitch window rows, 16-B units
       while (hk_next(p, u, u_hi, it)) {
         const int a = p.nacc == 2 ? (item & 1) : 0;
         hk_wait(tempty + a, (uint32_t)((item / p.nacc) & 1) ^ 1u);
@@ -601,7 +635,7 @@ __global__ void __launch_bounds__(kHkThreads, 1)
           if (wt) g_hk_wtrace[wi * 8 + 3] = global_ns();
           // descriptors: window row r of tap (i, j) = t*128 + pitch*i + j (the Hankel shift);
           // +1024 16-B units per 128-row tile, +2 per 32-byte K step
-          const uint64_t awin = make_sdesc(sW + (uint32_t)ws * p.wslot_bytes, 128u, 0);
+          const uint64_t awin = make_sdesc(sW + (uint32_t)ws * p.wslot_bytes, kRowB, 0);
           uint32_t rowoff = 0;
           int j = 0;
           for (int tap = 0; tap < p.RS; ++tap) {
@@ -611,17 +645,16 @@ __global__ void __launch_bounds__(kHkThreads, 1)
               tc_fence_after();
               if (trace && lane == 0 && item == 0 && ch == 0 && tap == 0) tr[3] = global_ns();
             }
-            const uint64_t bd = make_sdesc(sF + (uint32_t)slot * p.fblk_bytes, 128u, 0);
-            const uint64_t ad = awin + rowoff + (uint32_t)j * 8u;
+            const uint64_t bd = make_sdesc(sF + (uint32_t)slot * p.fblk_bytes, kRowB, 0);
+            const uint64_t ad = awin + rowoff + (uint32_t)j * kRow16;
             const uint32_t acc0 = (ch | tap) != 0 ? 1u : 0u;
             if (!(p.dbg & 4) && elect_one()) {
               for (int t = 0; t < it.T; ++t) {
-                const uint64_t at = ad + (uint64_t)(t * 1024);
+                const uint64_t at = ad + (uint64_t)(t * 128 * kRow16);
                 const uint32_t d = dacc + (uint32_t)(t * p.NN);
                 hk_mma<kTf32>(d, at, bd, p.idesc, acc0);
-                hk_mma<kTf32>(d, at + 2, bd + 2, p.idesc, 1u);
-                hk_mma<kTf32>(d, at + 4, bd + 4, p.idesc, 1u);
-                hk_mma<kTf32>(d, at + 6, bd + 6, p.idesc, 1u);
+#pragma unroll
+                for (int k = 1; k < kKSteps; ++k) hk_mma<kTf32>(d, at + 2 * k, bd + 2 * k, p.idesc, 1u);
               }
             }
             __syncwarp();
@@ -648,11 +681,14 @@ __global__ void __launch_bounds__(kHkThreads, 1)
     }
   } else if (role == kRoleLoader) {
     // ---- window loaders (a2) ----
-    const int lw = ridx & 7;
-    // row-pair half of every window this warp converts (split on a multiple of 32 pairs)
+    // 16-byte column group of every row this warp converts, and its slice of the row pairs
+    // (128-B rows: 8 groups x 2 halves; 32-B rows: 2 groups x 8 slices; split on 32 pairs)
+    constexpr int kGroups = (int)kRow16;
+    constexpr int kSlices = kHkLoadWarps / kGroups;
+    const int lw = ridx % kGroups, sl = ridx / kGroups;
     const int nrp_all = p.wrows >> 1;
-    const int split = ((nrp_all / 2 + 31) / 32) * 32;
-    const int rp_lo = (ridx >> 3) ? min(split, nrp_all) : 0, rp_hi = (ridx >> 3) ? nrp_all : min(split, nrp_all);
+    const int per = ((nrp_all + kSlices - 1) / kSlices + 31) / 32 * 32;
+    const int rp_lo = min(sl * per, nrp_all), rp_hi = min((sl + 1) * per, nrp_all);
     {
       long long u = u_lo;
       HkItem it;
@@ -666,8 +702,8 @@ __global__ void __launch_bounds__(kHkThreads, 1)
           hk_wait(wempty + ws, (uint32_t)(wuse & 1) ^ 1u);
           if (wt) g_hk_wtrace[wi * 8 + 1] = global_ns();
           if constexpr (kHW2 == -2 || kHW2 == -4)
-            hk_load_window_phase<kHW2 == -2>(p, sW + (uint32_t)ws * p.wslot_bytes, q0, ch * 64, lw, lane, rp_lo,
-                                             rp_hi);
+            hk_load_window_phase<kHW2 == -2, kRowB>(p, sW + (uint32_t)ws * p.wslot_bytes, q0, ch * kKC, lw, lane,
+                                                    rp_lo, rp_hi);
           else if constexpr (kHW2 >= 0)
             hk_load_window_pairs<IoT, kTf32, kHW2>(p, sW + (uint32_t)ws * p.wslot_bytes, q0, ch * (kTf32 ? 32 : 64), lw,
                                                    lane, rp_lo, rp_hi);
@@ -747,8 +783,13 @@ __global__ void __launch_bounds__(kHkThreads, 1)
         const uint32_t trow = tbase + ((uint32_t)(quad * 32) << 16) + (uint32_t)(a * p.T * p.NN + t * p.NN);
         for (int g = half; g * 16 < p.NN; g += 2) {
           uint32_t v[16];
-          hk_tmem_ld16(trow + (uint32_t)(g * 16), v);
-          tmem_ld_wait();
+          if (!(p.dbg & 512)) {
+            hk_tmem_ld16(trow + (uint32_t)(g * 16), v);
+            tmem_ld_wait();
+          } else {
+#pragma unroll
+            for (int c = 0; c < 16; ++c) v[c] = 0u;
+          }
           if (ybase >= 0 && !(p.dbg & 2)) {
             IoT* yp = y + ybase + (long long)(g * 16) * PQ;
             const int kleft = p.K - (it.nb * p.NN + g * 16);  // output channels left (warp-uniform)
@@ -817,12 +858,15 @@ size_t hankel_zero_bytes(const Geom& g) { return (size_t)32 * g.H * g.W + 256; }
 // window rebuilds per output-channel block); 128->128 28x28 NN=128/T=2 862.
 // The filter is resident in shared memory when its (single) block fits beside two windows,
 // else streamed by TMA through a ring of (chunk, tap) blocks.
-static HankelTiling hankel_tiling_core(const Geom& g, int fmt, int num_sms) {
+// kc16: 32-byte rows of 16 bf16 channels (SW32) for the small-C phase convolution (the stem)
+static HankelTiling hankel_tiling_core(const Geom& g, int fmt, int num_sms, int kc_small = 0) {
   HankelTiling t{};
   t.ok = false;
   if (fmt == FMT_F32) return t;
   const bool tf32 = fmt == FMT_TF32;
-  const int eb = tf32 ? 4 : 2, kc = 128 / eb;
+  if (kc_small && tf32) return t;
+  const int eb = tf32 ? 4 : 2, kc = kc_small ? kc_small : 128 / eb;
+  const uint32_t rowb = (uint32_t)(kc * eb);
   // row pitch: the paper's Wp = W + 2pw (even for even W, so position pairs are input
   // pairs), or W + pw (shared column padding, reading R16) for odd W;
   // POLYCONV_HK_PITCH=1 / 2 forces W + pw / W + 2pw
@@ -857,10 +901,10 @@ static HankelTiling hankel_tiling_core(const Geom& g, int fmt, int num_sms) {
     if ((forceT && T != forceT) || T * NN > (acc1 ? 512 : 256)) continue;
     const int NB = (g.K + NN - 1) / NN;
     if ((long long)RS * NB * NN >= (1LL << 31)) break;
-    const uint32_t fblk = (uint32_t)(NN / 2) * 128u;
+    const uint32_t fblk = (uint32_t)(NN / 2) * rowb;
     const int nblk = nchunks * RS;
     const int wrows = (128 * T + (g.R - 1) * pitch + g.S - 1 + 7) / 8 * 8;
-    const uint32_t wslot = (uint32_t)wrows * 128u;
+    const uint32_t wslot = (uint32_t)wrows * rowb;
     bool resident = false;
     int wslots = 0, fslots = 0;
     // Resident only when streaming would re-read more filter bytes per window than the window
@@ -891,7 +935,7 @@ static HankelTiling hankel_tiling_core(const Geom& g, int fmt, int num_sms) {
     t.npairs = (int)std::min<long long>(max_pairs, (long long)PT * NB);
   }
   if (!found) return t;
-  t.pitch = pitch; t.HS = HS; t.delta = delta; t.PT = PT; t.Cp = Cp; t.nchunks = nchunks;
+  t.pitch = pitch; t.HS = HS; t.delta = delta; t.PT = PT; t.Cp = Cp; t.nchunks = nchunks; t.kc = kc;
   // pair-aligned loader: every position pair is one aligned input pair or zeros
   t.aligned = (!(g.W & 1) && pitch == g.W + 2 * g.pw && delta == (g.pw & 1) && g.C % (tf32 ? 4 : 8) == 0 &&
                env_int("POLYCONV_HK_GENERAL", 0) == 0) ? 1 : 0;
@@ -929,12 +973,14 @@ static Geom hk_phase_geom(const Geom& g) {
 // math, even x width (x[2v], x[2v+1] one aligned word), C % 32 == 0 (a 64-channel chunk never
 // straddles the row phase a), R - 1 >= ph; POLYCONV_HK_PHASE=0 turns it off.
 HankelTiling hankel_tiling(const Geom& g, int fmt, int num_sms, bool io_bf16) {
-  if (g.sh == 2 && g.sw == 2 && fmt == FMT_BF16 && io_bf16 && g.W % 2 == 0 && g.C % 32 == 0 &&
+  if (g.sh == 2 && g.sw == 2 && fmt == FMT_BF16 && io_bf16 && g.W % 2 == 0 && (g.C % 32 == 0 || g.C <= 4) &&
       g.R - 1 >= g.ph && g.S - 1 >= g.pw && env_int("POLYCONV_HK_PHASE", 1) != 0) {
     const Geom e = hk_phase_geom(g);
-    HankelTiling t = hankel_tiling_core(e, fmt, num_sms);
+    HankelTiling t = hankel_tiling_core(e, fmt, num_sms, e.C <= 16 ? env_int("POLYCONV_HK_KC", 16) : 0);
     if (t.ok) {
       t.phase = 1;
+      // position pairs of the phase planes are both data of one row or both zero
+      t.aligned = (e.W % 2 == 0 && t.pitch == e.W + 2 * e.pw && t.delta == (e.pw & 1)) ? 1 : 0;
       t.eC = e.C; t.eH = e.H; t.eW = e.W; t.eR = e.R; t.eS = e.S; t.eph = e.ph; t.epw = e.pw;
       return t;
     }
@@ -962,11 +1008,13 @@ cudaError_t launch_mac_hankel(const Geom& g0, const HankelTiling& t, int fmt, co
     const uint32_t eb = tf32 ? 4 : 2;
     cuuint64_t dims[2] = {(cuuint64_t)t.Cp, (cuuint64_t)g.R * g.S * t.Kp};
     cuuint64_t strides[1] = {(cuuint64_t)t.Cp * eb};
-    cuuint32_t box[2] = {128u / eb, (cuuint32_t)(t.NN / 2)};
+    cuuint32_t box[2] = {(cuuint32_t)t.kc, (cuuint32_t)(t.NN / 2)};
     cuuint32_t estr[2] = {1, 1};
     if (!enc || enc(&tmU, tf32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2,
                     const_cast<void*>(U), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                    CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                    t.kc * eb == 32 ? CU_TENSOR_MAP_SWIZZLE_32B
+                    : t.kc * eb == 64 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B,
+                    CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
                     CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS) {
       snprintf(err, errlen, "mac_hankel: cuTensorMapEncodeTiled failed");
       return cudaErrorInvalidValue;
@@ -1001,7 +1049,13 @@ cudaError_t launch_mac_hankel(const Geom& g0, const HankelTiling& t, int fmt, co
   // plane size in words baked in (immediate channel offsets) for the ResNet / VGG planes
   void (*kern)(const CUtensorMap, const HkParams);
   const int hw2 = g.H * g.W / 2;
-  if (t.phase) {
+  if (t.phase && t.kc < 64) {
+    if (!t.aligned) {
+      snprintf(err, errlen, "mac_hankel: small-C phase mode needs pair-aligned phase planes");
+      return cudaErrorInvalidValue;
+    }
+    kern = t.kc == 16 ? mac_hankel_kernel<__nv_bfloat16, false, -2, 16> : mac_hankel_kernel<__nv_bfloat16, false, -2, 32>;
+  } else if (t.phase) {
     kern = t.aligned ? mac_hankel_kernel<__nv_bfloat16, false, -2> : mac_hankel_kernel<__nv_bfloat16, false, -4>;
   } else if (!t.aligned) {
     kern = tf32 ? mac_hankel_kernel<float, true, -1>

@@ -113,6 +113,8 @@ MX_SHAPES = [
     ConvShape("mx_s2_phase_p0", 2, 64, 16, 16, 40, 3, 3, 2, 2, 0, 0),
     ConvShape("mx_s2_phase_w14", 3, 64, 14, 14, 96, 3, 3, 2, 2, 1, 1),   # W/2 odd: per-position decode
     ConvShape("mx_k1_wide", 2, 512, 14, 14, 128, 1, 1, 1, 1, 0, 0),  # AUTO: tc_hankel from 24 units
+    ConvShape("mx_stem", 2, 3, 32, 32, 64, 7, 7, 2, 2, 3, 3),   # small-C phase mode, 32-byte rows
+    ConvShape("mx_stem_c4", 2, 4, 20, 24, 40, 7, 7, 2, 2, 3, 3),
 ]
 
 

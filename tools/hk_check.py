@@ -92,6 +92,12 @@ if which in ("tail", "all"):
                  (90, 512, 7, 7, 512, 3, 3, 1, 1), (70, 64, 28, 28, 96, 3, 3, 1, 1), (33, 96, 20, 21, 192, 3, 3, 1, 1)]:
         run(*args, name="tail")
         run(*args, math="tf32", io="f32", name="tail_tf32")
+if which in ("stem", "all"):
+    # 7x7 stride 2, C = 3: small-C phase mode, 32-byte window rows
+    for args in [(2, 3, 32, 32, 64, 7, 7, 2, 3), (3, 3, 30, 26, 40, 7, 7, 2, 3), (2, 4, 20, 20, 48, 7, 7, 2, 3),
+                 (2, 2, 16, 24, 64, 5, 5, 2, 2), (8, 3, 224, 224, 64, 7, 7, 2, 3)]:
+        run(*args, name="stem")
+    run(256, 3, 224, 224, 64, 7, 7, 2, 3, time_it=True, name="stem7x7")
 if which in ("s2", "all"):
     # stride 2: phase-split mode (reading R19) where W % 4 == 0 and C % 32 == 0
     for args in [(2, 64, 16, 16, 64, 3, 3, 2, 1), (3, 128, 56, 56, 128, 3, 3, 2, 1), (2, 256, 28, 28, 256, 3, 3, 2, 1),
