@@ -508,8 +508,53 @@ template <typename InT, int F> struct LFPlanar {
     return cudaGetLastError();
   }
 };
+// bf16 tap-major filter, one thread per (k, 8 consecutive channels): the 8*RS contiguous
+// elements w[k][c0..c0+7][*] as RS 16-byte loads, transposed in registers by byte permutes into
+// RS 16-byte rows U[tap][k][c0..c0+7].  A few hundred threads instead of one per (k, c): the
+// pack occupies a handful of SMs, so the MAC that follows it by programmatic dependent launch
+// starts on the others at once (conv3_x: 2048 threads in 16 blocks).  C % 8 == 0.
+template <int RS>
+__global__ void __launch_bounds__(128) pack_filter_tapmajor_oct_kernel(Geom g, const uint4* __restrict__ w,
+                                                                       uint4* __restrict__ dst, int Kp, int Cp) {
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+  const int noct = Cp >> 3;
+  const int idx = blockIdx.x * 128 + threadIdx.x;
+  if (idx >= Kp * noct) return;
+  const int k = idx / noct, oct = idx - k * noct;
+  const bool ok = k < g.K && oct * 8 < g.C;
+  uint4 v[RS];
+#pragma unroll
+  for (int i = 0; i < RS; ++i)
+    v[i] = ok ? __ldg(w + ((long long)k * (g.C >> 3) + oct) * RS + i) : make_uint4(0, 0, 0, 0);
+  const uint32_t* e = reinterpret_cast<const uint32_t*>(v);  // element j in word j/2, half j%2
+#pragma unroll
+  for (int t = 0; t < RS; ++t) {
+    uint32_t o[4];
+#pragma unroll
+    for (int m = 0; m < 4; ++m) {
+      const int a = (2 * m) * RS + t, b = (2 * m + 1) * RS + t;  // channels 2m, 2m+1 at tap t
+      const uint32_t sel = ((b & 1) ? 0x7600u : 0x5400u) | ((a & 1) ? 0x32u : 0x10u);
+      o[m] = __byte_perm(e[a >> 1], e[b >> 1], sel);
+    }
+    dst[((long long)t * Kp + k) * noct + oct] = make_uint4(o[0], o[1], o[2], o[3]);
+  }
+}
+
 template <typename InT, int F> struct LFTap {
   static cudaError_t run(const Geom& g, const void* w, void* dst, int Kp, int Cp, cudaStream_t st) {
+    if constexpr (sizeof(InT) == 2 && F == FMT_BF16) {
+      const int RS = g.R * g.S;
+      if (g.urep == 1 && g.C % 8 == 0 && Cp % 8 == 0 && (RS == 9 || RS == 25 || RS == 1) &&
+          ((uintptr_t)w & 15) == 0 && !getenv("POLYCONV_PACK_LEGACY")) {
+        const int n = Kp * (Cp / 8), blocks = (n + 127) / 128;
+        const uint4* wv = static_cast<const uint4*>(w);
+        uint4* dv = static_cast<uint4*>(dst);
+        if (RS == 9) pack_filter_tapmajor_oct_kernel<9><<<blocks, 128, 0, st>>>(g, wv, dv, Kp, Cp);
+        else if (RS == 25) pack_filter_tapmajor_oct_kernel<25><<<blocks, 128, 0, st>>>(g, wv, dv, Kp, Cp);
+        else pack_filter_tapmajor_oct_kernel<1><<<blocks, 128, 0, st>>>(g, wv, dv, Kp, Cp);
+        return cudaGetLastError();
+      }
+    }
     long long total = (long long)Kp * Cp;
     pack_filter_tapmajor_kernel<InT, F><<<grid_for(total, kThreads), kThreads, 0, st>>>(
         g, (const InT*)w, (typename Word<F>::T*)dst, Kp, Cp);
