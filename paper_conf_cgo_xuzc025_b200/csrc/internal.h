@@ -143,7 +143,7 @@ struct PairTiling {
   int ne_box, last_rows, in_bytes, obox_bytes, obox_bytes2;
   int tr, tpi, ntile;          // row-aligned CTA tiles: tr output rows of one image each
   int epi_tma, estage_bytes;   // epilogue staged in shared memory and written by TMA stores
-  int direct0, ne_w, u_img0, w0_off;  // first tile's windows from x in shared memory; A from image u_img0
+  int u_img0;  // first image whose bands the pack writes (0)
   int split, pack_grid, pack_smem;    // packing in its own grid, the pair kernel its programmatic dependent
 };
 PairTiling pair_tiling(const Geom& g, int fmt, bool io_bf16, int num_sms);
@@ -153,9 +153,7 @@ PairTiling pair_tiling(const Geom& g, int fmt, bool io_bf16, int num_sms);
 // flags (zeroed once; band u is published as `epoch` = launches so far); state: launch
 // cache from pair_state_new() (tensor maps + parameters per pointer set), or nullptr
 cudaError_t launch_mac_pair(const Geom& g, const PairTiling& t, const void* x, const void* w, bool io_bf16,
-                            void* A, void* U, void* y, unsigned long long* fcount, unsigned long long ftarget,
-                            unsigned long long* bflag, unsigned long long epoch, cudaStream_t st, char* err,
-                            size_t errlen, void* state);
+                            void* A, void* U, void* y, cudaStream_t st, char* err, size_t errlen, void* state);
 void* pair_state_new();
 void pair_state_free(void* s);
 

@@ -1,5 +1,7 @@
-// mac_pair.cu — the BF16 hot path in ONE launch on CTA pairs (tcgen05
-// cta_group::2): a2 + a3 packing, a4 coefficient MAC, a5 extraction.
+// mac_pair.cu — the round-1 BF16 path on CTA pairs (tcgen05 cta_group::2): a pack grid for
+// a2 + a3, then a4 coefficient MAC + a5 extraction as its programmatic dependent launch.
+// Since round 2 `mac_hankel` is the BF16 default; this kernel is selectable (TC_PAIR) and
+// kept as the ablation that packs A through HBM.
 //
 // The coefficient MAC
 //   p_{n,k}[m] = sum_c sum_{i,j} A_{n,c}[m - e(i,j)] * U_{k,c}[e(i,j)]   (P.965, P.1350-1352)
@@ -9,28 +11,23 @@
 //   D[pos][k] += sum_c A[pos + Wp*i + j][c] * U_tap(i,j)[k][c]
 // with pos = the base coefficient m - (L_U - 1) of an output (Eq. 12).
 //
-// Design (DESIGN.md §4 "mac_pair"):
-//  * Phase 1 (every CTA, all warps): pack a slice of the filter into the
-//    tap-major layout U[R*S][NN][Cp] (a3: the nonzero coefficients of the
-//    reversed, gap-padded U_{k,c}(t), Eq. 6, grouped by degree e(i,j)); the
-//    slices meet on a grid counter.  Then one band of rb padded rows of one
-//    image of the channel-interleaved input polynomial A[N*L_A][Cp] (a2:
-//    coefficient r*Wp + s of A_{n,c}(t) = xpad[n][c][r][s], Eq. 10 + zero
-//    padding P.1353-1356, BF16 RNE, reading R11): TMA boxes of the band's x
-//    rows (64 channel planes each), a shared-memory transpose into 128-byte
-//    swizzled rows, TMA stores, then the band is published on its own flag.
-//    The packed copies stay in L2.  All CTAs are co-resident (one per SM,
-//    checked when the launch is prepared).
-//  * Phase 2 (CTA pairs): UMMA M = 256 positions (128 per CTA = the TMEM lanes:
-//    a window of the interleaved input, K-major, TMA), N = NN output channels
-//    (B operand = the filter, each CTA holding NN/2 rows of every (chunk, tap)
-//    block -- RESIDENT in shared memory: loaded once, reused by every tile).
-//    One window of 128 + (R-1)*Wp + S-1 positions per channel chunk serves all
-//    R*S taps through descriptors shifted by (Wp*i + j) rows
-//    (tools/umma_probe.cu).  A window waits only for the bands it reads.  The
-//    leader CTA issues tcgen05.mma.cta_group::2 from a per-tap descriptor table;
-//    accumulators (fp32) live in TMEM, double buffered, so the epilogue of tile
-//    t overlaps the MMAs of tile t+1.  A CTA tile = tr output rows of one image.
+// Design:
+//  * Pack grid (pair_pack_kernel, several CTAs per SM): the tap-major filter
+//    U[R*S][NN][Cp] (a3: the nonzero coefficients of the reversed, gap-padded
+//    U_{k,c}(t), Eq. 6, grouped by degree e(i,j)) and bands of rb padded rows of the
+//    channel-interleaved input polynomial A[N*L_A][Cp] (a2: coefficient r*Wp + s of
+//    A_{n,c}(t) = xpad[n][c][r][s], Eq. 10 + zero padding P.1353-1356, BF16 RNE, reading
+//    R11): TMA boxes of x rows, a shared-memory transpose into 128-byte swizzled rows, TMA
+//    stores.  It triggers the dependent launch at once; the MAC's producer waits
+//    (griddepcontrol.wait) before its first TMA read of A / U.
+//  * MAC (CTA pairs): UMMA M = 256 positions (128 per CTA = the TMEM lanes: a window of
+//    the interleaved input, K-major, TMA), N = NN output channels (B operand = the filter,
+//    each CTA holding NN/2 rows of every (chunk, tap) block -- RESIDENT in shared memory:
+//    loaded once, reused by every tile).  One window of 128 + (R-1)*Wp + S-1 positions per
+//    channel chunk serves all R*S taps through descriptors shifted by (Wp*i + j) rows
+//    (tools/umma_probe.cu).  The leader CTA issues tcgen05.mma.cta_group::2 from a per-tap
+//    descriptor table; accumulators (fp32) live in TMEM, double buffered, so the epilogue
+//    of tile t overlaps the MMAs of tile t+1.  A CTA tile = tr output rows of one image.
 //  * Epilogue (a5, fused): positions are TMEM lanes; the Eq. 12 / reading R4
 //    extraction y[n][k][oh][ow] = p[Wp*sh*oh + sw*ow + L_U - 1] is a per-lane
 //    predicate; bf16 outputs are staged per channel half in shared memory and
@@ -38,10 +35,10 @@
 //    (direct stores for f32 outputs or K % 32 != 0).
 //  * Warp roles: warp 0 = TMA producer, warp 1 = TMEM allocator + MMA issuer
 //    (leader CTA), warps 2..9 = epilogue (2 per TMEM lane quadrant, each half
-//    of the channels).  All ten warps pack in phase 1.
-//  * Experiment switches (DESIGN.md §4 table; off by default): split packing
-//    grid, direct first-tile windows, filter built in shared memory, warm-up
-//    MMA chunk, per-CTA phase trace.
+//    of the channels).
+//  * Synchronisation is pair-local (mbarriers) plus the programmatic launch
+//    dependency: no grid-wide counters or flags (the round-1 one-launch variant with a
+//    grid counter and band flags, and its experiment switches, were removed).
 #include <cuda.h>
 #include <cstdio>
 #include <cstdlib>
@@ -69,10 +66,6 @@ struct PairParams {
   void* A;  // interleaved input polynomial [N*L_A][Cp] bf16 (plan workspace)
   void* U;  // tap-major filter [R*S][NN][Cp] bf16 (plan workspace)
   void* y;
-  unsigned long long* fcount;   // filter slices packed (all CTAs): reaches ftarget
-  unsigned long long ftarget;
-  unsigned long long* bflag;    // [N*nb] band u of A written in launch epoch
-  unsigned long long epoch;
   long long L_A, G, NLA;
   int N, C, H, W, K, R, S, sh, sw, ph, pw, Hp, Wp, P, Q, PQ;
   int Cp, NN, kc, row_bytes, nchunks, RS, nblk;
@@ -94,18 +87,10 @@ struct PairParams {
   // ntile CTA tiles in all); epilogue by TMA stores of [32 channels][tr*Q pixels]
   // boxes staged in shared memory (epi_tma) or by direct stores
   int tr, tpi, ntile, epi_tma;
-  int warm;   // warm-up MMA chunk at launch (code path + tensor pipe)
-  // direct0: every CTA builds its FIRST tile's windows in shared memory straight from x
-  // (one TMA box of ne_w plane elements x 64 channels per chunk, staged at sF + w0_off);
-  // the packed input A (bands) is written only for the images of later tiles, from u_img0 on
-  int direct0, ne_w, u_img0;
-  uint32_t w0_off;
+  int u_img0;  // first image the pack writes (0)
   // split: a2 + a3 run in a separate pack kernel (pair_pack_kernel) that this kernel
   // follows as a programmatic dependent launch: no grid counter, no band flags
   int split;
-  int fsmem;  // a3 straight into shared memory after the band packing (no global U, no counter):
-              // 1 = loads from w, 2 = bulk-copied slabs of frows rows of w
-  int frows;
   uint32_t estage_bytes;
   FastDiv ftpi;
 };
@@ -349,151 +334,6 @@ __device__ __forceinline__ void tma_store_2d(const void* tmap, uint32_t src, int
 // group when RS == 9 and C % 8 == 0), transposed in registers into one 16-byte
 // chunk per tap block.  Nothing goes to global memory.
 template <typename IoT>
-__device__ __forceinline__ void pair_filter_smem(const PairParams& p, uint8_t* sF, uint32_t rank) {
-  const int half = p.NN / 2, kb = (int)rank * half;
-  const int ncg = p.Cp / 8;
-  const int items = half * ncg;
-  const IoT* w = static_cast<const IoT*>(p.w);
-  const uint32_t M = (uint32_t)p.row_bytes / 16u - 1u;  // swizzle: 16-byte chunk ^= (row bits)
-  const bool vec9 = std::is_same<IoT, __nv_bfloat16>::value && p.RS == 9 && p.C % 8 == 0;
-  for (int it = threadIdx.x; it < items; it += blockDim.x) {
-    const int kl = it / ncg, cg = it - (it / ncg) * ncg;
-    const int k = kb + kl, c0 = cg * 8;
-    const int ch = c0 / p.kc, j = (c0 - ch * p.kc) >> 3;
-    const uint32_t o = (uint32_t)kl * (uint32_t)p.row_bytes + (uint32_t)j * 16u;
-    uint8_t* dst = sF + (size_t)(ch * p.RS) * p.fbytes + (o ^ (((o >> 7) & M) << 4));
-    if (vec9 && k < p.K && c0 + 8 <= p.C) {
-      // w[k][c0..c0+7][0..8]: 72 bf16 = 9 x 16 bytes, element c*9 + t
-      const uint4* src = reinterpret_cast<const uint4*>(w + ((long long)k * p.C + c0) * 9);
-      uint32_t e[36];
-#pragma unroll
-      for (int q = 0; q < 9; ++q) {
-        const uint4 v = __ldg(src + q);
-        e[4 * q] = v.x; e[4 * q + 1] = v.y; e[4 * q + 2] = v.z; e[4 * q + 3] = v.w;
-      }
-#pragma unroll
-      for (int t = 0; t < 9; ++t) {
-        uint32_t out[4];
-#pragma unroll
-        for (int m = 0; m < 4; ++m) {
-          const int i0 = (2 * m) * 9 + t, i1 = (2 * m + 1) * 9 + t;
-          const uint32_t lo = (e[i0 >> 1] >> ((i0 & 1) * 16)) & 0xFFFFu;
-          const uint32_t hi = (e[i1 >> 1] >> ((i1 & 1) * 16)) & 0xFFFFu;
-          out[m] = lo | (hi << 16);
-        }
-        *reinterpret_cast<uint4*>(dst + (size_t)t * p.fbytes) = make_uint4(out[0], out[1], out[2], out[3]);
-      }
-    } else {
-      for (int t = 0; t < p.RS; ++t) {
-        uint32_t out[4];
-#pragma unroll
-        for (int m = 0; m < 4; ++m) {
-          const int c = c0 + 2 * m;
-          const uint32_t lo =
-              (k < p.K && c < p.C) ? (uint32_t)to_bf16_bits<IoT>(w[((long long)k * p.C + c) * p.RS + t]) : 0u;
-          const uint32_t hi =
-              (k < p.K && c + 1 < p.C) ? (uint32_t)to_bf16_bits<IoT>(w[((long long)k * p.C + c + 1) * p.RS + t]) : 0u;
-          out[m] = lo | (hi << 16);
-        }
-        *reinterpret_cast<uint4*>(dst + (size_t)t * p.fbytes) = make_uint4(out[0], out[1], out[2], out[3]);
-      }
-    }
-  }
-}
-
-// a3 into shared memory from bulk-copied rows of w (fsmem == 2): slabs of `frows`
-// output-channel rows w[k][0..C*R*S) (contiguous in KCRS) land by cp.async.bulk in
-// a double-buffered staging area, and the warps transpose them into the resident
-// (chunk, tap) blocks: item (k, 8 channels) reads the 8*R*S contiguous coefficients
-// and writes one 16-byte chunk per tap block (same layout as pair_filter_smem).
-__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void* src, uint32_t bytes, uint64_t* bar) {
-  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
-               "l"(src), "r"(bytes), "r"(smem_u32(bar))
-               : "memory");
-}
-
-__device__ __forceinline__ void pair_filter_bulk(const PairParams& p, uint8_t* sF, uint8_t* stage, uint64_t* fb,
-                                                 uint32_t rank) {
-  const int half = p.NN / 2, kb = (int)rank * half;
-  const int ncg = p.Cp / 8;
-  const uint32_t rowb = (uint32_t)p.C * p.RS * 2u;  // bytes of one w row (bf16)
-  const uint32_t slab = (uint32_t)p.frows * rowb;
-  const int nslab = (half + p.frows - 1) / p.frows;
-  const uint32_t M = (uint32_t)p.row_bytes / 16u - 1u;
-  const __nv_bfloat16* w = static_cast<const __nv_bfloat16*>(p.w);
-  auto issue = [&](int sl) {
-    const int k0 = kb + sl * p.frows;
-    const int nk = min(p.frows, p.K - k0);
-    if (nk <= 0) return;
-    uint8_t* dst = stage + (size_t)(sl & 1) * slab;
-    mbar_arrive_expect_tx(fb + (sl & 1), (uint32_t)nk * rowb);
-    for (int r = 0; r < nk; ++r)
-      bulk_g2s(smem_u32(dst + (size_t)r * rowb), w + (size_t)(k0 + r) * p.C * p.RS, rowb, fb + (sl & 1));
-  };
-  if (threadIdx.x == 0) {
-    issue(0);
-    if (nslab > 1) issue(1);
-  }
-  for (int sl = 0; sl < nslab; ++sl) {
-    const int k0 = kb + sl * p.frows;
-    const int nk_valid = max(0, min(p.frows, p.K - k0));
-    if (nk_valid > 0) mbar_wait(fb + (sl & 1), (uint32_t)((sl >> 1) & 1));
-    const uint8_t* src = stage + (size_t)(sl & 1) * slab;
-    const int rows = min(p.frows, half - sl * p.frows);
-    for (int it = threadIdx.x; it < rows * ncg; it += blockDim.x) {
-      const int r = it / ncg, cg = it - (it / ncg) * ncg;
-      const int kl = sl * p.frows + r, k = kb + kl, c0 = cg * 8;
-      const int ch = c0 / p.kc, j = (c0 - ch * p.kc) >> 3;
-      const uint32_t o = (uint32_t)kl * (uint32_t)p.row_bytes + (uint32_t)j * 16u;
-      uint8_t* dst = sF + (size_t)(ch * p.RS) * p.fbytes + (o ^ (((o >> 7) & M) << 4));
-      const uint16_t* row = reinterpret_cast<const uint16_t*>(src + (size_t)r * rowb);
-      if (p.RS == 9 && k < p.K && c0 + 8 <= p.C) {
-        const uint4* v4 = reinterpret_cast<const uint4*>(row + c0 * 9);
-        uint32_t e[36];
-#pragma unroll
-        for (int q = 0; q < 9; ++q) {
-          const uint4 v = v4[q];
-          e[4 * q] = v.x; e[4 * q + 1] = v.y; e[4 * q + 2] = v.z; e[4 * q + 3] = v.w;
-        }
-#pragma unroll
-        for (int t = 0; t < 9; ++t) {
-          uint32_t out[4];
-#pragma unroll
-          for (int m = 0; m < 4; ++m) {
-            const int i0 = (2 * m) * 9 + t, i1 = (2 * m + 1) * 9 + t;
-            out[m] = ((e[i0 >> 1] >> ((i0 & 1) * 16)) & 0xFFFFu) | (((e[i1 >> 1] >> ((i1 & 1) * 16)) & 0xFFFFu) << 16);
-          }
-          *reinterpret_cast<uint4*>(dst + (size_t)t * p.fbytes) = make_uint4(out[0], out[1], out[2], out[3]);
-        }
-      } else {
-        for (int t = 0; t < p.RS; ++t) {
-          uint32_t out[4];
-#pragma unroll
-          for (int m = 0; m < 4; ++m) {
-            const int c = c0 + 2 * m;
-            const uint32_t lo = (k < p.K && c < p.C) ? (uint32_t)row[c * p.RS + t] : 0u;
-            const uint32_t hi = (k < p.K && c + 1 < p.C) ? (uint32_t)row[(c + 1) * p.RS + t] : 0u;
-            out[m] = lo | (hi << 16);
-          }
-          *reinterpret_cast<uint4*>(dst + (size_t)t * p.fbytes) = make_uint4(out[0], out[1], out[2], out[3]);
-        }
-      }
-    }
-    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // staging reads -> next bulk copy
-    __syncthreads();
-    if (threadIdx.x == 0 && sl + 2 < nslab) issue(sl + 2);
-  }
-}
-
-// Publish band u of this launch (epoch): its A rows are in global memory.
-__device__ __forceinline__ void publish_band(const PairParams& p, int u) {
-  asm volatile("fence.proxy.async.global;" ::: "memory");  // TMA-stored rows -> generic release
-  __threadfence();
-  asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p.bflag + u), "l"(p.epoch) : "memory");
-}
-
-// x-box bx (64 channel planes) of the band of unit u: TMA load, 16-byte aligned start
-template <typename IoT>
 __device__ __forceinline__ void pack_load(const PairParams& p, const CUtensorMap* tmX, uint8_t* stage,
                                           uint64_t* pbar, int u, int bx) {
   const int n = p.u_img0 + u / p.nb, b = u - (u / p.nb) * p.nb;
@@ -583,65 +423,12 @@ __device__ __forceinline__ void pair_pack_x_tma(const PairParams& p, uint8_t* st
     }
     if (tid == 0) {
       asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");  // written (before publishing / reuse)
-      if (!p.split) publish_band(p, u);
       if (ptr) g_pair_pk[blockIdx.x * 4 + 2] = global_ns();
     }
     __syncthreads();
   }
 }
 
-// direct0: the x rows of this CTA's first tile, one TMA box per 64-channel chunk
-// (start rounded down to 16 bytes), into the staging at sF + w0_off
-template <typename IoT>
-__device__ __forceinline__ void w0_load(const PairParams& p, const CUtensorMap* tmX0, uint8_t* stage,
-                                        uint64_t* bar, int tn, int h0w, int c) {
-  const uint32_t bytes = 64u * p.ne_w * (uint32_t)sizeof(IoT);
-  mbar_arrive_expect_tx(bar, bytes);
-  tma_load_2d(stage + (size_t)c * bytes, tmX0, bar, (h0w * p.W) & ~(16 / (int)sizeof(IoT) - 1), tn * p.C + c * 64);
-}
-
-// direct0: window slot c of the first tile = rows m of the interleaved input polynomial
-// from coefficient g0 = tn*L_A + r_lo*Wp on (Eq. 10: coefficient r*Wp + s of A_{n,c}(t)
-// is xpad[n][c][r][s]), 64 channel words per row, 128-byte swizzled exactly as the TMA
-// writes a window; rows past the image (junk positions) are zero.
-template <typename IoT>
-__device__ __forceinline__ void w0_gather(const PairParams& p, const uint8_t* stage, uint8_t* slot, int r_lo, int h0w,
-                                          int c) {
-  const IoT* in = reinterpret_cast<const IoT*>(stage + (size_t)c * 64u * p.ne_w * sizeof(IoT));
-  const int eoff = (h0w * p.W) & (16 / (int)sizeof(IoT) - 1);
-  const int rows = p.nbox * p.box_rows;
-  const int cbase = c * 64;
-  for (int m = threadIdx.x; m < rows; m += blockDim.x) {
-    const int rr = (int)p.fWp.div((uint32_t)m);
-    const int r = r_lo + rr, h = r - p.ph, ww = m - rr * p.Wp - p.pw;
-    uint8_t* drow = slot + (size_t)m * 128;
-    const uint32_t sw = (uint32_t)(m & 7);
-    if (r < p.Hp && h >= 0 && h < p.H && ww >= 0 && ww < p.W) {
-      const IoT* src = in + (h - h0w) * p.W + ww + eoff;
-#pragma unroll
-      for (int q8 = 0; q8 < 8; ++q8) {
-        const int c0 = cbase + q8 * 8;
-        uint32_t v[4];
-#pragma unroll
-        for (int mm = 0; mm < 4; ++mm) {
-          const int cc = c0 + 2 * mm;
-          const uint32_t lo = cc < p.C ? (uint32_t)to_bf16_bits<IoT>(src[(q8 * 8 + 2 * mm) * p.ne_w]) : 0u;
-          const uint32_t hi = cc + 1 < p.C ? (uint32_t)to_bf16_bits<IoT>(src[(q8 * 8 + 2 * mm + 1) * p.ne_w]) : 0u;
-          v[mm] = lo | (hi << 16);
-        }
-        *reinterpret_cast<uint4*>(drow + (((uint32_t)q8 ^ sw) << 4)) = make_uint4(v[0], v[1], v[2], v[3]);
-      }
-    } else {
-#pragma unroll
-      for (int q8 = 0; q8 < 8; ++q8)
-        *reinterpret_cast<uint4*>(drow + (((uint32_t)q8 ^ sw) << 4)) = make_uint4(0u, 0u, 0u, 0u);
-    }
-  }
-}
-
-// a2 + a3 as their own grid (split mode): every CTA packs a slice of the tap-major
-// filter U and one band of A (TMA in, transpose, TMA store); the pair kernel is its
-// programmatic dependent and starts its prologue as soon as every CTA here has begun.
 template <typename IoT>
 __global__ void __launch_bounds__(256) pair_pack_kernel(const __grid_constant__ CUtensorMap tmX,
                                                         const __grid_constant__ CUtensorMap tmS,
@@ -699,7 +486,7 @@ __global__ void __launch_bounds__(kPairThreads, 1)
     mac_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmU,
                     const __grid_constant__ CUtensorMap tmX, const __grid_constant__ CUtensorMap tmS,
                     const __grid_constant__ CUtensorMap tmS2, const __grid_constant__ CUtensorMap tmY,
-                    const __grid_constant__ CUtensorMap tmX0, const PairParams p) {
+                    const PairParams p) {
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw = smem_u32(smem_raw);
   uint8_t* smem = smem_raw + (((raw + 1023u) & ~1023u) - raw);
@@ -725,7 +512,6 @@ __global__ void __launch_bounds__(kPairThreads, 1)
     tr[0] = global_ns();
     g_pair_clk[blockIdx.x * 2] = clock64();
   }
-  if (p.dbg & 32) return;  // timing experiment: launch + teardown cost of this configuration
 
   if (warp == 0 && lane == 0) {
     prefetch_tmap(&tmA);
@@ -753,94 +539,7 @@ __global__ void __launch_bounds__(kPairThreads, 1)
     }
   }
   __syncthreads();  // pbar initialised
-  if (p.warm) {
-    // Warm-up: one chunk of MMAs on whatever shared memory holds, into accumulator 1
-    // (the first tile that uses it starts with accumulate = 0), so the issue path is
-    // fetched and the tensor pipe started while the packing runs.  The pair's TMEM
-    // must be allocated in both CTAs first.
-    tc_fence_before();
-    cluster_sync();
-    tc_fence_after();
-    if (warp == 1 && rank == 0)
-      issue_chunk(*tmem_slot + (uint32_t)p.NN, make_sdesc(smem_u32(sWin), (uint32_t)p.row_bytes, 0),
-                  make_sdesc(smem_u32(sF), (uint32_t)p.row_bytes, 0), mtab, p.RS, p.row_bytes / 32, p.idesc, 0u);
-  }
 
-  // phase 1: packing (all warps); the window ring and filter area are the staging buffer.
-  // The filter slices meet on the grid counter *fcount; every band of A is published
-  // on its own flag, so a tile's window waits only for the bands it reads.
-  if (p.fsmem == 2 && threadIdx.x == 0) {
-    // w (read by every CTA later) into L2 now: each CTA prefetches one slice
-    const size_t wb = (size_t)p.K * p.C * p.RS * 2;
-    const size_t per = ((wb + gridDim.x - 1) / gridDim.x + 15) & ~(size_t)15;
-    const size_t off = (size_t)blockIdx.x * per;
-    if (off < wb) {
-      const uint32_t n = (uint32_t)min(per, wb - off);
-      asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(static_cast<const char*>(p.w) + off), "r"(n)
-                   : "memory");
-    }
-  }
-  if (!p.split) {
-  // direct0: this CTA's first tile (CTA tile blockIdx.x) and the padded rows its windows read
-  const int w0_tn = (int)p.ftpi.div((uint32_t)blockIdx.x);
-  const int w0_rlo = ((int)blockIdx.x - w0_tn * p.tpi) * p.tr * p.sh;
-  const int w0_h0 = min(max(w0_rlo - p.ph, 0), p.H);
-  const bool w0_any = p.direct0 && (int)blockIdx.x < p.ntile && !(p.dbg & 2);
-  if (w0_any && threadIdx.x == 0) {
-    prefetch_tmap(&tmX0);
-    for (int c = 0; c < p.nchunks; ++c) w0_load<IoT>(p, &tmX0, sF + p.w0_off, pbar + 2 + c, w0_tn, w0_h0, c);
-  }
-  if (p.pack_tma) {
-    // the first band's input boxes fly while the filter is packed
-    const bool first = (int)blockIdx.x < p.nunits;
-    if (threadIdx.x == 0 && first && !(p.dbg & 2)) {
-      const int u = (int)blockIdx.x;
-      const int n = p.u_img0 + u / p.nb, b = u - (u / p.nb) * p.nb;
-      const int r0 = b * p.rb, r1 = min(p.Hp, r0 + p.rb);
-      const int h0 = min(max(r0 - p.ph, 0), p.H), h1 = min(max(r1 - p.ph, 0), p.H);
-      if (h1 > h0) {
-        prefetch_tmap(&tmX);
-        for (int bx = 0; bx < p.Cp / 64; ++bx) pack_load<IoT>(p, &tmX, sF, pbar, u, bx);
-      }
-    }
-    if (!p.fsmem) {
-      if (!(p.dbg & 2)) pair_pack<IoT>(p, nullptr, false);  // dbg&2: no packing (timing experiments only)
-      __syncthreads();
-      if (threadIdx.x == 0) {
-        __threadfence();
-        atomicAdd(p.fcount, 1ull);
-      }
-    }
-    if (p.direct0) {
-      // the first tile's windows, straight into window slots 0 .. nchunks-1
-      for (int c = 0; c < p.nchunks; ++c) {
-        if (w0_any) mbar_wait(pbar + 2 + c, 0u);
-        w0_gather<IoT>(p, sF + p.w0_off, sWin + (size_t)c * p.wbytes, w0_any ? w0_rlo : p.Hp, w0_h0, c);
-      }
-      if (trace && threadIdx.x == 0) g_pair_pk[blockIdx.x * 4 + 3] = global_ns();
-    }
-    pair_pack_x_tma<IoT>(p, sF, pbar, &tmX, &tmS, &tmS2, first);
-    if (p.fsmem) {
-      __syncthreads();  // the staging (filter area) is free: the bands' stores were read
-      if constexpr (std::is_same<IoT, __nv_bfloat16>::value) {
-        if (p.fsmem == 2) pair_filter_bulk(p, sF, sWin, pbar + 4, rank);
-        else pair_filter_smem<IoT>(p, sF, rank);
-      } else {
-        pair_filter_smem<IoT>(p, sF, rank);
-      }
-      if (trace && threadIdx.x == 0) g_pair_pk[blockIdx.x * 4] = global_ns();
-    }
-  } else {
-    if (!(p.dbg & 2)) pair_pack<IoT>(p, reinterpret_cast<uint16_t*>(sF), true);
-    __syncthreads();
-    if (threadIdx.x == 0) {
-      __threadfence();
-      atomicAdd(p.fcount, 1ull);
-      for (int u = blockIdx.x; u < p.nunits; u += gridDim.x)
-        asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p.bflag + u), "l"(p.epoch) : "memory");
-    }
-  }
-  }  // !split
   // the staging area is overwritten by TMA (async proxy) next
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
   __syncthreads();
@@ -857,39 +556,13 @@ __global__ void __launch_bounds__(kPairThreads, 1)
     const uint32_t lead_ffull = mapa_rank0(smem_u32(ffull));
     const uint32_t sW0 = smem_u32(sWin), sF0 = smem_u32(sF);
     const int half = p.NN / 2;
-    if (p.split) {
-      // the pack kernel (the programmatic-launch primary) has written A and U
-      asm volatile("griddepcontrol.wait;" ::: "memory");
-      asm volatile("fence.proxy.async.global;" ::: "memory");
-      if (trace && lane == 0) tr[2] = global_ns();
-    }
-    if (lane == 0 && !p.fsmem && !p.split) {
-      // every CTA's slice of the packed filter is in global memory
-      unsigned long long v;
-      uint64_t t0 = 0;
-      for (;;) {
-        asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p.fcount) : "memory");
-        if (v >= p.ftarget) break;
-        const uint64_t t = global_ns();
-        if (t0 == 0) t0 = t;
-      }
-      asm volatile("fence.proxy.async.global;" ::: "memory");  // generic writes -> TMA reads
-      if (trace) tr[2] = global_ns();
-      // dbg&64: the whole filter half right away (default: each chunk's blocks after
-      // its first window, so that the window is not queued behind them)
-      if ((p.dbg & 64) && pair < p.num_tiles) {
-        for (int blk = 0; blk < p.nblk; ++blk) {
-          const int ch = blk / p.RS, tap = blk - ch * p.RS;
-          if (rank == 0) mbar_arrive_expect_tx(ffull + blk, 2u * p.fbytes);
-          tma_load_2d_pair(sF0 + (uint32_t)blk * p.fbytes, &tmU, lead_ffull + 8u * (uint32_t)blk, ch * p.kc,
-                           tap * p.NN + (int)rank * half + (pair % p.urep) * p.RS * p.NN);
-        }
-      }
-    }
+    // the pack kernel (the programmatic-launch primary) has written A and U
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    asm volatile("fence.proxy.async.global;" ::: "memory");
+    if (trace && lane == 0) tr[2] = global_ns();
     __syncwarp();
-    // the first chunk's filter blocks go out before the first window's band wait (they
-    // depend only on the grid counter; measured +4%); dbg&4096 disables it
-    const bool f0_early = !(p.dbg & 4096) && !p.fsmem && !(p.dbg & 64) && pair < p.num_tiles;
+    // the first chunk's filter blocks go out before the first window (measured +4%)
+    const bool f0_early = pair < p.num_tiles;
     if (f0_early && elect_one()) {
       for (int tap = 0; tap < p.RS; ++tap) {
         if (rank == 0) mbar_arrive_expect_tx(ffull + tap, 2u * p.fbytes);
@@ -907,40 +580,14 @@ __global__ void __launch_bounds__(kPairThreads, 1)
       const int ct = 2 * t + (int)rank;
       const int tn = (int)p.ftpi.div((uint32_t)ct), tb = ct - tn * p.tpi;
       const int g0 = tn * (int)p.L_A + tb * p.tr * p.sh * p.Wp;
-      const bool direct = p.direct0 && lt == 0;  // windows already in shared memory (phase 1)
-      if (tn < p.N && !direct && !p.split) {
-        // the bands of image tn this tile's windows read (rows past the image are junk);
-        // lane i polls band b_lo + i, so the flags' round trips overlap
-        const int r_lo = tb * p.tr * p.sh, r_hi = min(p.Hp - 1, r_lo + wrows_img);
-        const int b_lo = r_lo / p.rb, nbw = r_hi / p.rb - b_lo + 1;
-        uint64_t t0 = 0;
-        for (int b0 = 0; b0 < nbw; b0 += 32) {
-          bool done = b0 + lane >= nbw;
-          const unsigned long long* f = p.bflag + (tn - p.u_img0) * p.nb + b_lo + b0 + lane;
-          while (!__all_sync(0xffffffffu, done)) {
-            if (!done) {
-              unsigned long long v;
-              asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(f) : "memory");
-              done = v >= p.epoch;
-            }
-            const uint64_t tt = global_ns();
-            if (t0 == 0) t0 = tt;
-          }
-        }
-        asm volatile("fence.acq_rel.gpu;" ::: "memory");   // acquire the bands' rows
-        asm volatile("fence.proxy.async.global;" ::: "memory");  // ... for the TMA reads
-        if (trace && lt == 0 && lane == 0) tr[14] = global_ns();
-      }
       __syncwarp();
       for (int ci = 0; ci < p.nchunks; ++ci, ++wi) {
         // one fixed (chunk, tap) order everywhere: every output sees the same
         // accumulation order whatever tile or batch it is computed in (reading R12)
         const int ch = ci;
         const int slot = wi % p.ring;
-        mbar_wait_cl(wempty + slot, (uint32_t)((wi / p.ring) & 1) ^ 1u, (p.dbg & 16) ? 500u : 0u);
-        if (direct) {
-          if (elect_one() && rank == 0) mbar_arrive(wfull + slot);  // built in phase 1 (cluster barrier since)
-        } else if (elect_one()) {
+        mbar_wait_cl(wempty + slot, (uint32_t)((wi / p.ring) & 1) ^ 1u);
+        if (elect_one()) {
           if (rank == 0) mbar_arrive_expect_tx(wfull + slot, 2u * p.wbytes_tx);
           for (int b = 0; b < p.nbox; ++b)
             tma_load_2d_pair(sW0 + (uint32_t)slot * p.wbytes + (uint32_t)(b * p.box_rows * p.row_bytes), &tmA,
@@ -948,13 +595,9 @@ __global__ void __launch_bounds__(kPairThreads, 1)
         }
         __syncwarp();
         if (elect_one()) {
-          if (lt == 0 && !(p.dbg & 64) && !p.fsmem && !(f0_early && ci == 0)) {  // this chunk's filter blocks
+          if (lt == 0 && !(f0_early && ci == 0)) {  // this chunk's filter blocks
             for (int tap = 0; tap < p.RS; ++tap) {
               const int blk = ch * p.RS + tap;
-              if ((p.dbg & 256) && (blk & 1)) {  // timing experiment: half the filter traffic (wrong results)
-                if (rank == 0) mbar_arrive(ffull + blk);
-                continue;
-              }
               if (rank == 0) mbar_arrive_expect_tx(ffull + blk, 2u * p.fbytes);
               tma_load_2d_pair(sF0 + (uint32_t)blk * p.fbytes, &tmU, lead_ffull + 8u * (uint32_t)blk, ch * p.kc,
                                tap * p.NN + (int)rank * half + (pair % p.urep) * p.RS * p.NN);
@@ -973,23 +616,16 @@ __global__ void __launch_bounds__(kPairThreads, 1)
       int wi = 0, lt = 0;
       for (int t = pair; t < p.num_tiles; t += p.num_pairs, ++lt) {
         const int a = lt & 1;
-        if (!(p.dbg & 4)) mbar_wait_cl(tempty + a, (uint32_t)((lt >> 1) & 1) ^ 1u);  // dbg&4: no waits (timing)
+        mbar_wait_cl(tempty + a, (uint32_t)((lt >> 1) & 1) ^ 1u);
         tc_fence_after();
         const uint32_t d_tmem = tmem_base + (uint32_t)(a * p.NN);
-        if (lt == 0 && (p.dbg & 1024) && !p.fsmem) {
-          // timing experiment: the whole first tile's operands resident before any MMA
-          // (TMA writes into shared memory are starved while the MMAs read it)
-          for (int b = 0; b < p.nblk; ++b) mbar_wait_cl(ffull + b, 0u);
-          for (int c = 0; c < p.nchunks && c < p.ring; ++c) mbar_wait_cl(wfull + c, 0u);
-          tc_fence_after();
-        }
         for (int ci = 0; ci < p.nchunks; ++ci, ++wi) {
           const int ch = ci;  // the producer's order
           const int slot = wi % p.ring;
-          if (!(p.dbg & 4)) mbar_wait_cl(wfull + slot, (uint32_t)((wi / p.ring) & 1));
+          mbar_wait_cl(wfull + slot, (uint32_t)((wi / p.ring) & 1));
           tc_fence_after();
           if (trace && lane == 0 && wi < 4) tr[3 + wi] = global_ns();
-          if (lt == 0 && !(p.dbg & 4) && !p.fsmem) {  // this chunk's filter blocks (first tile only; then resident)
+          if (lt == 0) {  // this chunk's filter blocks (first tile only; then resident)
             for (int tap = 0; tap < p.RS; ++tap) mbar_wait_cl(ffull + ch * p.RS + tap, 0u);
             tc_fence_after();
             if (trace && lane == 0 && ci == p.nchunks - 1) tr[12] = global_ns();
@@ -1017,7 +653,7 @@ __global__ void __launch_bounds__(kPairThreads, 1)
     int lt = 0;
     for (int t = pair; t < p.num_tiles; t += p.num_pairs, ++lt) {
       const int a = lt & 1;
-      mbar_wait_cl(tfull + a, (uint32_t)((lt >> 1) & 1), (p.dbg & 16) ? 1000u : 64u);
+      mbar_wait_cl(tfull + a, (uint32_t)((lt >> 1) & 1), 64u);
       tc_fence_after();
       if (trace && threadIdx.x == kEpi0 * 32 && lt < 2) tr[9 + 2 * lt] = global_ns();
       // this lane's position m (tile-relative coefficient) -> output pixel (Eq. 12 with
@@ -1203,11 +839,7 @@ PairTiling pair_tiling(const Geom& g, int fmt, bool io_bf16, int num_sms) {
   t.nb = (int)cdivp(g.Hp, t.rb);
   t.nunits = g.N * t.nb;
   // TMA pack path: x band by one TMA box, A rows out by TMA stores (64-channel SW128 boxes).
-  // direct0: the first round of tiles builds its windows in shared memory from x, so A is
-  // packed only for the images of later tiles (from u_img0 on), and the band staging
-  // shares the filter area with the first tile's x boxes.
   t.pack_tma = 0;
-  t.direct0 = 0;
   t.u_img0 = 0;
   {
     const int eb_in = io_bf16 ? 2 : 4;
@@ -1215,20 +847,14 @@ PairTiling pair_tiling(const Geom& g, int fmt, bool io_bf16, int num_sms) {
     const int rb_cap = std::min(256 / g.Wp, 256 / g.W);
     const bool tma_ok = t.Cp % 64 == 0 && t.Cp <= 256 && ((long long)g.H * g.W * eb_in) % 16 == 0 &&
                         !getenv("POLYCONV_PAIR_PACK_LD");
-    // the first tile's x rows: padded rows [r_lo, r_lo + rows_w) -> one box of ne_w elements
-    const int rows_w = (int)cdivp((long long)t.nbox * t.box_rows, g.Wp) + 1;
-    const int ne_w = (int)cdivp((long long)rows_w * g.W + ve - 1, ve) * ve;
-    const long long w0_b = (long long)t.nchunks * 64 * ne_w * eb_in;
-    const bool want_d0 = tma_ok && t.nchunks <= 2 && t.ring >= t.nchunks && ne_w <= 256 &&
-                         getenv("POLYCONV_PAIR_DIRECT0");  // measured no faster (filter waits for phase 1)
-    for (int d0 = want_d0 ? 1 : 0; d0 >= 0 && !t.pack_tma; --d0) {
-      const int img0 = d0 ? std::min(g.N, (2 * t.num_pairs) / t.tpi) : 0;
-      const int nimg = g.N - img0;
+    {
+      const int img0 = 0;
+      const int nimg = g.N;
       int nb2 = std::max(1, nimg > 0 ? t.grid / nimg : 1);
       if (nb2 > g.Hp) nb2 = g.Hp;
       int rb2 = (int)cdivp(g.Hp, nb2);
       if (rb2 > rb_cap) rb2 = rb_cap;
-      if (rb2 < 1 || !tma_ok) continue;
+      if (rb2 < 1 || !tma_ok) goto no_tma;
       const int nbb = (int)cdivp(g.Hp, rb2);
       const int last = g.Hp - (nbb - 1) * rb2;
       const int ne_box = (int)cdivp((long long)rb2 * g.W + ve - 1, ve) * ve;  // + the start's rounding
@@ -1236,17 +862,9 @@ PairTiling pair_tiling(const Geom& g, int fmt, bool io_bf16, int num_sms) {
       const long long ob = cdivp((long long)rb2 * g.Wp * 128, 1024) * 1024;
       const long long ob2 = cdivp((long long)last * g.Wp * 128, 1024) * 1024;
       const long long band_b = in_b + (long long)(t.Cp / 64) * std::max(ob, ob2);
-      if (ne_box > 256) continue;
-      if (d0) {
-        if (band_b + w0_b > fil) continue;  // both in the filter area (free during packing)
-      } else if (band_b > stage_cap) {
-        continue;
-      }
+      if (ne_box > 256 || band_b > stage_cap) goto no_tma;
       t.pack_tma = 1;
-      t.direct0 = d0;
       t.u_img0 = img0;
-      t.ne_w = ne_w;
-      t.w0_off = (int)band_b;
       t.rb = rb2;
       t.nb = nbb;
       t.nunits = nimg * nbb;
@@ -1256,6 +874,7 @@ PairTiling pair_tiling(const Geom& g, int fmt, bool io_bf16, int num_sms) {
       t.obox_bytes = (int)ob;
       t.obox_bytes2 = (int)ob2;
     }
+  no_tma:;
   }
   // split: the packing runs as its own grid (pair_pack_kernel, several CTAs per SM,
   // small bands), the pair kernel follows it as a programmatic dependent launch.  This is
@@ -1263,7 +882,7 @@ PairTiling pair_tiling(const Geom& g, int fmt, bool io_bf16, int num_sms) {
   // needed the whole grid co-resident and broke on CUDA-graph replay (the counters only
   // grew while the targets were baked into the captured launch); split measured 2% slower.
   t.split = 0;
-  if (t.pack_tma && !t.direct0) {
+  if (t.pack_tma) {
     const int eb_in = io_bf16 ? 2 : 4;
     const int ve = 16 / eb_in;
     const int rb_cap = std::min(256 / g.Wp, 256 / g.W);
@@ -1297,21 +916,18 @@ PairTiling pair_tiling(const Geom& g, int fmt, bool io_bf16, int num_sms) {
 }
 
 namespace {
-// Everything a launch needs except the grid-counter target, built once per
-// (x, w, y, workspace) pointer set: the host path of a repeated forward is one
-// cudaLaunchKernelEx (tensor-map encoding and the co-residency check cost
-// microseconds that an idle stream would wait for).
+// Everything a launch needs, built once per (x, w, y, workspace) pointer set: the host path
+// of a repeated forward is two cudaLaunchKernelEx calls (tensor-map encoding and the
+// cluster-occupancy check cost microseconds that an idle stream would wait for).
 struct PairLaunchState {
   const void *x = nullptr, *w = nullptr, *y = nullptr, *A = nullptr, *U = nullptr;
-  const unsigned long long* fcount = nullptr;
   bool io_bf16 = false, valid = false;
-  CUtensorMap tmA, tmU, tmX, tmS, tmS2, tmY, tmX0;
+  CUtensorMap tmA, tmU, tmX, tmS, tmS2, tmY;
   PairParams p;
 };
 
 cudaError_t prepare_mac_pair(PairLaunchState& S, const Geom& g, const PairTiling& t, const void* x, const void* w,
-                             bool io_bf16, void* A, void* U, void* y, unsigned long long* fcount, char* err,
-                             size_t errlen) {
+                             bool io_bf16, void* A, void* U, void* y, char* err, size_t errlen) {
   S.valid = false;
   CUtensorMap& tmA = S.tmA;
   CUtensorMap& tmU = S.tmU;
@@ -1359,43 +975,16 @@ cudaError_t prepare_mac_pair(PairLaunchState& S, const Geom& g, const PairTiling
       return cudaErrorInvalidValue;
     }
   }
-  CUtensorMap& tmX0 = S.tmX0;
-  memset(&tmX0, 0, sizeof(tmX0));
-  if (t.direct0) {
-    EncodeTiledFnPair enc = get_encode_pair();
-    const int eb_in = io_bf16 ? 2 : 4;
-    cuuint64_t dims[2] = {(cuuint64_t)g.H * g.W, (cuuint64_t)g.N * g.C};
-    cuuint64_t strides[1] = {(cuuint64_t)g.H * g.W * eb_in};
-    cuuint32_t box[2] = {(cuuint32_t)t.ne_w, 64};
-    cuuint32_t estr[2] = {1, 1};
-    if (!enc || enc(&tmX0, io_bf16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2,
-                    const_cast<void*>(x), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                    CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS) {
-      snprintf(err, errlen, "mac_pair: cuTensorMapEncodeTiled (first-tile input) failed");
-      return cudaErrorInvalidValue;
-    }
-  }
   PairParams& p = S.p;
   p = PairParams{};
   p.x = x; p.w = w; p.A = A; p.U = U; p.y = y;
   p.tr = t.tr; p.tpi = t.tpi; p.ntile = t.ntile; p.epi_tma = t.epi_tma;
-  p.warm = getenv("POLYCONV_PAIR_WARM") ? atoi(getenv("POLYCONV_PAIR_WARM")) : 0;
-  p.direct0 = t.direct0; p.ne_w = t.ne_w; p.u_img0 = t.u_img0; p.w0_off = (uint32_t)t.w0_off;
+  p.u_img0 = t.u_img0;
   p.split = t.split;
-  p.fsmem = (t.pack_tma && getenv("POLYCONV_PAIR_FSMEM")) ? atoi(getenv("POLYCONV_PAIR_FSMEM")) : 0;
-  {
-    // bulk-copied w slabs: two buffers of frows rows in the window ring + epilogue area
-    const long long rowb = (long long)g.C * g.R * g.S * 2;
-    const long long avail = (long long)t.ring * t.wbytes + t.estage_bytes;
-    p.frows = (int)std::min<long long>(32, avail / (2 * rowb));
-    if (p.fsmem == 2 && (!io_bf16 || p.frows < 1 || rowb % 16 != 0)) p.fsmem = 1;
-  }
   p.estage_bytes = (uint32_t)t.estage_bytes;
   p.ftpi.init((uint32_t)t.tpi);
   p.pack_tma = t.pack_tma; p.ne_box = t.ne_box; p.last_rows = t.last_rows;
   p.in_bytes = (uint32_t)t.in_bytes; p.obox_bytes = (uint32_t)t.obox_bytes; p.obox_bytes2 = (uint32_t)t.obox_bytes2;
-  p.fcount = fcount; p.ftarget = 0;
   p.L_A = g.L_A;
   p.G = (long long)(g.N - 1) * g.L_A + g.M_ext;
   p.NLA = (long long)g.N * g.L_A;
@@ -1442,7 +1031,7 @@ cudaError_t prepare_mac_pair(PairLaunchState& S, const Geom& g, const PairTiling
     return cudaErrorInvalidConfiguration;
   }
   cudaGetLastError();
-  S.x = x; S.w = w; S.y = y; S.A = A; S.U = U; S.fcount = fcount; S.io_bf16 = io_bf16;
+  S.x = x; S.w = w; S.y = y; S.A = A; S.U = U; S.io_bf16 = io_bf16;
   S.valid = true;
   return cudaSuccess;
 }
@@ -1452,23 +1041,18 @@ void* pair_state_new() { return new (std::nothrow) PairLaunchState(); }
 void pair_state_free(void* s) { delete static_cast<PairLaunchState*>(s); }
 
 cudaError_t launch_mac_pair(const Geom& g, const PairTiling& t, const void* x, const void* w, bool io_bf16,
-                            void* A, void* U, void* y, unsigned long long* fcount, unsigned long long ftarget,
-                            unsigned long long* bflag, unsigned long long epoch, cudaStream_t st, char* err,
-                            size_t errlen, void* state) {
+                            void* A, void* U, void* y, cudaStream_t st, char* err, size_t errlen, void* state) {
   if (!t.ok) {
     snprintf(err, errlen, "mac_pair: shape not supported");
     return cudaErrorInvalidValue;
   }
   PairLaunchState local;
   PairLaunchState& S = state ? *static_cast<PairLaunchState*>(state) : local;
-  if (!S.valid || S.x != x || S.w != w || S.y != y || S.A != A || S.U != U || S.fcount != fcount ||
+  if (!S.valid || S.x != x || S.w != w || S.y != y || S.A != A || S.U != U ||
       S.io_bf16 != io_bf16) {
-    cudaError_t e = prepare_mac_pair(S, g, t, x, w, io_bf16, A, U, y, fcount, err, errlen);
+    cudaError_t e = prepare_mac_pair(S, g, t, x, w, io_bf16, A, U, y, err, errlen);
     if (e != cudaSuccess) return e;
   }
-  S.p.ftarget = ftarget;
-  S.p.bflag = bflag;
-  S.p.epoch = epoch;
   const char* dbg = getenv("POLYCONV_PAIR_DEBUG");
   S.p.dbg = dbg ? atoi(dbg) : 0;
   if (t.split) {
@@ -1496,7 +1080,7 @@ cudaError_t launch_mac_pair(const Geom& g, const PairTiling& t, const void* x, c
   attr[1].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   cfg.numAttrs = t.split ? 2 : 1;
-  return cudaLaunchKernelEx(&cfg, kern, S.tmA, S.tmU, S.tmX, S.tmS, S.tmS2, S.tmY, S.tmX0, S.p);
+  return cudaLaunchKernelEx(&cfg, kern, S.tmA, S.tmU, S.tmX, S.tmS, S.tmS2, S.tmY, S.p);
 }
 
 }  // namespace polyconv

@@ -29,7 +29,6 @@ struct polyconv_plan_s {
   bool fft_tw_ready = false;  // twiddles computed into wsU
   void* hkzero = nullptr;  // mac_hankel: zero words read in place of padding (hankel_zero_bytes)
   void* pair_state = nullptr;  // mac_pair launch cache
-  unsigned long long* bflag = nullptr;  // mac_pair band flags [N * pair.nb]
   // stride s >= 2 (reading R4b): the stride-1 inner plan over the input's s*s phases
   polyconv_plan_s* inner = nullptr;
   int Hq = 0, Wq = 0, Rq = 0, Sq = 0;
@@ -59,9 +58,6 @@ struct polyconv_plan_s {
   // polyconv_plan_set_timing_events: recorded around the MAC launch
   cudaEvent_t ev_start = nullptr;
   cudaEvent_t ev_stop = nullptr;
-  // TC_FUSED: the MAC packs the filter in-kernel; its CTAs meet on this counter
-  unsigned long long* fcount = nullptr;
-  unsigned long long fepoch = 0;
   char err[512];
 };
 
@@ -432,7 +428,6 @@ polyconv_status_t polyconv_plan_set_kernel(polyconv_plan_t p, polyconv_kernel_t 
     return POLYCONV_STATUS_BAD_PARAM;
   }
   // workspace sizes (and the grid the pack counter counts) may have changed
-  if (p->fcount) { cudaFree(p->fcount); p->fcount = nullptr; }
   if (p->pair_state) { pair_state_free(p->pair_state); p->pair_state = nullptr; }
   if (p->wsA) { cudaFree(p->wsA); p->wsA = nullptr; }
   if (p->wsU) { cudaFree(p->wsU); p->wsU = nullptr; }
@@ -586,28 +581,12 @@ polyconv_status_t polyconv_forward(polyconv_plan_t p, const void* x, const void*
     return finish(p, e, "mac_1x1");
   }
   if (p->kernel == POLYCONV_KERNEL_TC_PAIR) {
-    // one launch: a3 (filter slices, every CTA; grid counter) + a2 (bands of A, each
-    // published on its own flag), then a4 + a5 on CTA pairs.  All CTAs are co-resident
-    // (checked when the launch is prepared).
-    if (!p->fcount) {
-      const size_t nflag = 1 + (size_t)g.N * p->pair.nb;
-      if (cudaMalloc(&p->fcount, nflag * sizeof(unsigned long long)) != cudaSuccess ||
-          cudaMemsetAsync(p->fcount, 0, nflag * sizeof(unsigned long long), st) != cudaSuccess) {
-        cudaGetLastError();
-        p->fcount = nullptr;
-        set_err(p, "cudaMalloc of the %s failed", "pack counters");
-        return POLYCONV_STATUS_ALLOC_FAILED;
-      }
-      p->bflag = p->fcount + 1;
-      p->fepoch = 0;
-    }
+    // a2 + a3 by the pack grid (pair_pack_kernel), then a4 + a5 on CTA pairs as its
+    // programmatic dependent launch (pair-local synchronisation only)
     if (p->ev_start) cudaEventRecord(p->ev_start, st);
-    const unsigned long long epoch = p->fepoch + 1;
     if (!p->pair_state) p->pair_state = pair_state_new();
-    e = launch_mac_pair(g, p->pair, x, w, p->io_bf16, p->wsA, p->wsU, y, p->fcount,
-                        epoch * (unsigned long long)p->pair.grid, p->bflag, epoch, st, p->err, sizeof(p->err),
+    e = launch_mac_pair(g, p->pair, x, w, p->io_bf16, p->wsA, p->wsU, y, st, p->err, sizeof(p->err),
                         p->pair_state);
-    if (e == cudaSuccess) ++p->fepoch;
     if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
     return finish(p, e, "mac_pair");
   }
@@ -814,7 +793,7 @@ polyconv_status_t polyconv_extract(polyconv_plan_t p, const float* coeffs, void*
 polyconv_status_t polyconv_destroy(polyconv_plan_t p) {
   if (!p) return POLYCONV_STATUS_SUCCESS;
   polyconv_status_t s = POLYCONV_STATUS_SUCCESS;
-  if (p->used || p->wsA || p->wsU || p->hx || p->hw || p->hy || p->fcount || p->hkzero) {
+  if (p->used || p->wsA || p->wsU || p->hx || p->hw || p->hy || p->hkzero) {
     DeviceGuard guard(p->device);
     if (p->used && cudaStreamSynchronize(p->last_stream) != cudaSuccess) {
       cudaGetLastError();
@@ -825,7 +804,6 @@ polyconv_status_t polyconv_destroy(polyconv_plan_t p) {
     if (p->hx) cudaFree(p->hx);
     if (p->hw) cudaFree(p->hw);
     if (p->hy) cudaFree(p->hy);
-    if (p->fcount) cudaFree(p->fcount);
     if (p->hkzero) cudaFree(p->hkzero);
   }
   if (p->pair_state) pair_state_free(p->pair_state);
