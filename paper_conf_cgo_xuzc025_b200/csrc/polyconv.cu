@@ -140,9 +140,12 @@ polyconv_status_t resolve(polyconv_plan_t p) {
   // under a third of a round of units (the synthetic nets at 4x4 / 8x8: 1-11 units; 14x14: 30).
   // The stem (7x7 stride 2, C = 3): its stride-1 phase convolution (reading R19: 12 virtual
   // channels, 4x4 taps) in 32-byte window rows (tools/hk_check.py stem).
-  const bool hk_stem = g.sh == 2 && g.R == 7 && 4 * g.C <= 16 && p->io_bf16;
-  if (k == POLYCONV_KERNEL_AUTO && p->math == POLYCONV_MATH_BF16 && g.K >= 16 && g.sh == g.sw && g.sh <= 2 &&
-      g.R == g.S && (g.R == 3 || g.R == 5 || hk_stem) && !getenv("POLYCONV_NO_HANKEL")) {
+  // TF32 (f32 I/O) takes the same kernel: against mac_tc2 with its pack (tools/kprof.py,
+  // N=256, us) l1 3x3 151 vs 300, l2 121 vs 171, l3 127 vs 151, l4 119 vs 168, l2 s2 406 vs 554,
+  // conv3_x N=32 33 vs 33.
+  const bool hk_stem = g.sh == 2 && g.R == 7 && 4 * g.C <= 16 && p->io_bf16 && p->math == POLYCONV_MATH_BF16;
+  if (k == POLYCONV_KERNEL_AUTO && (p->math == POLYCONV_MATH_BF16 || p->math == POLYCONV_MATH_TF32) && g.K >= 16 &&
+      g.sh == g.sw && g.sh <= 2 && g.R == g.S && (g.R == 3 || g.R == 5 || hk_stem) && !getenv("POLYCONV_NO_HANKEL")) {
     const HankelTiling h = hankel_tiling(g, p->fmt, p->num_sms, p->io_bf16);
     // odd widths use the general (element-load) window loader: it still wins for wide 3x3
     // layers (ResNet-50 l4 7x7, C = K = 512: 596 vs 572 TFLOP/s for mac_tc2)

@@ -80,7 +80,8 @@ def test_kernel_selection_and_forcing():
         pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="tf32", kernel="tc_pair")
     with pytest.raises(pc.PolyconvError):
         pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="fp32", kernel="tc_hankel")
-    assert pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="tf32").info()["kernel"] == "tc"
+    assert pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="tf32").info()["kernel"] == "tc_hankel"
+    assert pc.Plan((1, 64, 10, 10), (320, 64, 3, 3), padding=(1, 1), math="tf32").info()["kernel"] == "tc"
     assert pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="tf32",
                    kernel="tc_hankel").info()["kernel"] == "tc_hankel"
     assert pc.Plan((32, 128, 28, 28), (128, 128, 3, 3), padding=(1, 1), math="fp32").info()["kernel"] == "fp32"
