@@ -343,7 +343,7 @@ __device__ __forceinline__ void hk_load_window(const HkParams& p, uint32_t slot,
 // rows, channels past C) reads the plan's zero buffer through the same channel stride, so no
 // load is predicated and no value masked; kHW2 (the plane size in words, 0 = runtime) makes
 // the eight channel loads one base register plus immediate offsets.
-template <typename IoT, bool kTf32, int kHW2>
+template <typename IoT, bool kTf32, int kHW2, uint32_t kRowB = 128>
 __device__ __forceinline__ void hk_load_window_pairs(const HkParams& p, uint32_t slot, long long q0, int c0, int lw,
                                                      int lane, int rp_lo, int rp_hi) {
   constexpr bool kBf16In = sizeof(IoT) == 2;
@@ -364,8 +364,14 @@ __device__ __forceinline__ void hk_load_window_pairs(const HkParams& p, uint32_t
       if constexpr (kBf16In) {
         const uint32_t* base = e >= 0 ? static_cast<const uint32_t*>(p.x) + (((uint32_t)e >> 1) + cgo)
                                       : static_cast<const uint32_t*>(p.zero);
+        if constexpr (kRowB == 32) {
+          // small C (32-byte rows of 16 channels): channels past C read zeros, not x
 #pragma unroll
-        for (int c = 0; c < CPG; ++c) lo[b][c] = base[c * hw2];
+          for (int c = 0; c < CPG; ++c) lo[b][c] = cg + c < p.C ? base[c * hw2] : 0u;
+        } else {
+#pragma unroll
+          for (int c = 0; c < CPG; ++c) lo[b][c] = base[c * hw2];
+        }
       } else {
         const float2* base = e >= 0 ? static_cast<const float2*>(p.x) + (((uint32_t)e >> 1) + cgo)
                                     : static_cast<const float2*>(p.zero);
@@ -408,8 +414,10 @@ __device__ __forceinline__ void hk_load_window_pairs(const HkParams& p, uint32_t
         const uint32_t ra = 2u * (uint32_t)rp + sel, rb = 2u * (uint32_t)rp + (sel ^ 1u);
         const uint32_t* da = sel ? r1 : r0;
         const uint32_t* db = sel ? r0 : r1;
-        const uint32_t aa = slot + ra * 128u + (((uint32_t)lw ^ (ra & 7u)) << 4);
-        const uint32_t ab = slot + rb * 128u + (((uint32_t)lw ^ (rb & 7u)) << 4);
+        const uint32_t xa = kRowB == 128 ? (ra & 7u) : ((ra >> 2) & 1u);  // SW128 / SW32 chunk swizzle
+        const uint32_t xb = kRowB == 128 ? (rb & 7u) : ((rb >> 2) & 1u);
+        const uint32_t aa = slot + ra * kRowB + (((uint32_t)lw ^ xa) << 4);
+        const uint32_t ab = slot + rb * kRowB + (((uint32_t)lw ^ xb) << 4);
         asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(aa), "r"(da[0]), "r"(da[1]), "r"(da[2]),
                      "r"(da[3])
                      : "memory");
@@ -705,7 +713,7 @@ __global__ void __launch_bounds__(kHkThreads, 1)
             hk_load_window_phase<kHW2 == -2, kRowB>(p, sW + (uint32_t)ws * p.wslot_bytes, q0, ch * kKC, lw, lane,
                                                     rp_lo, rp_hi);
           else if constexpr (kHW2 >= 0)
-            hk_load_window_pairs<IoT, kTf32, kHW2>(p, sW + (uint32_t)ws * p.wslot_bytes, q0, ch * (kTf32 ? 32 : 64), lw,
+            hk_load_window_pairs<IoT, kTf32, kHW2, kRowB>(p, sW + (uint32_t)ws * p.wslot_bytes, q0, ch * kKC, lw,
                                                    lane, rp_lo, rp_hi);
           else
             hk_load_window<IoT, kTf32>(p, sW + (uint32_t)ws * p.wslot_bytes, q0, ch * (kTf32 ? 32 : 64), lw, lane,
@@ -985,6 +993,16 @@ HankelTiling hankel_tiling(const Geom& g, int fmt, int num_sms, bool io_bf16) {
       return t;
     }
   }
+  if (g.sh == 1 && g.sw == 1 && fmt == FMT_BF16 && io_bf16 && g.C <= 16 && env_int("POLYCONV_HK_SMALLC", 1) != 0) {
+    // small C at stride 1 (VGG conv1_1, C = 3): 32-byte window rows of 16 channels instead of
+    // 128-byte rows of 64 (4x less window and MMA K padding); the pair loader masks channels >= C
+    HankelTiling t = hankel_tiling_core(g, fmt, num_sms, 16);
+    if (t.ok) {
+      t.phase = 0;
+      t.aligned = (!(g.W & 1) && t.pitch == g.W + 2 * g.pw && t.delta == (g.pw & 1)) ? 1 : 0;
+      if (t.aligned) return t;
+    }
+  }
   HankelTiling t = hankel_tiling_core(g, fmt, num_sms);
   t.phase = 0;
   return t;
@@ -1049,7 +1067,13 @@ cudaError_t launch_mac_hankel(const Geom& g0, const HankelTiling& t, int fmt, co
   // plane size in words baked in (immediate channel offsets) for the ResNet / VGG planes
   void (*kern)(const CUtensorMap, const HkParams);
   const int hw2 = g.H * g.W / 2;
-  if (t.phase && t.kc < 64) {
+  if (!t.phase && t.kc == 16) {
+    if (!t.aligned) {
+      snprintf(err, errlen, "mac_hankel: small-C mode needs pair-aligned planes");
+      return cudaErrorInvalidValue;
+    }
+    kern = mac_hankel_kernel<__nv_bfloat16, false, 0, 16>;
+  } else if (t.phase && t.kc < 64) {
     if (!t.aligned) {
       snprintf(err, errlen, "mac_hankel: small-C phase mode needs pair-aligned phase planes");
       return cudaErrorInvalidValue;

@@ -115,6 +115,8 @@ MX_SHAPES = [
     ConvShape("mx_k1_wide", 2, 512, 14, 14, 128, 1, 1, 1, 1, 0, 0),  # AUTO: tc_hankel from 24 units
     ConvShape("mx_stem", 2, 3, 32, 32, 64, 7, 7, 2, 2, 3, 3),   # small-C phase mode, 32-byte rows
     ConvShape("mx_stem_c4", 2, 4, 20, 24, 40, 7, 7, 2, 2, 3, 3),
+    ConvShape("mx_smallc", 3, 3, 20, 22, 64, 3, 3, 1, 1, 1, 1),     # stride 1, C <= 16: 32-byte rows
+    ConvShape("mx_smallc16", 2, 16, 12, 16, 40, 3, 3, 1, 1, 1, 1),
 ]
 
 

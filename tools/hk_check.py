@@ -98,6 +98,11 @@ if which in ("stem", "all"):
                  (2, 2, 16, 24, 64, 5, 5, 2, 2), (8, 3, 224, 224, 64, 7, 7, 2, 3)]:
         run(*args, name="stem")
     run(256, 3, 224, 224, 64, 7, 7, 2, 3, time_it=True, name="stem7x7")
+    # stride 1, C <= 16: 32-byte rows (VGG conv1_1)
+    for args in [(2, 3, 32, 32, 64, 3, 3, 1, 1), (3, 5, 18, 20, 40, 3, 3, 1, 1), (2, 16, 16, 16, 48, 3, 3, 1, 1),
+                 (2, 3, 20, 24, 32, 5, 5, 1, 2), (4, 3, 224, 224, 64, 3, 3, 1, 1)]:
+        run(*args, name="smallc")
+    run(64, 3, 224, 224, 64, 3, 3, 1, 1, time_it=True, name="vgg_conv1_1")
 if which in ("s2", "all"):
     # stride 2: phase-split mode (reading R19) where W % 4 == 0 and C % 32 == 0
     for args in [(2, 64, 16, 16, 64, 3, 3, 2, 1), (3, 128, 56, 56, 128, 3, 3, 2, 1), (2, 256, 28, 28, 256, 3, 3, 2, 1),
