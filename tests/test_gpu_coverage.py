@@ -53,6 +53,14 @@ def test_resnet50_all_maths(shape, math):
     assert err <= GATE[math], (kern, err)
 
 
+# ... and BF16 with bf16 I/O, the bench's and the sweeps' configuration: the stride-2 phase
+# mode, the stem's 32-byte rows and the wide-input 1x1 routing of mac_hankel are bf16-I/O paths
+@pytest.mark.parametrize("shape", synth.RESNET50, ids=lambda s: s.name)
+def test_resnet50_bf16_io(shape):
+    err, kern = _full_launch_sampled(shape, "bf16", "bf16", seed=44)
+    assert err <= GATE["bf16"], (kern, err)
+
+
 # ---- BASELINE configs[3]: all 34 sweep points, BF16 (bf16 I/O) / TF32 / FP32 ----
 @pytest.mark.parametrize("shape", synth.SWEEP, ids=lambda s: s.name)
 @pytest.mark.parametrize("math,io", [("bf16", "bf16"), ("tf32", "f32"), ("fp32", "f32")])
