@@ -120,7 +120,8 @@ struct HkParams {
 
 // per-CTA trace (dbg & 8), globaltimer ns: 0 start, 1 setup done, 2 first window stored (loader
 // warp 0), 3 filter resident / first block (MMA), 4 first item's MMAs issued, 5 first item drained
-// (epilogue warp 0), 6 last item's MMAs issued, 7 last item drained, 8 end
+// (epilogue warp 0), 6 last item's MMAs issued, 7 last item drained, 8 end, 9 / 10 first / last
+// item's accumulator ready (epilogue warp 0)
 __device__ unsigned long long g_hk_trace[160 * 16];
 // dbg & 16: CTA 0 pipeline trace (globaltimer ns) of its first 64 windows: [w][0] loader warp 0
 // starts waiting for the slot, [1] slot free, [2] window stored, [3] MMA saw it full, [4] MMAs issued
@@ -772,6 +773,7 @@ __global__ void __launch_bounds__(kHkThreads, 1)
       const int a = p.nacc == 2 ? (item & 1) : 0;
       hk_wait(tfull + a, (uint32_t)((item / p.nacc) & 1));
       tc_fence_after();
+      if (trace && e == 0 && lane == 0) tr[item == 0 ? 9 : 10] = global_ns();
       for (int t = 0; t < it.T; ++t) {
         // position of this lane -> output pixel (Eq. 12 / reading R4 / R16)
         const long long q = (long long)it.pt * 256 + (long long)rank * 128 * it.T + t * 128 + quad * 32 + lane;

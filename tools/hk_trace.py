@@ -47,7 +47,7 @@ if os.environ.get("HK_CHILD"):
         rows = [r for r in rows if r[0]]
         t0 = min(r[0] for r in rows)
         summ = {}
-        for i in range(9):
+        for i in range(11):
             v = sorted((r[i] - t0) / 1e3 for r in rows if r[i])
             if v:
                 summ[i] = [round(v[len(v) // 2], 2), round(v[-1], 2)]
