@@ -70,8 +70,9 @@ cudaError_t launch_mac_thin(const Geom& g, const void* A, const void* U, int Kp,
 // ---- mac_fp32.cu ----------------------------------------------------------
 struct Fp32Tiling { int cc; int smem_bytes; int smax; };
 Fp32Tiling fp32_tiling(const Geom& g);
-cudaError_t launch_mac_fp32(const Geom& g, const Fp32Tiling& t, const float* A, const float* U,
-                            int Kp, int Cp, float* y, cudaStream_t st);
+// x: NCHW input (f32 or bf16); U: tap-major fp32 filter [RS][Kp][Cp]; y: NCHW output (x's dtype)
+cudaError_t launch_mac_fp32(const Geom& g, const Fp32Tiling& t, const void* x, bool io_bf16, const float* U,
+                            int Kp, int Cp, void* y, cudaStream_t st);
 inline int fp32_kp(int K) { return (K + 63) / 64 * 64; }
 
 // ---- mac_tc.cu ------------------------------------------------------------

@@ -105,10 +105,18 @@ bool fft_pays(const Geom& g) {
   if (getenv("POLYCONV_NO_FFT") || g.K < 16) return false;
   const FftTiling t = fft_tiling(g);
   if (!t.ok) return false;
-  const double work = (double)g.R * g.S * g.P * g.Q;
-  if (g.P * g.Q <= 64 && g.sh == 1 && (long long)g.C * g.K >= (1LL << 20)) return true;  // 1x1 on 7x7, C*K >= 1M
-  if (t.L <= 1024) return g.N >= 64 && work >= 0.8 * t.L;
-  return work >= 16.0 * t.L;
+  // r = taps x outputs per FFT bin.  Against the direct FFMA kernel (mac_fp32, round 2b),
+  // measured on all 71 FP32 layers (profiles/r03_fp32_cmp.jsonl, TFLOP/s FFT / FFMA): the FFT
+  // wins only on short transforms -- L <= 256 (l4 3x3 40 / 31), L = 512 at stride 2 or r >= 8
+  // (l4 3x3 s2 9.7 / 9.0, A_h14_s1 25.2 / 24.0; l3 3x3 29 / 34 loses), L = 1024 at stride 2
+  // or with C*K >= 128K (l3 3x3 s2 12.8 / 9.7, VGG conv4 56 / 38; conv3_x 20 / 32 loses).
+  const double r = (double)g.R * g.S * g.P * g.Q / t.L;
+  if (r < 0.8) return false;
+  const bool s2 = g.sh > 1;
+  if (t.L <= 256) return true;
+  if (t.L <= 512) return s2 || r >= 8.0;
+  if (t.L <= 1024) return (s2 && r >= 1.5) || ((long long)g.C * g.K >= 131072 && r >= 4.0);
+  return false;
 }
 
 // Resolve the MAC variant and fill the kernel-specific padded sizes.
@@ -228,7 +236,7 @@ polyconv_status_t resolve(polyconv_plan_t p) {
   // TC packs the input on the fly (no input workspace); TC_PERTAP needs the
   // interleaved copy, FP32/THIN the planar one
   const size_t a_elems = k == POLYCONV_KERNEL_TC_1X1 ? (size_t)g.N * g.C * mac1x1_pitch(g)
-                         : (k == POLYCONV_KERNEL_TC_FUSED || k == POLYCONV_KERNEL_TC_HANKEL) ? 0
+                         : (k == POLYCONV_KERNEL_TC_FUSED || k == POLYCONV_KERNEL_TC_HANKEL || k == POLYCONV_KERNEL_FP32) ? 0
                          : (k == POLYCONV_KERNEL_TC || k == POLYCONV_KERNEL_TC_PERTAP || k == POLYCONV_KERNEL_TC_PAIR) ? (size_t)g.N * g.L_A * g.Cp
                                                                                        : (size_t)g.N * g.C * g.L_A;
   p->wsA_bytes = a_elems * eb;
@@ -615,16 +623,20 @@ polyconv_status_t polyconv_forward(polyconv_plan_t p, const void* x, const void*
     if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
     return finish(p, e, "mac_tc_pertap");
   }
+  if (p->kernel == POLYCONV_KERNEL_FP32) {
+    // a3 (tap-major fp32 filter), then a2 + a4 + a5 in the FFMA kernel, which reads x directly
+    if (p->ev_start) cudaEventRecord(p->ev_start, st);
+    e = launch_pack_filter_tapmajor(g, w, p->io_bf16, p->wsU, p->fmt, g.Kp, g.Cp, st);
+    if (e != cudaSuccess) return finish(p, e, "pack_filter");
+    e = launch_mac_fp32(g, p->f32, x, p->io_bf16, (const float*)p->wsU, g.Kp, g.Cp, y, st);
+    if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
+    return finish(p, e, "mac_fp32");
+  }
   e = launch_pack_input_planar(g, x, p->io_bf16, p->wsA, p->fmt, st);
   if (e != cudaSuccess) return finish(p, e, "pack_input");
   e = launch_pack_filter_tapmajor(g, w, p->io_bf16, p->wsU, p->fmt, g.Kp, g.Cp, st);
   if (e != cudaSuccess) return finish(p, e, "pack_filter");
   if (p->ev_start) cudaEventRecord(p->ev_start, st);
-  if (p->kernel == POLYCONV_KERNEL_FP32) {
-    e = launch_mac_fp32(g, p->f32, (const float*)p->wsA, (const float*)p->wsU, g.Kp, g.Cp, (float*)y, st);
-    if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
-    return finish(p, e, "mac_fp32");
-  }
   e = launch_mac_thin(g, p->wsA, p->wsU, g.Kp, g.Cp, p->fmt, y, p->io_bf16, st);
   if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
   return finish(p, e, "mac_thin");

@@ -139,10 +139,15 @@ def test_fft_solver_planning():
     with pytest.raises(pc.PolyconvError):
         pc.Plan((1, 8, 20, 20), (8, 8, 3, 3), padding=(1, 1), math="tf32", kernel="fft")
     auto = lambda xs, ws, s=1: pc.Plan(xs, ws, (s, s), (ws[2] // 2, ws[3] // 2), math="fp32").info()["kernel"]
-    assert auto((256, 512, 7, 7), (512, 512, 3, 3)) == "fft"      # ResNet-50 l4 3x3: 40 vs 7 TFLOP/s
-    assert auto((256, 128, 28, 28), (128, 128, 3, 3)) == "fft"    # l2 3x3: 31 vs 26
-    assert auto((256, 64, 56, 56), (64, 64, 3, 3)) == "fp32"      # l1 3x3 (L = 4096): 12 vs 28
-    assert auto((32, 128, 28, 28), (128, 128, 3, 3)) == "fp32"    # conv3_x at N=32: 20 vs 22
+    # FFT / FFMA TFLOP/s, profiles/r03_fp32_cmp.jsonl
+    assert auto((256, 512, 7, 7), (512, 512, 3, 3)) == "fft"      # ResNet-50 l4 3x3 (L = 128): 40 vs 31
+    assert auto((256, 256, 28, 28), (256, 256, 3, 3), 2) == "fft"  # l3 3x3 s2 (L = 1024): 12.8 vs 9.7
+    assert auto((64, 512, 28, 28), (512, 512, 3, 3)) == "fft"     # VGG-16 conv4_2 (C*K = 256K): 56 vs 38
+    assert auto((256, 128, 28, 28), (128, 128, 3, 3)) == "fp32"   # l2 3x3: 31 vs 38
+    assert auto((256, 256, 14, 14), (256, 256, 3, 3)) == "fp32"   # l3 3x3 (L = 512): 29 vs 34
+    assert auto((256, 64, 56, 56), (64, 64, 3, 3)) == "fp32"      # l1 3x3 (L = 4096): 12 vs 38
+    assert auto((32, 128, 28, 28), (128, 128, 3, 3)) == "fp32"    # conv3_x at N=32: 20 vs 32
+    assert auto((256, 2048, 7, 7), (512, 2048, 1, 1)) == "fp32"   # l4 1x1 2048->512: 9.4 vs 18.3
 
 
 def test_tc_tiling_choices():
