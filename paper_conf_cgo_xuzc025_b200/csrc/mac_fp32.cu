@@ -21,6 +21,7 @@
 // tap): 8 conflict-free LDS.32 of the window (32 consecutive positions per instruction), two
 // broadcast LDS.128 of the filter, 64 FFMA.  Small tiles (256 x 32) keep the grid at several
 // CTAs per SM, so the work per SM is balanced to a few percent (conv3_x: 424 CTAs).
+#include <cstdlib>
 #include "common.cuh"
 
 namespace polyconv {
@@ -181,8 +182,13 @@ __global__ void __launch_bounds__(NT, 4) mac_fp32_kernel(Geom g, F32Geo f, const
 
 Fp32Tiling fp32_tiling(const Geom& g) {
   Fp32Tiling t{8, 0, 0};
-  // channel chunk: 8, fewer for large kernels (two buffers of CC x R*S x 32 filter words)
-  for (int cc = 8; cc >= 1; cc >>= 1) {
+  // channel chunk: 8 (16 for 1x1: the per-position decode and the chunk barrier amortise over
+  // more channels, ResNet-50 1x1 layers 21-22 -> 24-25 TFLOP/s; 3x3 layers lose 2-7% with 16),
+  // fewer for large kernels (two buffers of CC x R*S x 32 filter words); POLYCONV_F32_CC
+  // overrides the starting value (experiments)
+  const char* ev = getenv("POLYCONV_F32_CC");
+  const int cc0 = ev ? atoi(ev) : (g.R * g.S == 1 ? 16 : 8);
+  for (int cc = cc0; cc >= 1; cc >>= 1) {
     t.cc = cc;
     t.smem_bytes = smem_bytes_for(g, cc);
     if (t.smem_bytes <= 100 * 1024) break;
