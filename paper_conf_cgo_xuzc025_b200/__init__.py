@@ -357,15 +357,16 @@ def wgrad(x, dy, w_shape, stride=(1, 1), padding=(0, 0), stream=None):
     return dw
 
 
-def conv2d(x, w, stride=(1, 1), padding=(0, 0), math="bf16", kernel="auto"):
-    """One-shot convenience: plan + forward (the plan is cached per shape)."""
+def conv2d(x, w, stride=(1, 1), padding=(0, 0), math="bf16", kernel="auto", out=None):
+    """One-shot convenience: plan + forward (the plan is cached per shape); `out` (optional)
+    receives y in place."""
     key = (tuple(x.shape), tuple(w.shape), tuple(stride), tuple(padding), math,
            "bf16" if str(x.dtype) == "torch.bfloat16" else "f32", x.device.index or 0, kernel)
     plan = _PLANS.get(key)
     if plan is None:
         plan = Plan(x.shape, w.shape, stride, padding, math, key[5], key[6], kernel)
         _PLANS[key] = plan
-    return plan.forward(x, w)
+    return plan.forward(x, w, out)
 
 
 _PLANS: dict = {}

@@ -46,9 +46,10 @@ def shard_plan(N: int, K: int, world: int, rank: int) -> Shard:
     return Shard("kshard", 0, N, k0, k1, kb * world)
 
 
-def _cuda_compute(x, w, stride, padding, math):
+def _cuda_compute(x, w, stride, padding, math, out=None):
+    """The CUDA path; `out` (optional) receives the result in place (polyconv_forward writes it)."""
     from . import conv2d
-    return conv2d(x, w, stride=stride, padding=padding, math=math)
+    return conv2d(x, w, stride=stride, padding=padding, math=math, out=out)
 
 
 def sharded_forward(x, w, stride=(1, 1), padding=(0, 0), math="bf16", group=None, compute=None):
@@ -56,7 +57,13 @@ def sharded_forward(x, w, stride=(1, 1), padding=(0, 0), math="bf16", group=None
     rank (batch mode slices it; pass only the local images with N >= world for
     zero-copy use through `local_batch`), w: full filters.  Returns
     (shard, y): in batch mode y is the local shard [n1-n0][K][P][Q]; in
-    output-channel mode y is the full gathered output [N][K][P][Q]."""
+    output-channel mode y is the full gathered output [N][K][P][Q].
+
+    `compute(x, w, stride, padding, math, out)` runs one shard and writes `out` when given.
+    Output-channel mode computes the local block straight into the all-gather's send buffer
+    (the last rank's filter block is zero-padded to the common block size, so its padding
+    channels come out zero without a fill); for N = 1 the rank-ordered blocks are NCHW and
+    NCCL gathers straight into the output."""
     import torch
     import torch.distributed as dist
     compute = compute or _cuda_compute
@@ -67,22 +74,27 @@ def sharded_forward(x, w, stride=(1, 1), padding=(0, 0), math="bf16", group=None
     if sh.mode == "batch":
         return sh, compute(x[sh.n0:sh.n1].contiguous(), w, stride, padding, math)
     kb = sh.k_pad // world
-    y_loc = compute(x, w[sh.k0:sh.k1].contiguous(), stride, padding, math) if sh.k1 > sh.k0 else None
-    P, Q = (y_loc.shape[2], y_loc.shape[3]) if y_loc is not None else _out_hw(x, w, stride, padding)
-    buf = torch.zeros((N, kb, P, Q), dtype=x.dtype, device=x.device)
-    if y_loc is not None:
-        buf[:, : sh.k1 - sh.k0] = y_loc
+    P, Q = _out_hw(x, w, stride, padding)
+    w_loc = w[sh.k0:sh.k1]
+    if sh.k1 - sh.k0 < kb:  # tail block: zero filters for the padding channels
+        w_loc = torch.cat([w_loc, w.new_zeros((kb - (sh.k1 - sh.k0),) + tuple(w.shape[1:]))])
+    send = torch.empty((N, kb, P, Q), dtype=x.dtype, device=x.device)
+    compute(x, w_loc.contiguous(), stride, padding, math, send)
     # gather the K blocks: [world][N][kb][P][Q] -> [N][K][P][Q]
     if dist.is_initialized() and dist.get_backend(group) == "nccl":
+        if N == 1:
+            y = torch.empty((1, world * kb, P, Q), dtype=x.dtype, device=x.device)
+            dist.all_gather_into_tensor(y.view(world, kb, P, Q), send.view(kb, P, Q), group=group)
+            return sh, y[:, :K]
         out = torch.empty((world * N, kb, P, Q), dtype=x.dtype, device=x.device)
-        dist.all_gather_into_tensor(out, buf.reshape(N, kb, P, Q).contiguous(), group=group)
+        dist.all_gather_into_tensor(out, send, group=group)
         blocks = out.reshape(world, N, kb, P, Q)
     else:
-        parts = [torch.empty_like(buf) for _ in range(world)]
+        parts = [torch.empty_like(send) for _ in range(world)]
         if dist.is_initialized():
-            dist.all_gather(parts, buf, group=group)
+            dist.all_gather(parts, send, group=group)
         else:
-            parts = [buf]
+            parts = [send]
         blocks = torch.stack(parts)
     y = blocks.permute(1, 0, 2, 3, 4).reshape(N, world * kb, P, Q)[:, :K]
     return sh, y.contiguous()

@@ -29,8 +29,12 @@ def test_shard_plan_partitions_work(N, K, world):
     assert (seen == 1).all()
 
 
-def _oracle_compute(x, w, stride, padding, math):
-    return torch.from_numpy(oracle.conv2d(x.numpy(), w.numpy(), stride, padding))
+def _oracle_compute(x, w, stride, padding, math, out=None):
+    y = torch.from_numpy(oracle.conv2d(x.numpy(), w.numpy(), stride, padding))
+    if out is None:
+        return y
+    out.copy_(y)
+    return out
 
 
 def _free_port():
