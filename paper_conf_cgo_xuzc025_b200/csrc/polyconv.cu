@@ -111,7 +111,7 @@ bool fft_pays(const Geom& g) {
   // (l4 3x3 s2 9.7 / 9.0, A_h14_s1 25.2 / 24.0; l3 3x3 29 / 34 loses), L = 1024 at stride 2
   // or with C*K >= 128K (l3 3x3 s2 12.8 / 9.7, VGG conv4 56 / 38; conv3_x 20 / 32 loses).
   const double r = (double)g.R * g.S * g.P * g.Q / t.L;
-  if (r < 0.8) return false;
+  if (r < 0.8 || g.N < 64) return false;  // every measured FFT win had N >= 64
   const bool s2 = g.sh > 1;
   if (t.L <= 256) return true;
   if (t.L <= 512) return s2 || r >= 8.0;
