@@ -155,6 +155,20 @@ polyconv_status_t polyconv_plan_info(polyconv_plan_t plan, polyconv_info_t *info
 polyconv_status_t polyconv_forward(polyconv_plan_t plan, const void *x, const void *w,
                                    void *y, void *stream);
 
+/* Output-channel-sharded forward with the all-gather fused into the MAC epilogue (SURVEY
+ * §8(e)/(f) f4; the paper is single-GPU, P.1431-1433).  ys[0..n_out-1] are device pointers to
+ * outputs [N][k_total][P][Q] in the io dtype -- local buffers, or every rank's buffer mapped
+ * over NVLink (e.g. torch symmetric memory); this plan's K output channels (a block of the
+ * layer's k_total) are stored at channel offset k_offset of EVERY ys[r] straight from the
+ * epilogue: no local copy, no separate collective.  1 <= n_out <= 8, 0 <= k_offset,
+ * k_offset + K <= k_total; all pointers 16-byte aligned (else NOT_SUPPORTED).  The caller
+ * orders the peers' reads after this forward (stream order plus a cross-rank barrier).  Only
+ * the TC_HANKEL kernel stores to peers: NOT_SUPPORTED (nothing enqueued) for plans that
+ * resolved to another kernel.  Other errors as polyconv_forward. */
+polyconv_status_t polyconv_forward_scatter(polyconv_plan_t plan, const void *x, const void *w,
+                                           void *const *ys, int n_out, int k_total, int k_offset,
+                                           void *stream);
+
 /* polyconv_forward from HOST buffers (the end-to-end call): x, w, y are host
  * pointers (pinned for asynchronous copies; pageable works but serialises).
  * Enqueues on `stream`: H2D copy of x and w into plan-owned device buffers

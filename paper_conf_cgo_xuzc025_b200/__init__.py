@@ -45,7 +45,7 @@ class Info(ctypes.Structure):
 
 
 EXPORTS = ["polyconv_plan", "polyconv_plan_set_kernel", "polyconv_output_dims", "polyconv_plan_info",
-           "polyconv_forward", "polyconv_forward_host", "polyconv_plan_set_timing_events", "polyconv_pack_input", "polyconv_pack_filter", "polyconv_packed_bytes",
+           "polyconv_forward", "polyconv_forward_scatter", "polyconv_forward_host", "polyconv_plan_set_timing_events", "polyconv_pack_input", "polyconv_pack_filter", "polyconv_packed_bytes",
            "polyconv_extract", "polyconv_destroy", "polyconv_status_string", "polyconv_last_error",
            "polyconv_abi_version", "polyconv_flip_filter", "polyconv_swap_nc",
            "polyconv_dilate", "polyconv_wgrad"]
@@ -70,6 +70,7 @@ def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
     lib.polyconv_plan_info.argtypes = [vp, ctypes.POINTER(Info)]
     lib.polyconv_forward.argtypes = [vp, vp, vp, vp, vp]
     lib.polyconv_forward_host.argtypes = [vp, vp, vp, vp, vp]
+    lib.polyconv_forward_scatter.argtypes = [vp, vp, vp, ctypes.POINTER(vp), i, i, i, vp]
     lib.polyconv_plan_set_timing_events.argtypes = [vp, vp, vp]
     lib.polyconv_pack_input.argtypes = [vp, vp, vp, i, vp]
     lib.polyconv_pack_filter.argtypes = [vp, vp, vp, i, vp]
@@ -189,6 +190,19 @@ class Plan:
         self._check(self._lib.polyconv_forward(self._h, ctypes.c_void_p(x.data_ptr()), ctypes.c_void_p(w.data_ptr()),
                                                ctypes.c_void_p(y.data_ptr()), _stream_ptr(stream, self.device)), "forward")
         return y
+
+    def forward_scatter(self, x, w, y_ptrs, k_total, k_offset, stream=None):
+        """Output-channel shard with the all-gather fused into the epilogue (f4): this plan's
+        K channels are stored at channel offset `k_offset` of every buffer in `y_ptrs`
+        (device addresses of [N][k_total][P][Q] outputs: local, or peers' mapped over NVLink,
+        e.g. torch symmetric memory's buffer_ptrs).  Only TC_HANKEL plans (NOT_SUPPORTED else)."""
+        self._check_tensor(x, self.x_shape, "x")
+        self._check_tensor(w, self.w_shape, "w")
+        ptrs = (ctypes.c_void_p * len(y_ptrs))(*[int(v) for v in y_ptrs])
+        self._check(self._lib.polyconv_forward_scatter(self._h, ctypes.c_void_p(x.data_ptr()),
+                                                       ctypes.c_void_p(w.data_ptr()), ptrs, len(y_ptrs),
+                                                       int(k_total), int(k_offset), _stream_ptr(stream, self.device)),
+                    "forward_scatter")
 
     def forward_host(self, x, w, y, stream=None):
         """End-to-end call: x, w, y are (pinned) CPU tensors; the library copies

@@ -181,8 +181,10 @@ HankelTiling hankel_tiling(const Geom& g, int fmt, int num_sms, bool io_bf16);
 // the preceding launch, which this one follows as a programmatic dependent
 // zero: device buffer of hankel_zero_bytes(g) zero bytes (read in place of padding)
 size_t hankel_zero_bytes(const Geom& g);
+// ys[0..nys-1]: outputs [N][ktot][P][Q]; this plan's K channels go to channel offset koff of each
 cudaError_t launch_mac_hankel(const Geom& g, const HankelTiling& t, int fmt, const void* x, bool io_bf16,
-                              const void* U, void* y, const void* zero, cudaStream_t st, char* err, size_t errlen);
+                              const void* U, void* const* ys, int nys, int ktot, int koff, const void* zero,
+                              cudaStream_t st, char* err, size_t errlen);
 
 // ---- fft.cu (R = IFFT(FFT(A) . FFT(U)) per channel, summed in frequency) ----
 struct FftTiling {

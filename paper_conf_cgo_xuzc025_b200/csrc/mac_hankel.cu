@@ -89,10 +89,13 @@ constexpr int kHkSmemMax = 232448;                         // 227 KB dynamic
 constexpr int kHkMaxFBlk = 64;                             // filter ring slots (max)
 constexpr int kHkMaxWSlots = 4;
 
+constexpr int kHkMaxOut = 8;  // output buffers of one forward (polyconv_forward_scatter)
+
 struct HkParams {
   const void* x;
   const void* zero;     // plan-owned zero words (>= 8 planes of float2), read for zero pairs
-  void* y;
+  void* ys[kHkMaxOut];  // outputs [N][Ktot][P][Q]: y, or every rank's (peer-mapped) buffer
+  int nys, Ktot, koff;  // number of outputs; their channel count and this plan's channel offset
   int N, C, H, W, K, P, Q, sh, sw, ph, pw;
   int HW, CHW;          // plane size, image size (elements)
   int pitch, HS, delta; // input polynomial layout (reading R16)
@@ -762,7 +765,6 @@ __global__ void __launch_bounds__(kHkThreads, 1)
     const int quad = warp & 3;      // TMEM lane quadrant this warp may access
     const int half = e & 1;         // column groups half, half + 2, ...
     const uint32_t tbase = *tmem_slot;
-    IoT* y = static_cast<IoT*>(p.y);
     const long long PQ = (long long)p.P * p.Q;
     // plane size of y as a compile-time constant when the output has the input's size
     const bool pq_const = kHW2 > 0 && PQ == 2LL * kHW2;
@@ -788,7 +790,7 @@ __global__ void __launch_bounds__(kHkThreads, 1)
           const uint32_t oh = p.fsh.div(ohs), ow = p.fsw.div(col);
           if ((int)n < p.N && oh * (uint32_t)p.sh == ohs && ow * (uint32_t)p.sw == col && (int)oh < p.P &&
               (int)ow < p.Q)
-            ybase = ((long long)n * p.K + it.nb * p.NN) * PQ + (long long)oh * p.Q + ow;
+            ybase = ((long long)n * p.Ktot + p.koff + it.nb * p.NN) * PQ + (long long)oh * p.Q + ow;
         }
         const uint32_t trow = tbase + ((uint32_t)(quad * 32) << 16) + (uint32_t)(a * p.T * p.NN + t * p.NN);
         for (int g = half; g * 16 < p.NN; g += 2) {
@@ -801,17 +803,20 @@ __global__ void __launch_bounds__(kHkThreads, 1)
             for (int c = 0; c < 16; ++c) v[c] = 0u;
           }
           if (ybase >= 0 && !(p.dbg & 2)) {
-            IoT* yp = y + ybase + (long long)(g * 16) * PQ;
             const int kleft = p.K - (it.nb * p.NN + g * 16);  // output channels left (warp-uniform)
-            if (kHW2 > 0 && pq_const && kleft >= 16) {
-              // same-size output with a baked-in plane size: one base register, immediate offsets
+            // every output buffer (f4: the K-shard all-gather as peer stores over NVLink)
+            for (int o = 0; o < p.nys; ++o) {
+              IoT* yp = static_cast<IoT*>(p.ys[o]) + ybase + (long long)(g * 16) * PQ;
+              if (kHW2 > 0 && pq_const && kleft >= 16) {
+                // same-size output with a baked-in plane size: one base register, immediate offsets
 #pragma unroll
-              for (int c = 0; c < 16; ++c)
-                hk_store<IoT>(yp, (long long)c * (2 * (kHW2 > 0 ? kHW2 : 1)), __uint_as_float(v[c]));
-            } else {
+                for (int c = 0; c < 16; ++c)
+                  hk_store<IoT>(yp, (long long)c * (2 * (kHW2 > 0 ? kHW2 : 1)), __uint_as_float(v[c]));
+              } else {
 #pragma unroll
-              for (int c = 0; c < 16; ++c)
-                if (c < kleft) hk_store<IoT>(yp, (long long)c * PQ, __uint_as_float(v[c]));
+                for (int c = 0; c < 16; ++c)
+                  if (c < kleft) hk_store<IoT>(yp, (long long)c * PQ, __uint_as_float(v[c]));
+              }
             }
           }
         }
@@ -1011,7 +1016,12 @@ HankelTiling hankel_tiling(const Geom& g, int fmt, int num_sms, bool io_bf16) {
 }
 
 cudaError_t launch_mac_hankel(const Geom& g0, const HankelTiling& t, int fmt, const void* x, bool io_bf16,
-                              const void* U, void* y, const void* zero, cudaStream_t st, char* err, size_t errlen) {
+                              const void* U, void* const* ys, int nys, int ktot, int koff, const void* zero,
+                              cudaStream_t st, char* err, size_t errlen) {
+  if (nys < 1 || nys > kHkMaxOut || koff < 0 || koff + g0.K > ktot) {
+    snprintf(err, errlen, "mac_hankel: bad output list");
+    return cudaErrorInvalidValue;
+  }
   if (!t.ok) {
     snprintf(err, errlen, "mac_hankel: shape not supported");
     return cudaErrorInvalidValue;
@@ -1043,7 +1053,10 @@ cudaError_t launch_mac_hankel(const Geom& g0, const HankelTiling& t, int fmt, co
   HkParams p{};
   p.x = x;
   p.zero = zero;
-  p.y = y;
+  for (int o = 0; o < nys; ++o) p.ys[o] = ys[o];
+  p.nys = nys;
+  p.Ktot = ktot;
+  p.koff = koff;
   p.N = g.N; p.C = g.C; p.H = g.H; p.W = g.W; p.K = g.K; p.P = g.P; p.Q = g.Q;
   p.sh = g.sh; p.sw = g.sw; p.ph = g.ph; p.pw = g.pw;
   p.HW = g.H * g.W;

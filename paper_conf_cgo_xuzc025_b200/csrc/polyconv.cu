@@ -499,6 +499,57 @@ polyconv_status_t polyconv_plan_info(polyconv_plan_t p, polyconv_info_t* info) {
   return POLYCONV_STATUS_SUCCESS;
 }
 
+// a3 (tap-major filter, one small launch), then a2 + a4 + a5 in the persistent pair kernel,
+// which reads x directly and follows the pack as a programmatic dependent; its epilogue stores
+// the plan's K channels at channel offset koff of each of the nys outputs [N][ktot][P][Q]
+static polyconv_status_t forward_hankel(polyconv_plan_t p, const void* x, const void* w, void* const* ys, int nys,
+                                        int ktot, int koff, cudaStream_t st) {
+  const Geom& g = p->g;
+  cudaError_t e;
+  if (!p->hkzero) {
+    const size_t zb = hankel_zero_bytes(g);
+    if (cudaMalloc(&p->hkzero, zb) != cudaSuccess || cudaMemsetAsync(p->hkzero, 0, zb, st) != cudaSuccess) {
+      cudaGetLastError();
+      if (p->hkzero) cudaFree(p->hkzero);
+      p->hkzero = nullptr;
+      set_err(p, "cudaMalloc of the %s failed", "zero buffer");
+      return POLYCONV_STATUS_ALLOC_FAILED;
+    }
+  }
+  if (p->ev_start) cudaEventRecord(p->ev_start, st);
+  if (p->hk.phase)
+    e = launch_pack_filter_phase(g, w, p->wsU, p->hk.eR, p->hk.eS, p->hk.eph, p->hk.epw, g.Kp, g.Cp, st);
+  else
+    e = launch_pack_filter_tapmajor(g, w, p->io_bf16, p->wsU, p->fmt, g.Kp, g.Cp, st);
+  if (e != cudaSuccess) return finish(p, e, "pack_filter");
+  e = launch_mac_hankel(g, p->hk, p->fmt, x, p->io_bf16, p->wsU, ys, nys, ktot, koff, p->hkzero, st, p->err,
+                        sizeof(p->err));
+  if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
+  return finish(p, e, "mac_hankel");
+}
+
+polyconv_status_t polyconv_forward_scatter(polyconv_plan_t p, const void* x, const void* w, void* const* ys,
+                                           int n_out, int k_total, int k_offset, void* stream) {
+  if (!p || !x || !w || !ys || n_out < 1 || n_out > 8 || k_offset < 0 || k_total < k_offset + p->g.K)
+    return POLYCONV_STATUS_BAD_PARAM;
+  if (!aligned(x, 16) || !aligned(w, 16)) return POLYCONV_STATUS_NOT_SUPPORTED;
+  for (int o = 0; o < n_out; ++o) {
+    if (!ys[o] || ys[o] == x || ys[o] == w) return POLYCONV_STATUS_BAD_PARAM;
+    if (!aligned(ys[o], 16)) return POLYCONV_STATUS_NOT_SUPPORTED;
+  }
+  if (p->kernel != POLYCONV_KERNEL_TC_HANKEL || p->inner) {
+    set_err(p, "forward_scatter: the %s kernel does not store to peers", "plan's");
+    return POLYCONV_STATUS_NOT_SUPPORTED;
+  }
+  PC_BEGIN(p);
+  polyconv_status_t s = ensure_workspace(p);
+  if (s != POLYCONV_STATUS_SUCCESS) return s;
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  p->last_stream = st;
+  p->used = true;
+  return forward_hankel(p, x, w, ys, n_out, k_total, k_offset, st);
+}
+
 polyconv_status_t polyconv_forward(polyconv_plan_t p, const void* x, const void* w, void* y, void* stream) {
   if (!p) return POLYCONV_STATUS_BAD_PARAM;
   if (!x || !w || !y || x == y || w == y) return POLYCONV_STATUS_BAD_PARAM;
@@ -554,29 +605,7 @@ polyconv_status_t polyconv_forward(polyconv_plan_t p, const void* x, const void*
     if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
     return finish(p, e, "fft_conv");
   }
-  if (p->kernel == POLYCONV_KERNEL_TC_HANKEL) {
-    // a3 (tap-major filter, one small launch), then a2 + a4 + a5 in the persistent pair
-    // kernel, which reads x directly and follows the pack as a programmatic dependent
-    if (!p->hkzero) {
-      const size_t zb = hankel_zero_bytes(g);
-      if (cudaMalloc(&p->hkzero, zb) != cudaSuccess || cudaMemsetAsync(p->hkzero, 0, zb, st) != cudaSuccess) {
-        cudaGetLastError();
-        if (p->hkzero) cudaFree(p->hkzero);
-        p->hkzero = nullptr;
-        set_err(p, "cudaMalloc of the %s failed", "zero buffer");
-        return POLYCONV_STATUS_ALLOC_FAILED;
-      }
-    }
-    if (p->ev_start) cudaEventRecord(p->ev_start, st);
-    if (p->hk.phase)
-      e = launch_pack_filter_phase(g, w, p->wsU, p->hk.eR, p->hk.eS, p->hk.eph, p->hk.epw, g.Kp, g.Cp, st);
-    else
-      e = launch_pack_filter_tapmajor(g, w, p->io_bf16, p->wsU, p->fmt, g.Kp, g.Cp, st);
-    if (e != cudaSuccess) return finish(p, e, "pack_filter");
-    e = launch_mac_hankel(g, p->hk, p->fmt, x, p->io_bf16, p->wsU, y, p->hkzero, st, p->err, sizeof(p->err));
-    if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
-    return finish(p, e, "mac_hankel");
-  }
+  if (p->kernel == POLYCONV_KERNEL_TC_HANKEL) return forward_hankel(p, x, w, &y, 1, g.K, 0, st);
   if (p->kernel == POLYCONV_KERNEL_TC_1X1) {
     // a3 (the [1][Kp][Cp] filter), then the GEMM over the NCHW planes as its programmatic dependent
     if (p->ev_start) cudaEventRecord(p->ev_start, st);
