@@ -17,12 +17,22 @@ CASES = {  # kernel: [(x_shape, w_shape, stride, pad, math, io)]
     "tc_pair": [((2, 64, 16, 16), (64, 64, 3, 3), 1, 1, "bf16", "bf16")],
     "tc_1x1": [((2, 64, 16, 16), (128, 64, 1, 1), 1, 0, "bf16", "bf16")],
     "tc_pertap": [((2, 64, 12, 12), (64, 64, 3, 3), 1, 1, "bf16", "f32")],
-    "fp32": [((2, 16, 12, 12), (32, 16, 3, 3), 1, 1, "fp32", "f32")],
+    "fp32": [((2, 16, 12, 12), (32, 16, 3, 3), 1, 1, "fp32", "f32"), ((2, 24, 9, 13), (40, 24, 5, 5), 2, 2, "fp32", "f32"),
+             ((2, 20, 7, 7), (36, 20, 1, 1), 1, 0, "fp32", "f32")],
     "thin": [((1, 1, 8, 8), (1, 1, 3, 3), 1, 0, "fp32", "f32")],
     "fft": [((2, 16, 12, 12), (32, 16, 3, 3), 1, 1, "fp32", "f32"), ((2, 8, 9, 9), (16, 8, 5, 5), 2, 2, "fp32", "f32")],
 }
-which = sys.argv[1:] or list(CASES)
+which = sys.argv[1:] or list(CASES) + ["scatter"]
 for kern in which:
+    if kern == "scatter":  # f4: the K-shard block stored into three output buffers
+        x = (torch.rand((2, 64, 12, 12), device="cuda") * 2 - 1).bfloat16()
+        w = (torch.rand((64, 64, 3, 3), device="cuda") * 2 - 1).bfloat16()
+        plan = pc.Plan(x.shape, w.shape, (1, 1), (1, 1), math="bf16", io_dtype="bf16", kernel="tc_hankel")
+        ys = [torch.zeros((2, 160, 12, 12), dtype=torch.bfloat16, device="cuda") for _ in range(3)]
+        plan.forward_scatter(x, w, [t.data_ptr() for t in ys], 160, 64)
+        torch.cuda.synchronize()
+        print("scatter ok", float(ys[2].float().abs().sum()) > 0, flush=True)
+        continue
     for xs, ws, s, p, math, io in CASES[kern]:
         dt = torch.bfloat16 if io == "bf16" else torch.float32
         x = (torch.rand(xs, device="cuda") * 2 - 1).to(dt)
