@@ -115,11 +115,13 @@ __global__ void __launch_bounds__(NT, 4) mac_fp32_kernel(Geom g, F32Geo f, const
     cp_async_commit();
   };
 
-  float acc[8][8];
+  // accumulators as position pairs: one packed FFMA2 (fma.rn.f32x2, sm_100) per channel and
+  // pair -- the same round-to-nearest fp32 FMAs as two FFMA, half the issue slots
+  float2 acc[8][4];
 #pragma unroll
   for (int a = 0; a < 8; ++a)
 #pragma unroll
-    for (int b = 0; b < 8; ++b) acc[a][b] = 0.f;
+    for (int b = 0; b < 4; ++b) acc[a][b] = make_float2(0.f, 0.f);
 
   const int nch = (g.C + CC - 1) / CC;
   stage(0, 0);
@@ -143,13 +145,14 @@ __global__ void __launch_bounds__(NT, 4) mac_fp32_kernel(Geom g, F32Geo f, const
           const float4 w0 = *reinterpret_cast<const float4*>(wr + (i * S + j) * BK);
           const float4 w1 = *reinterpret_cast<const float4*>(wr + (i * S + j) * BK + 4);
           const float wv[8] = {w0.x, w0.y, w0.z, w0.w, w1.x, w1.y, w1.z, w1.w};
-          float av[8];
+          float2 av[4];
 #pragma unroll
-          for (int bb = 0; bb < 8; ++bb) av[bb] = win[i * f.pitch + j + 32 * bb];
+          for (int bb = 0; bb < 4; ++bb)
+            av[bb] = make_float2(win[i * f.pitch + j + 64 * bb], win[i * f.pitch + j + 64 * bb + 32]);
 #pragma unroll
           for (int a = 0; a < 8; ++a)
 #pragma unroll
-            for (int bb = 0; bb < 8; ++bb) acc[a][bb] = fmaf(wv[a], av[bb], acc[a][bb]);
+            for (int bb = 0; bb < 4; ++bb) acc[a][bb] = __ffma2_rn(make_float2(wv[a], wv[a]), av[bb], acc[a][bb]);
         }
       }
     }
@@ -173,7 +176,7 @@ __global__ void __launch_bounds__(NT, 4) mac_fp32_kernel(Geom g, F32Geo f, const
 #pragma unroll
     for (int a = 0; a < 8; ++a) {
       const int k = k0 + warp * 8 + a;
-      if (k < g.K) y[ybase + (long long)k * PQ] = acc[a][bb];
+      if (k < g.K) y[ybase + (long long)k * PQ] = (bb & 1) ? acc[a][bb >> 1].y : acc[a][bb >> 1].x;
     }
   }
 }

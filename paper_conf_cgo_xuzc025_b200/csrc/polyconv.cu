@@ -105,16 +105,16 @@ bool fft_pays(const Geom& g) {
   if (getenv("POLYCONV_NO_FFT") || g.K < 16) return false;
   const FftTiling t = fft_tiling(g);
   if (!t.ok) return false;
-  // r = taps x outputs per FFT bin.  Against the direct FFMA kernel (mac_fp32, round 2b),
-  // measured on all 71 FP32 layers (profiles/r03_fp32_cmp.jsonl, TFLOP/s FFT / FFMA): the FFT
-  // wins only on short transforms -- L <= 256 (l4 3x3 40 / 31), L = 512 at stride 2 or r >= 8
-  // (l4 3x3 s2 9.7 / 9.0, A_h14_s1 25.2 / 24.0; l3 3x3 29 / 34 loses), L = 1024 at stride 2
-  // or with C*K >= 128K (l3 3x3 s2 12.8 / 9.7, VGG conv4 56 / 38; conv3_x 20 / 32 loses).
+  // r = taps x outputs per FFT bin.  Against the direct FFMA kernel (mac_fp32 with packed FFMA2,
+  // round 2b), measured on all 71 FP32 layers (profiles/r03_fp32_cmp.jsonl, TFLOP/s FFT / FFMA):
+  // the FFT wins only on short transforms -- L <= 256 (l4 3x3 40 / 32), L = 512 at stride 2
+  // (l4 3x3 s2 9.7 / 9.4; l3 3x3 29 / 35 and A_h14_s1 25.5 / 26.8 lose), L = 1024 at stride 2
+  // or with C*K >= 128K (l3 3x3 s2 12.8 / 10.1, VGG conv4 56 / 40; conv3_x 20 / 32 loses).
   const double r = (double)g.R * g.S * g.P * g.Q / t.L;
   if (r < 0.8 || g.N < 64) return false;  // every measured FFT win had N >= 64
   const bool s2 = g.sh > 1;
   if (t.L <= 256) return true;
-  if (t.L <= 512) return s2 || r >= 8.0;
+  if (t.L <= 512) return s2;
   if (t.L <= 1024) return (s2 && r >= 1.5) || ((long long)g.C * g.K >= 131072 && r >= 4.0);
   return false;
 }
