@@ -49,7 +49,29 @@ struct P1x1 {
   int epi_tma;  // 1: stage each warp's 32 channels x NT pixels (SW128) and TMA-store them;
                 // 2: whole planes (one position block): stage the warp's 32 channel planes densely
                 //    (a contiguous run of y) and write them with one bulk copy
+  int resA;     // 1: each CTA keeps one 128-channel filter block resident (loaded once) and walks
+                //    its images / position blocks, so only the x planes stream through the ring
+  int groups;   // resA: CTAs per filter block (gridDim.x = groups * num_kt)
 };
+
+// The CTA's i-th tile: (filter block kt, position block pb, image n).  resA: a CTA's tiles
+// share kt = blockIdx.x % num_kt; else tiles t = blockIdx.x + i * gridDim.x, kt fastest.
+__device__ __forceinline__ bool tile_of(const P1x1& p, int i, int& kt, int& pb, int& n) {
+  int rest;
+  if (p.resA) {
+    kt = blockIdx.x % p.num_kt;
+    rest = blockIdx.x / p.num_kt + i * p.groups;
+    if (rest >= p.N * p.num_pb) return false;
+  } else {
+    const long long t = blockIdx.x + (long long)i * gridDim.x;
+    if (t >= p.num_tiles) return false;
+    kt = (int)(t % p.num_kt);
+    rest = (int)(t / p.num_kt);
+  }
+  pb = rest % p.num_pb;
+  n = rest / p.num_pb;
+  return true;
+}
 
 __device__ __forceinline__ uint64_t desc_mn(uint32_t saddr) {
   // MN-major, 128-byte swizzle: LBO = 8192 (next 64-position box), SBO = 1024 (next 8 k-rows)
@@ -75,14 +97,15 @@ __global__ void __launch_bounds__(k1Threads, 1)
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw = smem_u32(smem_raw);
   uint8_t* smem = smem_raw + (((raw + 1023u) & ~1023u) - raw);
-  uint8_t* sA = smem;                                      // [stages][128 rows][128 B]
-  uint8_t* sB = sA + (size_t)p.stages * p.a_bytes;         // [stages][nbox][64 ch][128 B]
+  uint8_t* sA = smem;  // [stages][128 rows][128 B], resA: [kchunks][128 rows][128 B] resident
+  uint8_t* sB = sA + (p.resA ? (size_t)p.kchunks * p.a_bytes : (size_t)p.stages * p.a_bytes);  // [stages][nbox][64 ch][128 B]
   uint8_t* sE = sB + (size_t)p.stages * p.b_bytes;          // epi_tma: [4 warps][nbox][32 ch][128 B]
   uint64_t* full = reinterpret_cast<uint64_t*>(sE + (p.epi_tma ? (size_t)p.nbox * 16384 : 0));
   uint64_t* empty = full + k1MaxStages;
   uint64_t* tfull = empty + k1MaxStages;
   uint64_t* tempty = tfull + 2;
-  uint32_t* tslot = reinterpret_cast<uint32_t*>(tempty + 2);
+  uint64_t* afull = tempty + 2;  // resA: the resident filter block landed
+  uint32_t* tslot = reinterpret_cast<uint32_t*>(afull + 1);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     prefetch_tmap(&tmU);
@@ -96,6 +119,7 @@ __global__ void __launch_bounds__(k1Threads, 1)
       mbar_init(tfull + a, 1);
       mbar_init(tempty + a, 4);
     }
+    mbar_init(afull, 1);
     fence_barrier_init();
   }
   if (warp == 1) tmem_alloc(tslot, (uint32_t)p.tmem_cols);
@@ -109,14 +133,19 @@ __global__ void __launch_bounds__(k1Threads, 1)
   if (warp == 0) {
     int st = 0;
     uint32_t ph = 0;
-    for (int t = blockIdx.x; t < p.num_tiles; t += gridDim.x) {
-      const int kt = t % p.num_kt, rest = t / p.num_kt;
-      const int pb = rest % p.num_pb, n = rest / p.num_pb;
+    int kt, pb, n;
+    if (p.resA && tile_of(p, 0, kt, pb, n) && elect_one()) {
+      mbar_arrive_expect_tx(afull, (uint32_t)p.kchunks * p.a_bytes);
+      for (int kc = 0; kc < p.kchunks; ++kc)
+        tma_load_2d(sA + (size_t)kc * p.a_bytes, &tmU, afull, kc * 64, kt * 128);
+    }
+    __syncwarp();
+    for (int i = 0; tile_of(p, i, kt, pb, n); ++i) {
       for (int kc = 0; kc < p.kchunks; ++kc) {
         mbar_wait(empty + st, ph ^ 1u);
         if (elect_one()) {
-          mbar_arrive_expect_tx(full + st, p.a_bytes + (uint32_t)p.nbox * 8192u);
-          tma_load_2d(sA + (size_t)st * p.a_bytes, &tmU, full + st, kc * 64, kt * 128);
+          mbar_arrive_expect_tx(full + st, (p.resA ? 0u : p.a_bytes) + (uint32_t)p.nbox * 8192u);
+          if (!p.resA) tma_load_2d(sA + (size_t)st * p.a_bytes, &tmU, full + st, kc * 64, kt * 128);
           for (int b = 0; b < p.nbox; ++b)
             tma_load_2d(sB + (size_t)st * p.b_bytes + (size_t)b * 8192, &tmX, full + st, pb * p.NT + b * 64,
                         n * p.C + kc * 64);
@@ -128,7 +157,12 @@ __global__ void __launch_bounds__(k1Threads, 1)
   } else if (warp == 1) {
     int st = 0, lt = 0;
     uint32_t ph = 0;
-    for (int t = blockIdx.x; t < p.num_tiles; t += gridDim.x, ++lt) {
+    int kt, pb, n;
+    if (p.resA && tile_of(p, 0, kt, pb, n)) {
+      mbar_wait(afull, 0);
+      tc_fence_after();
+    }
+    for (; tile_of(p, lt, kt, pb, n); ++lt) {
       const int a = lt & 1;
       mbar_wait(tempty + a, (uint32_t)((lt >> 1) & 1) ^ 1u);
       tc_fence_after();
@@ -136,7 +170,7 @@ __global__ void __launch_bounds__(k1Threads, 1)
       for (int kc = 0; kc < p.kchunks; ++kc) {
         mbar_wait(full + st, ph);
         tc_fence_after();
-        const uint64_t ad = make_sdesc(smem_u32(sA + (size_t)st * p.a_bytes), 128, 0);
+        const uint64_t ad = make_sdesc(smem_u32(sA + (size_t)(p.resA ? kc : st) * p.a_bytes), 128, 0);
         const uint64_t bd = desc_mn(smem_u32(sB + (size_t)st * p.b_bytes));
         if (elect_one()) {
 #pragma unroll
@@ -154,10 +188,8 @@ __global__ void __launch_bounds__(k1Threads, 1)
     // epilogue: lane = output channel (quadrant warp % 4), 32 positions per TMEM load
     const int q = warp & 3;
     __nv_bfloat16* y = static_cast<__nv_bfloat16*>(p.y);
-    int lt = 0;
-    for (int t = blockIdx.x; t < p.num_tiles; t += gridDim.x, ++lt) {
-      const int kt = t % p.num_kt, rest = t / p.num_kt;
-      const int pb = rest % p.num_pb, n = rest / p.num_pb;
+    int lt = 0, kt, pb, n;
+    for (; tile_of(p, lt, kt, pb, n); ++lt) {
       const int a = lt & 1;
       mbar_wait_sleep(tfull + a, (uint32_t)((lt >> 1) & 1), 64);
       tc_fence_after();
@@ -384,7 +416,15 @@ cudaError_t launch_mac_1x1(const Geom& g, const void* x, const void* U, int Kp, 
   const bool ep_ok = g.K % 32 == 0 && (reinterpret_cast<uintptr_t>(y) & 15) == 0 && (ev == nullptr || ev[0] != '0');
   p.epi_tma = !ep_ok ? 0 : (p.num_pb == 1 && g.K % 8 == 0) ? 2 : (p.HWo % 8 == 0 ? 1 : 0);
   const int estage = p.epi_tma ? p.nbox * 16384 : 0;
-  p.stages = std::min(k1MaxStages, (227 * 1024 - 2048 - estage) / per);
+  // resident filter block: every CTA's tiles share one 128-channel block, which is loaded
+  // once, so only x streams (C <= 384: at most 96 KB; POLYCONV_1X1_RESA=0 turns it off)
+  const char* er = getenv("POLYCONV_1X1_RESA");
+  const int resA_bytes = p.kchunks * (int)p.a_bytes;
+  p.resA = (er == nullptr || er[0] != '0') && resA_bytes <= 96 * 1024 && p.num_kt <= num_sms &&
+           (long long)g.N * p.num_pb >= num_sms / p.num_kt;
+  p.groups = p.resA ? num_sms / p.num_kt : 0;
+  p.stages = p.resA ? std::min(k1MaxStages, (227 * 1024 - 2048 - estage - resA_bytes) / (int)p.b_bytes)
+                    : std::min(k1MaxStages, (227 * 1024 - 2048 - estage) / per);
   if (p.stages < 2) {
     snprintf(err, errlen, "mac_1x1: shared memory");
     return cudaErrorInvalidValue;
@@ -400,11 +440,12 @@ cudaError_t launch_mac_1x1(const Geom& g, const void* x, const void* U, int Kp, 
     snprintf(err, errlen, "mac_1x1: cuTensorMapEncodeTiled failed");
     return cudaErrorInvalidValue;
   }
-  const int smem = 1024 + p.stages * per + estage + 1024;
+  const int smem = p.resA ? 1024 + resA_bytes + p.stages * (int)p.b_bytes + estage + 1024
+                         : 1024 + p.stages * per + estage + 1024;
   cudaError_t e = cudaFuncSetAttribute(mac_1x1_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   if (e != cudaSuccess) return e;
   cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3((unsigned)std::min(p.num_tiles, num_sms));
+  cfg.gridDim = dim3((unsigned)(p.resA ? p.groups * p.num_kt : std::min(p.num_tiles, num_sms)));
   cfg.blockDim = dim3(k1Threads);
   cfg.dynamicSmemBytes = (size_t)smem;
   cfg.stream = st;
