@@ -198,13 +198,6 @@ __device__ __forceinline__ void hk_tmem_alloc2(uint32_t* slot, uint32_t ncols) {
 __device__ __forceinline__ void hk_tmem_dealloc2(uint32_t taddr, uint32_t ncols) {
   asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(taddr), "r"(ncols) : "memory");
 }
-// 32 lanes x 8 consecutive 32-bit columns
-__device__ __forceinline__ void hk_tmem_ld8(uint32_t taddr, uint32_t (&v)[8]) {
-  asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
-               : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7])
-               : "r"(taddr)
-               : "memory");
-}
 // 32 lanes x 16 consecutive 32-bit columns
 __device__ __forceinline__ void hk_tmem_ld16(uint32_t taddr, uint32_t (&v)[16]) {
   asm volatile(
@@ -800,45 +793,33 @@ __global__ void __launch_bounds__(kHkThreads, 1)
             ybase = ((long long)n * p.Ktot + p.koff + it.nb * p.NN) * PQ + (long long)oh * p.Q + ow;
         }
         const uint32_t trow = tbase + ((uint32_t)(quad * 32) << 16) + (uint32_t)(a * p.T * p.NN + t * p.NN);
-        // this warp's 8-column chunks (16-column groups half, half + 2, ...), the TMEM load of
-        // chunk i + 1 in flight while chunk i is stored (tcgen05.wait::ld after the stores)
-        const int nchunk = 2 * ((p.NN / 16 - half + 1) / 2);
-#define HK_STORE8(V, I)                                                                              \
-  do {                                                                                               \
-    const int col_ = (half + 2 * ((I) >> 1)) * 16 + ((I) & 1) * 8;                                   \
-    if (ybase >= 0 && !(p.dbg & 2)) {                                                                \
-      const int kleft_ = p.K - (it.nb * p.NN + col_); /* output channels left (warp-uniform) */      \
-      for (int o = 0; o < p.nys; ++o) { /* f4: every output buffer (peer stores over NVLink) */      \
-        IoT* yp_ = static_cast<IoT*>(p.ys[o]) + ybase + (long long)col_ * PQ;                         \
-        if (kHW2 > 0 && pq_const && kleft_ >= 8) { /* baked-in plane size: immediate offsets */       \
-          _Pragma("unroll") for (int c = 0; c < 8; ++c)                                              \
-              hk_store<IoT>(yp_, (long long)c * (2 * (kHW2 > 0 ? kHW2 : 1)), __uint_as_float(V[c]));  \
-        } else {                                                                                     \
-          _Pragma("unroll") for (int c = 0; c < 8; ++c) if (c < kleft_)                              \
-              hk_store<IoT>(yp_, (long long)c * PQ, __uint_as_float(V[c]));                           \
-        }                                                                                            \
-      }                                                                                              \
-    }                                                                                                \
-  } while (0)
-#define HK_LD8(V, I)                                                                                 \
-  do {                                                                                               \
-    const int col_ = (half + 2 * ((I) >> 1)) * 16 + ((I) & 1) * 8;                                   \
-    if (!(p.dbg & 512)) hk_tmem_ld8(trow + (uint32_t)col_, V);                                       \
-    else { _Pragma("unroll") for (int c = 0; c < 8; ++c) V[c] = 0u; }                                \
-  } while (0)
-        uint32_t va[8], vb[8];
-        if (nchunk > 0) HK_LD8(va, 0);
-        tmem_ld_wait();
-        for (int i = 0; i < nchunk; i += 2) {
-          if (i + 1 < nchunk) HK_LD8(vb, i + 1);
-          HK_STORE8(va, i);
-          tmem_ld_wait();
-          if (i + 2 < nchunk) HK_LD8(va, i + 2);
-          if (i + 1 < nchunk) HK_STORE8(vb, i + 1);
-          tmem_ld_wait();
+        for (int g = half; g * 16 < p.NN; g += 2) {
+          uint32_t v[16];
+          if (!(p.dbg & 512)) {
+            hk_tmem_ld16(trow + (uint32_t)(g * 16), v);
+            tmem_ld_wait();
+          } else {
+#pragma unroll
+            for (int c = 0; c < 16; ++c) v[c] = 0u;
+          }
+          if (ybase >= 0 && !(p.dbg & 2)) {
+            const int kleft = p.K - (it.nb * p.NN + g * 16);  // output channels left (warp-uniform)
+            // every output buffer (f4: the K-shard all-gather as peer stores over NVLink)
+            for (int o = 0; o < p.nys; ++o) {
+              IoT* yp = static_cast<IoT*>(p.ys[o]) + ybase + (long long)(g * 16) * PQ;
+              if (kHW2 > 0 && pq_const && kleft >= 16) {
+                // same-size output with a baked-in plane size: one base register, immediate offsets
+#pragma unroll
+                for (int c = 0; c < 16; ++c)
+                  hk_store<IoT>(yp, (long long)c * (2 * (kHW2 > 0 ? kHW2 : 1)), __uint_as_float(v[c]));
+              } else {
+#pragma unroll
+                for (int c = 0; c < 16; ++c)
+                  if (c < kleft) hk_store<IoT>(yp, (long long)c * PQ, __uint_as_float(v[c]));
+              }
+            }
+          }
         }
-#undef HK_STORE8
-#undef HK_LD8
       }
       tc_fence_before();
       __syncwarp();
