@@ -163,8 +163,9 @@ polyconv_status_t polyconv_forward(polyconv_plan_t plan, const void *x, const vo
  * epilogue: no local copy, no separate collective.  1 <= n_out <= 8, 0 <= k_offset,
  * k_offset + K <= k_total; all pointers 16-byte aligned (else NOT_SUPPORTED).  The caller
  * orders the peers' reads after this forward (stream order plus a cross-rank barrier).  Only
- * the TC_HANKEL kernel stores to peers: NOT_SUPPORTED (nothing enqueued) for plans that
- * resolved to another kernel.  Other errors as polyconv_forward. */
+ * the TC_HANKEL kernel of stride-1 plans stores to peers: NOT_SUPPORTED for plans that resolved
+ * to another kernel or to its stride-2 phase mode (nothing written to ys).  Other errors as
+ * polyconv_forward. */
 polyconv_status_t polyconv_forward_scatter(polyconv_plan_t plan, const void *x, const void *w,
                                            void *const *ys, int n_out, int k_total, int k_offset,
                                            void *stream);

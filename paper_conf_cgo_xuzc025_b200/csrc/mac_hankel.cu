@@ -535,7 +535,10 @@ __device__ __forceinline__ void hk_store<__nv_bfloat16>(__nv_bfloat16* y, long l
   y[i] = __float2bfloat16_rn(v);
 }
 
-template <typename IoT, bool kTf32, int kHW2, int kKC = (kTf32 ? 32 : 64)>
+// kScatter: the epilogue stores to every buffer of p.ys at channel offset p.koff of p.Ktot
+// (polyconv_forward_scatter); the plain forward (one output, its own channels) keeps the single
+// store path (a runtime output loop there cost up to 4 us per ResNet-50 layer, same-box A/B)
+template <typename IoT, bool kTf32, int kHW2, int kKC = (kTf32 ? 32 : 64), bool kScatter = false>
 __global__ void __launch_bounds__(kHkThreads, 1)
     mac_hankel_kernel(const __grid_constant__ CUtensorMap tmU, const HkParams p) {
   extern __shared__ uint8_t smem_raw[];
@@ -765,6 +768,7 @@ __global__ void __launch_bounds__(kHkThreads, 1)
     const int quad = warp & 3;      // TMEM lane quadrant this warp may access
     const int half = e & 1;         // column groups half, half + 2, ...
     const uint32_t tbase = *tmem_slot;
+    IoT* y = static_cast<IoT*>(p.ys[0]);
     const long long PQ = (long long)p.P * p.Q;
     // plane size of y as a compile-time constant when the output has the input's size
     const bool pq_const = kHW2 > 0 && PQ == 2LL * kHW2;
@@ -790,7 +794,8 @@ __global__ void __launch_bounds__(kHkThreads, 1)
           const uint32_t oh = p.fsh.div(ohs), ow = p.fsw.div(col);
           if ((int)n < p.N && oh * (uint32_t)p.sh == ohs && ow * (uint32_t)p.sw == col && (int)oh < p.P &&
               (int)ow < p.Q)
-            ybase = ((long long)n * p.Ktot + p.koff + it.nb * p.NN) * PQ + (long long)oh * p.Q + ow;
+            ybase = kScatter ? ((long long)n * p.Ktot + p.koff + it.nb * p.NN) * PQ + (long long)oh * p.Q + ow
+                             : ((long long)n * p.K + it.nb * p.NN) * PQ + (long long)oh * p.Q + ow;
         }
         const uint32_t trow = tbase + ((uint32_t)(quad * 32) << 16) + (uint32_t)(a * p.T * p.NN + t * p.NN);
         for (int g = half; g * 16 < p.NN; g += 2) {
@@ -804,9 +809,16 @@ __global__ void __launch_bounds__(kHkThreads, 1)
           }
           if (ybase >= 0 && !(p.dbg & 2)) {
             const int kleft = p.K - (it.nb * p.NN + g * 16);  // output channels left (warp-uniform)
-            // every output buffer (f4: the K-shard all-gather as peer stores over NVLink)
-            for (int o = 0; o < p.nys; ++o) {
-              IoT* yp = static_cast<IoT*>(p.ys[o]) + ybase + (long long)(g * 16) * PQ;
+            if constexpr (kScatter) {
+              // every output buffer (f4: the K-shard all-gather as peer stores over NVLink)
+              for (int o = 0; o < p.nys; ++o) {
+                IoT* yp = static_cast<IoT*>(p.ys[o]) + ybase + (long long)(g * 16) * PQ;
+#pragma unroll
+                for (int c = 0; c < 16; ++c)
+                  if (c < kleft) hk_store<IoT>(yp, (long long)c * PQ, __uint_as_float(v[c]));
+              }
+            } else {
+              IoT* yp = y + ybase + (long long)(g * 16) * PQ;
               if (kHW2 > 0 && pq_const && kleft >= 16) {
                 // same-size output with a baked-in plane size: one base register, immediate offsets
 #pragma unroll
@@ -1081,6 +1093,7 @@ cudaError_t launch_mac_hankel(const Geom& g0, const HankelTiling& t, int fmt, co
   // kHW2: -1 = general loader, 0 = pair-aligned loader with a runtime plane size, > 0 = the
   // plane size in words baked in (immediate channel offsets) for the ResNet / VGG planes
   void (*kern)(const CUtensorMap, const HkParams);
+  const bool scatter = nys > 1 || ktot != g0.K || koff != 0;
   const int hw2 = g.H * g.W / 2;
   if (!t.phase && t.kc == 16) {
     if (!t.aligned) {
@@ -1108,6 +1121,15 @@ cudaError_t launch_mac_hankel(const Geom& g0, const HankelTiling& t, int fmt, co
            : hw2 == 392 ? mac_hankel_kernel<__nv_bfloat16, false, 392>
            : hw2 == 98  ? mac_hankel_kernel<__nv_bfloat16, false, 98>
                         : mac_hankel_kernel<__nv_bfloat16, false, 0>;
+  }
+  if (scatter) {
+    // the scatter epilogue: stride-1 plans with 128-byte window rows, the general loader
+    if (t.phase || t.kc * (tf32 ? 4 : 2) != 128) {
+      snprintf(err, errlen, "mac_hankel: forward_scatter needs a stride-1 plan with 128-byte window rows");
+      return cudaErrorNotSupported;
+    }
+    kern = tf32 ? mac_hankel_kernel<float, true, -1, 32, true>
+                : (io_bf16 ? mac_hankel_kernel<__nv_bfloat16, false, -1, 64, true> : mac_hankel_kernel<float, false, -1, 64, true>);
   }
   cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, t.smem_bytes);
   if (e != cudaSuccess) return e;

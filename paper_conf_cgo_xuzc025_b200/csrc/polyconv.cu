@@ -525,6 +525,7 @@ static polyconv_status_t forward_hankel(polyconv_plan_t p, const void* x, const 
   e = launch_mac_hankel(g, p->hk, p->fmt, x, p->io_bf16, p->wsU, ys, nys, ktot, koff, p->hkzero, st, p->err,
                         sizeof(p->err));
   if (p->ev_stop) cudaEventRecord(p->ev_stop, st);
+  if (e == cudaErrorNotSupported) return POLYCONV_STATUS_NOT_SUPPORTED;  // (the filter pack is harmless)
   return finish(p, e, "mac_hankel");
 }
 

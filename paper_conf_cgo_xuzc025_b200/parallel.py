@@ -112,7 +112,12 @@ def sharded_forward(x, w, stride=(1, 1), padding=(0, 0), math="bf16", group=None
     if sh.k1 - sh.k0 < kb:  # tail block: zero filters for the padding channels
         w_loc = torch.cat([w_loc, w.new_zeros((kb - (sh.k1 - sh.k0),) + tuple(w.shape[1:]))])
     if fused:
-        return _fused_kshard(x, w_loc.contiguous(), sh, kb, K, stride, padding, math, group, world, rank)
+        from . import PolyconvError, NOT_SUPPORTED
+        try:
+            return _fused_kshard(x, w_loc.contiguous(), sh, kb, K, stride, padding, math, group, world, rank)
+        except PolyconvError as e:  # a plan whose kernel does not store to peers: the NCCL gather
+            if e.status != NOT_SUPPORTED:
+                raise
     send = torch.empty((N, kb, P, Q), dtype=x.dtype, device=x.device)
     compute(x, w_loc.contiguous(), stride, padding, math, send)
     # gather the K blocks: [world][N][kb][P][Q] -> [N][K][P][Q]

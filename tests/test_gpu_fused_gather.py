@@ -22,7 +22,7 @@ pytestmark = pytest.mark.gpu
 @pytest.mark.parametrize("shape,k_total,k_off", [
     (synth.ConvShape("blk64", 2, 64, 14, 14, 64, 3, 3, 1, 1, 1, 1), 160, 64),   # middle block
     (synth.ConvShape("blk32", 3, 32, 28, 28, 32, 3, 3, 1, 1, 1, 1), 96, 64),    # last block
-    (synth.ConvShape("blk_s2", 2, 64, 16, 16, 64, 3, 3, 2, 2, 1, 1), 128, 0)])  # stride 2 (phase mode)
+    (synth.ConvShape("blk_oddw", 2, 64, 9, 7, 64, 3, 3, 1, 1, 1, 1), 128, 0)])  # odd width
 def test_forward_scatter_into_several_outputs(shape, k_total, k_off):
     x, w = synth.make_inputs(shape, synth.seed_for(41, shape.K), "int")
     ref = bf16_round(oracle.conv2d(x, w, shape.stride, shape.padding))
@@ -52,6 +52,11 @@ def test_forward_scatter_errors():
         plan.forward_scatter(xt, wt, [y.data_ptr()], 128, 96)
     with pytest.raises(pc.PolyconvError):      # more than 8 outputs
         plan.forward_scatter(xt, wt, [y.data_ptr()] * 9, 128, 0)
+    x2 = torch.zeros((1, 64, 16, 16), dtype=torch.bfloat16, device="cuda")   # stride 2: phase mode
+    p2 = pc.Plan(x2.shape, wt.shape, (2, 2), (1, 1), math="bf16", io_dtype="bf16", kernel="tc_hankel")
+    with pytest.raises(pc.PolyconvError) as ei:
+        p2.forward_scatter(x2, wt, [y.data_ptr()], 128, 0)
+    assert ei.value.status == pc.NOT_SUPPORTED
     x32, w32 = xt.float(), wt.float()          # FP32_FMA plan: not the hankel kernel
     p32 = pc.Plan(x32.shape, w32.shape, shape.stride, shape.padding, math="fp32", io_dtype="f32")
     with pytest.raises(pc.PolyconvError) as ei:
