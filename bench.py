@@ -75,14 +75,20 @@ def _roofline_peak(math, peaks):
         "148 SM x 128 FP32 lanes x 2 FLOP x sm_max_mhz"
 
 
-def _traffic(kernel_key):
-    """dram bytes per launch of the dominant kernel from the committed ncu
-    --set full summary (profiles/ncu_summary.json), else None."""
+def _traffic(kernel_key, field="dram"):
+    """Bytes per launch of the dominant kernel from the committed ncu --set full summary
+    (profiles/ncu_summary.json), else None.  field "dram": dram read + write; "l2_write": the
+    bytes the kernel writes into L2 (32-byte sectors) -- the output y stays dirty in L2 when
+    the kernel ends, so its DRAM write-back is not in the kernel's own dram counters."""
     try:
         with open(os.path.join(PROFILES, "ncu_summary.json")) as f:
             d = json.load(f)
         e = d.get(kernel_key)
-        return int(e["dram_bytes_read"] + e["dram_bytes_write"]) if e else None
+        if not e:
+            return None
+        if field == "l2_write":
+            return int(e["l2_write_sectors"] * 32)
+        return int(e["dram_bytes_read"] + e["dram_bytes_write"])
     except (OSError, ValueError, KeyError, TypeError):
         return None
 
@@ -482,6 +488,10 @@ def main():
                    "l2": "flushed between steps (256 MiB write, then 256 MiB read so no dirty lines remain)", "inputs": "seeded synth 'uniform'"},
         "roofline": {"bound": bound, "achieved": achieved, "peak": peak,
                      "unit": "TFLOP/s", "frac": achieved / peak, "traffic": _traffic("mac_%s_%s" % (info["kernel"], args.math)),
+                     "traffic_l2_write": _traffic("mac_%s_%s" % (info["kernel"], args.math), "l2_write"),
+                     "traffic_note": "traffic = the launch's dram read + write (ncu); y stays dirty in L2 at the "
+                                     "end of the launch, so its write-back shows in traffic_l2_write instead",
+                     "algorithmic_bytes": alg_bytes,
                      "kernel": "mac_%s" % info["kernel"], "kernel_ms": t_kern_ms,
                      "kernel_timing": "CUDA events recorded by the library around its launch (own pass of K steps)",
                      "algorithmic": "2*N*K*C*R*S*P*Q = %.4g FLOP per launch" % F,
