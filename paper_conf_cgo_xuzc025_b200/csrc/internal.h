@@ -175,6 +175,9 @@ struct HankelTiling {
   // stride-2 phase mode (reading R19): the kernel runs on the phase-split geometry
   int phase, eC, eH, eW, eR, eS, eph, epw;
   int kc;  // channels per window row: 64 bf16 / 32 tf32 (128 B), 16 bf16 (32 B, small-C phase mode)
+  // plane-staged loader: whole (image, 64-channel) blocks of x by bulk copy, two staging buffers
+  int planes, pimg_max;
+  uint32_t pimg_bytes;
 };
 HankelTiling hankel_tiling(const Geom& g, int fmt, int num_sms, bool io_bf16);
 // x: NCHW input (io dtype); U: tap-major packed filter [RS][Kp][Cp] (t.Kp, t.Cp), packed by

@@ -117,6 +117,9 @@ struct HkParams {
   // phase-split input; N, C, H, W, ph, pw, sh, sw above are that convolution's, these are x's
   int phase;            // 0 / 1
   int xC, xH, xW;       // x dims (phase mode)
+  // plane-staged loader (kHW2 == kHkPlanes): whole (image, 64-channel) blocks of x, bulk-copied
+  uint32_t pimg_bytes;  // 64 * H * W * 2: one image's 64-channel block (16-byte multiple)
+  int pimg_max;         // images a window can touch (staging buffer = pimg_max blocks)
   int dbg;  // POLYCONV_HK_DEBUG (timing ablations, results wrong): 1 loaders store zeros without
             // loading, 2 epilogue skips stores, 4 no MMAs (commits only), 8 per-CTA trace
 };
@@ -523,6 +526,54 @@ __device__ __forceinline__ void hk_load_window_phase(const HkParams& p, uint32_t
   }
 }
 
+// Plane-staged window (bf16 in and math, stride 1, C % 64 == 0; small planes such as 7x7,
+// where the element loader above does two 4-byte loads per element): each window touches a few
+// whole images, and one image's block of 64 channel planes is one contiguous, 16-byte aligned
+// run of x (64*H*W*2 bytes), so the window forwarder bulk-copies those blocks into a staging
+// buffer (two buffers, one window ahead) and the loader warps transpose from shared memory:
+// 8 two-byte reads (one per channel of the warp's 16-byte group) per position, one 16-byte
+// swizzled store per window row (zeros for padding rows / columns).
+constexpr int kHkPlanes = -9;
+// first image of the window at origin q0 (images before it hold no element of the window)
+__device__ __forceinline__ int hk_window_img0(const HkParams& p, long long q0) {
+  const long long qq = max(q0 - p.delta, 0LL);
+  const int vr = (int)p.fpitch.div((uint32_t)qq) - p.ph;
+  return vr < 0 ? 0 : (int)p.fHS.div((uint32_t)vr);
+}
+__device__ __forceinline__ void hk_planes_issue(const HkParams& p, long long q0, int c0, uint32_t stg, uint64_t* bar) {
+  const int n0 = hk_window_img0(p, q0);
+  const int nimg = max(0, min(p.pimg_max, p.N - n0));
+  mbar_arrive_expect_tx(bar, (uint32_t)nimg * p.pimg_bytes);
+  for (int i = 0; i < nimg; ++i) {
+    const char* src = static_cast<const char*>(p.x) + ((long long)(n0 + i) * p.C + c0) * p.HW * 2;
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                     stg + (uint32_t)i * p.pimg_bytes),
+                 "l"(src), "r"(p.pimg_bytes), "r"(smem_u32(bar))
+                 : "memory");
+  }
+}
+__device__ __forceinline__ void hk_planes_transpose(const HkParams& p, long long q0, uint32_t stg, uint32_t slot,
+                                                    int lw, int lane, int r_lo, int r_hi) {
+  const int n0 = hk_window_img0(p, q0);
+  for (int r = r_lo + lane; r < r_hi; r += 32) {
+    int n, h, w;
+    uint32_t d[4] = {0u, 0u, 0u, 0u};
+    if (hk_pos(p, q0 + r, n, h, w) && n - n0 < p.pimg_max) {
+      const uint32_t e = stg + (((uint32_t)(n - n0) * 64u + (uint32_t)lw * 8u) * (uint32_t)p.HW + (uint32_t)(h * p.W + w)) * 2u;
+#pragma unroll
+      for (int c = 0; c < 4; ++c) {
+        uint16_t lo, hi;
+        asm volatile("ld.shared.u16 %0, [%1];" : "=h"(lo) : "r"(e + (uint32_t)(2 * c) * (uint32_t)p.HW * 2u));
+        asm volatile("ld.shared.u16 %0, [%1];" : "=h"(hi) : "r"(e + (uint32_t)(2 * c + 1) * (uint32_t)p.HW * 2u));
+        d[c] = (uint32_t)lo | ((uint32_t)hi << 16);
+      }
+    }
+    const uint32_t a = slot + (uint32_t)r * 128u + ((((uint32_t)lw) ^ ((uint32_t)r & 7u)) << 4);
+    asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(a), "r"(d[0]), "r"(d[1]), "r"(d[2]), "r"(d[3])
+                 : "memory");
+  }
+}
+
 // ---- a5: one accumulator tile to NCHW y -------------------------------------------------
 template <typename IoT>
 __device__ __forceinline__ void hk_store(IoT* y, long long i, float v);
@@ -547,7 +598,8 @@ __global__ void __launch_bounds__(kHkThreads, 1)
   const uint32_t sF = smem_u32(smem);                                   // filter blocks
   const uint32_t sW = sF + (uint32_t)p.fslots * p.fblk_bytes;           // window ring (1 KB aligned)
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + (size_t)p.fslots * p.fblk_bytes +
-                                               (size_t)p.wslots * p.wslot_bytes);
+                                               (size_t)p.wslots * p.wslot_bytes +
+                                               (kHW2 == kHkPlanes ? 2 * (size_t)p.pimg_max * p.pimg_bytes : 0));
   uint64_t* ffull = bars;                    // [kHkMaxFBlk] leader: both halves landed
   uint64_t* fempty = ffull + kHkMaxFBlk;     // [kHkMaxFBlk] both: MMAs done with the block
   uint64_t* wfull = fempty + kHkMaxFBlk;     // [kHkMaxWSlots] leader: both CTAs' loaders done
@@ -560,7 +612,9 @@ __global__ void __launch_bounds__(kHkThreads, 1)
   // (ncu: ERRBAR / membar was the loaders' largest stall after the loads themselves).
   uint64_t* wloc = tempty + 2;               // [kHkMaxWSlots] this CTA's loaders done
   uint64_t* eloc = wloc + kHkMaxWSlots;      // [2] this CTA's epilogue warps drained
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(eloc + 2);
+  uint64_t* sfull = eloc + 2;                // [2] plane-staged loader: a window's blocks landed
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(sfull + 2);
+  const uint32_t sS = sW + (uint32_t)p.wslots * p.wslot_bytes;  // plane-staged loader: 2 staging buffers
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   // window / filter rows: kKC channels of 128 B (SW128) or, for the small-C phase convolution
@@ -591,6 +645,7 @@ __global__ void __launch_bounds__(kHkThreads, 1)
       mbar_init(tfull + i, 1);
       mbar_init(tempty + i, 2);
       mbar_init(eloc + i, kHkEpiWarps);
+      mbar_init(sfull + i, 1);
     }
     fence_barrier_init();
   }
@@ -704,7 +759,26 @@ __global__ void __launch_bounds__(kHkThreads, 1)
     const int nrp_all = p.wrows >> 1;
     const int per = ((nrp_all + kSlices - 1) / kSlices + 31) / 32 * 32;
     const int rp_lo = min(sl * per, nrp_all), rp_hi = min((sl + 1) * per, nrp_all);
-    {
+    if constexpr (kHW2 == kHkPlanes) {
+      long long u = u_lo;
+      HkItem it;
+      int ws = 0, wuse = 0, sb = 0, suse = 0;
+      while (hk_next(p, u, u_hi, it)) {
+        const long long q0 = (long long)it.pt * 256 + (long long)rank * 128 * it.T;
+        for (int ch = 0; ch < p.nchunks; ++ch) {
+          hk_wait(wempty + ws, (uint32_t)(wuse & 1) ^ 1u);
+          hk_wait(sfull + sb, (uint32_t)(suse & 1));
+          if (!(p.dbg & 1))
+            hk_planes_transpose(p, q0, sS + (uint32_t)sb * (uint32_t)p.pimg_max * p.pimg_bytes,
+                                sW + (uint32_t)ws * p.wslot_bytes, lw, lane, 2 * rp_lo, 2 * rp_hi);
+          if (++sb == 2) { sb = 0; ++suse; }
+          asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> MMA reads
+          __syncwarp();
+          if (lane == 0) mbar_arrive(wloc + ws);
+          if (++ws == p.wslots) { ws = 0; ++wuse; }
+        }
+      }
+    } else {
       long long u = u_lo;
       HkItem it;
       int ws = 0, wuse = 0;
@@ -741,12 +815,39 @@ __global__ void __launch_bounds__(kHkThreads, 1)
     long long u = u_lo;
     HkItem it;
     int ws = 0, wuse = 0;
-    while (hk_next(p, u, u_hi, it)) {
-      for (int ch = 0; ch < p.nchunks; ++ch) {
-        hk_wait(wloc + ws, (uint32_t)(wuse & 1));
-        if (lane == 0) hk_arrive_cluster(wfull0 + (uint32_t)ws * 8u);
+    if constexpr (kHW2 == kHkPlanes) {
+      // plane-staged loader: window w's blocks go to staging buffer w % 2; window w + 2's are
+      // fetched once the loaders are done with window w (= this window stored)
+      long long ua = u_lo;
+      HkItem ita;
+      bool hava = hk_next(p, ua, u_hi, ita);
+      int cha = 0, sb = 0;
+      auto issue = [&]() {
+        if (lane == 0)
+          hk_planes_issue(p, (long long)ita.pt * 256 + (long long)rank * 128 * ita.T, cha * kKC,
+                          sS + (uint32_t)sb * (uint32_t)p.pimg_max * p.pimg_bytes, sfull + sb);
         __syncwarp();
-        if (++ws == p.wslots) { ws = 0; ++wuse; }
+        sb ^= 1;
+        if (++cha == p.nchunks) { cha = 0; hava = hk_next(p, ua, u_hi, ita); }
+      };
+      for (int k = 0; k < 2 && hava; ++k) issue();
+      while (hk_next(p, u, u_hi, it)) {
+        for (int ch = 0; ch < p.nchunks; ++ch) {
+          hk_wait(wloc + ws, (uint32_t)(wuse & 1));
+          if (lane == 0) hk_arrive_cluster(wfull0 + (uint32_t)ws * 8u);
+          __syncwarp();
+          if (++ws == p.wslots) { ws = 0; ++wuse; }
+          if (hava) issue();
+        }
+      }
+    } else {
+      while (hk_next(p, u, u_hi, it)) {
+        for (int ch = 0; ch < p.nchunks; ++ch) {
+          hk_wait(wloc + ws, (uint32_t)(wuse & 1));
+          if (lane == 0) hk_arrive_cluster(wfull0 + (uint32_t)ws * 8u);
+          __syncwarp();
+          if (++ws == p.wslots) { ws = 0; ++wuse; }
+        }
       }
     }
   } else if (role == kRoleFwdE) {
@@ -886,7 +987,7 @@ size_t hankel_zero_bytes(const Geom& g) { return (size_t)32 * g.H * g.W + 256; }
 // The filter is resident in shared memory when its (single) block fits beside two windows,
 // else streamed by TMA through a ring of (chunk, tap) blocks.
 // kc16: 32-byte rows of 16 bf16 channels (SW32) for the small-C phase convolution (the stem)
-static HankelTiling hankel_tiling_core(const Geom& g, int fmt, int num_sms, int kc_small = 0) {
+static HankelTiling hankel_tiling_core(const Geom& g, int fmt, int num_sms, int kc_small = 0, bool planes = false) {
   HankelTiling t{};
   t.ok = false;
   if (fmt == FMT_F32) return t;
@@ -915,7 +1016,7 @@ static HankelTiling hankel_tiling_core(const Geom& g, int fmt, int num_sms, int 
   const bool no_res = env_int("POLYCONV_HK_STREAM", 0) != 0;
   const int acc1_mode = env_int("POLYCONV_HK_ACC1", -1);
   const int max_pairs = std::max(1, num_sms / 2);
-  const uint32_t fixed = 3072;  // alignment + barriers
+  const uint32_t fixed0 = 3072;  // alignment + barriers
   int NN = forceNN ? forceNN : (K16 <= 256 ? K16 : 256);
   bool found = false;
   for (int T = 4; T >= 1 && !found; T >>= 1) {
@@ -932,6 +1033,10 @@ static HankelTiling hankel_tiling_core(const Geom& g, int fmt, int num_sms, int 
     const int nblk = nchunks * RS;
     const int wrows = (128 * T + (g.R - 1) * pitch + g.S - 1 + 7) / 8 * 8;
     const uint32_t wslot = (uint32_t)wrows * rowb;
+    // plane-staged loader: two staging buffers of the images a window touches
+    const int pimg_max = planes ? (wrows + HS * pitch - 1) / (HS * pitch) + 1 : 0;
+    const uint32_t pimg_bytes = (uint32_t)(64 * g.H * g.W * 2);
+    const uint32_t fixed = fixed0 + (planes ? 2u * (uint32_t)pimg_max * pimg_bytes : 0u);
     bool resident = false;
     int wslots = 0, fslots = 0;
     // Resident only when streaming would re-read more filter bytes per window than the window
@@ -958,6 +1063,7 @@ static HankelTiling hankel_tiling_core(const Geom& g, int fmt, int num_sms, int 
     if (wslots < 2) continue;
     found = true;
     t.NN = NN; t.NB = NB; t.T = T; t.wrows = wrows; t.wslot_bytes = wslot; t.wslots = wslots;
+    t.planes = planes ? 1 : 0; t.pimg_max = pimg_max; t.pimg_bytes = pimg_bytes;
     t.resident = resident ? 1 : 0; t.fslots = fslots; t.fblk_bytes = fblk;
     t.npairs = (int)std::min<long long>(max_pairs, (long long)PT * NB);
   }
@@ -967,7 +1073,8 @@ static HankelTiling hankel_tiling_core(const Geom& g, int fmt, int num_sms, int 
   t.aligned = (!(g.W & 1) && pitch == g.W + 2 * g.pw && delta == (g.pw & 1) && g.C % (tf32 ? 4 : 8) == 0 &&
                env_int("POLYCONV_HK_GENERAL", 0) == 0) ? 1 : 0;
   t.Kp = t.NB * t.NN;
-  t.smem_bytes = (int)((size_t)t.fslots * t.fblk_bytes + (size_t)t.wslots * t.wslot_bytes + fixed);
+  t.smem_bytes = (int)((size_t)t.fslots * t.fblk_bytes + (size_t)t.wslots * t.wslot_bytes + fixed0 +
+                       (t.planes ? 2 * (size_t)t.pimg_max * t.pimg_bytes : 0));
   t.nacc = t.T * t.NN > 256 ? 1 : 2;
   const int tc = t.nacc * t.T * t.NN;
   t.tmem_cols = tc <= 32 ? 32 : tc <= 64 ? 64 : tc <= 128 ? 128 : tc <= 256 ? 256 : 512;
@@ -1024,6 +1131,16 @@ HankelTiling hankel_tiling(const Geom& g, int fmt, int num_sms, bool io_bf16) {
   }
   HankelTiling t = hankel_tiling_core(g, fmt, num_sms);
   t.phase = 0;
+  if (t.ok && !t.aligned && fmt == FMT_BF16 && io_bf16 && g.C % 64 == 0 && env_int("POLYCONV_HK_PLANES", 1) != 0) {
+    // small odd planes (7x7): whole (image, 64-channel) blocks by bulk copy instead of the
+    // element loader's two 4-byte loads per element
+    HankelTiling tp = hankel_tiling_core(g, fmt, num_sms, 0, true);
+    if (tp.ok && tp.T == t.T && tp.NN == t.NN) {
+      tp.phase = 0;
+      tp.aligned = 0;
+      return tp;
+    }
+  }
   return t;
 }
 
@@ -1089,6 +1206,7 @@ cudaError_t launch_mac_hankel(const Geom& g0, const HankelTiling& t, int fmt, co
   p.fsw.init((uint32_t)g.sw);
   p.phase = t.phase;
   p.xC = g0.C; p.xH = g0.H; p.xW = g0.W;
+  p.pimg_bytes = t.pimg_bytes; p.pimg_max = t.pimg_max;
   p.dbg = env_int("POLYCONV_HK_DEBUG", 0);
   // kHW2: -1 = general loader, 0 = pair-aligned loader with a runtime plane size, > 0 = the
   // plane size in words baked in (immediate channel offsets) for the ResNet / VGG planes
@@ -1109,6 +1227,8 @@ cudaError_t launch_mac_hankel(const Geom& g0, const HankelTiling& t, int fmt, co
     kern = t.kc == 16 ? mac_hankel_kernel<__nv_bfloat16, false, -2, 16> : mac_hankel_kernel<__nv_bfloat16, false, -2, 32>;
   } else if (t.phase) {
     kern = t.aligned ? mac_hankel_kernel<__nv_bfloat16, false, -2> : mac_hankel_kernel<__nv_bfloat16, false, -4>;
+  } else if (t.planes) {
+    kern = mac_hankel_kernel<__nv_bfloat16, false, kHkPlanes>;
   } else if (!t.aligned) {
     kern = tf32 ? mac_hankel_kernel<float, true, -1>
                 : (io_bf16 ? mac_hankel_kernel<__nv_bfloat16, false, -1> : mac_hankel_kernel<float, false, -1>);
