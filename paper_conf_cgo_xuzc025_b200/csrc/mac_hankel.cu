@@ -120,6 +120,7 @@ struct HkParams {
   // plane-staged loader (kHW2 == kHkPlanes): whole (image, 64-channel) blocks of x, bulk-copied
   uint32_t pimg_bytes;  // 64 * H * W * 2: one image's 64-channel block (16-byte multiple)
   int pimg_max;         // images a window can touch (staging buffer = pimg_max blocks)
+  int psbufs;           // staging buffers (2: the copies run one window ahead; 1 when smem is short)
   int dbg;  // POLYCONV_HK_DEBUG (timing ablations, results wrong): 1 loaders store zeros without
             // loading, 2 epilogue skips stores, 4 no MMAs (commits only), 8 per-CTA trace
 };
@@ -599,7 +600,7 @@ __global__ void __launch_bounds__(kHkThreads, 1)
   const uint32_t sW = sF + (uint32_t)p.fslots * p.fblk_bytes;           // window ring (1 KB aligned)
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + (size_t)p.fslots * p.fblk_bytes +
                                                (size_t)p.wslots * p.wslot_bytes +
-                                               (kHW2 == kHkPlanes ? 2 * (size_t)p.pimg_max * p.pimg_bytes : 0));
+                                               (kHW2 == kHkPlanes ? (size_t)p.psbufs * p.pimg_max * p.pimg_bytes : 0));
   uint64_t* ffull = bars;                    // [kHkMaxFBlk] leader: both halves landed
   uint64_t* fempty = ffull + kHkMaxFBlk;     // [kHkMaxFBlk] both: MMAs done with the block
   uint64_t* wfull = fempty + kHkMaxFBlk;     // [kHkMaxWSlots] leader: both CTAs' loaders done
@@ -771,7 +772,7 @@ __global__ void __launch_bounds__(kHkThreads, 1)
           if (!(p.dbg & 1))
             hk_planes_transpose(p, q0, sS + (uint32_t)sb * (uint32_t)p.pimg_max * p.pimg_bytes,
                                 sW + (uint32_t)ws * p.wslot_bytes, lw, lane, 2 * rp_lo, 2 * rp_hi);
-          if (++sb == 2) { sb = 0; ++suse; }
+          if (++sb == p.psbufs) { sb = 0; ++suse; }
           asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> MMA reads
           __syncwarp();
           if (lane == 0) mbar_arrive(wloc + ws);
@@ -816,8 +817,8 @@ __global__ void __launch_bounds__(kHkThreads, 1)
     HkItem it;
     int ws = 0, wuse = 0;
     if constexpr (kHW2 == kHkPlanes) {
-      // plane-staged loader: window w's blocks go to staging buffer w % 2; window w + 2's are
-      // fetched once the loaders are done with window w (= this window stored)
+      // plane-staged loader: window w's blocks go to staging buffer w % psbufs; window
+      // w + psbufs's are fetched once the loaders are done with window w (= this window stored)
       long long ua = u_lo;
       HkItem ita;
       bool hava = hk_next(p, ua, u_hi, ita);
@@ -827,10 +828,10 @@ __global__ void __launch_bounds__(kHkThreads, 1)
           hk_planes_issue(p, (long long)ita.pt * 256 + (long long)rank * 128 * ita.T, cha * kKC,
                           sS + (uint32_t)sb * (uint32_t)p.pimg_max * p.pimg_bytes, sfull + sb);
         __syncwarp();
-        sb ^= 1;
+        if (++sb == p.psbufs) sb = 0;
         if (++cha == p.nchunks) { cha = 0; hava = hk_next(p, ua, u_hi, ita); }
       };
-      for (int k = 0; k < 2 && hava; ++k) issue();
+      for (int k = 0; k < p.psbufs && hava; ++k) issue();
       while (hk_next(p, u, u_hi, it)) {
         for (int ch = 0; ch < p.nchunks; ++ch) {
           hk_wait(wloc + ws, (uint32_t)(wuse & 1));
@@ -987,7 +988,7 @@ size_t hankel_zero_bytes(const Geom& g) { return (size_t)32 * g.H * g.W + 256; }
 // The filter is resident in shared memory when its (single) block fits beside two windows,
 // else streamed by TMA through a ring of (chunk, tap) blocks.
 // kc16: 32-byte rows of 16 bf16 channels (SW32) for the small-C phase convolution (the stem)
-static HankelTiling hankel_tiling_core(const Geom& g, int fmt, int num_sms, int kc_small = 0, bool planes = false) {
+static HankelTiling hankel_tiling_core(const Geom& g, int fmt, int num_sms, int kc_small = 0, int planes = 0) {
   HankelTiling t{};
   t.ok = false;
   if (fmt == FMT_F32) return t;
@@ -1036,7 +1037,7 @@ static HankelTiling hankel_tiling_core(const Geom& g, int fmt, int num_sms, int 
     // plane-staged loader: two staging buffers of the images a window touches
     const int pimg_max = planes ? (wrows + HS * pitch - 1) / (HS * pitch) + 1 : 0;
     const uint32_t pimg_bytes = (uint32_t)(64 * g.H * g.W * 2);
-    const uint32_t fixed = fixed0 + (planes ? 2u * (uint32_t)pimg_max * pimg_bytes : 0u);
+    const uint32_t fixed = fixed0 + (uint32_t)planes * (uint32_t)pimg_max * pimg_bytes;  // planes = staging buffers
     bool resident = false;
     int wslots = 0, fslots = 0;
     // Resident only when streaming would re-read more filter bytes per window than the window
@@ -1063,7 +1064,7 @@ static HankelTiling hankel_tiling_core(const Geom& g, int fmt, int num_sms, int 
     if (wslots < 2) continue;
     found = true;
     t.NN = NN; t.NB = NB; t.T = T; t.wrows = wrows; t.wslot_bytes = wslot; t.wslots = wslots;
-    t.planes = planes ? 1 : 0; t.pimg_max = pimg_max; t.pimg_bytes = pimg_bytes;
+    t.planes = planes; t.pimg_max = pimg_max; t.pimg_bytes = pimg_bytes;
     t.resident = resident ? 1 : 0; t.fslots = fslots; t.fblk_bytes = fblk;
     t.npairs = (int)std::min<long long>(max_pairs, (long long)PT * NB);
   }
@@ -1074,7 +1075,7 @@ static HankelTiling hankel_tiling_core(const Geom& g, int fmt, int num_sms, int 
                env_int("POLYCONV_HK_GENERAL", 0) == 0) ? 1 : 0;
   t.Kp = t.NB * t.NN;
   t.smem_bytes = (int)((size_t)t.fslots * t.fblk_bytes + (size_t)t.wslots * t.wslot_bytes + fixed0 +
-                       (t.planes ? 2 * (size_t)t.pimg_max * t.pimg_bytes : 0));
+                       (size_t)t.planes * t.pimg_max * t.pimg_bytes);
   t.nacc = t.T * t.NN > 256 ? 1 : 2;
   const int tc = t.nacc * t.T * t.NN;
   t.tmem_cols = tc <= 32 ? 32 : tc <= 64 ? 64 : tc <= 128 ? 128 : tc <= 256 ? 256 : 512;
@@ -1131,14 +1132,17 @@ HankelTiling hankel_tiling(const Geom& g, int fmt, int num_sms, bool io_bf16) {
   }
   HankelTiling t = hankel_tiling_core(g, fmt, num_sms);
   t.phase = 0;
-  if (t.ok && !t.aligned && fmt == FMT_BF16 && io_bf16 && g.C % 64 == 0 && env_int("POLYCONV_HK_PLANES", 1) != 0) {
-    // small odd planes (7x7): whole (image, 64-channel) blocks by bulk copy instead of the
-    // element loader's two 4-byte loads per element
-    HankelTiling tp = hankel_tiling_core(g, fmt, num_sms, 0, true);
-    if (tp.ok && tp.T == t.T && tp.NN == t.NN) {
-      tp.phase = 0;
-      tp.aligned = 0;
-      return tp;
+  const int pl_mode = env_int("POLYCONV_HK_PLANES", 1);  // 0 off, 1 odd widths, 2 also even widths
+  if (t.ok && (!t.aligned || pl_mode >= 2) && fmt == FMT_BF16 && io_bf16 && g.C % 64 == 0 && pl_mode != 0) {
+    // small planes (7x7): whole (image, 64-channel) blocks by bulk copy instead of the element
+    // loader's two 4-byte loads per element; two staging buffers, else one
+    for (int nb = 2; nb >= 1; --nb) {
+      HankelTiling tp = hankel_tiling_core(g, fmt, num_sms, 0, nb);
+      if (tp.ok && tp.T == t.T && tp.NN == t.NN) {
+        tp.phase = 0;
+        tp.aligned = 0;
+        return tp;
+      }
     }
   }
   return t;
@@ -1206,7 +1210,7 @@ cudaError_t launch_mac_hankel(const Geom& g0, const HankelTiling& t, int fmt, co
   p.fsw.init((uint32_t)g.sw);
   p.phase = t.phase;
   p.xC = g0.C; p.xH = g0.H; p.xW = g0.W;
-  p.pimg_bytes = t.pimg_bytes; p.pimg_max = t.pimg_max;
+  p.pimg_bytes = t.pimg_bytes; p.pimg_max = t.pimg_max; p.psbufs = t.planes;
   p.dbg = env_int("POLYCONV_HK_DEBUG", 0);
   // kHW2: -1 = general loader, 0 = pair-aligned loader with a runtime plane size, > 0 = the
   // plane size in words baked in (immediate channel offsets) for the ResNet / VGG planes
