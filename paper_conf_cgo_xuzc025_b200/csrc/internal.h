@@ -178,6 +178,7 @@ struct HankelTiling {
   // plane-staged loader: whole (image, 64-channel) blocks of x by bulk copy, two staging buffers
   int planes, pimg_max;
   uint32_t pimg_bytes;
+  int rowtile;  // the stem: pitch 128, one output row per tile, TMA-stored epilogue
 };
 HankelTiling hankel_tiling(const Geom& g, int fmt, int num_sms, bool io_bf16);
 // x: NCHW input (io dtype); U: tap-major packed filter [RS][Kp][Cp] (t.Kp, t.Cp), packed by

@@ -117,6 +117,7 @@ struct HkParams {
   // phase-split input; N, C, H, W, ph, pw, sh, sw above are that convolution's, these are x's
   int phase;            // 0 / 1
   int xC, xH, xW;       // x dims (phase mode)
+  uint32_t rt_stage;    // kRowTile: bytes of one staged output tile (NN channels x Q pixels, bf16)
   // plane-staged loader (kHW2 == kHkPlanes): whole (image, 64-channel) blocks of x, bulk-copied
   uint32_t pimg_bytes;  // 64 * H * W * 2: one image's 64-channel block (16-byte multiple)
   int pimg_max;         // images a window can touch (staging buffer = pimg_max blocks)
@@ -590,9 +591,15 @@ __device__ __forceinline__ void hk_store<__nv_bfloat16>(__nv_bfloat16* y, long l
 // kScatter: the epilogue stores to every buffer of p.ys at channel offset p.koff of p.Ktot
 // (polyconv_forward_scatter); the plain forward (one output, its own channels) keeps the single
 // store path (a runtime output loop there cost up to 4 us per ResNet-50 layer, same-box A/B)
-template <typename IoT, bool kTf32, int kHW2, int kKC = (kTf32 ? 32 : 64), bool kScatter = false>
+// kRowTile (the stem): pitch 128 makes every 128-position tile one output row; the epilogue
+// stages the tile's NN channel rows (Q pixels each) in shared memory and one thread writes them
+// with a TMA tensor store (y as [N*K][P][Q]) instead of 2-byte stores (the stem was bound by
+// its epilogue stores)
+template <typename IoT, bool kTf32, int kHW2, int kKC = (kTf32 ? 32 : 64), bool kScatter = false,
+          bool kRowTile = false>
 __global__ void __launch_bounds__(kHkThreads, 1)
-    mac_hankel_kernel(const __grid_constant__ CUtensorMap tmU, const HkParams p) {
+    mac_hankel_kernel(const __grid_constant__ CUtensorMap tmU, const __grid_constant__ CUtensorMap tmY,
+                      const HkParams p) {
   extern __shared__ uint8_t smem_raw[];
   const uint32_t raw = smem_u32(smem_raw);
   uint8_t* smem = smem_raw + (((raw + 1023u) & ~1023u) - raw);
@@ -600,7 +607,9 @@ __global__ void __launch_bounds__(kHkThreads, 1)
   const uint32_t sW = sF + (uint32_t)p.fslots * p.fblk_bytes;           // window ring (1 KB aligned)
   uint64_t* bars = reinterpret_cast<uint64_t*>(smem + (size_t)p.fslots * p.fblk_bytes +
                                                (size_t)p.wslots * p.wslot_bytes +
-                                               (kHW2 == kHkPlanes ? (size_t)p.psbufs * p.pimg_max * p.pimg_bytes : 0));
+                                               (kHW2 == kHkPlanes ? (size_t)p.psbufs * p.pimg_max * p.pimg_bytes : 0) +
+                                               (kRowTile ? 2 * (size_t)p.rt_stage : 0));
+  const uint32_t sY = sW + (uint32_t)p.wslots * p.wslot_bytes;  // kRowTile: two staged output tiles
   uint64_t* ffull = bars;                    // [kHkMaxFBlk] leader: both halves landed
   uint64_t* fempty = ffull + kHkMaxFBlk;     // [kHkMaxFBlk] both: MMAs done with the block
   uint64_t* wfull = fempty + kHkMaxFBlk;     // [kHkMaxWSlots] leader: both CTAs' loaders done
@@ -876,12 +885,51 @@ __global__ void __launch_bounds__(kHkThreads, 1)
     const bool pq_const = kHW2 > 0 && PQ == 2LL * kHW2;
     long long u = u_lo;
     HkItem it;
-    int item = 0;
+    int item = 0, rt_buf = 0;
     while (hk_next(p, u, u_hi, it)) {
       const int a = p.nacc == 2 ? (item & 1) : 0;
       hk_wait(tfull + a, (uint32_t)((item / p.nacc) & 1));
       tc_fence_after();
       if (trace && e == 0 && lane == 0) tr[item == 0 ? 9 : 10] = global_ns();
+      if constexpr (kRowTile) {
+        // tile t = output row (n, oh) of the item's block of NN channels; lanes = pixels ow
+        for (int t = 0; t < it.T; ++t) {
+          const long long qt = (long long)it.pt * 256 + (long long)rank * 128 * it.T + t * 128;
+          const uint32_t vr = (uint32_t)(qt >> 7);
+          const uint32_t n = p.fHS.div(vr), oh = vr - n * (uint32_t)p.HS;
+          const bool row_ok = (int)n < p.N && (int)oh < p.P;
+          const uint32_t stg = sY + (uint32_t)(rt_buf & 1) * p.rt_stage;
+          if (e == 0 && lane == 0) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");  // buffer free
+          asm volatile("bar.sync 1, %0;" ::"n"(32 * kHkEpiWarps) : "memory");
+          const int ow = quad * 32 + lane;
+          const uint32_t trow = tbase + ((uint32_t)(quad * 32) << 16) + (uint32_t)(a * p.T * p.NN + t * p.NN);
+          for (int g = half; g * 16 < p.NN; g += 2) {
+            uint32_t v[16];
+            hk_tmem_ld16(trow + (uint32_t)(g * 16), v);
+            tmem_ld_wait();
+            if (row_ok && ow < p.Q && !(p.dbg & 2)) {
+#pragma unroll
+              for (int c = 0; c < 16; ++c) {
+                const uint32_t ad = stg + ((uint32_t)(g * 16 + c) * (uint32_t)p.Q + (uint32_t)ow) * 2u;
+                const unsigned short h = __bfloat16_as_ushort(__float2bfloat16_rn(__uint_as_float(v[c])));
+                asm volatile("st.shared.u16 [%0], %1;" ::"r"(ad), "h"(h) : "memory");
+              }
+            }
+          }
+          asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+          asm volatile("bar.sync 1, %0;" ::"n"(32 * kHkEpiWarps) : "memory");
+          if (e == 0 && lane == 0 && row_ok && !(p.dbg & 2)) {
+            const int c2 = (int)n * p.K + it.nb * p.NN;
+            asm volatile(
+                "cp.async.bulk.tensor.3d.global.shared::cta.bulk_group [%0, {%2, %3, %4}], [%1];" ::"l"(
+                    reinterpret_cast<uint64_t>(&tmY)),
+                "r"(stg), "r"(0), "r"((int)oh), "r"(c2)
+                : "memory");
+            asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+          }
+          ++rt_buf;
+        }
+      } else
       for (int t = 0; t < it.T; ++t) {
         // position of this lane -> output pixel (Eq. 12 / reading R4 / R16)
         const long long q = (long long)it.pt * 256 + (long long)rank * 128 * it.T + t * 128 + quad * 32 + lane;
@@ -941,6 +989,8 @@ __global__ void __launch_bounds__(kHkThreads, 1)
       if (trace && e == 0 && lane == 0) tr[item == 0 ? 5 : 7] = global_ns();
       ++item;
     }
+    (void)rt_buf;
+    if (kRowTile && e == 0 && lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
   }
   // teardown: every role done in both CTAs (remote arrivals land before the peer exits)
   tc_fence_before();
@@ -988,7 +1038,8 @@ size_t hankel_zero_bytes(const Geom& g) { return (size_t)32 * g.H * g.W + 256; }
 // The filter is resident in shared memory when its (single) block fits beside two windows,
 // else streamed by TMA through a ring of (chunk, tap) blocks.
 // kc16: 32-byte rows of 16 bf16 channels (SW32) for the small-C phase convolution (the stem)
-static HankelTiling hankel_tiling_core(const Geom& g, int fmt, int num_sms, int kc_small = 0, int planes = 0) {
+static HankelTiling hankel_tiling_core(const Geom& g, int fmt, int num_sms, int kc_small = 0, int planes = 0,
+                                       int force_pitch = 0, uint32_t extra_smem = 0, bool force_res = false) {
   HankelTiling t{};
   t.ok = false;
   if (fmt == FMT_F32) return t;
@@ -1001,7 +1052,7 @@ static HankelTiling hankel_tiling_core(const Geom& g, int fmt, int num_sms, int 
   // POLYCONV_HK_PITCH=1 / 2 forces W + pw / W + 2pw
   const int mode = env_int("POLYCONV_HK_PITCH", 0);
   const bool shared_cols = mode == 1 || (mode == 0 && (g.W & 1));
-  const int pitch = std::max(shared_cols ? g.W + g.pw : g.W + 2 * g.pw, g.S);
+  const int pitch = force_pitch ? force_pitch : std::max(shared_cols ? g.W + g.pw : g.W + 2 * g.pw, g.S);
   const int HS = g.H + g.ph;
   const int delta = (!(pitch & 1) && (g.pw & 1)) ? 1 : 0;
   const long long q_last = ((long long)(g.N - 1) * HS + (long long)g.sh * (g.P - 1)) * pitch +
@@ -1017,7 +1068,7 @@ static HankelTiling hankel_tiling_core(const Geom& g, int fmt, int num_sms, int 
   const bool no_res = env_int("POLYCONV_HK_STREAM", 0) != 0;
   const int acc1_mode = env_int("POLYCONV_HK_ACC1", -1);
   const int max_pairs = std::max(1, num_sms / 2);
-  const uint32_t fixed0 = 3072;  // alignment + barriers
+  const uint32_t fixed0 = 3072 + extra_smem;  // alignment + barriers (+ kRowTile staging)
   int NN = forceNN ? forceNN : (K16 <= 256 ? K16 : 256);
   bool found = false;
   for (int T = 4; T >= 1 && !found; T >>= 1) {
@@ -1044,7 +1095,7 @@ static HankelTiling hankel_tiling_core(const Geom& g, int fmt, int num_sms, int 
     // itself holds: otherwise a short filter ring leaves shared memory to L1, which the window
     // loaders' global loads hit (tools/hk_slots.sh: 64->64 56x56 resident 583 vs streamed 650
     // TFLOP/s; 128->128 28x28 resident 862 vs streamed 838).
-    const bool want_res = (size_t)nblk * fblk > wslot || env_int("POLYCONV_HK_RESIDENT", 0) != 0;
+    const bool want_res = (size_t)nblk * fblk > wslot || force_res || env_int("POLYCONV_HK_RESIDENT", 0) != 0;
     if (NB == 1 && nblk <= kHkMaxFBlk && !no_res && want_res &&
         (size_t)nblk * fblk + 2 * wslot + fixed <= (size_t)kHkSmemMax) {
       resident = true;
@@ -1111,6 +1162,19 @@ HankelTiling hankel_tiling(const Geom& g, int fmt, int num_sms, bool io_bf16) {
   if (g.sh == 2 && g.sw == 2 && fmt == FMT_BF16 && io_bf16 && g.W % 2 == 0 && (g.C % 32 == 0 || g.C <= 4) &&
       g.R - 1 >= g.ph && g.S - 1 >= g.pw && env_int("POLYCONV_HK_PHASE", 1) != 0) {
     const Geom e = hk_phase_geom(g);
+    if (e.C <= 16 && e.W + 2 * e.pw <= 128 && e.pw % 2 == 0 && (g.Q * 2) % 16 == 0 && g.K <= 256 &&
+        env_int("POLYCONV_HK_ROWTILE", 1) != 0) {
+      // the stem: one output row per 128-position tile, TMA-stored epilogue (kRowTile)
+      const int NNr = (g.K + 15) / 16 * 16;
+      HankelTiling t = hankel_tiling_core(e, fmt, num_sms, 16, 0, 128, 2u * (uint32_t)(NNr * g.Q * 2), true);
+      if (t.ok && t.NN == g.K && t.delta == 0) {
+        t.phase = 1;
+        t.rowtile = 1;
+        t.aligned = (e.W % 2 == 0 && t.delta == (e.pw & 1)) ? 1 : 0;
+        t.eC = e.C; t.eH = e.H; t.eW = e.W; t.eR = e.R; t.eS = e.S; t.eph = e.ph; t.epw = e.pw;
+        if (t.aligned) return t;
+      }
+    }
     HankelTiling t = hankel_tiling_core(e, fmt, num_sms, e.C <= 16 ? env_int("POLYCONV_HK_KC", 16) : 0);
     if (t.ok) {
       t.phase = 1;
@@ -1214,7 +1278,21 @@ cudaError_t launch_mac_hankel(const Geom& g0, const HankelTiling& t, int fmt, co
   p.dbg = env_int("POLYCONV_HK_DEBUG", 0);
   // kHW2: -1 = general loader, 0 = pair-aligned loader with a runtime plane size, > 0 = the
   // plane size in words baked in (immediate channel offsets) for the ResNet / VGG planes
-  void (*kern)(const CUtensorMap, const HkParams);
+  void (*kern)(const CUtensorMap, const CUtensorMap, const HkParams);
+  CUtensorMap tmY = tmU;  // kRowTile: y as [N*K][P][Q] bf16, boxes of Q pixels x 1 row x NN channels
+  if (t.rowtile) {
+    cuuint64_t dims[3] = {(cuuint64_t)g0.Q, (cuuint64_t)g0.P, (cuuint64_t)g0.N * g0.K};
+    cuuint64_t strides[2] = {(cuuint64_t)g0.Q * 2, (cuuint64_t)g0.P * g0.Q * 2};
+    cuuint32_t box[3] = {(cuuint32_t)g0.Q, 1, (cuuint32_t)t.NN};
+    cuuint32_t estr[3] = {1, 1, 1};
+    if (!enc || enc(&tmY, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 3, ys[0], dims, strides, box, estr,
+                    CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_NONE,
+                    CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS) {
+      snprintf(err, errlen, "mac_hankel: cuTensorMapEncodeTiled (y) failed");
+      return cudaErrorInvalidValue;
+    }
+  }
+  p.rt_stage = t.rowtile ? (uint32_t)(t.NN * g0.Q * 2) : 0u;
   const bool scatter = nys > 1 || ktot != g0.K || koff != 0;
   const int hw2 = g.H * g.W / 2;
   if (!t.phase && t.kc == 16) {
@@ -1223,6 +1301,12 @@ cudaError_t launch_mac_hankel(const Geom& g0, const HankelTiling& t, int fmt, co
       return cudaErrorInvalidValue;
     }
     kern = mac_hankel_kernel<__nv_bfloat16, false, 0, 16>;
+  } else if (t.phase && t.kc == 16 && t.rowtile) {
+    if (!io_bf16 || scatter) {
+      snprintf(err, errlen, "mac_hankel: row-tile mode needs bf16 output and one output buffer");
+      return cudaErrorInvalidValue;
+    }
+    kern = mac_hankel_kernel<__nv_bfloat16, false, -2, 16, false, true>;
   } else if (t.phase && t.kc < 64) {
     if (!t.aligned) {
       snprintf(err, errlen, "mac_hankel: small-C phase mode needs pair-aligned phase planes");
@@ -1280,7 +1364,7 @@ cudaError_t launch_mac_hankel(const Geom& g0, const HankelTiling& t, int fmt, co
   attr[1].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 2;
-  return cudaLaunchKernelEx(&cfg, kern, tmU, p);
+  return cudaLaunchKernelEx(&cfg, kern, tmU, tmY, p);
 }
 
 }  // namespace polyconv
