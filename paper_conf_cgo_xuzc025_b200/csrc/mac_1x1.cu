@@ -52,6 +52,7 @@ struct P1x1 {
   int resA;     // 1: each CTA keeps one 128-channel filter block resident (loaded once) and walks
                 //    its images / position blocks, so only the x planes stream through the ring
   int groups;   // resA: CTAs per filter block (gridDim.x = groups * num_kt)
+  int dbg;      // POLYCONV_1X1_DEBUG ablations (timing probes only): 1 no stores, 2 no MMA, 4 no x loads
 };
 
 // The CTA's i-th tile: (filter block kt, position block pb, image n).  resA: a CTA's tiles
@@ -144,8 +145,9 @@ __global__ void __launch_bounds__(k1Threads, 1)
       for (int kc = 0; kc < p.kchunks; ++kc) {
         mbar_wait(empty + st, ph ^ 1u);
         if (elect_one()) {
-          mbar_arrive_expect_tx(full + st, (p.resA ? 0u : p.a_bytes) + (uint32_t)p.nbox * 8192u);
+          mbar_arrive_expect_tx(full + st, (p.resA ? 0u : p.a_bytes) + ((p.dbg & 4) ? 0u : (uint32_t)p.nbox * 8192u));
           if (!p.resA) tma_load_2d(sA + (size_t)st * p.a_bytes, &tmU, full + st, kc * 64, kt * 128);
+          if (!(p.dbg & 4))
           for (int b = 0; b < p.nbox; ++b)
             tma_load_2d(sB + (size_t)st * p.b_bytes + (size_t)b * 8192, &tmX, full + st, pb * p.NT + b * 64,
                         n * p.C + kc * 64);
@@ -175,7 +177,7 @@ __global__ void __launch_bounds__(k1Threads, 1)
         if (elect_one()) {
 #pragma unroll
           for (int ks = 0; ks < 4; ++ks)  // K step: +32 B (K-major A), +2048 B (MN-major B)
-            umma<false>(d, ad + 2 * ks, bd + 128 * ks, p.idesc, (kc | ks) != 0 ? 1u : 0u);
+            if (!(p.dbg & 2)) umma<false>(d, ad + 2 * ks, bd + 128 * ks, p.idesc, (kc | ks) != 0 ? 1u : 0u);
           umma_commit(empty + st);
         }
         __syncwarp();
@@ -198,7 +200,7 @@ __global__ void __launch_bounds__(k1Threads, 1)
       const int nvalid = min(p.NT, p.HWo - pb * p.NT);
       const bool vec = (p.HWo & 7) == 0;  // 16-byte aligned 8-pixel groups
       // epi_tma (K % 32 == 0): the warp's 32 channels are all valid or all past K
-      const bool wvalid = kt * 128 + q * 32 < p.K;
+      const bool wvalid = kt * 128 + q * 32 < p.K && !(p.dbg & 1);
       uint8_t* stg = sE + (size_t)q * p.nbox * 4096;
       if (p.epi_tma) {
         if (lane == 0) asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");  // staging free
@@ -264,6 +266,7 @@ __global__ void __launch_bounds__(k1Threads, 1)
               asm volatile("cp.async.bulk.commit_group;" ::: "memory");
             }
           }
+        } else if (p.dbg & 1) {
         } else if (k < p.K && c < nvalid && (p.HWo & 3) != 0) {
 #pragma unroll
           for (int j = 0; j < 32; ++j)
@@ -439,6 +442,10 @@ cudaError_t launch_mac_1x1(const Geom& g, const void* x, const void* U, int Kp, 
   p.resA = (er == nullptr || er[0] != '0') && resA_bytes <= 96 * 1024 && p.num_kt <= num_sms &&
            (long long)g.N * p.num_pb >= num_sms / p.num_kt;
   p.groups = p.resA ? num_sms / p.num_kt : 0;
+  {
+    const char* ed = getenv("POLYCONV_1X1_DEBUG");
+    p.dbg = ed ? atoi(ed) : 0;
+  }
   p.stages = p.resA ? std::min(k1MaxStages, (227 * 1024 - 2048 - estage - resA_bytes) / (int)p.b_bytes)
                     : std::min(k1MaxStages, (227 * 1024 - 2048 - estage) / per);
   if (p.stages < 2) {

@@ -135,7 +135,7 @@ polyconv_status_t resolve(polyconv_plan_t p) {
       g.sh == 1 && g.sw == 1 && g.ph == 0 && g.pw == 0 && mac1x1_pitch(g) != 0 && g.C >= 512 &&
       g.C >= 2 * g.K && !getenv("POLYCONV_NO_HANKEL")) {
     const HankelTiling h = hankel_tiling(g, p->fmt, p->num_sms, p->io_bf16);
-    if (h.ok && h.aligned && (long long)h.PT * h.NB >= 24) k = POLYCONV_KERNEL_TC_HANKEL;
+    if (h.ok && (h.aligned || h.planes) && (long long)h.PT * h.NB >= 24) k = POLYCONV_KERNEL_TC_HANKEL;
   }
   if (k == POLYCONV_KERNEL_AUTO && mac1x1_supported(g, p->fmt, p->io_bf16) && !getenv("POLYCONV_NO_1X1") &&
       mac1x1_auto(g))

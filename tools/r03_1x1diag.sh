@@ -1,0 +1,7 @@
+# 1x1 layers on 14x14 / 7x7 planes: kernel choice and mac_1x1 ablations (POLYCONV_1X1_DEBUG)
+python -c "import __graft_entry__ as g; g.build()" > gpurun_out/r03_build.log 2>&1 || exit 1
+L=gpurun_out/r03_1x1diag.log; rm -f $L
+for SHAPE in "256 256 14 14 1024 1 1 1 0" "256 1024 14 14 256 1 1 1 0" "256 512 7 7 2048 1 1 1 0" "256 2048 7 7 512 1 1 1 0" "256 1024 14 14 512 1 1 1 0" "256 1024 14 14 2048 1 1 2 0" "256 128 28 28 512 1 1 1 0"; do
+  for KER in auto tc_1x1 tc_hankel tc tc_pair; do echo "== $SHAPE $KER" >> $L; HK_KERNEL=$KER HK_DBGS="0" timeout 120 python tools/hk_trace.py $SHAPE >> $L 2>&1; done
+  for D in 1 2 4 7; do echo "== $SHAPE tc_1x1 dbg=$D" >> $L; POLYCONV_1X1_DEBUG=$D HK_KERNEL=tc_1x1 HK_DBGS="0" timeout 120 python tools/hk_trace.py $SHAPE >> $L 2>&1; done
+done
