@@ -28,7 +28,11 @@ namespace polyconv {
 
 namespace {
 
-constexpr int BP = 256, BK = 32, NT = 128;
+#ifndef PC_F32_KW
+#define PC_F32_KW 8
+#endif
+constexpr int KW = PC_F32_KW;            // output channels per warp
+constexpr int BP = 256, BK = 4 * KW, NT = 128;
 
 struct F32Geo {
   int pitch, HS, WU, CC;
@@ -117,9 +121,9 @@ __global__ void __launch_bounds__(NT, 4) mac_fp32_kernel(Geom g, F32Geo f, const
 
   // accumulators as position pairs: one packed FFMA2 (fma.rn.f32x2, sm_100) per channel and
   // pair -- the same round-to-nearest fp32 FMAs as two FFMA, half the issue slots
-  float2 acc[8][4];
+  float2 acc[KW][4];
 #pragma unroll
-  for (int a = 0; a < 8; ++a)
+  for (int a = 0; a < KW; ++a)
 #pragma unroll
     for (int b = 0; b < 4; ++b) acc[a][b] = make_float2(0.f, 0.f);
 
@@ -137,20 +141,23 @@ __global__ void __launch_bounds__(NT, 4) mac_fp32_kernel(Geom g, F32Geo f, const
     const int ccn = min(CC, g.C - ch * CC);
     for (int cc = 0; cc < ccn; ++cc) {
       const float* win = s_win + (b * CC + cc) * WU + lane;
-      const float* wr = s_w + ((b * CC + cc) * RS) * BK + warp * 8;
+      const float* wr = s_w + ((b * CC + cc) * RS) * BK + warp * KW;
 #pragma unroll(RT ? RT : 1)
       for (int i = 0; i < R; ++i) {
 #pragma unroll(ST ? ST : 1)
         for (int j = 0; j < S; ++j) {
-          const float4 w0 = *reinterpret_cast<const float4*>(wr + (i * S + j) * BK);
-          const float4 w1 = *reinterpret_cast<const float4*>(wr + (i * S + j) * BK + 4);
-          const float wv[8] = {w0.x, w0.y, w0.z, w0.w, w1.x, w1.y, w1.z, w1.w};
+          float wv[KW];
+#pragma unroll
+          for (int a4 = 0; a4 < KW; a4 += 4) {
+            const float4 w4 = *reinterpret_cast<const float4*>(wr + (i * S + j) * BK + a4);
+            wv[a4] = w4.x; wv[a4 + 1] = w4.y; wv[a4 + 2] = w4.z; wv[a4 + 3] = w4.w;
+          }
           float2 av[4];
 #pragma unroll
           for (int bb = 0; bb < 4; ++bb)
             av[bb] = make_float2(win[i * f.pitch + j + 64 * bb], win[i * f.pitch + j + 64 * bb + 32]);
 #pragma unroll
-          for (int a = 0; a < 8; ++a)
+          for (int a = 0; a < KW; ++a)
 #pragma unroll
             for (int bb = 0; bb < 4; ++bb) acc[a][bb] = __ffma2_rn(make_float2(wv[a], wv[a]), av[bb], acc[a][bb]);
         }
@@ -174,8 +181,8 @@ __global__ void __launch_bounds__(NT, 4) mac_fp32_kernel(Geom g, F32Geo f, const
     const long long PQ = (long long)g.P * g.Q;
     const long long ybase = (long long)n * g.K * PQ + (long long)oh * g.Q + ow;
 #pragma unroll
-    for (int a = 0; a < 8; ++a) {
-      const int k = k0 + warp * 8 + a;
+    for (int a = 0; a < KW; ++a) {
+      const int k = k0 + warp * KW + a;
       if (k < g.K) y[ybase + (long long)k * PQ] = (bb & 1) ? acc[a][bb >> 1].y : acc[a][bb >> 1].x;
     }
   }
