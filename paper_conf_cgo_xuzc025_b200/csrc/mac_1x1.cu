@@ -330,9 +330,47 @@ __global__ void __launch_bounds__(256) gather1x1_kernel(const __nv_bfloat16* __r
   // stride 1: the plane is one contiguous run, copied with 8-byte loads when its element
   // offsets are multiples of 4 (ResNet-50 14x14: 18.4 -> 9 us for 25.7 MB)
   const bool contig = sh == 1 && sw == 1 && Q == W && (PQ & 3) == 0;
+  // stride 1, any plane size: the 8 elements of a vector are consecutive in x (offset e, any
+  // alignment) -- two aligned 16-byte loads and a funnel shift (adjacent lanes' loads overlap
+  // in L1; x is read from HBM once)
+  const bool funnel = sh == 1 && sw == 1 && Q == W && (PQ & 3) != 0;
+  const long long xtotal = rows * H * W;
   for (long long v = (long long)blockIdx.x * 256 + threadIdx.x; v < nvec; v += (long long)gridDim.x * 256) {
     const long long r = v / vpr;
     const int m0 = (int)(v - r * vpr) * 8;
+    if (funnel) {
+      uint32_t o4[4] = {0u, 0u, 0u, 0u};
+      if (m0 < PQ) {
+        const long long e = r * PQ + m0, a = e & ~7LL;
+        const int sft = (int)(e - a);
+        const uint4* x4 = reinterpret_cast<const uint4*>(xs);
+        auto vec = [&](long long a8) {  // x[a8 .. a8 + 8), nothing read past the tensor
+          if (a8 + 8 <= xtotal) return __ldg(x4 + (a8 >> 3));
+          uint32_t t[4] = {0u, 0u, 0u, 0u};
+          for (int j = 0; j < 8 && a8 + j < xtotal; ++j) t[j >> 1] |= (uint32_t)xs[a8 + j] << (16 * (j & 1));
+          return make_uint4(t[0], t[1], t[2], t[3]);
+        };
+        const uint4 lo = vec(a);
+        const uint4 hi = vec(a + 8);
+        const uint32_t w[8] = {lo.x, lo.y, lo.z, lo.w, hi.x, hi.y, hi.z, hi.w};
+        const int hw = sft >> 1;
+        uint32_t o[5];
+#pragma unroll
+        for (int i = 0; i < 5; ++i)
+          o[i] = hw == 0 ? w[i] : hw == 1 ? w[i + 1] : hw == 2 ? w[i + 2] : w[i + 3 < 8 ? i + 3 : 7];
+#pragma unroll
+        for (int i = 0; i < 4; ++i) o4[i] = (sft & 1) ? __funnelshift_r(o[i], o[i + 1], 16) : o[i];
+        if (m0 + 8 > PQ) {  // the plane's last vector: zeros past PQ
+#pragma unroll
+          for (int i = 0; i < 4; ++i) {
+            if (m0 + 2 * i >= PQ) o4[i] = 0u;
+            else if (m0 + 2 * i + 1 >= PQ) o4[i] &= 0xFFFFu;
+          }
+        }
+      }
+      xq[v] = make_uint4(o4[0], o4[1], o4[2], o4[3]);
+      continue;
+    }
     const uint16_t* src = xs + r * H * W;
     if (contig && m0 + 8 <= PQ) {
       const uint2* s2 = reinterpret_cast<const uint2*>(src + m0);
