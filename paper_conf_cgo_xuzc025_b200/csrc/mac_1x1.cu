@@ -53,6 +53,7 @@ struct P1x1 {
                 //    its images / position blocks, so only the x planes stream through the ring
   int groups;   // resA: CTAs per filter block (gridDim.x = groups * num_kt)
   int dbg;      // POLYCONV_1X1_DEBUG ablations (timing probes only): 1 no stores, 2 no MMA, 4 no x loads
+  int gimg, NG; // images per tile (planes of <= 64 pixels: one 64-position box each) and image groups
 };
 
 // The CTA's i-th tile: (filter block kt, position block pb, image n).  resA: a CTA's tiles
@@ -62,7 +63,7 @@ __device__ __forceinline__ bool tile_of(const P1x1& p, int i, int& kt, int& pb, 
   if (p.resA) {
     kt = blockIdx.x % p.num_kt;
     rest = blockIdx.x / p.num_kt + i * p.groups;
-    if (rest >= p.N * p.num_pb) return false;
+    if (rest >= p.NG * p.num_pb) return false;
   } else {
     const long long t = blockIdx.x + (long long)i * gridDim.x;
     if (t >= p.num_tiles) return false;
@@ -149,8 +150,9 @@ __global__ void __launch_bounds__(k1Threads, 1)
           if (!p.resA) tma_load_2d(sA + (size_t)st * p.a_bytes, &tmU, full + st, kc * 64, kt * 128);
           if (!(p.dbg & 4))
           for (int b = 0; b < p.nbox; ++b)
-            tma_load_2d(sB + (size_t)st * p.b_bytes + (size_t)b * 8192, &tmX, full + st, pb * p.NT + b * 64,
-                        n * p.C + kc * 64);
+            tma_load_2d(sB + (size_t)st * p.b_bytes + (size_t)b * 8192, &tmX, full + st,
+                        p.gimg > 1 ? 0 : pb * p.NT + b * 64,
+                        (p.gimg > 1 ? (n * p.gimg + b) * p.C : n * p.C) + kc * 64);  // past N: zero fill
         }
         __syncwarp();
         if (++st == p.stages) { st = 0; ph ^= 1u; }
@@ -212,20 +214,22 @@ __global__ void __launch_bounds__(k1Threads, 1)
         tmem_ld_wait();
         if (p.epi_tma == 2) {
           // plane `lane` of the warp's dense [32][HWo] run; positions past HWo are not stored
+          // gimg > 1: box c/64 is image n*gimg + c/64, staged as its own dense run
+          const int cb = p.gimg > 1 ? (c & 63) : c;
           if (wvalid) {
-            uint8_t* row = stg + (size_t)lane * p.HWo * 2;
+            uint8_t* row = stg + (size_t)(p.gimg > 1 ? (c >> 6) * 4096 : 0) + (size_t)lane * p.HWo * 2;
             if ((p.HWo & 1) == 0) {
 #pragma unroll
               for (int j = 0; j < 32; j += 2)
-                if (c + j < p.HWo) {
+                if (cb + j < p.HWo) {
                   const __nv_bfloat162 h2 = __floats2bfloat162_rn(__uint_as_float(v[j]), __uint_as_float(v[j + 1]));
-                  *reinterpret_cast<__nv_bfloat162*>(row + (c + j) * 2) = h2;
+                  *reinterpret_cast<__nv_bfloat162*>(row + (cb + j) * 2) = h2;
                 }
             } else {
 #pragma unroll
               for (int j = 0; j < 32; ++j)
-                if (c + j < p.HWo)
-                  *reinterpret_cast<__nv_bfloat16*>(row + (c + j) * 2) = __float2bfloat16_rn(__uint_as_float(v[j]));
+                if (cb + j < p.HWo)
+                  *reinterpret_cast<__nv_bfloat16*>(row + (cb + j) * 2) = __float2bfloat16_rn(__uint_as_float(v[j]));
             }
           }
           if (c + 32 >= p.NT) {
@@ -233,10 +237,14 @@ __global__ void __launch_bounds__(k1Threads, 1)
             __syncwarp();
             if (lane == 0 && wvalid) {
               const uint32_t bytes = 64u * (uint32_t)p.HWo;  // 32 planes x HWo x 2 B, a multiple of 16
-              __nv_bfloat16* dst = y + ((long long)n * p.K + kt * 128 + q * 32) * p.HWo;
-              asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst),
-                           "r"(smem_u32(stg)), "r"(bytes)
-                           : "memory");
+              for (int b = 0; b < p.gimg; ++b) {
+                const int ni = n * p.gimg + b;
+                if (ni >= p.N) break;
+                __nv_bfloat16* dst = y + ((long long)ni * p.K + kt * 128 + q * 32) * p.HWo;
+                asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst),
+                             "r"(smem_u32(stg + (size_t)b * 4096)), "r"(bytes)
+                             : "memory");
+              }
               asm volatile("cp.async.bulk.commit_group;" ::: "memory");
             }
           }
@@ -455,11 +463,19 @@ cudaError_t launch_mac_1x1(const Geom& g, const void* x, const void* U, int Kp, 
   p.HW = pitch ? pitch : g.H * g.W;  // x (direct) or the gathered copy
   p.HWo = g.P * g.Q;
   p.NT = p.HWo >= 256 ? 256 : (p.HWo + 63) / 64 * 64;
+  // planes of <= 64 pixels: four images per tile (one 64-position box each), so a streamed
+  // filter block serves four images and the MMAs run at N = 256 (POLYCONV_1X1_GIMG=0: one image)
+  const char* eg = getenv("POLYCONV_1X1_GIMG");
+  const bool gep = g.K % 32 == 0 && (reinterpret_cast<uintptr_t>(y) & 15) == 0 &&
+                   (getenv("POLYCONV_1X1_EPI_TMA") == nullptr || getenv("POLYCONV_1X1_EPI_TMA")[0] != '0');
+  p.gimg = (p.HWo <= 64 && g.N > 1 && gep && (eg == nullptr || eg[0] != '0')) ? 4 : 1;
+  if (p.gimg > 1) p.NT = 256;
+  p.NG = (g.N + p.gimg - 1) / p.gimg;
   p.nbox = p.NT / 64;
   p.kchunks = Cp / 64;
-  p.num_pb = (p.HWo + p.NT - 1) / p.NT;
+  p.num_pb = p.gimg > 1 ? 1 : (p.HWo + p.NT - 1) / p.NT;
   p.num_kt = Kp / 128;
-  const long long tiles = (long long)g.N * p.num_pb * p.num_kt;
+  const long long tiles = (long long)p.NG * p.num_pb * p.num_kt;
   if (tiles >= (1LL << 31) || p.kchunks < 1) {
     snprintf(err, errlen, "mac_1x1: unsupported shape");
     return cudaErrorInvalidValue;
@@ -472,13 +488,17 @@ cudaError_t launch_mac_1x1(const Geom& g, const void* x, const void* U, int Kp, 
   const char* ev = getenv("POLYCONV_1X1_EPI_TMA");
   const bool ep_ok = g.K % 32 == 0 && (reinterpret_cast<uintptr_t>(y) & 15) == 0 && (ev == nullptr || ev[0] != '0');
   p.epi_tma = !ep_ok ? 0 : (p.num_pb == 1 && g.K % 8 == 0) ? 2 : (p.HWo % 8 == 0 ? 1 : 0);
+  if (p.gimg > 1 && p.epi_tma != 2) {
+    snprintf(err, errlen, "mac_1x1: multi-image tiles need the staged epilogue");
+    return cudaErrorInvalidValue;
+  }
   const int estage = p.epi_tma ? p.nbox * 16384 : 0;
   // resident filter block: every CTA's tiles share one 128-channel block, which is loaded
   // once, so only x streams (C <= 384: at most 96 KB; POLYCONV_1X1_RESA=0 turns it off)
   const char* er = getenv("POLYCONV_1X1_RESA");
   const int resA_bytes = p.kchunks * (int)p.a_bytes;
   p.resA = (er == nullptr || er[0] != '0') && resA_bytes <= 96 * 1024 && p.num_kt <= num_sms &&
-           (long long)g.N * p.num_pb >= num_sms / p.num_kt;
+           (long long)p.NG * p.num_pb >= num_sms / p.num_kt;
   p.groups = p.resA ? num_sms / p.num_kt : 0;
   {
     const char* ed = getenv("POLYCONV_1X1_DEBUG");

@@ -78,6 +78,10 @@ bool mac1x1_auto(const Geom& g) {
   if (mac1x1_pitch(g) == 0 || g.sh > 1 || g.sw > 1) return true;
   const char* ev = getenv("POLYCONV_1X1_SMALL");
   if (ev) return ev[0] != '0';
+  // planes of <= 64 pixels run four images per tile (mac_1x1 gimg) when K % 32 == 0: then the
+  // expansion layers win too (ResNet-50 512->2048 7x7 N=256: 63.6 vs 80.9 us for mac_tc2; N=32:
+  // 21.5 vs 31.8); one image per tile lost them to mac_tc2
+  if ((long long)g.P * g.Q <= 64 && g.N > 1 && g.K % 32 == 0) return true;
   return !((long long)g.P * g.Q < 64 && g.K > g.C);
 }
 

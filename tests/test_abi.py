@@ -106,7 +106,11 @@ def test_kernel_selection_and_forcing():
     assert k1((256, 256, 14, 14), (1024, 256, 1, 1))["kernel"] == "tc_1x1"
     assert k1((4, 256, 28, 28), (512, 256, 1, 1), 2)["kernel"] == "tc_1x1"
     assert k1((4, 1024, 7, 7), (512, 1024, 1, 1))["kernel"] == "tc_1x1"
-    assert k1((4, 512, 7, 7), (2048, 512, 1, 1))["kernel"] == "tc"
+    # planes of <= 64 pixels with K % 32 == 0: four images per mac_1x1 tile, expansions included
+    # (ResNet-50 512->2048 7x7 N=256: 63.6 us vs 80.9 for mac_tc2, profiles/r03_1x1_gimg.log)
+    assert k1((4, 512, 7, 7), (2048, 512, 1, 1))["kernel"] == "tc_1x1"
+    assert k1((1, 512, 7, 7), (2048, 512, 1, 1))["kernel"] == "tc"     # one image: the old rule
+    assert k1((4, 512, 7, 7), (2040, 512, 1, 1))["kernel"] == "tc"     # K % 32 != 0
     # bf16 in/out (profiles/r02_kcmp_*.jsonl): mac_hankel for 3x3 / 5x5 from 24 pair
     # units, stride 1 or 2; odd plane widths, 7x7 kernels and sub-round problems keep the
     # earlier rules (pack + mac_tc2 below one round of pair tiles, in-kernel packing for 3x3

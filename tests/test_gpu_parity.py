@@ -405,6 +405,7 @@ def test_1x1_planes_as_operand(shape, epi, monkeypatch):
                                    ConvShape("k1g_10x9", 2, 130, 10, 9, 160, 1, 1),            # 90 px, 3 chunks
                                    ConvShape("k1g_rows", 80, 1024, 7, 7, 32, 1, 1),            # many planes, odd size
                                    ConvShape("k1g_5x5_tail", 1, 3, 5, 5, 16, 1, 1),            # x ends mid-vector
+                                   ConvShape("k1g_7_n7", 7, 64, 7, 7, 64, 1, 1),               # 4-image tiles, ragged group
                                    ConvShape("k1g_big", 1, 2, 160, 160, 32, 1, 1, 2, 2, 0, 0)],  # plane past the stage
                          ids=lambda s: s.name)
 def test_1x1_gathered(shape):
