@@ -15,5 +15,6 @@ run hk_conv3x mac_hankel python tools/hk_one.py 32 128 28 28 128 3 3
 run hk_l4 mac_hankel python tools/hk_one.py 256 512 7 7 512 3 3
 run hk_l1 mac_hankel python tools/hk_one.py 256 64 56 56 64 3 3
 run hk_stem mac_hankel python tools/hk_one.py 256 3 224 224 64 7 7 2 3
-run hk_l2 mac_hankel python tools/hk_one.py 256 128 28 28 128 3 3
-run hk_l3 mac_hankel python tools/hk_one.py 256 256 14 14 256 3 3
+
+
+run 1x1_l4x mac_1x1 python tools/hk_one.py 256 512 7 7 2048 1 1 1 0
