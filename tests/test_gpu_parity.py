@@ -406,6 +406,8 @@ def test_1x1_planes_as_operand(shape, epi, monkeypatch):
                                    ConvShape("k1g_rows", 80, 1024, 7, 7, 32, 1, 1),            # many planes, odd size
                                    ConvShape("k1g_5x5_tail", 1, 3, 5, 5, 16, 1, 1),            # x ends mid-vector
                                    ConvShape("k1g_7_n7", 7, 64, 7, 7, 64, 1, 1),               # 4-image tiles, ragged group
+                                   ConvShape("k1g_5x5_c8", 5, 8, 5, 5, 32, 1, 1),              # 4-image tiles, C < 64, 25 px
+                                   ConvShape("k1g_s2_8x8", 6, 64, 16, 16, 160, 1, 1, 2, 2, 0, 0),  # 4-image, 2 k-tiles
                                    ConvShape("k1g_s2_56", 2, 64, 56, 56, 96, 1, 1, 2, 2, 0, 0),  # s2, 16-byte groups
                                    ConvShape("k1g_s2_24", 3, 40, 24, 20, 64, 1, 1, 2, 2, 0, 0),  # s2, Q = 10: 8-byte
                                    ConvShape("k1g_big", 1, 2, 160, 160, 32, 1, 1, 2, 2, 0, 0)],  # plane past the stage
