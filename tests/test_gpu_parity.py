@@ -427,7 +427,8 @@ def test_1x1_gathered(shape):
     (ConvShape("host_pair", 7, 64, 28, 28, 64, 3, 3, 1, 1, 1, 1), "bf16", "bf16"),   # 4 chunks, tail of 1
     (ConvShape("host_1x1", 6, 64, 16, 16, 128, 1, 1), "bf16", "bf16"),              # 3 chunks of 2
     (ConvShape("host_fp32", 5, 16, 12, 12, 32, 3, 3, 1, 1, 1, 1), "fp32", "f32"),  # 3 chunks, tail 1
-    (ConvShape("host_s2", 4, 16, 15, 15, 32, 7, 7, 2, 2, 3, 3), "bf16", "bf16")],    # polyphase: one piece
+    (ConvShape("host_s2", 4, 16, 15, 15, 32, 7, 7, 2, 2, 3, 3), "bf16", "bf16"),    # polyphase: one piece
+    (ConvShape("host_n18", 18, 32, 12, 12, 64, 3, 3, 1, 1, 1, 1), "bf16", "bf16")],  # chunks 5,5,5,3
     ids=lambda v: v.name if isinstance(v, ConvShape) else str(v))
 @pytest.mark.parametrize("chunks", ["default", "1"])
 def test_forward_host_pipeline(shape, math, io, chunks, monkeypatch):
