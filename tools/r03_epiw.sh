@@ -1,6 +1,6 @@
 python -c "import __graft_entry__ as g; g.build()" > gpurun_out/r03_build.log 2>&1 || exit 1
 timeout 600 python -m pytest tests/test_gpu_parity.py tests/test_gpu_coverage.py -m gpu -x -q -k "1x1" > gpurun_out/r03_pytest_1x1.log 2>&1; echo "pytest rc=$?"; tail -2 gpurun_out/r03_pytest_1x1.log
-L=gpurun_out/r03_epiw2.log; rm -f $L
+L=gpurun_out/r03_epi2ld.log; rm -f $L
 for SHAPE in "256 128 28 28 512 1 1 1 0" "256 512 28 28 128 1 1 1 0" "256 64 56 56 256 1 1 1 0" "256 256 56 56 64 1 1 1 0" "256 256 56 56 128 1 1 1 0" "256 64 56 56 64 1 1 1 0"; do
   for V in v1 new v1 new; do
     if [ $V = v1 ]; then lib=$PWD/ab_tmp/libs/v1.so; else lib=""; fi
